@@ -1,0 +1,147 @@
+"""CPU oracle for exhaustive best-improvement 2-opt (TEST INFRASTRUCTURE ONLY).
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl
+reference legs may import this package.  It wraps oracle/tsp2opt_oracle.c
+(plain C, int64, OpenMP over the j loop) via ctypes and shares no code with
+the CUDA path in paper_conf_ipps_rockis13_b200/.
+
+Functions mirror the C file; each cites the passage it follows there.
+Parity pins: tests/test_oracle.py.  `parity unpinned`: none.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "tsp2opt_oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+_lock = threading.Lock()
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile the oracle with gcc (plain -O2, OpenMP)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(
+            ["gcc", "-O2", "-fopenmp", "-shared", "-fPIC", "-std=c11", "-o", tmp, _SRC, "-lm"]
+        )
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+def _load():
+    global _lib
+    with _lock:
+        if _lib is None:
+            build()
+            lib = ctypes.CDLL(_LIB)
+            i64 = ctypes.c_int64
+            p = ctypes.c_void_p
+            lib.oracle_isqrt.argtypes = [i64]
+            lib.oracle_isqrt.restype = i64
+            lib.oracle_nint_sqrt.argtypes = [i64]
+            lib.oracle_nint_sqrt.restype = i64
+            lib.oracle_dist.argtypes = [i64, i64, i64, i64]
+            lib.oracle_dist.restype = i64
+            lib.oracle_tour_length.argtypes = [p, i64, p]
+            lib.oracle_tour_length.restype = i64
+            lib.oracle_delta.argtypes = [p, i64, p, i64, i64]
+            lib.oracle_delta.restype = i64
+            lib.oracle_cell.argtypes = [i64, i64]
+            lib.oracle_cell.restype = i64
+            lib.oracle_best_move.argtypes = [p, i64, p, p, p, p]
+            lib.oracle_best_move.restype = None
+            lib.oracle_apply.argtypes = [p, i64, i64]
+            lib.oracle_apply.restype = None
+            lib.oracle_local_search.argtypes = [p, i64, p, i64, p, p, p, i64]
+            lib.oracle_local_search.restype = ctypes.c_int
+            lib.oracle_num_threads.argtypes = []
+            lib.oracle_num_threads.restype = ctypes.c_int
+            _lib = lib
+    return _lib
+
+
+def _xy(coords) -> np.ndarray:
+    a = np.ascontiguousarray(np.asarray(coords, dtype=np.int32).reshape(-1, 2))
+    return a
+
+
+def _ptr(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+def nint_sqrt(s: int) -> int:
+    return int(_load().oracle_nint_sqrt(int(s)))
+
+
+def isqrt(s: int) -> int:
+    return int(_load().oracle_isqrt(int(s)))
+
+
+def dist(a, b) -> int:
+    return int(_load().oracle_dist(int(a[0]), int(a[1]), int(b[0]), int(b[1])))
+
+
+def tour_length(coords, tour) -> int:
+    xy = _xy(coords)
+    t = np.ascontiguousarray(tour, dtype=np.int32)
+    return int(_load().oracle_tour_length(_ptr(xy), xy.shape[0], _ptr(t)))
+
+
+def delta(coords, tour, i: int, j: int) -> int:
+    xy = _xy(coords)
+    t = np.ascontiguousarray(tour, dtype=np.int32)
+    return int(_load().oracle_delta(_ptr(xy), xy.shape[0], _ptr(t), i, j))
+
+
+def cell(i: int, j: int) -> int:
+    return int(_load().oracle_cell(i, j))
+
+
+def best_move(coords, tour):
+    """(i, j, delta) of the best 2-opt move of `tour` (Fig. 3 tie-break)."""
+    xy = _xy(coords)
+    t = np.ascontiguousarray(tour, dtype=np.int32)
+    out = np.zeros(3, dtype=np.int64)
+    _load().oracle_best_move(
+        _ptr(xy), xy.shape[0], _ptr(t),
+        _ptr(out[0:1]), _ptr(out[1:2]), _ptr(out[2:3]),
+    )
+    return int(out[0]), int(out[1]), int(out[2])
+
+
+def apply(tour, i: int, j: int) -> np.ndarray:
+    """Return a copy of `tour` with positions i+1..j reversed."""
+    t = np.array(tour, dtype=np.int32, copy=True)
+    _load().oracle_apply(_ptr(t), i, j)
+    return t
+
+
+def local_search(coords, tour, max_iters: int = -1, trace_cap: int = 0):
+    """Best-improvement 2-opt to a local minimum.
+
+    Returns dict(tour, length, iterations, status, trace) where status is 0 at
+    a local minimum and 1 when `max_iters` moves were applied and an improving
+    move still remains; trace is int64[min(iterations, trace_cap), 3] (i, j, delta).
+    """
+    xy = _xy(coords)
+    t = np.array(tour, dtype=np.int32, copy=True)
+    out = np.zeros(2, dtype=np.int64)
+    tr = np.zeros((max(trace_cap, 1), 3), dtype=np.int64)
+    st = _load().oracle_local_search(
+        _ptr(xy), xy.shape[0], _ptr(t), int(max_iters),
+        _ptr(out[0:1]), _ptr(out[1:2]), _ptr(tr) if trace_cap > 0 else None, int(trace_cap),
+    )
+    it = int(out[1])
+    return dict(tour=t, length=int(out[0]), iterations=it, status=int(st),
+                trace=tr[: min(it, trace_cap)].copy())
+
+
+def num_threads() -> int:
+    return int(_load().oracle_num_threads())

@@ -1,0 +1,205 @@
+/*
+ * oracle/tsp2opt_oracle.c -- plain CPU oracle for exhaustive best-improvement
+ * 2-opt on the symmetric Euclidean TSP (Rocki & Suda, IPDPSW 2013).
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and the
+ * cpu_baseline / --impl reference legs of bench.py may load this library.
+ * The product path (paper_conf_ipps_rockis13_b200/, libtsp2opt.so) never
+ * links, imports or calls it, and this file shares no code, header, table or
+ * constant generator with the CUDA path.
+ *
+ * Everything is int64 integer arithmetic (the paper fixes no float precision
+ * for the oracle; distances are TSPLIB EUC_2D on integer coordinates, so every
+ * quantity the method computes is an integer and the oracle is exact).
+ *
+ * Citations: PAPER.md is one physical line per paper page:
+ *   L12 = p.2 (§I.B 2-opt, Fig. 1, Fig. 2), L14 = p.3 (§IV, Fig. 3, Alg. 2),
+ *   L16 = p.4 (Listing 1, §IV.A), L18 = p.5 (Fig. 6, §IV.B).
+ * Readings R1..R13 of garbled / silent passages are listed in DESIGN.md §3.
+ *
+ * Parity pins (tests/test_oracle.py, tests/test_oracle_dist.py):
+ *   oracle_dist       -- closed form nint = (isqrt(4s)+1)//2 (Python, exhaustive
+ *                        boundaries), exhaustive C cross-check over all s.
+ *   oracle_best_move  -- brute force: every 2-opt neighbour built by explicit
+ *                        reversal and full length recomputation, n <= 9;
+ *                        Fig. 2 worked example; Fig. 3 cell order.
+ *   oracle_apply      -- Fig. 2 worked example; permutation invariant.
+ *   oracle_local_search -- delta == full recomputation after every move,
+ *                        local-minimum certificate, convex-position hull order,
+ *                        brute-force global optimum is a 2-opt local minimum.
+ */
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+/* ---------------------------------------------------------------------------
+ * Distance.  L16 Listing 1: "return (int)(sqrtf(dx*dx+dy*dy) + 0.5f); //
+ * return Euclidean distance" -- the intent is the TSPLIB EUC_2D rounded
+ * Euclidean distance nint(sqrt(dx^2+dy^2)).  Reading R3: we compute that
+ * integer exactly (Listing 1's float formula is not exact for large s).
+ * nint(sqrt(s)) = r+1 if s > r^2 + r else r, where r = floor(sqrt(s)):
+ * sqrt(s) >= r + 1/2  <=>  s >= r^2 + r + 1/4  <=>  s > r^2 + r (integers).
+ * ------------------------------------------------------------------------- */
+int64_t oracle_isqrt(int64_t s)
+{
+    int64_t r = (int64_t)sqrt((double)s);
+    while (r > 0 && r * r > s) r--;
+    while ((r + 1) * (r + 1) <= s) r++;
+    return r;
+}
+
+int64_t oracle_nint_sqrt(int64_t s)
+{
+    int64_t r = oracle_isqrt(s);
+    return (s > r * r + r) ? r + 1 : r;
+}
+
+int64_t oracle_dist(int64_t xa, int64_t ya, int64_t xb, int64_t yb)
+{
+    int64_t dx = xa - xb, dy = ya - yb;
+    return oracle_nint_sqrt(dx * dx + dy * dy);
+}
+
+/* d(tour[a], tour[b]) with positions taken modulo n: position n is position 0,
+ * the closed tour of L18 Fig. 6 ("ordered coordinates") -- reading R10. */
+static int64_t dpos(const int32_t *xy, const int32_t *tour, int64_t n,
+                    int64_t a, int64_t b)
+{
+    int64_t ca = tour[a % n], cb = tour[b % n];
+    return oracle_dist(xy[2 * ca], xy[2 * ca + 1], xy[2 * cb], xy[2 * cb + 1]);
+}
+
+/* Tour length: sum of the n closing edges d(t[k], t[k+1 mod n]). */
+int64_t oracle_tour_length(const int32_t *xy, int64_t n, const int32_t *tour)
+{
+    int64_t L = 0;
+    for (int64_t k = 0; k < n; k++) L += dpos(xy, tour, n, k, k + 1);
+    return L;
+}
+
+/* 2-opt delta of pair (i, j), 0 <= i < j <= n-1 (north_star; L12 Fig. 2
+ * "distance(b,f) + distance(g,d) > distance(b,d) + distance(g,f)" with
+ * b = t[i], f = t[i+1], d = t[j], g = t[j+1]; reading R2):
+ *   delta = d(i,j) + d(i+1,j+1) - d(i,i+1) - d(j,j+1);  improving iff < 0. */
+int64_t oracle_delta(const int32_t *xy, int64_t n, const int32_t *tour,
+                     int64_t i, int64_t j)
+{
+    return dpos(xy, tour, n, i, j) + dpos(xy, tour, n, i + 1, j + 1)
+         - dpos(xy, tour, n, i, i + 1) - dpos(xy, tour, n, j, j + 1);
+}
+
+/* Fig. 3 cell number of pair (i, j), i < j: cells are numbered column by
+ * column, "0,1 0  0,2 1  1,2 2  0,3 3 ..." (L14), i.e. k = j(j-1)/2 + i. */
+int64_t oracle_cell(int64_t i, int64_t j) { return j * (j - 1) / 2 + i; }
+
+/* ---------------------------------------------------------------------------
+ * One exhaustive sweep (L14 Alg. 2 steps 2-5: "Calculate swap effect of one
+ * pair ... Find the best value").  Neighbourhood: all pairs 0 <= i < j <= n-1
+ * of the closed tour (reading R1, C(n,2) checks).  Best = lowest delta, ties
+ * to the lowest Fig. 3 cell number (reading R5).  Scanning j ascending, then
+ * i ascending, visits cells in increasing k, so a strict '<' keeps the lowest
+ * cell among equal deltas.  At a 2-opt local minimum the winner is pair
+ * (0, 1) with delta 0 (cell 0, a degenerate pair; reading R7).
+ *
+ * OpenMP splits the j loop; each thread keeps its own (delta, k) minimum and
+ * the minima are combined with the same total order, which is independent of
+ * the split.
+ * ------------------------------------------------------------------------- */
+void oracle_best_move(const int32_t *xy, int64_t n, const int32_t *tour,
+                      int64_t *bi, int64_t *bj, int64_t *bdelta)
+{
+    int64_t best_d = 0, best_i = 0, best_j = 1;   /* pair (0,1): delta == 0 */
+    /* route-ordered coordinates P[k] = coords[t[k]], P[n] = P[0] (L18 Fig. 6) */
+    int64_t *px = (int64_t *)malloc(sizeof(int64_t) * (n + 1));
+    int64_t *py = (int64_t *)malloc(sizeof(int64_t) * (n + 1));
+    int64_t *e = (int64_t *)malloc(sizeof(int64_t) * n);
+    for (int64_t k = 0; k <= n; k++) {
+        int64_t c = tour[k % n];
+        px[k] = xy[2 * c];
+        py[k] = xy[2 * c + 1];
+    }
+    for (int64_t k = 0; k < n; k++) e[k] = oracle_dist(px[k], py[k], px[k + 1], py[k + 1]);
+
+#pragma omp parallel
+    {
+        int64_t td = 0, ti = 0, tj = 1;
+#pragma omp for schedule(dynamic, 16) nowait
+        for (int64_t j = 1; j < n; j++) {
+            for (int64_t i = 0; i < j; i++) {
+                int64_t d = oracle_dist(px[i], py[i], px[j], py[j])
+                          + oracle_dist(px[i + 1], py[i + 1], px[j + 1], py[j + 1])
+                          - e[i] - e[j];
+                if (d < td || (d == td && oracle_cell(i, j) < oracle_cell(ti, tj))) {
+                    td = d; ti = i; tj = j;
+                }
+            }
+        }
+#pragma omp critical
+        {
+            if (td < best_d || (td == best_d && oracle_cell(ti, tj) < oracle_cell(best_i, best_j))) {
+                best_d = td; best_i = ti; best_j = tj;
+            }
+        }
+    }
+    free(px); free(py); free(e);
+    *bi = best_i; *bj = best_j; *bdelta = best_d;
+}
+
+/* The 2-opt move (L12 §I.B "removes two edges ... reconnects ... reversing
+ * order of sub-tour"; Fig. 1): reverse tour positions i+1..j (reading R6:
+ * never the complement, so tour[0] never moves). */
+void oracle_apply(int32_t *tour, int64_t i, int64_t j)
+{
+    for (int64_t a = i + 1, b = j; a < b; a++, b--) {
+        int32_t t = tour[a]; tour[a] = tour[b]; tour[b] = t;
+    }
+}
+
+/* Best-improvement 2-opt local search (L12: "This step is applied only if the
+ * new tour would be shorter. Repeating removing and reconnecting the tour until
+ * no 2-opt improvements can be found leads to ... (local minimum)").
+ * Returns 0 at a local minimum, 1 when max_iters moves were applied first
+ * (max_iters < 0: unbounded).  trace (may be NULL) receives (i, j, delta) of
+ * every applied move, up to trace_cap moves. */
+int oracle_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64_t max_iters,
+                        int64_t *length, int64_t *iterations,
+                        int64_t *trace, int64_t trace_cap)
+{
+    int64_t L = oracle_tour_length(xy, n, tour);
+    int64_t it = 0;
+    int status = 0;
+    for (;;) {
+        if (max_iters >= 0 && it >= max_iters) {
+            /* reading R8: report MAXITER only if an improving move remains */
+            int64_t i, j, d;
+            oracle_best_move(xy, n, tour, &i, &j, &d);
+            status = (d < 0) ? 1 : 0;
+            break;
+        }
+        int64_t i, j, d;
+        oracle_best_move(xy, n, tour, &i, &j, &d);
+        if (d >= 0) break;
+        oracle_apply(tour, i, j);
+        L += d;
+        if (trace && it < trace_cap) {
+            trace[3 * it] = i; trace[3 * it + 1] = j; trace[3 * it + 2] = d;
+        }
+        it++;
+    }
+    *length = L;
+    *iterations = it;
+    return status;
+}
+
+int oracle_num_threads(void)
+{
+#ifdef _OPENMP
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
+}
