@@ -1,0 +1,347 @@
+#!/usr/bin/env python
+"""Benchmark of the exhaustive best-improvement 2-opt hot path on B200.
+
+Metric (BASELINE.json): 2-opt pair checks/sec (and time to local minimum) at
+1/2/4/8 B200.  One timed STEP = one pass of every SURVEY.md §8(a) row over the
+workload: load the tour from HBM (a2 reorder + a3 edges), the sweep over all
+C(n,2) pairs (a4 + a5 reduce), the allreduce-min across ranks (a6, N > 1), the
+segment-reversal apply (a7) and the loop-control state (a8).  Every step
+reloads the same seeded random tour, so every step does identical work.
+
+Workload (N=1 and N>1): config C5, n = 85900 pla-shaped lattice, random tour
+(BASELINE.json configs[4]; the metric names 1/2/4/8 GPUs, which only the
+sharded configs have).  `value` = C(n,2) * K / (max over ranks of the device
+time of the K steps); `e2e` = the same through the C ABI with host buffers.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_ipps_rockis13_b200 import inputs  # noqa: E402
+
+METRIC = "2-opt pair checks/sec and time-to-local-minimum at 1/2/4/8 B200 vs roofline"
+UNIT = "pair checks/s"
+PAIRS_PER_CLK_SM = 8  # north_star roofline: ~2 distance evaluations (16 issue slots, 2 XU ops) per pair
+N_SM = 148
+
+
+def peaks():
+    p = {}
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+    except OSError:
+        pass
+    return p
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, smax, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 8:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                smax = float(parts[1])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": smax,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- distributed
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def l2_flush(buf):
+    buf.add_(1)  # writes 256 MiB > 126 MB L2
+
+
+# ----------------------------------------------------------------------------- our arm
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_rockis13_b200 import tsp2opt
+
+    rank, world, local = dist_env()
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    cfg = inputs.CONFIGS[args.config]
+    n = cfg["n"]
+    coords, tour = inputs.config_instance(args.config, args.tour)
+    total_pairs = n * (n - 1) // 2
+
+    if world > 1:
+        obj = [tsp2opt.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        g = tsp2opt.TSP2Opt(coords, rank, world, obj[0])
+    else:
+        g = tsp2opt.TSP2Opt(coords)
+    stream = torch.cuda.current_stream()
+    g.set_stream(stream.cuda_stream)
+    d_tour = torch.from_numpy(tour).cuda()
+    flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device="cuda")
+
+    def step():
+        g.set_tour_device_async(d_tour.data_ptr())
+        g.iterate_async(1)
+
+    for _ in range(args.warmup):
+        step()
+    s = g.sync()
+    first_move = s["last_move"]
+
+    sampler = ClockSampler(local)
+    sampler.start()
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    g.profile(True)
+    launches0 = tsp2opt.launch_count()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for k in range(args.steps):
+        l2_flush(flush)  # between timed steps, outside the events
+        starts[k].record(stream)
+        step()
+        ends[k].record(stream)
+    torch.cuda.synchronize()
+    launches = tsp2opt.launch_count() - launches0
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop()
+    sweep_ms, sweep_n = g.profile_read()
+    g.profile(False)
+    step_ms = [a.elapsed_time(b) for a, b in zip(starts, ends)]
+    total_ms = sum(step_ms)
+    s = g.sync()
+    assert s["iterations"] == 1 and s["last_move"] == first_move, "steps must be identical"
+
+    # e2e: same metric through the public C ABI with HOST buffers each step
+    # (H2D of the tour, device sweep + apply, D2H of the move and the state).
+    geo = g.geometry()
+    g.set_stream(None)
+    e2e_ms = []
+    for k in range(max(2, args.steps // 2) + 1):
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        i, j, d = g.best_move(tour)
+        if d < 0:
+            g.apply(i, j)
+        e2e_ms.append((time.perf_counter() - t0) * 1e3)
+    e2e_ms = e2e_ms[1:]
+
+    t = torch.tensor([total_ms, sweep_ms / max(sweep_n, 1), sum(e2e_ms)], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    total_ms, sweep_avg_ms, e2e_total = t.tolist()
+
+    ls = None
+    if rank == 0 and world == 1 and not args.no_ls:
+        ls = time_to_local_min(tsp2opt, args.ls_config)
+
+    if rank == 0:
+        pk = peaks()
+        sm_max = clocks.get("sm_max_mhz") or pk.get("sm_max_mhz") or 1965.0
+        peak = PAIRS_PER_CLK_SM * N_SM * sm_max * 1e6 * world  # aggregate over ranks
+        achieved = geo["pairs"] * world / (sweep_avg_ms * 1e-3)  # per launch, all ranks
+        value = total_pairs * args.steps / (total_ms * 1e-3)
+        line = {
+            "metric": METRIC,
+            "value": value,
+            "unit": UNIT,
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": total_ms / args.steps,
+            "higher_is_better": True,
+            "scaling": "strong" if world > 1 else "weak",
+            "vs_baseline": None,
+            "dtype": "int32+f32",
+            "data": "synthetic",
+            "config": {"workload": f"{args.config} n={n} {cfg['coords']} coords seed={cfg['seed']}, "
+                                   f"{args.tour} tour; one step = load tour + sweep C(n,2) pairs + "
+                                   f"{'allreduce-min + ' if world > 1 else ''}apply",
+                       "n": n, "pairs_per_step": total_pairs, "l2": "flushed (256 MiB write) between timed steps",
+                       "geometry": geo, "parallelism": f"tile-shard x{world}"},
+            "roofline": {"bound": "alu", "achieved": achieved / 1e9, "peak": peak / 1e9, "unit": "Gpair/s",
+                         "frac": achieved / peak, "traffic": None,
+                         "kernel": "sweep_kernel", "peak_def": f"{PAIRS_PER_CLK_SM} pairs/clk/SM x {N_SM} SMs x "
+                         f"{sm_max:.0f} MHz (north_star: ~2 distance evaluations per pair; DESIGN.md §7)",
+                         "sweep_ms_avg": sweep_avg_ms, "sweep_share_of_step": sweep_avg_ms / (total_ms / args.steps)},
+            "e2e": {"value": total_pairs * len(e2e_ms) / (e2e_total * 1e-3), "unit": UNIT,
+                    "h2d_bytes_per_step": 4 * n, "d2h_bytes_per_step": 2 * 64,
+                    "api": "tsp2opt_best_move(host tour) + tsp2opt_apply"},
+            "gpu_launches": launches,
+            "clocks": clocks,
+            "first_move": list(first_move),
+        }
+        if ls:
+            line["time_to_local_minimum"] = ls
+        if world == 1 and not args.no_cpu:
+            line["cpu_baseline"] = cpu_baseline(args, coords, tour, total_pairs)
+        print(json.dumps(line), flush=True)
+    g.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def time_to_local_min(tsp2opt, cfg_name):
+    """Wall time of tsp2opt_local_search (host tour in, host tour out) per config."""
+    out = []
+    for name in cfg_name.split(","):
+        name, _, tk = name.partition(":")
+        coords, tour = inputs.config_instance(name, tk or None)
+        with tsp2opt.TSP2Opt(coords) as g:
+            g.local_search(tour, max_iters=2)  # warm-up
+            t0 = time.perf_counter()
+            r = g.local_search(tour)
+            dt = time.perf_counter() - t0
+        n = len(tour)
+        out.append({"config": name, "n": n, "start": tk or inputs.CONFIGS[name]["tour"], "seconds": dt,
+                    "iterations": r["iterations"], "length": r["length"],
+                    "pair_checks_per_s": (r["iterations"] + 1) * n * (n - 1) / 2 / dt})
+    return out
+
+
+# ----------------------------------------------------------------------------- oracle timing
+def cpu_baseline(args, coords, tour, total_pairs):
+    import oracle
+
+    t0 = time.perf_counter()
+    sweeps = 0
+    while True:
+        oracle.best_move(coords, tour)
+        sweeps += 1
+        if time.perf_counter() - t0 > args.cpu_seconds or sweeps >= 3:
+            break
+    dt = time.perf_counter() - t0
+    return {"value": sweeps * total_pairs / dt, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": f"{sweeps} full sweep(s) of the same workload (best_move over C(n,2) pairs), "
+                      f"{dt:.1f} s, plain C oracle, OpenMP", "seconds": dt}
+
+
+def run_reference(args):
+    """--impl reference: the oracle (plain C, host cores) on our arm's config/metric."""
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    import oracle
+
+    cfg = inputs.CONFIGS[args.config]
+    n = cfg["n"]
+    coords, tour = inputs.config_instance(args.config, args.tour)
+    total_pairs = n * (n - 1) // 2
+    oracle.build()
+    for _ in range(min(args.warmup, 1)):
+        oracle.best_move(coords, tour)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        i, j, d = oracle.best_move(coords, tour)
+        t2 = oracle.apply(tour, i, j) if d < 0 else tour  # noqa: F841  (apply is part of the step)
+        times.append(time.perf_counter() - t0)
+        if sum(times) > args.ref_seconds:
+            break
+    k = len(times)
+    value = total_pairs * k / sum(times)
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": k, "warmup": args.warmup,
+            "ms_per_step": 1e3 * sum(times) / k, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "int64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": f"{args.config} n={n} {cfg['coords']} coords, {args.tour} tour; one step = "
+                                   "oracle best_move (C(n,2) pairs) + apply", "n": n},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
+                             "sample": f"{k} step(s) of the workload (capped at {args.ref_seconds:.0f} s)"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C5")
+    ap.add_argument("--tour", default="random", choices=["random", "hilbert"])
+    ap.add_argument("--ls-config", default="C2,C3", help="configs timed to a local minimum (rank 0, N=1)")
+    ap.add_argument("--no-ls", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--ref-seconds", type=float, default=120.0)
+    args = ap.parse_args()
+    if args.warmup < 3 and args.impl == "ours":
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

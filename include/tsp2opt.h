@@ -1,0 +1,165 @@
+/*
+ * include/tsp2opt.h -- C ABI of the B200 (sm_100a) exhaustive best-improvement
+ * 2-opt library (libtsp2opt.so), after Rocki & Suda, "High Performance GPU
+ * Accelerated Local Optimization in TSP", IPDPSW 2013.
+ *
+ * Citations "Lnn" are lines of the paper text PAPER.md (one line per page;
+ * SURVEY.md §0); readings R1..R13 of garbled passages are in DESIGN.md §3.
+ *
+ * The operation (north_star; L12 §I.B Fig. 1-2; L14 §IV Fig. 3, Alg. 2):
+ *   P[k] = coords[tour[k]] (k < n), P[n] = P[0]      (route-ordered coordinates, L18 Fig. 6)
+ *   e[k] = d(P[k], P[k+1])                            (tour edges)
+ *   d(a,b) = nint(sqrt((xa-xb)^2 + (ya-yb)^2))        (TSPLIB EUC_2D, exact integer; R3)
+ *   for every pair 0 <= i < j <= n-1 (C(n,2) pairs; R1):
+ *       delta(i,j) = d(P[i],P[j]) + d(P[i+1],P[j+1]) - e[i] - e[j]
+ *   best = lowest delta, ties to the lowest Fig. 3 cell k = j(j-1)/2 + i   (R5)
+ *   move = reverse tour positions i+1..j (tour[0] never moves)            (R6)
+ *   local search = repeat {best; apply if delta < 0} until best delta >= 0 (R7)
+ *
+ * Conventions for every function:
+ *   - Return TSP2OPT_OK (0) on success, a negative TSP2OPT_E* code on error,
+ *     TSP2OPT_MAXITER (1) from local_search when capped.  On a validation error
+ *     (EINVAL/ERANGE/ENOTPERM/ESTATE) the handle's state is unchanged.
+ *   - Host pointers are only read/written during the call; the library never
+ *     retains caller buffers.  All device memory is owned by the handle.
+ *   - Functions are synchronous (they return after the device work finished)
+ *     unless named *_async.  A handle is not thread-safe: one handle per
+ *     device (and per rank); the CUDA device current at create time is used.
+ *   - Coordinates are integers in [0, 2^15) (R4); 3 <= n <= 2^22 (key width, R5).
+ */
+#ifndef TSP2OPT_H
+#define TSP2OPT_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct tsp2opt_ctx *tsp2opt_t;
+
+enum {
+    TSP2OPT_OK = 0,
+    TSP2OPT_MAXITER = 1,    /* local_search applied max_iters moves and an improving move remains */
+    TSP2OPT_EINVAL = -1,    /* NULL pointer, n out of range, bad rank/world, max_iters < 0, !(0<=i<j<n) */
+    TSP2OPT_ERANGE = -2,    /* a coordinate outside [0, 2^15) */
+    TSP2OPT_ENOTPERM = -3,  /* tour is not a permutation of 0..n-1 */
+    TSP2OPT_ESTATE = -4,    /* operation needs a loaded tour (set_tour / best_move with a tour) first */
+    TSP2OPT_ECUDA = -5,     /* a CUDA runtime error (message via tsp2opt_last_error) */
+    TSP2OPT_ENCCL = -6,     /* an NCCL error (sharded handles) */
+    TSP2OPT_ENOMEM = -7     /* device or pinned host allocation failed */
+};
+
+#define TSP2OPT_MAX_N (1 << 22)
+#define TSP2OPT_COORD_LIMIT (1 << 15)
+#define TSP2OPT_NCCL_ID_BYTES 128
+
+/* Create a single-GPU handle.  coords_xy: host int32[2n] = x0,y0,x1,y1,...
+ * (copied to the device once, L14 Alg. 2 step 1).  *out receives the handle. */
+int tsp2opt_create(const int32_t *coords_xy, int32_t n, tsp2opt_t *out);
+
+/* Sharded handle for one rank of `world` ranks (one GPU each, one node).
+ * The triangular tile space of the sweep is split into `world` contiguous
+ * ranges of equal pair count; coordinates, tour and edges are replicated; one
+ * ncclAllReduce(int64, MIN) of the packed best-move key per sweep (SURVEY.md
+ * §8(e); L18 §VI "dividing the 2-opt task between multiple devices").
+ * nccl_id: TSP2OPT_NCCL_ID_BYTES bytes from tsp2opt_nccl_unique_id() on rank 0,
+ * broadcast by the caller.  Every rank must make the same sequence of calls;
+ * outputs are identical on all ranks.  world == 1 is allowed (no NCCL). */
+int tsp2opt_create_sharded(const int32_t *coords_xy, int32_t n, int32_t rank, int32_t world,
+                           const void *nccl_id, tsp2opt_t *out);
+
+/* Write an NCCL unique id (TSP2OPT_NCCL_ID_BYTES bytes) into out. */
+int tsp2opt_nccl_unique_id(void *out);
+
+/* Release all device memory, streams, graphs and the NCCL communicator. */
+void tsp2opt_destroy(tsp2opt_t h);
+
+/* Use `cuda_stream` (a cudaStream_t, e.g. torch.cuda.current_stream().cuda_stream)
+ * for all subsequent work; NULL selects the handle's own non-blocking stream. */
+int tsp2opt_set_stream(tsp2opt_t h, void *cuda_stream);
+
+/* Load a tour: host int32[n] permutation (validated on the host, O(n)), then
+ * the route-order gather P[k] = coords[tour[k]] and the edge pass e[k] run on
+ * the device (L18 Fig. 6 "array of ordered coordinates").  */
+int tsp2opt_set_tour(tsp2opt_t h, const int32_t *tour);
+
+/* Same with a DEVICE pointer (int32[n] in this GPU's memory), enqueued on the
+ * handle's stream without a host sync; the permutation check runs on the device
+ * and a violation surfaces as TSP2OPT_ENOTPERM from the next synchronous call
+ * (tsp2opt_sync / best_move / get_tour), which also clears the loaded tour. */
+int tsp2opt_set_tour_device_async(tsp2opt_t h, const int32_t *d_tour);
+
+/* One exhaustive sweep (L14 Alg. 2 steps 2-6): if tour != NULL it is loaded
+ * first (as tsp2opt_set_tour), else the current tour is used.  Returns the best
+ * move (i, j, delta); at a 2-opt local minimum this is (0, 1, 0) (R7).
+ * Does not modify the tour. */
+int tsp2opt_best_move(tsp2opt_t h, const int32_t *tour, int32_t *i, int32_t *j, int32_t *delta);
+
+/* Apply the 2-opt move (i, j), 0 <= i < j <= n-1: reverse positions i+1..j of
+ * the tour (L12 "reversing order of sub-tour"); edges and length are updated
+ * on the device.  Any valid pair is accepted (improving or not). */
+int tsp2opt_apply(tsp2opt_t h, int32_t i, int32_t j);
+
+/* Enqueue `count` device-resident iterations {sweep; [allreduce]; apply if
+ * delta < 0} on the handle's stream, no host sync (the bench's timed step).
+ * Iterations after convergence are no-ops.  Needs a loaded tour. */
+int tsp2opt_iterate_async(tsp2opt_t h, int32_t count);
+
+/* Wait for the handle's stream; report the device-side status:
+ * *iterations = moves applied since the tour was loaded, *length = current
+ * tour length, *converged = 1 at a local minimum, 2 if capped, 0 otherwise;
+ * *last_i/_j/_delta = the most recent sweep's best move.  Any pointer may be NULL. */
+int tsp2opt_sync(tsp2opt_t h, int64_t *iterations, int64_t *length, int32_t *converged,
+                 int32_t *last_i, int32_t *last_j, int32_t *last_delta);
+
+/* Best-improvement 2-opt local search (L12 §I.B; north_star).  tour: host
+ * int32[n], in: start tour, out: tour at the local minimum (or after
+ * max_iters moves).  max_iters >= 0 caps the number of applied moves
+ * (TSP2OPT_MAX_ITERS_UNBOUNDED = no cap).  *length = final tour length,
+ * *iterations = applied moves.  Returns TSP2OPT_OK at a local minimum,
+ * TSP2OPT_MAXITER if max_iters moves were applied and an improving move remains. */
+#define TSP2OPT_MAX_ITERS_UNBOUNDED INT64_MAX
+int tsp2opt_local_search(tsp2opt_t h, int32_t *tour, int64_t max_iters, int64_t *length,
+                         int64_t *iterations);
+
+/* Copy the current tour (host int32[n]) and its length out. */
+int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
+
+/* Diagnostics / test hooks ------------------------------------------------ */
+
+/* Restrict this handle's sweep to shard `rank` of `world` of the tile space
+ * WITHOUT any collective (world = 1 restores the full sweep).  Used to check on
+ * one GPU that the min over shards equals the unsharded result. */
+int tsp2opt_debug_set_shard(tsp2opt_t h, int32_t rank, int32_t world);
+
+/* Sweep geometry actually used: rows per thread R, warps per CTA, columns per
+ * tile TJ, number of tiles and pairs of this handle's shard. */
+int tsp2opt_get_geometry(tsp2opt_t h, int32_t *R, int32_t *warps, int32_t *tj,
+                         int64_t *tiles, int64_t *pairs);
+
+/* Exhaustive device self-test of the sweep kernel's arithmetic (same inline
+ * device functions): (a) the exact distance d(s) over every s in [0, 2*32767^2]
+ * against m^2 - m < s <= m^2 + m; (b) the squared-distance prefilter never
+ * rejects: for every (dx, dy) in [0, 32767]^2 the float s(dx,dy) passes the
+ * float threshold built from t = d(dx,dy).  Writes the violation counts. */
+int tsp2opt_selftest(int64_t *dist_violations, int64_t *filter_violations);
+
+/* Sweep-kernel timing: enable != 0 starts recording a CUDA event pair around
+ * every sweep launch of this handle (previous records are dropped); enable == 0
+ * stops.  tsp2opt_profile_read waits for the stream and returns the summed
+ * device time (ms) of the recorded sweep launches and their number. */
+int tsp2opt_profile(tsp2opt_t h, int32_t enable);
+int tsp2opt_profile_read(tsp2opt_t h, double *total_ms, int64_t *launches);
+
+/* Number of this library's kernel launches since load (for gpu_launches). */
+int64_t tsp2opt_launch_count(void);
+
+/* Human-readable message for a return code; last CUDA/NCCL error text. */
+const char *tsp2opt_strerror(int code);
+const char *tsp2opt_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TSP2OPT_H */

@@ -1,0 +1,544 @@
+// tsp2opt_api.cu -- C ABI (include/tsp2opt.h) and host runtime of libtsp2opt.so.
+//
+// Owns the device state of one instance (one GPU, one rank): coordinates,
+// tour, route-ordered coordinates P, edges E, the ping-pong Slot pair, the
+// sweep's tile table; drives the kernels of tsp2opt_kernels.cu on one stream;
+// for sharded handles owns an NCCL communicator and performs one 8-byte
+// ncclAllReduce(MIN) of the packed best-move key per sweep.
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include <nccl.h>
+
+#include "../../include/tsp2opt.h"
+#include "tsp2opt_internal.h"
+
+using namespace tsp2opt;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+int cuda_fail(cudaError_t e, const char* what)
+{
+    g_last_error = std::string(what) + ": " + cudaGetErrorString(e);
+    return e == cudaErrorMemoryAllocation ? TSP2OPT_ENOMEM : TSP2OPT_ECUDA;
+}
+int nccl_fail(ncclResult_t r, const char* what)
+{
+    g_last_error = std::string(what) + ": " + ncclGetErrorString(r);
+    return TSP2OPT_ENCCL;
+}
+
+#define CUDA_TRY(call)                                   \
+    do {                                                 \
+        cudaError_t e_ = (call);                         \
+        if (e_ != cudaSuccess) return cuda_fail(e_, #call); \
+    } while (0)
+
+struct Tile {
+    int i0, j0;
+    long long pairs;
+};
+
+}  // namespace
+
+struct tsp2opt_ctx {
+    int n = 0;
+    int rank = 0, world = 1;          // NCCL sharding
+    int shard_rank = 0, shard_world = 1;  // tile range actually swept (== rank/world unless debug)
+    int device = 0;
+    cudaStream_t own_stream = nullptr;
+    cudaStream_t stream = nullptr;
+    int* d_coords = nullptr;    // int32[2n]
+    int* d_tour = nullptr;      // int32[n + pad]
+    int* d_tour_in = nullptr;   // int32[n] staging for host tours
+    float2* d_P = nullptr;      // [n + 1 + pad] biased route-ordered coordinates
+    int* d_E = nullptr;         // [n + pad] edges
+    Slot* d_slots = nullptr;    // [2]
+    unsigned* d_stamp = nullptr;  // [n] permutation check
+    int2* d_tiles = nullptr;    // this shard's tiles
+    Slot* h_slot = nullptr;     // pinned readback
+    unsigned epoch = 0;
+    int parity = 0;             // iteration t reads slot[parity]
+    bool has_tour = false;
+    Geometry geo{};
+    std::vector<Tile> all_tiles;  // sorted, all shards
+    int ntiles = 0;               // tiles of this shard
+    long long shard_pairs = 0;
+    ncclComm_t comm = nullptr;
+    bool profiling = false;
+    std::vector<cudaEvent_t> ev_pool;  // pairs (start, stop) of recorded sweep launches
+    size_t ev_used = 0;
+};
+
+namespace {
+
+Geometry choose_geometry(long long pairs_per_rank)
+{
+    Geometry best{kRows, 1, 32};
+    const char* ew = getenv("TSP2OPT_WARPS");
+    const char* et = getenv("TSP2OPT_TJ");
+    if (ew && et) {
+        Geometry g{kRows, atoi(ew), atoi(et)};
+        if (g.warps >= 1 && g.warps <= kMaxWarps && g.tj >= 2 && g.tj <= kMaxTJ) return g;
+    }
+    const long long target = 24LL * 148;  // tiles per shard: >= ~6 waves of 4 CTAs/SM
+    long long best_area = -1;
+    for (int w : {4, 2, 1})
+        for (int tj : {1024, 512, 256, 128, 64, 32}) {
+            Geometry g{kRows, w, tj};
+            long long area = (long long)g.ti() * tj;
+            if (pairs_per_rank / area >= target && area > best_area) {
+                best = g;
+                best_area = area;
+            }
+        }
+    return best;
+}
+
+// Tiles over the upper triangle only (L20 Fig. 8 "Skip unnecessary computation"):
+// row blocks [I0, I0+TI) with I0 <= n-2, column chunks [J0, J0+TJ) containing a
+// column j > I0; pairs = #{(i, j): I0 <= i < min(I0+TI, n-1), J0 <= j < min(J0+TJ, n), i < j}.
+std::vector<Tile> build_tiles(int n, const Geometry& g)
+{
+    std::vector<Tile> t;
+    const int TI = g.ti(), TJ = g.tj;
+    for (int I0 = 0; I0 <= n - 2; I0 += TI) {
+        const int rows = std::min(I0 + TI, n - 1) - I0;
+        for (int J0 = ((I0 + 1) / TJ) * TJ; J0 < n; J0 += TJ) {
+            const int J1 = std::min(J0 + TJ, n);
+            long long p = 0;
+            for (int j = J0; j < J1; j++) p += std::max(0, std::min(j - I0, rows));
+            if (p > 0) t.push_back({I0, J0, p});
+        }
+    }
+    std::stable_sort(t.begin(), t.end(), [](const Tile& a, const Tile& b) { return a.pairs > b.pairs; });
+    return t;
+}
+
+// Greedy LPT split of the (size-sorted) tile list into `world` shards of equal
+// pair count; each shard keeps the largest-first order.
+std::vector<Tile> shard_tiles(const std::vector<Tile>& all, int rank, int world, long long* pairs)
+{
+    std::vector<long long> load(world, 0);
+    std::vector<Tile> mine;
+    for (const Tile& t : all) {
+        int r = (int)(std::min_element(load.begin(), load.end()) - load.begin());
+        load[r] += t.pairs;
+        if (r == rank) mine.push_back(t);
+    }
+    *pairs = load[rank];
+    return mine;
+}
+
+int upload_shard(tsp2opt_ctx* h, int rank, int world)
+{
+    long long pairs = 0;
+    std::vector<Tile> mine = shard_tiles(h->all_tiles, rank, world, &pairs);
+    std::vector<int2> host(mine.size());
+    for (size_t k = 0; k < mine.size(); k++) host[k] = make_int2(mine[k].i0, mine[k].j0);
+    if (h->d_tiles) cudaFree(h->d_tiles);
+    h->d_tiles = nullptr;
+    if (!host.empty()) {
+        CUDA_TRY(cudaMalloc(&h->d_tiles, host.size() * sizeof(int2)));
+        CUDA_TRY(cudaMemcpy(h->d_tiles, host.data(), host.size() * sizeof(int2), cudaMemcpyHostToDevice));
+    }
+    h->ntiles = (int)host.size();
+    h->shard_pairs = pairs;
+    h->shard_rank = rank;
+    h->shard_world = world;
+    return TSP2OPT_OK;
+}
+
+void free_ctx(tsp2opt_ctx* h)
+{
+    if (!h) return;
+    if (h->comm) ncclCommDestroy(h->comm);
+    cudaFree(h->d_coords);
+    cudaFree(h->d_tour);
+    cudaFree(h->d_tour_in);
+    cudaFree(h->d_P);
+    cudaFree(h->d_E);
+    cudaFree(h->d_slots);
+    cudaFree(h->d_stamp);
+    cudaFree(h->d_tiles);
+    if (h->h_slot) cudaFreeHost(h->h_slot);
+    for (cudaEvent_t e : h->ev_pool) cudaEventDestroy(e);
+    if (h->own_stream) cudaStreamDestroy(h->own_stream);
+    delete h;
+}
+
+int validate_coords(const int32_t* xy, int32_t n)
+{
+    if (!xy) return TSP2OPT_EINVAL;
+    if (n < 3 || n > TSP2OPT_MAX_N) return TSP2OPT_EINVAL;
+    for (long long k = 0; k < 2LL * n; k++)
+        if (xy[k] < 0 || xy[k] >= TSP2OPT_COORD_LIMIT) return TSP2OPT_ERANGE;
+    return TSP2OPT_OK;
+}
+
+int validate_tour(const int32_t* t, int n)
+{
+    if (!t) return TSP2OPT_EINVAL;
+    std::vector<unsigned char> seen(n, 0);
+    for (int k = 0; k < n; k++) {
+        if (t[k] < 0 || t[k] >= n || seen[t[k]]) return TSP2OPT_ENOTPERM;
+        seen[t[k]] = 1;
+    }
+    return TSP2OPT_OK;
+}
+
+int read_slot(tsp2opt_ctx* h)
+{
+    CUDA_TRY(cudaMemcpyAsync(h->h_slot, h->d_slots + h->parity, sizeof(Slot), cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    if (h->h_slot->done & 4) {
+        h->has_tour = false;
+        g_last_error = "device tour is not a permutation";
+        return TSP2OPT_ENOTPERM;
+    }
+    return TSP2OPT_OK;
+}
+
+int load_device_tour(tsp2opt_ctx* h, const int32_t* d_src)
+{
+    h->parity = 0;
+    if (++h->epoch == 0) {  // stamp wrap-around: clear and restart epochs
+        CUDA_TRY(cudaMemsetAsync(h->d_stamp, 0, sizeof(unsigned) * h->n, h->stream));
+        h->epoch = 1;
+    }
+    CUDA_TRY(launch_load_tour(h->d_coords, d_src, h->d_tour, h->d_P, h->d_E, h->n, h->d_slots + 0, h->d_stamp,
+                              h->epoch, h->stream));
+    h->has_tour = true;
+    return TSP2OPT_OK;
+}
+
+int load_host_tour(tsp2opt_ctx* h, const int32_t* tour)
+{
+    int rc = validate_tour(tour, h->n);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(h->d_tour_in, tour, sizeof(int32_t) * h->n, cudaMemcpyHostToDevice, h->stream));
+    return load_device_tour(h, h->d_tour_in);
+}
+
+// One iteration: sweep (a4/a5) -> allreduce-min (a6) -> apply (a7/a8).
+int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
+{
+    Slot* in = h->d_slots + h->parity;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    if (h->profiling) {
+        while (h->ev_pool.size() < h->ev_used + 2) {
+            cudaEvent_t e;
+            CUDA_TRY(cudaEventCreate(&e));
+            h->ev_pool.push_back(e);
+        }
+        ev0 = h->ev_pool[h->ev_used];
+        ev1 = h->ev_pool[h->ev_used + 1];
+        h->ev_used += 2;
+        CUDA_TRY(cudaEventRecord(ev0, h->stream));
+    }
+    CUDA_TRY(launch_sweep(h->geo, h->d_P, h->d_E, h->n, h->d_tiles, h->ntiles, in, apply ? 1 : 0, h->stream));
+    if (ev1) CUDA_TRY(cudaEventRecord(ev1, h->stream));
+    if (h->comm) {
+        ncclResult_t r = ncclAllReduce(&in->key, &in->key, 1, ncclUint64, ncclMin, h->comm, h->stream);
+        if (r != ncclSuccess) return nccl_fail(r, "ncclAllReduce");
+    }
+    if (apply) {
+        Slot* out = h->d_slots + (h->parity ^ 1);
+        CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, max_moves, 0, 0, 0, h->stream));
+        h->parity ^= 1;
+    }
+    return TSP2OPT_OK;
+}
+
+int create_common(const int32_t* xy, int32_t n, int rank, int world, const void* nccl_id, tsp2opt_t* out)
+{
+    if (!out) return TSP2OPT_EINVAL;
+    *out = nullptr;
+    int rc = validate_coords(xy, n);
+    if (rc) return rc;
+    if (world < 1 || rank < 0 || rank >= world || (world > 1 && !nccl_id)) return TSP2OPT_EINVAL;
+    tsp2opt_ctx* h = new tsp2opt_ctx();
+    h->n = n;
+    h->rank = rank;
+    h->world = world;
+    auto fail = [&](int code) {
+        free_ctx(h);
+        return code;
+    };
+#define CTRY(call)                                               \
+    do {                                                         \
+        cudaError_t e_ = (call);                                 \
+        if (e_ != cudaSuccess) return fail(cuda_fail(e_, #call)); \
+    } while (0)
+    CTRY(cudaGetDevice(&h->device));
+    CTRY(cudaStreamCreateWithFlags(&h->own_stream, cudaStreamNonBlocking));
+    h->stream = h->own_stream;
+    const size_t np = (size_t)n + 1 + kPad;
+    CTRY(cudaMalloc(&h->d_coords, sizeof(int) * 2 * (size_t)n));
+    CTRY(cudaMalloc(&h->d_tour, sizeof(int) * np));
+    CTRY(cudaMalloc(&h->d_tour_in, sizeof(int) * (size_t)n));
+    CTRY(cudaMalloc(&h->d_P, sizeof(float2) * np));
+    CTRY(cudaMalloc(&h->d_E, sizeof(int) * np));
+    CTRY(cudaMalloc(&h->d_slots, sizeof(Slot) * 2));
+    CTRY(cudaMalloc(&h->d_stamp, sizeof(unsigned) * (size_t)n));
+    CTRY(cudaHostAlloc(&h->h_slot, sizeof(Slot), cudaHostAllocDefault));
+    CTRY(cudaMemset(h->d_tour, 0, sizeof(int) * np));
+    CTRY(cudaMemset(h->d_E, 0, sizeof(int) * np));
+    CTRY(cudaMemset(h->d_stamp, 0, sizeof(unsigned) * (size_t)n));
+    CTRY(cudaMemset(h->d_slots, 0, sizeof(Slot) * 2));
+    {
+        std::vector<float2> pad(np, make_float2(kCoordBias, kCoordBias));
+        CTRY(cudaMemcpy(h->d_P, pad.data(), sizeof(float2) * np, cudaMemcpyHostToDevice));
+    }
+    CTRY(cudaMemcpy(h->d_coords, xy, sizeof(int) * 2 * (size_t)n, cudaMemcpyHostToDevice));
+    CTRY(sweep_prepare());
+    const long long total_pairs = (long long)n * (n - 1) / 2;
+    h->geo = choose_geometry(total_pairs / world);
+    h->all_tiles = build_tiles(n, h->geo);
+    rc = upload_shard(h, rank, world);
+    if (rc) return fail(rc);
+    if (world > 1) {
+        ncclUniqueId id;
+        memcpy(&id, nccl_id, sizeof(id));
+        ncclResult_t r = ncclCommInitRank(&h->comm, world, id, rank);
+        if (r != ncclSuccess) {
+            h->comm = nullptr;
+            return fail(nccl_fail(r, "ncclCommInitRank"));
+        }
+    }
+#undef CTRY
+    *out = h;
+    return TSP2OPT_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int tsp2opt_create(const int32_t* coords_xy, int32_t n, tsp2opt_t* out)
+{
+    return create_common(coords_xy, n, 0, 1, nullptr, out);
+}
+
+int tsp2opt_create_sharded(const int32_t* coords_xy, int32_t n, int32_t rank, int32_t world, const void* nccl_id,
+                           tsp2opt_t* out)
+{
+    return create_common(coords_xy, n, rank, world, nccl_id, out);
+}
+
+int tsp2opt_nccl_unique_id(void* out)
+{
+    if (!out) return TSP2OPT_EINVAL;
+    static_assert(sizeof(ncclUniqueId) == TSP2OPT_NCCL_ID_BYTES, "NCCL id size");
+    ncclUniqueId id;
+    ncclResult_t r = ncclGetUniqueId(&id);
+    if (r != ncclSuccess) return nccl_fail(r, "ncclGetUniqueId");
+    memcpy(out, &id, sizeof(id));
+    return TSP2OPT_OK;
+}
+
+void tsp2opt_destroy(tsp2opt_t h)
+{
+    if (!h) return;
+    cudaStreamSynchronize(h->stream);
+    free_ctx(h);
+}
+
+int tsp2opt_set_stream(tsp2opt_t h, void* cuda_stream)
+{
+    if (!h) return TSP2OPT_EINVAL;
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    h->stream = cuda_stream ? (cudaStream_t)cuda_stream : h->own_stream;
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_set_tour(tsp2opt_t h, const int32_t* tour)
+{
+    if (!h || !tour) return TSP2OPT_EINVAL;
+    int rc = load_host_tour(h, tour);
+    if (rc) return rc;
+    return read_slot(h);
+}
+
+int tsp2opt_set_tour_device_async(tsp2opt_t h, const int32_t* d_tour)
+{
+    if (!h || !d_tour) return TSP2OPT_EINVAL;
+    return load_device_tour(h, d_tour);
+}
+
+int tsp2opt_best_move(tsp2opt_t h, const int32_t* tour, int32_t* i, int32_t* j, int32_t* delta)
+{
+    if (!h || !i || !j || !delta) return TSP2OPT_EINVAL;
+    if (tour) {
+        int rc = load_host_tour(h, tour);
+        if (rc) return rc;
+    }
+    if (!h->has_tour) return TSP2OPT_ESTATE;
+    CUDA_TRY(launch_reset_key(h->d_slots + h->parity, h->stream));
+    int rc = enqueue_iteration(h, 0, false);
+    if (rc) return rc;
+    rc = read_slot(h);
+    if (rc) return rc;
+    const unsigned long long k = h->h_slot->key;
+    *i = key_i(k);
+    *j = key_j(k);
+    *delta = key_delta(k);
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_apply(tsp2opt_t h, int32_t i, int32_t j)
+{
+    if (!h) return TSP2OPT_EINVAL;
+    if (!(0 <= i && i < j && j < h->n)) return TSP2OPT_EINVAL;
+    if (!h->has_tour) return TSP2OPT_ESTATE;
+    Slot* in = h->d_slots + h->parity;
+    Slot* out = h->d_slots + (h->parity ^ 1);
+    CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, 0, 1, i, j, h->stream));
+    h->parity ^= 1;
+    return read_slot(h);
+}
+
+int tsp2opt_iterate_async(tsp2opt_t h, int32_t count)
+{
+    if (!h || count < 0) return TSP2OPT_EINVAL;
+    if (!h->has_tour) return TSP2OPT_ESTATE;
+    for (int c = 0; c < count; c++) {
+        int rc = enqueue_iteration(h, TSP2OPT_MAX_ITERS_UNBOUNDED, true);
+        if (rc) return rc;
+    }
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_sync(tsp2opt_t h, int64_t* iterations, int64_t* length, int32_t* converged, int32_t* last_i,
+                 int32_t* last_j, int32_t* last_delta)
+{
+    if (!h) return TSP2OPT_EINVAL;
+    if (!h->has_tour) return TSP2OPT_ESTATE;
+    int rc = read_slot(h);
+    if (rc) return rc;
+    const Slot& s = *h->h_slot;
+    if (iterations) *iterations = s.moves;
+    if (length) *length = s.length;
+    if (converged) *converged = s.done & 3;
+    if (last_i) *last_i = key_i(s.last_key);
+    if (last_j) *last_j = key_j(s.last_key);
+    if (last_delta) *last_delta = key_delta(s.last_key);
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_local_search(tsp2opt_t h, int32_t* tour, int64_t max_iters, int64_t* length, int64_t* iterations)
+{
+    if (!h || !tour || !length || !iterations || max_iters < 0) return TSP2OPT_EINVAL;
+    int rc = load_host_tour(h, tour);
+    if (rc) return rc;
+    // Device-resident loop: batches of K iterations between host checks; an
+    // iteration after convergence is a no-op (sweep CTAs exit on the done flag).
+    long long k = 4;
+    for (;;) {
+        for (long long c = 0; c < k; c++) {
+            rc = enqueue_iteration(h, max_iters, true);
+            if (rc) return rc;
+        }
+        rc = read_slot(h);
+        if (rc) return rc;
+        if (h->h_slot->done & 3) break;
+        if (k < 64) k *= 2;
+    }
+    CUDA_TRY(cudaMemcpyAsync(tour, h->d_tour, sizeof(int32_t) * h->n, cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    *length = h->h_slot->length;
+    *iterations = h->h_slot->moves;
+    return (h->h_slot->done & 3) == 2 ? TSP2OPT_MAXITER : TSP2OPT_OK;
+}
+
+int tsp2opt_get_tour(tsp2opt_t h, int32_t* tour_out, int64_t* length)
+{
+    if (!h || !tour_out) return TSP2OPT_EINVAL;
+    if (!h->has_tour) return TSP2OPT_ESTATE;
+    int rc = read_slot(h);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(tour_out, h->d_tour, sizeof(int32_t) * h->n, cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    if (length) *length = h->h_slot->length;
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_debug_set_shard(tsp2opt_t h, int32_t rank, int32_t world)
+{
+    if (!h || world < 1 || rank < 0 || rank >= world) return TSP2OPT_EINVAL;
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    return upload_shard(h, rank, world);
+}
+
+int tsp2opt_get_geometry(tsp2opt_t h, int32_t* R, int32_t* warps, int32_t* tj, int64_t* tiles, int64_t* pairs)
+{
+    if (!h) return TSP2OPT_EINVAL;
+    if (R) *R = h->geo.rows;
+    if (warps) *warps = h->geo.warps;
+    if (tj) *tj = h->geo.tj;
+    if (tiles) *tiles = h->ntiles;
+    if (pairs) *pairs = h->shard_pairs;
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_selftest(int64_t* dist_violations, int64_t* filter_violations)
+{
+    if (!dist_violations || !filter_violations) return TSP2OPT_EINVAL;
+    long long a = -1, b = -1;
+    CUDA_TRY(run_selftest(&a, &b));
+    *dist_violations = a;
+    *filter_violations = b;
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_profile(tsp2opt_t h, int32_t enable)
+{
+    if (!h) return TSP2OPT_EINVAL;
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    h->profiling = enable != 0;
+    h->ev_used = 0;
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_profile_read(tsp2opt_t h, double* total_ms, int64_t* launches)
+{
+    if (!h || !total_ms || !launches) return TSP2OPT_EINVAL;
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    double sum = 0;
+    for (size_t k = 0; k + 1 < h->ev_used; k += 2) {
+        float ms = 0;
+        CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_pool[k], h->ev_pool[k + 1]));
+        sum += ms;
+    }
+    *total_ms = sum;
+    *launches = (int64_t)(h->ev_used / 2);
+    return TSP2OPT_OK;
+}
+
+int64_t tsp2opt_launch_count(void) { return launch_count(); }
+
+const char* tsp2opt_strerror(int code)
+{
+    switch (code) {
+    case TSP2OPT_OK: return "ok";
+    case TSP2OPT_MAXITER: return "max_iters reached with an improving move left";
+    case TSP2OPT_EINVAL: return "invalid argument";
+    case TSP2OPT_ERANGE: return "coordinate outside [0, 2^15)";
+    case TSP2OPT_ENOTPERM: return "tour is not a permutation of 0..n-1";
+    case TSP2OPT_ESTATE: return "no tour loaded";
+    case TSP2OPT_ECUDA: return "CUDA error";
+    case TSP2OPT_ENCCL: return "NCCL error";
+    case TSP2OPT_ENOMEM: return "out of memory";
+    default: return "unknown error";
+    }
+}
+
+const char* tsp2opt_last_error(void) { return g_last_error.c_str(); }
+
+}  // extern "C"

@@ -1,0 +1,152 @@
+// tsp2opt_device.cuh -- device-side arithmetic of the sm_100a 2-opt path.
+//
+// Shared by the sweep, apply, load and self-test kernels of libtsp2opt.so only
+// (never by oracle/).  Citations: PAPER.md line = page;
+// readings R1..R13 in DESIGN.md §3.
+#pragma once
+
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace tsp2opt {
+
+// ---------------------------------------------------------------------------
+// Packed best-move key (reading R5: lowest delta, then lowest Fig. 3 cell
+// k = j(j-1)/2 + i, i.e. lowest j then lowest i):
+//   key = (delta + 2^18) << 44 | j << 22 | i,  bit 63 == 0,
+// so unsigned and signed int64 order agree (atomicMin(u64), NCCL MIN on int64).
+// |delta| <= 2 * 46340 < 2^18 and n <= 2^22.
+// ---------------------------------------------------------------------------
+constexpr int kKeyDeltaShift = 44;
+constexpr int kKeyJShift = 22;
+constexpr int kDeltaBias = 1 << 18;
+constexpr unsigned long long kKeyNone = ~0ULL;
+
+__host__ __device__ __forceinline__ unsigned long long pack_key(int delta, int i, int j)
+{
+    return ((unsigned long long)(unsigned)(delta + kDeltaBias) << kKeyDeltaShift) |
+           ((unsigned long long)(unsigned)j << kKeyJShift) | (unsigned long long)(unsigned)i;
+}
+__host__ __device__ __forceinline__ int key_delta(unsigned long long k)
+{
+    return (int)(k >> kKeyDeltaShift) - kDeltaBias;
+}
+__host__ __device__ __forceinline__ int key_j(unsigned long long k) { return (int)((k >> kKeyJShift) & 0x3FFFFF); }
+__host__ __device__ __forceinline__ int key_i(unsigned long long k) { return (int)(k & 0x3FFFFF); }
+
+// The degenerate pair (0,1) has delta 0 and cell 0 (reading R7): every sweep
+// starts from it, so a sweep at a local minimum returns (0, 1, 0).
+__host__ __device__ __forceinline__ unsigned long long seed_key() { return pack_key(0, 0, 1); }
+
+// ---------------------------------------------------------------------------
+// Coordinates live on the device as float(x + 2^23): the float difference of
+// two such values is the exact integer difference (same exponent, ulp 1), and
+// the raw bits minus 0x4B000000 give x back for the exact integer path.
+// ---------------------------------------------------------------------------
+constexpr float kCoordBias = 8388608.0f;  // 2^23
+__host__ __device__ __forceinline__ float bias_coord(int x) { return (float)(x + (1 << 23)); }
+__device__ __forceinline__ int unbias(float f) { return __float_as_int(f) - 0x4B000000; }
+
+__device__ __forceinline__ float sqrt_approx(float x)
+{
+    float r;
+    asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+    return r;
+}
+
+// Exact TSPLIB EUC_2D nint(sqrt(s)) for 0 <= s <= 2*32767^2 (reading R3/R4):
+// one MUFU.SQRT estimate rounded to the nearest integer m, then one integer
+// correction step using  nint(sqrt(s)) = m  <=>  m^2 - m < s <= m^2 + m.
+// Exhaustively verified on the device over every s (tsp2opt_selftest).
+__device__ __forceinline__ int nint_sqrt_exact(int s)
+{
+    float r = sqrt_approx(__int2float_rn(s));
+    int m = __float2int_rn(r);
+    long long ss = s, mm = (long long)m * m;
+    if (ss > mm + m) m += 1;
+    else if (ss <= mm - m) m -= 1;
+    return m;
+}
+
+__device__ __forceinline__ int exact_dist_xy(int xa, int ya, int xb, int yb)
+{
+    int dx = xa - xb, dy = ya - yb;
+    return nint_sqrt_exact(dx * dx + dy * dy);
+}
+
+__device__ __forceinline__ int exact_dist_biased(float2 a, float2 b)
+{
+    return exact_dist_xy(unbias(a.x), unbias(a.y), unbias(b.x), unbias(b.y));
+}
+
+// ---------------------------------------------------------------------------
+// Squared-distance prefilter.  For an integer t:
+//   nint(sqrt(s)) <= t  <=>  s <= t^2 + t   (t >= 0; impossible for t < 0).
+// sq_threshold(t) returns a float S_f >= (t^2 + t)(1 + 2^-21) for t >= 0 and a
+// negative value for t < 0.  The float squared distance s_f = fma(dx,dx,dy*dy)
+// satisfies s_f <= s (1 + 2^-23 + 2^-48) (two roundings, exact dx, dy), so
+// s <= t^2 + t  implies  s_f <= S_f: the filter never rejects a pair the exact
+// test would accept.  Exhaustively verified on the device (tsp2opt_selftest).
+// ---------------------------------------------------------------------------
+constexpr float kThrScale = 1.00000095367431640625f;  // 1 + 2^-20
+__device__ __forceinline__ float sq_threshold(float t)
+{
+    float tt = fmaxf(t, -0.5f);            // t < 0  ->  tt^2 + tt = -0.25 < 0
+    return fmaf(tt, tt, tt) * kThrScale;
+}
+
+// ---------------------------------------------------------------------------
+// Blackwell packed FP32x2 arithmetic (FADD2 / FMUL2 / FFMA2): one issue slot
+// for two lanes' worth of FP32 work.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ float2 add2(float2 a, float2 b)
+{
+    float2 r;
+    asm("{\n\t.reg .b64 ra, rb, rd;\n\t"
+        "mov.b64 ra, {%2, %3};\n\tmov.b64 rb, {%4, %5};\n\t"
+        "add.rn.f32x2 rd, ra, rb;\n\tmov.b64 {%0, %1}, rd;\n\t}"
+        : "=f"(r.x), "=f"(r.y) : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y));
+    return r;
+}
+__device__ __forceinline__ float2 mul2(float2 a, float2 b)
+{
+    float2 r;
+    asm("{\n\t.reg .b64 ra, rb, rd;\n\t"
+        "mov.b64 ra, {%2, %3};\n\tmov.b64 rb, {%4, %5};\n\t"
+        "mul.rn.f32x2 rd, ra, rb;\n\tmov.b64 {%0, %1}, rd;\n\t}"
+        : "=f"(r.x), "=f"(r.y) : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y));
+    return r;
+}
+__device__ __forceinline__ float2 fma2(float2 a, float2 b, float2 c)
+{
+    float2 r;
+    asm("{\n\t.reg .b64 ra, rb, rc, rd;\n\t"
+        "mov.b64 ra, {%2, %3};\n\tmov.b64 rb, {%4, %5};\n\tmov.b64 rc, {%6, %7};\n\t"
+        "fma.rn.f32x2 rd, ra, rb, rc;\n\tmov.b64 {%0, %1}, rd;\n\t}"
+        : "=f"(r.x), "=f"(r.y)
+        : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y), "f"(c.x), "f"(c.y));
+    return r;
+}
+
+// Squared distances of two row cities (packed) to one column city given as
+// negated biased coordinates (-x, -x) / (-y, -y):  s = dx*dx + dy*dy.
+__device__ __forceinline__ float2 sq2(float2 xr, float2 yr, float2 ncx, float2 ncy)
+{
+    float2 dx = add2(xr, ncx);
+    float2 dy = add2(yr, ncy);
+    return fma2(dx, dx, mul2(dy, dy));
+}
+
+// Per-rank / per-handle device state, ping-ponged between iterations: the
+// kernels of iteration t read slot[t & 1] and write slot[(t + 1) & 1], so no
+// kernel ever reads a field another block of the same kernel writes.
+struct __align__(64) Slot {
+    unsigned long long key;       // best-move key of the sweep reading this slot (atomicMin target)
+    unsigned long long last_key;  // key of the most recent finished sweep
+    long long moves;              // moves applied since the tour was loaded
+    long long length;             // current tour length (int64: n * 46340 > 2^31)
+    int done;                     // 0 running, 1 local minimum, 2 capped, bit 2 (4): invalid tour
+    int pad[7];
+};
+
+}  // namespace tsp2opt

@@ -1,0 +1,37 @@
+// tsp2opt_internal.h -- host-side declarations shared by the kernels and the
+// C-ABI runtime of libtsp2opt.so (not part of the public ABI; see include/tsp2opt.h).
+#pragma once
+
+#include <atomic>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "tsp2opt_device.cuh"
+
+namespace tsp2opt {
+
+constexpr int kRows = 15;     // R: rows per lane (R + 1 = 16 cities, 8 packed FP32x2 pairs)
+constexpr int kMaxTJ = 1024;  // columns per tile, upper bound (shared memory sizing)
+constexpr int kMaxWarps = 4;  // warps per CTA, upper bound (__launch_bounds__(128))
+constexpr int kPad = 32 * kRows * kMaxWarps + kMaxTJ + 8;  // P/E/tour padding beyond n
+
+struct Geometry {
+    int rows;   // R
+    int warps;  // warps per CTA
+    int tj;     // columns per tile
+    int ti() const { return 32 * rows * warps; }
+};
+
+long long launch_count();
+size_t sweep_smem_bytes(int TJ);
+cudaError_t sweep_prepare();
+cudaError_t launch_load_tour(const int* coords, const int* tour_src, int* tour_dst, float2* P, int* E, int n,
+                             Slot* slot, unsigned* stamp, unsigned epoch, cudaStream_t st);
+cudaError_t launch_reset_key(Slot* slot, cudaStream_t st);
+cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
+                         Slot* slot, int respect_done, cudaStream_t st);
+cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Slot* out, long long max_moves,
+                         int explicit_move, int ei, int ej, cudaStream_t st);
+cudaError_t run_selftest(long long* dist_bad, long long* filter_bad);
+
+}  // namespace tsp2opt

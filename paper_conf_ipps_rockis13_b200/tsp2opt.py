@@ -1,0 +1,277 @@
+"""Thin ctypes binding of libtsp2opt.so (include/tsp2opt.h).
+
+Argument marshalling only: every step of the 2-opt path runs in the library's
+CUDA kernels.  There is no CPU fallback: if the shared library is missing or
+no CUDA device is present, calls raise.  Function names mirror the C ABI
+without the `tsp2opt_` prefix; `TSP2Opt` is a convenience wrapper that owns a
+handle.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+from ._build import LIB
+
+OK, MAXITER = 0, 1
+EINVAL, ERANGE, ENOTPERM, ESTATE, ECUDA, ENCCL, ENOMEM = -1, -2, -3, -4, -5, -6, -7
+NCCL_ID_BYTES = 128
+MAX_ITERS_UNBOUNDED = (1 << 63) - 1
+
+_lib = None
+
+
+class TSP2OptError(RuntimeError):
+    def __init__(self, code: int, where: str):
+        self.code = code
+        msg = _L().tsp2opt_strerror(code).decode()
+        extra = _L().tsp2opt_last_error().decode()
+        super().__init__(f"{where}: {msg} ({code})" + (f" [{extra}]" if extra else ""))
+
+
+def _L():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB):
+            raise RuntimeError(
+                f"{LIB} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'` "
+                "(no CPU fallback exists)")
+        lib = ctypes.CDLL(LIB)
+        P, I32, I64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+        pI32, pI64 = ctypes.POINTER(I32), ctypes.POINTER(I64)
+        sig = {
+            "tsp2opt_create": ([P, I32, ctypes.POINTER(P)], I32),
+            "tsp2opt_create_sharded": ([P, I32, I32, I32, P, ctypes.POINTER(P)], I32),
+            "tsp2opt_nccl_unique_id": ([P], I32),
+            "tsp2opt_destroy": ([P], None),
+            "tsp2opt_set_stream": ([P, P], I32),
+            "tsp2opt_set_tour": ([P, P], I32),
+            "tsp2opt_set_tour_device_async": ([P, P], I32),
+            "tsp2opt_best_move": ([P, P, pI32, pI32, pI32], I32),
+            "tsp2opt_apply": ([P, I32, I32], I32),
+            "tsp2opt_iterate_async": ([P, I32], I32),
+            "tsp2opt_sync": ([P, pI64, pI64, pI32, pI32, pI32, pI32], I32),
+            "tsp2opt_local_search": ([P, P, I64, pI64, pI64], I32),
+            "tsp2opt_get_tour": ([P, P, pI64], I32),
+            "tsp2opt_debug_set_shard": ([P, I32, I32], I32),
+            "tsp2opt_get_geometry": ([P, pI32, pI32, pI32, pI64, pI64], I32),
+            "tsp2opt_selftest": ([pI64, pI64], I32),
+            "tsp2opt_profile": ([P, I32], I32),
+            "tsp2opt_profile_read": ([P, ctypes.POINTER(ctypes.c_double), pI64], I32),
+            "tsp2opt_launch_count": ([], I64),
+            "tsp2opt_strerror": ([I32], ctypes.c_char_p),
+            "tsp2opt_last_error": ([], ctypes.c_char_p),
+        }
+        for name, (args, res) in sig.items():
+            f = getattr(lib, name)
+            f.argtypes = args
+            f.restype = res
+        _lib = lib
+    return _lib
+
+
+def exported_symbols():
+    """Names of the C-ABI entry points the binding expects (all declared in include/tsp2opt.h)."""
+    _L()
+    return [n for n in dir(_lib) if n.startswith("tsp2opt_")]
+
+
+def _check(code: int, where: str) -> int:
+    if code < 0:
+        raise TSP2OptError(code, where)
+    return code
+
+
+def _i32(a) -> np.ndarray:
+    return np.ascontiguousarray(np.asarray(a, dtype=np.int32))
+
+
+def _ptr(a: np.ndarray):
+    return ctypes.c_void_p(a.ctypes.data)
+
+
+# ----------------------------------------------------------------------------- C-ABI mirrors
+
+def create(coords) -> ctypes.c_void_p:
+    xy = _i32(coords).reshape(-1)
+    h = ctypes.c_void_p()
+    _check(_L().tsp2opt_create(_ptr(xy), xy.size // 2, ctypes.byref(h)), "tsp2opt_create")
+    return h
+
+
+def create_sharded(coords, rank: int, world: int, nccl_id: bytes | None) -> ctypes.c_void_p:
+    xy = _i32(coords).reshape(-1)
+    h = ctypes.c_void_p()
+    idbuf = None if nccl_id is None else ctypes.create_string_buffer(bytes(nccl_id), NCCL_ID_BYTES)
+    _check(_L().tsp2opt_create_sharded(_ptr(xy), xy.size // 2, rank, world, idbuf, ctypes.byref(h)),
+           "tsp2opt_create_sharded")
+    return h
+
+
+def nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(NCCL_ID_BYTES)
+    _check(_L().tsp2opt_nccl_unique_id(buf), "tsp2opt_nccl_unique_id")
+    return buf.raw
+
+
+def destroy(h) -> None:
+    _L().tsp2opt_destroy(h)
+
+
+def set_stream(h, stream_handle: int | None) -> None:
+    _check(_L().tsp2opt_set_stream(h, ctypes.c_void_p(stream_handle or 0)), "tsp2opt_set_stream")
+
+
+def set_tour(h, tour) -> None:
+    t = _i32(tour)
+    _check(_L().tsp2opt_set_tour(h, _ptr(t)), "tsp2opt_set_tour")
+
+
+def set_tour_device_async(h, device_ptr: int) -> None:
+    _check(_L().tsp2opt_set_tour_device_async(h, ctypes.c_void_p(device_ptr)), "tsp2opt_set_tour_device_async")
+
+
+def best_move(h, tour=None):
+    i, j, d = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+    if tour is None:
+        tp = None
+    else:
+        t = _i32(tour)
+        tp = _ptr(t)
+    _check(_L().tsp2opt_best_move(h, tp, ctypes.byref(i), ctypes.byref(j), ctypes.byref(d)), "tsp2opt_best_move")
+    return i.value, j.value, d.value
+
+
+def apply(h, i: int, j: int) -> None:
+    _check(_L().tsp2opt_apply(h, int(i), int(j)), "tsp2opt_apply")
+
+
+def iterate_async(h, count: int) -> None:
+    _check(_L().tsp2opt_iterate_async(h, int(count)), "tsp2opt_iterate_async")
+
+
+def sync(h) -> dict:
+    it, L = ctypes.c_int64(), ctypes.c_int64()
+    cv, li, lj, ld = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+    _check(_L().tsp2opt_sync(h, ctypes.byref(it), ctypes.byref(L), ctypes.byref(cv), ctypes.byref(li),
+                             ctypes.byref(lj), ctypes.byref(ld)), "tsp2opt_sync")
+    return dict(iterations=it.value, length=L.value, converged=cv.value, last_move=(li.value, lj.value, ld.value))
+
+
+def local_search(h, tour, max_iters: int | None = None):
+    """Returns dict(tour, length, iterations, status) with status OK (0) or MAXITER (1)."""
+    t = np.array(tour, dtype=np.int32, copy=True)
+    L, it = ctypes.c_int64(), ctypes.c_int64()
+    mi = MAX_ITERS_UNBOUNDED if max_iters is None else int(max_iters)
+    st = _check(_L().tsp2opt_local_search(h, _ptr(t), mi, ctypes.byref(L), ctypes.byref(it)), "tsp2opt_local_search")
+    return dict(tour=t, length=L.value, iterations=it.value, status=st)
+
+
+def get_tour(h, n: int):
+    """(tour int32[n], length) of handle h (n = the handle's city count)."""
+    t = np.empty(n, dtype=np.int32)
+    L = ctypes.c_int64()
+    _check(_L().tsp2opt_get_tour(h, _ptr(t), ctypes.byref(L)), "tsp2opt_get_tour")
+    return t, L.value
+
+
+def debug_set_shard(h, rank: int, world: int) -> None:
+    _check(_L().tsp2opt_debug_set_shard(h, rank, world), "tsp2opt_debug_set_shard")
+
+
+def get_geometry(h) -> dict:
+    R, w, tj = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+    tiles, pairs = ctypes.c_int64(), ctypes.c_int64()
+    _check(_L().tsp2opt_get_geometry(h, ctypes.byref(R), ctypes.byref(w), ctypes.byref(tj), ctypes.byref(tiles),
+                                     ctypes.byref(pairs)), "tsp2opt_get_geometry")
+    return dict(rows=R.value, warps=w.value, tj=tj.value, tiles=tiles.value, pairs=pairs.value)
+
+
+def selftest() -> tuple[int, int]:
+    a, b = ctypes.c_int64(), ctypes.c_int64()
+    _check(_L().tsp2opt_selftest(ctypes.byref(a), ctypes.byref(b)), "tsp2opt_selftest")
+    return a.value, b.value
+
+
+def profile(h, enable: bool) -> None:
+    _check(_L().tsp2opt_profile(h, 1 if enable else 0), "tsp2opt_profile")
+
+
+def profile_read(h):
+    """(summed device ms of the recorded sweep launches, number of launches)."""
+    ms, n = ctypes.c_double(), ctypes.c_int64()
+    _check(_L().tsp2opt_profile_read(h, ctypes.byref(ms), ctypes.byref(n)), "tsp2opt_profile_read")
+    return ms.value, n.value
+
+
+def launch_count() -> int:
+    return int(_L().tsp2opt_launch_count())
+
+
+# ----------------------------------------------------------------------------- convenience wrapper
+
+class TSP2Opt:
+    """One library handle (one GPU / one rank)."""
+
+    def __init__(self, coords, rank: int = 0, world: int = 1, nccl_id: bytes | None = None):
+        xy = _i32(coords).reshape(-1, 2)
+        self.n = xy.shape[0]
+        self.h = create(xy) if world == 1 else create_sharded(xy, rank, world, nccl_id)
+
+    def close(self):
+        if self.h:
+            destroy(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def set_stream(self, stream_handle: int | None):
+        set_stream(self.h, stream_handle)
+
+    def set_tour(self, tour):
+        set_tour(self.h, tour)
+
+    def set_tour_device_async(self, device_ptr: int):
+        set_tour_device_async(self.h, device_ptr)
+
+    def best_move(self, tour=None):
+        return best_move(self.h, tour)
+
+    def apply(self, i, j):
+        apply(self.h, i, j)
+
+    def iterate_async(self, count: int):
+        iterate_async(self.h, count)
+
+    def sync(self):
+        return sync(self.h)
+
+    def local_search(self, tour, max_iters=None):
+        return local_search(self.h, tour, max_iters)
+
+    def get_tour(self):
+        return get_tour(self.h, self.n)
+
+    def debug_set_shard(self, rank, world):
+        debug_set_shard(self.h, rank, world)
+
+    def geometry(self):
+        return get_geometry(self.h)
+
+    def profile(self, enable: bool):
+        profile(self.h, enable)
+
+    def profile_read(self):
+        return profile_read(self.h)

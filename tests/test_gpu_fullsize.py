@@ -1,0 +1,42 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py
+times: one sweep per config vs the oracle (the oracle computes one sweep of
+n = 85900 in seconds on the box's cores), plus properties that hold at any size."""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_ipps_rockis13_b200 import inputs, tsp2opt
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("cfg", ["C3", "C4", "C5"])
+def test_full_size_first_sweep(gpu, cfg):
+    c, t = inputs.config_instance(cfg)
+    with tsp2opt.TSP2Opt(c) as g:
+        assert g.best_move(t) == oracle.best_move(c, t)
+
+
+@pytest.mark.parametrize("cfg", ["C4", "C5"])
+def test_full_size_iterations_invariants(gpu, cfg):
+    """A few device-resident iterations: length bookkeeping == full recomputation,
+    tour stays a permutation with tour[0] fixed, and the next sweep matches the oracle."""
+    c, t = inputs.config_instance(cfg)
+    with tsp2opt.TSP2Opt(c) as g:
+        g.set_tour(t)
+        L0 = oracle.tour_length(c, t)
+        assert g.sync()["length"] == L0
+        g.iterate_async(5)
+        s = g.sync()
+        tour, L = g.get_tour()
+        assert s["iterations"] == 5
+        assert sorted(tour.tolist()) == list(range(len(t))) and tour[0] == t[0]
+        assert L == oracle.tour_length(c, tour) < L0
+        assert g.best_move() == oracle.best_move(c, tour)
+
+
+def test_C5_hilbert_start_sweep(gpu):
+    c, _ = inputs.config_instance("C5")
+    th = inputs.hilbert_tour(c)
+    with tsp2opt.TSP2Opt(c) as g:
+        assert g.best_move(th) == oracle.best_move(c, th)
