@@ -141,10 +141,12 @@ def run_ours(args):
         g = tsp2opt.TSP2Opt(coords, rank, world, obj[0])
     else:
         g = tsp2opt.TSP2Opt(coords)
-    stream = torch.cuda.current_stream()
+    stream = torch.cuda.Stream()  # a real stream: events and the library's launches share it
+    torch.cuda.set_stream(stream)
     g.set_stream(stream.cuda_stream)
     d_tour = torch.from_numpy(tour).cuda()
     flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device="cuda")
+    torch.cuda.synchronize()
 
     def step():
         g.set_tour_device_async(d_tour.data_ptr())
@@ -329,7 +331,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C5")
     ap.add_argument("--tour", default="random", choices=["random", "hilbert"])
-    ap.add_argument("--ls-config", default="C2,C3", help="configs timed to a local minimum (rank 0, N=1)")
+    ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert", help="configs timed to a local minimum (rank 0, N=1)")
     ap.add_argument("--no-ls", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)

@@ -142,8 +142,10 @@ int tsp2opt_get_geometry(tsp2opt_t h, int32_t *R, int32_t *warps, int32_t *tj,
  * device functions): (a) the exact distance d(s) over every s in [0, 2*32767^2]
  * against m^2 - m < s <= m^2 + m; (b) the squared-distance prefilter never
  * rejects: for every (dx, dy) in [0, 32767]^2 the float s(dx,dy) passes the
- * float threshold built from t = d(dx,dy).  Writes the violation counts. */
-int tsp2opt_selftest(int64_t *dist_violations, int64_t *filter_violations);
+ * float threshold built from t = d(dx,dy).  Writes the violation counts and
+ * (may be NULL) the smallest violating s and (dx << 15 | dy), or -1. */
+int tsp2opt_selftest(int64_t *dist_violations, int64_t *filter_violations, int64_t *first_bad_s,
+                     int64_t *first_bad_dxdy);
 
 /* Sweep-kernel timing: enable != 0 starts recording a CUDA event pair around
  * every sweep launch of this handle (previous records are dropped); enable == 0

@@ -487,13 +487,16 @@ int tsp2opt_get_geometry(tsp2opt_t h, int32_t* R, int32_t* warps, int32_t* tj, i
     return TSP2OPT_OK;
 }
 
-int tsp2opt_selftest(int64_t* dist_violations, int64_t* filter_violations)
+int tsp2opt_selftest(int64_t* dist_violations, int64_t* filter_violations, int64_t* first_bad_s,
+                     int64_t* first_bad_dxdy)
 {
     if (!dist_violations || !filter_violations) return TSP2OPT_EINVAL;
-    long long a = -1, b = -1;
-    CUDA_TRY(run_selftest(&a, &b));
-    *dist_violations = a;
-    *filter_violations = b;
+    long long r[4] = {-1, -1, -1, -1};
+    CUDA_TRY(run_selftest(r));
+    *dist_violations = r[0];
+    *filter_violations = r[1];
+    if (first_bad_s) *first_bad_s = r[0] ? r[2] : -1;
+    if (first_bad_dxdy) *first_bad_dxdy = r[1] ? r[3] : -1;
     return TSP2OPT_OK;
 }
 

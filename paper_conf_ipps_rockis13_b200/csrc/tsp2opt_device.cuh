@@ -64,7 +64,7 @@ __device__ __forceinline__ int nint_sqrt_exact(int s)
     int m = __float2int_rn(r);
     long long ss = s, mm = (long long)m * m;
     if (ss > mm + m) m += 1;
-    else if (ss <= mm - m) m -= 1;
+    else if (m > 0 && ss <= mm - m) m -= 1;  // m = 0: nothing is below 0
     return m;
 }
 

@@ -32,6 +32,6 @@ cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n
                          Slot* slot, int respect_done, cudaStream_t st);
 cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Slot* out, long long max_moves,
                          int explicit_move, int ei, int ej, cudaStream_t st);
-cudaError_t run_selftest(long long* dist_bad, long long* filter_bad);
+cudaError_t run_selftest(long long* out4);  // dist_bad, filter_bad, first bad s, first bad dx<<15|dy
 
 }  // namespace tsp2opt

@@ -81,9 +81,8 @@ __global__ void reset_key_kernel(Slot* slot) { slot->key = seed_key(); }
 // ===========================================================================
 template <int R>
 struct Rows {
-    float2 xp[(R + 1) / 2];  // (x_r, x_{r+1}) packed pairs, biased floats
+    float2 xp[(R + 1) / 2];  // (x_r, x_{r+1}) packed pairs, biased floats, r = 0..R
     float2 yp[(R + 1) / 2];
-    float ef[R];             // e_{i_r} as float (exact integers)
 };
 
 template <int R>
@@ -98,97 +97,128 @@ __device__ __forceinline__ void column_sq(float (&s)[R + 1], const Rows<R>& rows
     }
 }
 
-__device__ __forceinline__ float row_x(const float2* xp, int r) { return (r & 1) ? xp[r >> 1].y : xp[r >> 1].x; }
-
 template <int R>
 struct Bound {
-    int B;      // accept delta < B
-    float a1f;  // row offset  a1 = floor((B - 2) / 2)
+    int B;      // accept delta < B (lane-local running bound)
     float a2f;  // column offset a2 = (B - 2) - a1
-    float srow[R];
+    float srow[R];  // row thresholds: D(i_r, j) <= e_{i_r} + a1  <=>  s <= srow[r]
 };
 
+// Thresholds of the exact necessary condition for bound B:
+// delta <= B - 1 = c  ==>  D(i,j) <= e_i + a1  or  D(i+1,j+1) <= e_j + a2,
+// a1 = floor((c - 1) / 2), a2 = c - 1 - a1.  Row edges are re-read from E
+// (L1-resident; this runs once per tile and when B drops).
 template <int R>
-__device__ __forceinline__ void set_bound(Bound<R>& b, const Rows<R>& rows, int B)
+__device__ __forceinline__ void set_bound(Bound<R>& b, const int* __restrict__ E, int row0, int B)
 {
     b.B = B;
-    const int c = B - 1;          // need delta <= c
-    const int a1 = (c - 1) >> 1;  // floor((c - 1) / 2)
+    const int c = B - 1;
+    const int a1 = (c - 1) >> 1;
     const int a2 = c - 1 - a1;
-    b.a1f = (float)a1;
     b.a2f = (float)a2;
 #pragma unroll
-    for (int r = 0; r < R; r++) b.srow[r] = sq_threshold(rows.ef[r] + b.a1f);
+    for (int r = 0; r < R; r++) b.srow[r] = sq_threshold((float)(E[row0 + r] + a1));
 }
 
-// Exact evaluation of the candidate pairs of one column step (rare path).
+// The fast test of one column step: does any pair (i_r, j), r < R, of this
+// lane pass the necessary condition?  Four independent predicate chains keep
+// the dependency depth short.
 template <int R, bool MASK>
-__device__ __forceinline__ void exact_step(const Rows<R>& rows, Bound<R>& b, const float (&cur)[R + 1],
-                                        const float (&nxt)[R + 1], float scol, int row0, int j,
-                                        float4 c0, float4 c1, float ej, unsigned long long& mykey)
+__device__ __forceinline__ bool step_any(const Bound<R>& b, const float (&cur)[R + 1], const float (&nxt)[R + 1],
+                                         float scol, int row0, int j)
 {
-    const int xj = unbias(-c0.x), yj = unbias(-c0.z);
-    const int xj1 = unbias(-c1.x), yj1 = unbias(-c1.z);
-    const int ejn = (int)ej;
-    bool changed = false;
+    if (!MASK) {
+        float m = nxt[1];
+#pragma unroll
+        for (int r = 2; r <= R; r++) m = fminf(m, nxt[r]);
+        bool a0 = m <= scol, a1 = false, a2 = false, a3 = false;
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            const bool t = cur[r] <= b.srow[r];
+            if ((r & 3) == 0) a0 |= t;
+            else if ((r & 3) == 1) a1 |= t;
+            else if ((r & 3) == 2) a2 |= t;
+            else a3 |= t;
+        }
+        return (a0 | a1) | (a2 | a3);
+    } else {
+        bool any = false;
+#pragma unroll
+        for (int r = 0; r < R; r++) any |= ((cur[r] <= b.srow[r]) || (nxt[r + 1] <= scol)) && (row0 + r < j);
+        return any;
+    }
+}
+
+// Exact evaluation of this lane's candidate pairs of column step j (rare path;
+// only lanes with a candidate run it).  Integer nint distances, identical
+// arithmetic to the oracle; accept delta < B in increasing cell order.
+template <int R, bool MASK>
+__device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1], const float (&nxt)[R + 1],
+                                           float scol, int row0, int j, float4 c0, float4 c1, float ej,
+                                           const float2* __restrict__ P, const int* __restrict__ E,
+                                           unsigned long long& mykey)
+{
+    unsigned mask = 0;
 #pragma unroll
     for (int r = 0; r < R; r++) {
         bool cand = (cur[r] <= b.srow[r]) || (nxt[r + 1] <= scol);
         if (MASK) cand = cand && (row0 + r < j);
-        if (cand) {
-            const int xi = unbias(row_x(rows.xp, r)), yi = unbias(row_x(rows.yp, r));
-            const int xi1 = unbias(row_x(rows.xp, r + 1)), yi1 = unbias(row_x(rows.yp, r + 1));
-            const int d = exact_dist_xy(xi, yi, xj, yj) + exact_dist_xy(xi1, yi1, xj1, yj1) -
-                          (int)rows.ef[r] - ejn;
-            if (d < b.B) {
-                b.B = d;
-                mykey = pack_key(d, row0 + r, j);
-                changed = true;
-            }
+        mask |= (cand ? 1u : 0u) << r;
+    }
+    const int xj = unbias(-c0.x), yj = unbias(-c0.z);
+    const int xj1 = unbias(-c1.x), yj1 = unbias(-c1.z);
+    const int ejn = (int)ej;
+    int B = b.B;
+    while (mask) {  // ascending r == ascending cell number
+        const int r = __ffs(mask) - 1;
+        mask &= mask - 1;
+        const float2 pi = P[row0 + r], pi1 = P[row0 + r + 1];
+        const int d = exact_dist_xy(unbias(pi.x), unbias(pi.y), xj, yj) +
+                      exact_dist_xy(unbias(pi1.x), unbias(pi1.y), xj1, yj1) - E[row0 + r] - ejn;
+        if (d < B) {
+            B = d;
+            mykey = pack_key(d, row0 + r, j);
         }
     }
-    if (changed) set_bound<R>(b, rows, b.B);
+    b.B = B;
 }
 
 template <int R, bool MASK>
 __device__ __forceinline__ void column_step(const Rows<R>& rows, Bound<R>& b, const float (&cur)[R + 1],
                                             float (&nxt)[R + 1], int row0, int j, int J0,
                                             const float4* __restrict__ colxy, const float* __restrict__ cole,
+                                            const float2* __restrict__ P, const int* __restrict__ E,
                                             unsigned long long& mykey)
 {
     const float4 c1 = colxy[j + 1 - J0];
     column_sq<R>(nxt, rows, c1);
     const float ej = cole[j - J0];
     const float scol = sq_threshold(ej + b.a2f);
-    bool any;
-    if (!MASK) {
-        float m = nxt[1];
-#pragma unroll
-        for (int r = 2; r <= R; r++) m = fminf(m, nxt[r]);
-        any = m <= scol;
-#pragma unroll
-        for (int r = 0; r < R; r++) any |= cur[r] <= b.srow[r];
-    } else {
-        any = false;
-#pragma unroll
-        for (int r = 0; r < R; r++) any |= ((cur[r] <= b.srow[r]) || (nxt[r + 1] <= scol)) && (row0 + r < j);
+    const bool any = step_any<R, MASK>(b, cur, nxt, scol, row0, j);
+    if (__builtin_expect(__any_sync(0xffffffffu, any), 0)) {
+        const int B0 = b.B;
+        if (any) exact_step<R, MASK>(b, cur, nxt, scol, row0, j, colxy[j - J0], c1, ej, P, E, mykey);
+        // share the warp's best: a lane may accept delta <= (best of another lane)
+        const int wb = __reduce_min_sync(0xffffffffu, b.B);
+        const int nb = min(b.B, wb + 1);
+        if (nb < B0) set_bound<R>(b, E, row0, nb);
     }
-    if (any) exact_step<R, MASK>(rows, b, cur, nxt, scol, row0, j, colxy[j - J0], c1, ej, mykey);
 }
 
 template <int R, bool MASK>
 __device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0, int jstart, int J0, int J1,
                                      const float4* __restrict__ colxy, const float* __restrict__ cole,
+                                     const float2* __restrict__ P, const int* __restrict__ E,
                                      unsigned long long& mykey)
 {
     float sa[R + 1], sb[R + 1];
     column_sq<R>(sa, rows, colxy[jstart - J0]);
     int j = jstart;
     for (; j + 1 < J1; j += 2) {
-        column_step<R, MASK>(rows, b, sa, sb, row0, j, J0, colxy, cole, mykey);
-        column_step<R, MASK>(rows, b, sb, sa, row0, j + 1, J0, colxy, cole, mykey);
+        column_step<R, MASK>(rows, b, sa, sb, row0, j, J0, colxy, cole, P, E, mykey);
+        column_step<R, MASK>(rows, b, sb, sa, row0, j + 1, J0, colxy, cole, P, E, mykey);
     }
-    if (j < J1) column_step<R, MASK>(rows, b, sa, sb, row0, j, J0, colxy, cole, mykey);
+    if (j < J1) column_step<R, MASK>(rows, b, sa, sb, row0, j, J0, colxy, cole, P, E, mykey);
 }
 
 template <int R>
@@ -197,9 +227,8 @@ __global__ void __launch_bounds__(128) sweep_kernel(const float2* __restrict__ P
                                                      int respect_done)
 {
     extern __shared__ float4 smem[];
-    float4* colxy = smem;                          // [TJ + 1]: (-x, -x, -y, -y) of column cities J0..J1
+    float4* colxy = smem;                                    // [TJ + 1]: (-x, -x, -y, -y) of columns J0..J1
     float* cole = reinterpret_cast<float*>(smem + TJ + 1);  // [TJ + 1]: e_j as float
-    __shared__ unsigned long long red[32];
 
     if (respect_done && *(volatile int*)&slot->done) return;  // converged: iteration is a no-op
     const int2 tile = tiles[blockIdx.x];
@@ -217,43 +246,34 @@ __global__ void __launch_bounds__(128) sweep_kernel(const float2* __restrict__ P
     const int wrow0 = I0 + warp * 32 * R;
     const int row0 = wrow0 + lane * R;
     const int jstart = max(J0, wrow0 + 1);  // no pair of this warp has j <= wrow0
+    if (jstart >= J1) return;                // warp-uniform: nothing to do
     unsigned long long mykey = kKeyNone;
-    if (jstart < J1) {
-        Rows<R> rows;
+    Rows<R> rows;
 #pragma unroll
-        for (int q = 0; q < (R + 1) / 2; q++) {
-            const float2 p0 = P[row0 + 2 * q], p1 = P[row0 + 2 * q + 1];
-            rows.xp[q] = make_float2(p0.x, p1.x);
-            rows.yp[q] = make_float2(p0.y, p1.y);
-        }
-#pragma unroll
-        for (int r = 0; r < R; r++) rows.ef[r] = (float)E[row0 + r];
-        // Start from the best key any CTA of this sweep has published so far.
-        // The slot key is the seed (0, cell 0) or a real pair of this sweep, so a
-        // pair of ours can only win with delta < 0 (if the key's delta is 0) or
-        // delta <= key delta otherwise.
-        const unsigned long long g = *(volatile unsigned long long*)&slot->key;
-        const int dg = key_delta(g);
-        Bound<R> b;
-        set_bound<R>(b, rows, dg == 0 ? 0 : dg + 1);
-        const bool masked = (wrow0 + 32 * R - 1) >= jstart;  // warp-uniform: some row >= some j
-        if (masked) walk<R, true>(rows, b, row0, jstart, J0, J1, colxy, cole, mykey);
-        else walk<R, false>(rows, b, row0, jstart, J0, J1, colxy, cole, mykey);
+    for (int q = 0; q < (R + 1) / 2; q++) {
+        const float2 p0 = P[row0 + 2 * q], p1 = P[row0 + 2 * q + 1];
+        rows.xp[q] = make_float2(p0.x, p1.x);
+        rows.yp[q] = make_float2(p0.y, p1.y);
     }
-    // a5: warp -> CTA -> one atomicMin per CTA (L16 Fig. 4 "Get best local pair ...
-    // Get best global pair"); min is order-independent, so the result is deterministic.
+    // Start from the best key any CTA of this sweep has published so far.  The
+    // slot key is the seed (0, cell 0) or a real pair of this sweep, so a pair of
+    // ours can only win with delta < 0 (key delta 0) or delta <= key delta.
+    const unsigned long long g = *(volatile unsigned long long*)&slot->key;
+    const int dg = key_delta(g);
+    Bound<R> b;
+    set_bound<R>(b, E, row0, dg == 0 ? 0 : dg + 1);
+    const bool masked = (wrow0 + 32 * R - 1) >= jstart;  // warp-uniform: some row >= some j
+    if (masked) walk<R, true>(rows, b, row0, jstart, J0, J1, colxy, cole, P, E, mykey);
+    else walk<R, false>(rows, b, row0, jstart, J0, J1, colxy, cole, P, E, mykey);
+
+    // a5: warp min, one atomicMin per warp (L16 Fig. 4 "Get best local pair ...
+    // Get best global pair"); min is order-independent -> deterministic result.
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
         const unsigned long long other = __shfl_xor_sync(0xffffffffu, mykey, o);
         mykey = other < mykey ? other : mykey;
     }
-    if (lane == 0) red[warp] = mykey;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        unsigned long long m = red[0];
-        for (int w = 1; w < (int)(blockDim.x >> 5); w++) m = red[w] < m ? red[w] : m;
-        if (m < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, m);
-    }
+    if (lane == 0 && mykey < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, mykey);
 }
 
 // ===========================================================================
@@ -327,18 +347,21 @@ __global__ void __launch_bounds__(256) apply_kernel(float2* __restrict__ P, int*
 // ===========================================================================
 // Exhaustive self-test kernels (tsp2opt_selftest).
 // ===========================================================================
-__global__ void selftest_dist_kernel(long long smax, unsigned long long* bad)
+__global__ void selftest_dist_kernel(long long smax, unsigned long long* bad, unsigned long long* first)
 {
     unsigned long long nbad = 0;
     for (long long s = (long long)blockIdx.x * blockDim.x + threadIdx.x; s <= smax;
          s += (long long)gridDim.x * blockDim.x) {
         const long long m = nint_sqrt_exact((int)s);
-        if (!(m * m - m < s && s <= m * m + m) && !(s == 0 && m == 0)) nbad++;
+        if (!(m * m - m < s && s <= m * m + m) && !(s == 0 && m == 0)) {
+            nbad++;
+            atomicMin(first, (unsigned long long)s);
+        }
     }
     if (nbad) atomicAdd(bad, nbad);
 }
 
-__global__ void selftest_filter_kernel(unsigned long long* bad)
+__global__ void selftest_filter_kernel(unsigned long long* bad, unsigned long long* first)
 {
     // every (dx, dy) in [0, 32767]^2; the float s is computed exactly as the
     // sweep does it (biased coordinates, FADD2 / FMUL2 / FFMA2)
@@ -355,8 +378,10 @@ __global__ void selftest_filter_kernel(unsigned long long* bad)
         const float2 s = sq2(xr, yr, ncx, ncy);
         const int t = nint_sqrt_exact(dx * dx + dy * dy);  // smallest t with "D <= t"
         const float S = sq_threshold((float)t);
-        if (!(s.x <= S)) nbad++;
-        if (!(s.y <= S)) nbad++;
+        if (!(s.x <= S) || !(s.y <= S)) {
+            nbad++;
+            atomicMin(first, (unsigned long long)id);
+        }
     }
     if (nbad) atomicAdd(bad, nbad);
 }
@@ -412,20 +437,20 @@ cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Sl
     return cudaGetLastError();
 }
 
-cudaError_t run_selftest(long long* dist_bad, long long* filter_bad)
+cudaError_t run_selftest(long long* out4)
 {
     unsigned long long* d = nullptr;
-    cudaError_t err = cudaMalloc(&d, 2 * sizeof(unsigned long long));
+    cudaError_t err = cudaMalloc(&d, 4 * sizeof(unsigned long long));
     if (err != cudaSuccess) return err;
-    cudaMemset(d, 0, 2 * sizeof(unsigned long long));
-    selftest_dist_kernel<<<148 * 8, 256>>>(2LL * 32767 * 32767, d);
-    selftest_filter_kernel<<<148 * 8, 256>>>(d + 1);
+    unsigned long long init[4] = {0, 0, ~0ULL, ~0ULL};
+    cudaMemcpy(d, init, sizeof(init), cudaMemcpyHostToDevice);
+    selftest_dist_kernel<<<148 * 8, 256>>>(2LL * 32767 * 32767, d, d + 2);
+    selftest_filter_kernel<<<148 * 8, 256>>>(d + 1, d + 3);
     g_launches += 2;
-    unsigned long long h[2] = {0, 0};
+    unsigned long long h[4];
     err = cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
     cudaFree(d);
-    *dist_bad = (long long)h[0];
-    *filter_bad = (long long)h[1];
+    for (int k = 0; k < 4; k++) out4[k] = (long long)h[k];
     return err;
 }
 

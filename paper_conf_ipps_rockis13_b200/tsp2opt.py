@@ -57,7 +57,7 @@ def _L():
             "tsp2opt_get_tour": ([P, P, pI64], I32),
             "tsp2opt_debug_set_shard": ([P, I32, I32], I32),
             "tsp2opt_get_geometry": ([P, pI32, pI32, pI32, pI64, pI64], I32),
-            "tsp2opt_selftest": ([pI64, pI64], I32),
+            "tsp2opt_selftest": ([pI64, pI64, pI64, pI64], I32),
             "tsp2opt_profile": ([P, I32], I32),
             "tsp2opt_profile_read": ([P, ctypes.POINTER(ctypes.c_double), pI64], I32),
             "tsp2opt_launch_count": ([], I64),
@@ -189,10 +189,11 @@ def get_geometry(h) -> dict:
     return dict(rows=R.value, warps=w.value, tj=tj.value, tiles=tiles.value, pairs=pairs.value)
 
 
-def selftest() -> tuple[int, int]:
-    a, b = ctypes.c_int64(), ctypes.c_int64()
-    _check(_L().tsp2opt_selftest(ctypes.byref(a), ctypes.byref(b)), "tsp2opt_selftest")
-    return a.value, b.value
+def selftest() -> dict:
+    a, b, c, d = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+    _check(_L().tsp2opt_selftest(ctypes.byref(a), ctypes.byref(b), ctypes.byref(c), ctypes.byref(d)),
+           "tsp2opt_selftest")
+    return dict(dist_violations=a.value, filter_violations=b.value, first_bad_s=c.value, first_bad_dxdy=d.value)
 
 
 def profile(h, enable: bool) -> None:

@@ -21,9 +21,9 @@ def _inst(kind, n, seed, tour="random"):
 
 
 def test_selftest_exhaustive_distance_and_filter(gpu):
-    dist_bad, filt_bad = tsp2opt.selftest()
-    assert dist_bad == 0, "exact nint(sqrt(s)) wrong for some s in [0, 2*32767^2]"
-    assert filt_bad == 0, "squared-distance prefilter rejects a reachable (dx, dy)"
+    r = tsp2opt.selftest()
+    assert r["dist_violations"] == 0, f"exact nint(sqrt(s)) wrong for some s in [0, 2*32767^2]: {r}"
+    assert r["filter_violations"] == 0, f"squared-distance prefilter rejects a reachable (dx, dy): {r}"
 
 
 SIZES = [3, 4, 5, 7, 16, 31, 32, 33, 100, 101, 479, 480, 481, 961, 1002, 1921, 2500]
