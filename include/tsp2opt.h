@@ -133,6 +133,15 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
  * one GPU that the min over shards equals the unsharded result. */
 int tsp2opt_debug_set_shard(tsp2opt_t h, int32_t rank, int32_t world);
 
+/* Host-only planning (no GPU needed): the tile shard a handle with n cities
+ * would sweep as `rank` of `world`.  *R, *warps, *tj: geometry; *ntiles,
+ * *pairs: this shard's tile count and pair count.  If tiles_out != NULL it
+ * receives 2 * min(*ntiles, cap) int32 (row start I0, column start J0) in
+ * launch order; a tile covers rows [I0, min(I0 + 32*R*warps, n-1)) x columns
+ * [J0, min(J0 + tj, n)), pairs i < j only. */
+int tsp2opt_plan_shard(int32_t n, int32_t rank, int32_t world, int32_t *R, int32_t *warps, int32_t *tj,
+                       int32_t *tiles_out, int64_t cap, int64_t *ntiles, int64_t *pairs);
+
 /* Sweep geometry actually used: rows per thread R, warps per CTA, columns per
  * tile TJ, number of tiles and pairs of this handle's shard. */
 int tsp2opt_get_geometry(tsp2opt_t h, int32_t *R, int32_t *warps, int32_t *tj,

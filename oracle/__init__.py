@@ -57,6 +57,8 @@ def _load():
             lib.oracle_cell.restype = i64
             lib.oracle_best_move.argtypes = [p, i64, p, p, p, p]
             lib.oracle_best_move.restype = None
+            lib.oracle_best_move_tiles.argtypes = [p, i64, p, p, i64, i64, i64, p, p, p]
+            lib.oracle_best_move_tiles.restype = None
             lib.oracle_apply.argtypes = [p, i64, i64]
             lib.oracle_apply.restype = None
             lib.oracle_local_search.argtypes = [p, i64, p, i64, p, p, p, i64]
@@ -113,6 +115,17 @@ def best_move(coords, tour):
         _ptr(xy), xy.shape[0], _ptr(t),
         _ptr(out[0:1]), _ptr(out[1:2]), _ptr(out[2:3]),
     )
+    return int(out[0]), int(out[1]), int(out[2])
+
+
+def best_move_tiles(coords, tour, tiles, ti: int, tj: int):
+    """(i, j, delta): best move over the pairs of the given tiles only."""
+    xy = _xy(coords)
+    t = np.ascontiguousarray(tour, dtype=np.int32)
+    tl = np.ascontiguousarray(np.asarray(tiles, dtype=np.int32).reshape(-1, 2))
+    out = np.zeros(3, dtype=np.int64)
+    _load().oracle_best_move_tiles(_ptr(xy), xy.shape[0], _ptr(t), _ptr(tl), tl.shape[0], ti, tj,
+                                   _ptr(out[0:1]), _ptr(out[1:2]), _ptr(out[2:3]))
     return int(out[0]), int(out[1]), int(out[2])
 
 

@@ -149,6 +149,29 @@ void oracle_best_move(const int32_t *xy, int64_t n, const int32_t *tour,
     *bi = best_i; *bj = best_j; *bdelta = best_d;
 }
 
+/* The same argmin restricted to a list of rectangular tiles of the pair
+ * matrix (L18 §IV.B problem division; L20 Fig. 7 "It is possible to calculate
+ * distances in arbitrary segments"): tile t covers rows [I0, min(I0+TI, n-1)) x
+ * columns [J0, min(J0+TJ, n)), pairs i < j only.  Used to check a shard of
+ * the multi-GPU split.  Returns (0, 1, 0) if no pair in the tiles beats it. */
+void oracle_best_move_tiles(const int32_t *xy, int64_t n, const int32_t *tour, const int32_t *tiles,
+                            int64_t ntiles, int64_t TI, int64_t TJ, int64_t *bi, int64_t *bj, int64_t *bdelta)
+{
+    int64_t best_d = 0, best_i = 0, best_j = 1;
+    for (int64_t t = 0; t < ntiles; t++) {
+        int64_t I0 = tiles[2 * t], J0 = tiles[2 * t + 1];
+        int64_t I1 = I0 + TI < n - 1 ? I0 + TI : n - 1, J1 = J0 + TJ < n ? J0 + TJ : n;
+        for (int64_t j = J0; j < J1; j++)
+            for (int64_t i = I0; i < I1 && i < j; i++) {
+                int64_t d = oracle_delta(xy, n, tour, i, j);
+                if (d < best_d || (d == best_d && oracle_cell(i, j) < oracle_cell(best_i, best_j))) {
+                    best_d = d; best_i = i; best_j = j;
+                }
+            }
+    }
+    *bi = best_i; *bj = best_j; *bdelta = best_d;
+}
+
 /* The 2-opt move (L12 §I.B "removes two edges ... reconnects ... reversing
  * order of sub-tour"; Fig. 1): reverse tour positions i+1..j (reading R6:
  * never the complement, so tour[0] never moves). */

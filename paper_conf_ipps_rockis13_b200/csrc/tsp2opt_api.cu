@@ -476,6 +476,27 @@ int tsp2opt_debug_set_shard(tsp2opt_t h, int32_t rank, int32_t world)
     return upload_shard(h, rank, world);
 }
 
+int tsp2opt_plan_shard(int32_t n, int32_t rank, int32_t world, int32_t* R, int32_t* warps, int32_t* tj,
+                       int32_t* tiles_out, int64_t cap, int64_t* ntiles, int64_t* pairs)
+{
+    if (n < 3 || n > TSP2OPT_MAX_N || world < 1 || rank < 0 || rank >= world || !ntiles || !pairs)
+        return TSP2OPT_EINVAL;
+    const Geometry g = choose_geometry((long long)n * (n - 1) / 2 / world);
+    long long p = 0;
+    std::vector<Tile> mine = shard_tiles(build_tiles(n, g), rank, world, &p);
+    if (R) *R = g.rows;
+    if (warps) *warps = g.warps;
+    if (tj) *tj = g.tj;
+    *ntiles = (int64_t)mine.size();
+    *pairs = p;
+    if (tiles_out)
+        for (size_t k = 0; k < mine.size() && (int64_t)k < cap; k++) {
+            tiles_out[2 * k] = mine[k].i0;
+            tiles_out[2 * k + 1] = mine[k].j0;
+        }
+    return TSP2OPT_OK;
+}
+
 int tsp2opt_get_geometry(tsp2opt_t h, int32_t* R, int32_t* warps, int32_t* tj, int64_t* tiles, int64_t* pairs)
 {
     if (!h) return TSP2OPT_EINVAL;

@@ -56,6 +56,7 @@ def _L():
             "tsp2opt_local_search": ([P, P, I64, pI64, pI64], I32),
             "tsp2opt_get_tour": ([P, P, pI64], I32),
             "tsp2opt_debug_set_shard": ([P, I32, I32], I32),
+            "tsp2opt_plan_shard": ([I32, I32, I32, pI32, pI32, pI32, P, I64, pI64, pI64], I32),
             "tsp2opt_get_geometry": ([P, pI32, pI32, pI32, pI64, pI64], I32),
             "tsp2opt_selftest": ([pI64, pI64, pI64, pI64], I32),
             "tsp2opt_profile": ([P, I32], I32),
@@ -179,6 +180,19 @@ def get_tour(h, n: int):
 
 def debug_set_shard(h, rank: int, world: int) -> None:
     _check(_L().tsp2opt_debug_set_shard(h, rank, world), "tsp2opt_debug_set_shard")
+
+
+def plan_shard(n: int, rank: int, world: int) -> dict:
+    """Host-only: geometry and tile list (int32[ntiles, 2] of (I0, J0)) of one shard."""
+    R, w, tj = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+    nt, pairs = ctypes.c_int64(), ctypes.c_int64()
+    _check(_L().tsp2opt_plan_shard(n, rank, world, ctypes.byref(R), ctypes.byref(w), ctypes.byref(tj), None, 0,
+                                   ctypes.byref(nt), ctypes.byref(pairs)), "tsp2opt_plan_shard")
+    tiles = np.zeros((nt.value, 2), dtype=np.int32)
+    _check(_L().tsp2opt_plan_shard(n, rank, world, None, None, None, _ptr(tiles), nt.value, ctypes.byref(nt),
+                                   ctypes.byref(pairs)), "tsp2opt_plan_shard")
+    return dict(rows=R.value, warps=w.value, tj=tj.value, ti=32 * R.value * w.value, tiles=tiles,
+                pairs=pairs.value)
 
 
 def get_geometry(h) -> dict:
