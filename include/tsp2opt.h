@@ -163,6 +163,16 @@ int tsp2opt_selftest(int64_t *dist_violations, int64_t *filter_violations, int64
 int tsp2opt_profile(tsp2opt_t h, int32_t enable);
 int tsp2opt_profile_read(tsp2opt_t h, double *total_ms, int64_t *launches);
 
+/* Exhaustive bound of the sweep's sqrt-sum prefilter input: the max relative
+ * error of the kernel's MUFU.SQRT over every float in [1, 2^31] (*max_rel_err)
+ * and whether sqrt(0) == 0 (*zero_ok).  DESIGN.md §5.2 needs <= 2^-21. */
+int tsp2opt_selftest_sqrt(double *max_rel_err, int32_t *zero_ok);
+
+/* Sweep counters of an instrumented build (-DTSP2OPT_STATS): out4[0] warp column
+ * steps, [1] steps that took the exact path, [2] candidate pairs evaluated
+ * exactly; -1 in product builds.  reset != 0 zeroes them afterwards. */
+int tsp2opt_debug_stats(int64_t *out4, int32_t reset);
+
 /* Number of this library's kernel launches since load (for gpu_launches). */
 int64_t tsp2opt_launch_count(void);
 

@@ -61,6 +61,10 @@ struct tsp2opt_ctx {
     int* d_E = nullptr;         // [n + pad] edges
     Slot* d_slots = nullptr;    // [2]
     unsigned* d_stamp = nullptr;  // [n] permutation check
+    unsigned* d_bar = nullptr;    // [2] grid barrier of the persistent local search (count, generation)
+    int* d_ctl = nullptr;         // [1] parity the persistent local search ended on
+    int* h_ctl = nullptr;         // pinned readback of d_ctl
+    int persistent = 2;           // local_search loop: 0 per-iteration kernels, 1 persistent launch, 2 auto
     int2* d_tiles = nullptr;    // this shard's tiles
     Slot* h_slot = nullptr;     // pinned readback
     unsigned epoch = 0;
@@ -166,6 +170,9 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_E);
     cudaFree(h->d_slots);
     cudaFree(h->d_stamp);
+    cudaFree(h->d_bar);
+    cudaFree(h->d_ctl);
+    if (h->h_ctl) cudaFreeHost(h->h_ctl);
     cudaFree(h->d_tiles);
     if (h->h_slot) cudaFreeHost(h->h_slot);
     for (cudaEvent_t e : h->ev_pool) cudaEventDestroy(e);
@@ -291,6 +298,11 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     CTRY(cudaMemset(h->d_tour, 0, sizeof(int) * np));
     CTRY(cudaMemset(h->d_E, 0, sizeof(int) * np));
     CTRY(cudaMemset(h->d_stamp, 0, sizeof(unsigned) * (size_t)n));
+    CTRY(cudaMalloc(&h->d_bar, sizeof(unsigned) * 2));
+    CTRY(cudaMemset(h->d_bar, 0, sizeof(unsigned) * 2));
+    CTRY(cudaMalloc(&h->d_ctl, sizeof(int)));
+    CTRY(cudaHostAlloc(&h->h_ctl, sizeof(int), cudaHostAllocDefault));
+    if (const char* ep = getenv("TSP2OPT_PERSISTENT")) h->persistent = atoi(ep);
     CTRY(cudaMemset(h->d_slots, 0, sizeof(Slot) * 2));
     {
         std::vector<float2> pad(np, make_float2(kCoordBias, kCoordBias));
@@ -437,8 +449,41 @@ int tsp2opt_local_search(tsp2opt_t h, int32_t* tour, int64_t max_iters, int64_t*
     if (!h || !tour || !length || !iterations || max_iters < 0) return TSP2OPT_EINVAL;
     int rc = load_host_tour(h, tour);
     if (rc) return rc;
-    // Device-resident loop: batches of K iterations between host checks; an
-    // iteration after convergence is a no-op (sweep CTAs exit on the done flag).
+    // Persistent single launch pays off while the per-iteration launch/sync
+    // overhead dominates the sweep (measured: faster up to n ~ 1e3, slower from
+    // n ~ 7e3 where the per-sweep kernels pack tiles better); TSP2OPT_PERSISTENT
+    // = 0 / 1 forces either loop, 2 (default) chooses by pair count.
+    const bool use_persistent =
+        !h->comm && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
+    if (use_persistent) {
+        // One persistent cooperative launch runs sweep -> apply to the local
+        // minimum; the per-launch iteration budget bounds a launch to roughly
+        // 2e12 pair checks (~0.5 s), after which the host relaunches.
+        const long long pairs = std::max(1LL, h->shard_pairs);
+        const long long budget = std::min(1LL << 20, std::max(16LL, 2000000000000LL / pairs));
+        for (long long launches = 0;; launches++) {
+            if (launches * budget > 1000LL * h->n + (1LL << 24)) {  // cannot happen: delta < 0 shortens the tour
+                g_last_error = "local search did not converge";
+                return TSP2OPT_ECUDA;
+            }
+            CUDA_TRY(launch_local_search(h->geo, h->d_P, h->d_E, h->d_tour, h->n, h->d_tiles, h->ntiles, h->d_slots,
+                                         h->parity, max_iters, budget, h->d_bar, h->d_ctl, h->stream));
+            CUDA_TRY(cudaMemcpyAsync(h->h_ctl, h->d_ctl, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+            CUDA_TRY(cudaStreamSynchronize(h->stream));
+            h->parity = *h->h_ctl;
+            rc = read_slot(h);
+            if (rc) return rc;
+            if (h->h_slot->done & 3) break;
+        }
+        CUDA_TRY(cudaMemcpyAsync(tour, h->d_tour, sizeof(int32_t) * h->n, cudaMemcpyDeviceToHost, h->stream));
+        CUDA_TRY(cudaStreamSynchronize(h->stream));
+        *length = h->h_slot->length;
+        *iterations = h->h_slot->moves;
+        return (h->h_slot->done & 3) == 2 ? TSP2OPT_MAXITER : TSP2OPT_OK;
+    }
+    // Multi-kernel loop (sharded handles): batches of K iterations between host
+    // checks; an iteration after convergence is a no-op (sweep CTAs exit on the
+    // done flag).
     long long k = 4;
     for (;;) {
         for (long long c = 0; c < k; c++) {
@@ -546,6 +591,25 @@ int tsp2opt_profile_read(tsp2opt_t h, double* total_ms, int64_t* launches)
 }
 
 int64_t tsp2opt_launch_count(void) { return launch_count(); }
+
+int tsp2opt_selftest_sqrt(double* max_rel_err, int32_t* zero_ok)
+{
+    if (!max_rel_err || !zero_ok) return TSP2OPT_EINVAL;
+    int z = 0;
+    CUDA_TRY(run_selftest_sqrt(max_rel_err, &z));
+    *zero_ok = z;
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_debug_stats(int64_t* out4, int32_t reset)
+{
+    if (!out4) return TSP2OPT_EINVAL;
+    long long r[4];
+    CUDA_TRY(cudaDeviceSynchronize());
+    CUDA_TRY(read_stats(r, reset));
+    for (int k = 0; k < 4; k++) out4[k] = r[k];
+    return TSP2OPT_OK;
+}
 
 const char* tsp2opt_strerror(int code)
 {

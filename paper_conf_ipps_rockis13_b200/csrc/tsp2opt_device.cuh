@@ -146,7 +146,8 @@ struct __align__(64) Slot {
     long long moves;              // moves applied since the tour was loaded
     long long length;             // current tour length (int64: n * 46340 > 2^31)
     int done;                     // 0 running, 1 local minimum, 2 capped, bit 2 (4): invalid tour
-    int pad[7];
+    unsigned next_tile;           // dynamic tile counter of the persistent sweep reading this slot
+    int pad[6];
 };
 
 }  // namespace tsp2opt

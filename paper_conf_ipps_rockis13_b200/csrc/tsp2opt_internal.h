@@ -23,7 +23,7 @@ struct Geometry {
 };
 
 long long launch_count();
-size_t sweep_smem_bytes(int TJ);
+size_t sweep_smem_bytes(const Geometry& g);
 cudaError_t sweep_prepare();
 cudaError_t launch_load_tour(const int* coords, const int* tour_src, int* tour_dst, float2* P, int* E, int n,
                              Slot* slot, unsigned* stamp, unsigned epoch, cudaStream_t st);
@@ -32,6 +32,11 @@ cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n
                          Slot* slot, int respect_done, cudaStream_t st);
 cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Slot* out, long long max_moves,
                          int explicit_move, int ei, int ej, cudaStream_t st);
+cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
+                                Slot* slots, int parity, long long max_moves, long long budget, unsigned* bar,
+                                int* ctl, cudaStream_t st);
+cudaError_t read_stats(long long* out4, int reset);
+cudaError_t run_selftest_sqrt(double* max_rel, int* zero_ok);
 cudaError_t run_selftest(long long* out4);  // dist_bad, filter_bad, first bad s, first bad dx<<15|dy
 
 }  // namespace tsp2opt

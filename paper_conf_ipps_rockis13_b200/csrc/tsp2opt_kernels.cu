@@ -9,6 +9,7 @@
 // tiles over the upper triangle only).  Design and B200 rationale: DESIGN.md §5.
 #include "tsp2opt_device.cuh"
 #include "tsp2opt_internal.h"
+#include "tsp2opt_sweep.cuh"
 
 namespace tsp2opt {
 
@@ -60,220 +61,25 @@ __global__ void init_slot_kernel(Slot* slot, int clear_length)
     slot->moves = 0;
     if (clear_length) slot->length = 0;
     slot->done = 0;
+    slot->next_tile = 0;
 }
 
 __global__ void reset_key_kernel(Slot* slot) { slot->key = seed_key(); }
 
-// ===========================================================================
-// a4 + a5: the sweep.  One CTA = one tile = rows [I0, I0 + 32*R*NW) x columns
-// [J0, J0 + TJ).  Each lane owns R consecutive rows (R+1 cities in registers),
-// the warp walks the tile's columns; column city j is a shared-memory broadcast.
-// Per column step the lane computes the R+1 squared distances of its rows to
-// column j+1 (diagonal reuse: s(i+1, j+1) of pair (i, j) is s(i', j') of pair
-// (i', j') = (i+1, j+1)), and tests every pair (i, j) with the exact
-// necessary condition of DESIGN.md §5.2:
-//     delta(i,j) <= B - 1   ==>   D(i,j) <= e_i + a1   or   D(i+1,j+1) <= e_j + a2
-// (a1 + a2 = B - 2), evaluated on squared distances (no sqrt).  Pairs that pass
-// are evaluated exactly (integer nint, same as the oracle) and accepted iff
-// delta < B; B is the lane's running bound, started from the global best.
-// Pairs are visited in increasing Fig. 3 cell order per lane, so a strict '<'
-// keeps the lowest cell among equal deltas (reading R5).
-// ===========================================================================
+// a4 + a5: the sweep of one tile lives in tsp2opt_sweep.cuh.
+
+#ifndef TSP2OPT_MINB
+#define TSP2OPT_MINB 4  // CTAs of 128 threads per SM the register allocation must allow
+#endif
 template <int R>
-struct Rows {
-    float2 xp[(R + 1) / 2];  // (x_r, x_{r+1}) packed pairs, biased floats, r = 0..R
-    float2 yp[(R + 1) / 2];
-};
-
-template <int R>
-__device__ __forceinline__ void column_sq(float (&s)[R + 1], const Rows<R>& rows, float4 c)
-{
-    const float2 ncx = make_float2(c.x, c.y), ncy = make_float2(c.z, c.w);
-#pragma unroll
-    for (int q = 0; q < (R + 1) / 2; q++) {
-        float2 v = sq2(rows.xp[q], rows.yp[q], ncx, ncy);
-        s[2 * q] = v.x;
-        s[2 * q + 1] = v.y;
-    }
-}
-
-template <int R>
-struct Bound {
-    int B;      // accept delta < B (lane-local running bound)
-    float a2f;  // column offset a2 = (B - 2) - a1
-    float srow[R];  // row thresholds: D(i_r, j) <= e_{i_r} + a1  <=>  s <= srow[r]
-};
-
-// Thresholds of the exact necessary condition for bound B:
-// delta <= B - 1 = c  ==>  D(i,j) <= e_i + a1  or  D(i+1,j+1) <= e_j + a2,
-// a1 = floor((c - 1) / 2), a2 = c - 1 - a1.  Row edges are re-read from E
-// (L1-resident; this runs once per tile and when B drops).
-template <int R>
-__device__ __forceinline__ void set_bound(Bound<R>& b, const int* __restrict__ E, int row0, int B)
-{
-    b.B = B;
-    const int c = B - 1;
-    const int a1 = (c - 1) >> 1;
-    const int a2 = c - 1 - a1;
-    b.a2f = (float)a2;
-#pragma unroll
-    for (int r = 0; r < R; r++) b.srow[r] = sq_threshold((float)(E[row0 + r] + a1));
-}
-
-// The fast test of one column step: does any pair (i_r, j), r < R, of this
-// lane pass the necessary condition?  Four independent predicate chains keep
-// the dependency depth short.
-template <int R, bool MASK>
-__device__ __forceinline__ bool step_any(const Bound<R>& b, const float (&cur)[R + 1], const float (&nxt)[R + 1],
-                                         float scol, int row0, int j)
-{
-    if (!MASK) {
-        float m = nxt[1];
-#pragma unroll
-        for (int r = 2; r <= R; r++) m = fminf(m, nxt[r]);
-        bool a0 = m <= scol, a1 = false, a2 = false, a3 = false;
-#pragma unroll
-        for (int r = 0; r < R; r++) {
-            const bool t = cur[r] <= b.srow[r];
-            if ((r & 3) == 0) a0 |= t;
-            else if ((r & 3) == 1) a1 |= t;
-            else if ((r & 3) == 2) a2 |= t;
-            else a3 |= t;
-        }
-        return (a0 | a1) | (a2 | a3);
-    } else {
-        bool any = false;
-#pragma unroll
-        for (int r = 0; r < R; r++) any |= ((cur[r] <= b.srow[r]) || (nxt[r + 1] <= scol)) && (row0 + r < j);
-        return any;
-    }
-}
-
-// Exact evaluation of this lane's candidate pairs of column step j (rare path;
-// only lanes with a candidate run it).  Integer nint distances, identical
-// arithmetic to the oracle; accept delta < B in increasing cell order.
-template <int R, bool MASK>
-__device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1], const float (&nxt)[R + 1],
-                                           float scol, int row0, int j, float4 c0, float4 c1, float ej,
-                                           const float2* __restrict__ P, const int* __restrict__ E,
-                                           unsigned long long& mykey)
-{
-    unsigned mask = 0;
-#pragma unroll
-    for (int r = 0; r < R; r++) {
-        bool cand = (cur[r] <= b.srow[r]) || (nxt[r + 1] <= scol);
-        if (MASK) cand = cand && (row0 + r < j);
-        mask |= (cand ? 1u : 0u) << r;
-    }
-    const int xj = unbias(-c0.x), yj = unbias(-c0.z);
-    const int xj1 = unbias(-c1.x), yj1 = unbias(-c1.z);
-    const int ejn = (int)ej;
-    int B = b.B;
-    while (mask) {  // ascending r == ascending cell number
-        const int r = __ffs(mask) - 1;
-        mask &= mask - 1;
-        const float2 pi = P[row0 + r], pi1 = P[row0 + r + 1];
-        const int d = exact_dist_xy(unbias(pi.x), unbias(pi.y), xj, yj) +
-                      exact_dist_xy(unbias(pi1.x), unbias(pi1.y), xj1, yj1) - E[row0 + r] - ejn;
-        if (d < B) {
-            B = d;
-            mykey = pack_key(d, row0 + r, j);
-        }
-    }
-    b.B = B;
-}
-
-template <int R, bool MASK>
-__device__ __forceinline__ void column_step(const Rows<R>& rows, Bound<R>& b, const float (&cur)[R + 1],
-                                            float (&nxt)[R + 1], int row0, int j, int J0,
-                                            const float4* __restrict__ colxy, const float* __restrict__ cole,
-                                            const float2* __restrict__ P, const int* __restrict__ E,
-                                            unsigned long long& mykey)
-{
-    const float4 c1 = colxy[j + 1 - J0];
-    column_sq<R>(nxt, rows, c1);
-    const float ej = cole[j - J0];
-    const float scol = sq_threshold(ej + b.a2f);
-    const bool any = step_any<R, MASK>(b, cur, nxt, scol, row0, j);
-    if (__builtin_expect(__any_sync(0xffffffffu, any), 0)) {
-        const int B0 = b.B;
-        if (any) exact_step<R, MASK>(b, cur, nxt, scol, row0, j, colxy[j - J0], c1, ej, P, E, mykey);
-        // share the warp's best: a lane may accept delta <= (best of another lane)
-        const int wb = __reduce_min_sync(0xffffffffu, b.B);
-        const int nb = min(b.B, wb + 1);
-        if (nb < B0) set_bound<R>(b, E, row0, nb);
-    }
-}
-
-template <int R, bool MASK>
-__device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0, int jstart, int J0, int J1,
-                                     const float4* __restrict__ colxy, const float* __restrict__ cole,
-                                     const float2* __restrict__ P, const int* __restrict__ E,
-                                     unsigned long long& mykey)
-{
-    float sa[R + 1], sb[R + 1];
-    column_sq<R>(sa, rows, colxy[jstart - J0]);
-    int j = jstart;
-    for (; j + 1 < J1; j += 2) {
-        column_step<R, MASK>(rows, b, sa, sb, row0, j, J0, colxy, cole, P, E, mykey);
-        column_step<R, MASK>(rows, b, sb, sa, row0, j + 1, J0, colxy, cole, P, E, mykey);
-    }
-    if (j < J1) column_step<R, MASK>(rows, b, sa, sb, row0, j, J0, colxy, cole, P, E, mykey);
-}
-
-template <int R>
-__global__ void __launch_bounds__(128) sweep_kernel(const float2* __restrict__ P, const int* __restrict__ E, int n,
+__global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* __restrict__ P, const int* __restrict__ E, int n,
                                                      const int2* __restrict__ tiles, int TJ, Slot* __restrict__ slot,
                                                      int respect_done)
 {
     extern __shared__ float4 smem[];
-    float4* colxy = smem;                                    // [TJ + 1]: (-x, -x, -y, -y) of columns J0..J1
-    float* cole = reinterpret_cast<float*>(smem + TJ + 1);  // [TJ + 1]: e_j as float
-
+    const TileSmem sm(smem, TJ);
     if (respect_done && *(volatile int*)&slot->done) return;  // converged: iteration is a no-op
-    const int2 tile = tiles[blockIdx.x];
-    const int I0 = tile.x, J0 = tile.y;
-    const int J1 = min(J0 + TJ, n);  // columns j in [J0, J1), j <= n-1
-    const int ncol = J1 - J0;
-    for (int c = threadIdx.x; c <= ncol; c += blockDim.x) {  // J1 <= n: P[n] = P[0] closes the tour
-        const float2 p = P[J0 + c];
-        colxy[c] = make_float4(-p.x, -p.x, -p.y, -p.y);
-        cole[c] = (float)E[J0 + c];
-    }
-    __syncthreads();
-
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int wrow0 = I0 + warp * 32 * R;
-    const int row0 = wrow0 + lane * R;
-    const int jstart = max(J0, wrow0 + 1);  // no pair of this warp has j <= wrow0
-    if (jstart >= J1) return;                // warp-uniform: nothing to do
-    unsigned long long mykey = kKeyNone;
-    Rows<R> rows;
-#pragma unroll
-    for (int q = 0; q < (R + 1) / 2; q++) {
-        const float2 p0 = P[row0 + 2 * q], p1 = P[row0 + 2 * q + 1];
-        rows.xp[q] = make_float2(p0.x, p1.x);
-        rows.yp[q] = make_float2(p0.y, p1.y);
-    }
-    // Start from the best key any CTA of this sweep has published so far.  The
-    // slot key is the seed (0, cell 0) or a real pair of this sweep, so a pair of
-    // ours can only win with delta < 0 (key delta 0) or delta <= key delta.
-    const unsigned long long g = *(volatile unsigned long long*)&slot->key;
-    const int dg = key_delta(g);
-    Bound<R> b;
-    set_bound<R>(b, E, row0, dg == 0 ? 0 : dg + 1);
-    const bool masked = (wrow0 + 32 * R - 1) >= jstart;  // warp-uniform: some row >= some j
-    if (masked) walk<R, true>(rows, b, row0, jstart, J0, J1, colxy, cole, P, E, mykey);
-    else walk<R, false>(rows, b, row0, jstart, J0, J1, colxy, cole, P, E, mykey);
-
-    // a5: warp min, one atomicMin per warp (L16 Fig. 4 "Get best local pair ...
-    // Get best global pair"); min is order-independent -> deterministic result.
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        const unsigned long long other = __shfl_xor_sync(0xffffffffu, mykey, o);
-        mykey = other < mykey ? other : mykey;
-    }
-    if (lane == 0 && mykey < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, mykey);
+    sweep_tile<R, false>(P, E, n, tiles[blockIdx.x], TJ, slot, sm);
 }
 
 // ===========================================================================
@@ -283,9 +89,10 @@ __global__ void __launch_bounds__(128) sweep_kernel(const float2* __restrict__ P
 // pre-reversal cities (thread 0 reads them before doing its own swap; no other
 // thread touches P[i], P[i+1], P[j], P[j+1], e[i], e[j]).
 // ===========================================================================
-__global__ void __launch_bounds__(256) apply_kernel(float2* __restrict__ P, int* __restrict__ E, int* __restrict__ tour,
-                                                    const Slot* __restrict__ in, Slot* __restrict__ out,
-                                                    long long max_moves, int explicit_move, int ei, int ej)
+// Returns whether a move was applied (false: converged / capped / already done).
+__device__ __forceinline__ bool apply_phase(float2* __restrict__ P, int* __restrict__ E, int* __restrict__ tour,
+                                            const Slot* __restrict__ in, Slot* __restrict__ out, long long max_moves,
+                                            int explicit_move, int ei, int ej, int gtid, int stride)
 {
     const unsigned long long key = in->key;
     const int done = in->done;
@@ -301,47 +108,125 @@ __global__ void __launch_bounds__(256) apply_kernel(float2* __restrict__ P, int*
         j = key_j(key);
         apply = !done && key_delta(key) < 0 && moves < max_moves;
     }
-    const int gtid = blockIdx.x * blockDim.x + threadIdx.x;
-    const int stride = gridDim.x * blockDim.x;
     if (gtid == 0) {
         Slot o;
         o.key = seed_key();
         o.last_key = explicit_move ? in->last_key : key;
         o.moves = moves;
         o.length = in->length;
-        o.done = done;
+        o.done = explicit_move ? (done & 4) : done;  // an explicit move makes the tour unconverged
+        o.next_tile = 0;
         if (!explicit_move && !done) {
             if (key_delta(key) >= 0) o.done = 1;        // local minimum (reading R7)
             else if (moves >= max_moves) o.done = 2;    // capped with an improving move left (R8)
         }
         if (apply) {
-            const float2 pi = P[i], pj = P[j], pi1 = P[i + 1], pj1 = P[j + 1];
+            const float2 pi = __ldcg(P + i), pj = __ldcg(P + j), pi1 = __ldcg(P + i + 1), pj1 = __ldcg(P + j + 1);
             const int ni = exact_dist_biased(pi, pj), nj = exact_dist_biased(pi1, pj1);
-            o.length += (long long)ni + nj - E[i] - E[j];
+            o.length += (long long)ni + nj - __ldcg(E + i) - __ldcg(E + j);
             o.moves = moves + 1;
             E[i] = ni;
             E[j] = nj;
         }
         *out = o;
     }
-    if (!apply) return;
+    if (!apply) return false;
     const int half = (j - i) >> 1;  // swap P/tour positions i+1+t <-> j-t
     for (int t = gtid; t < half; t += stride) {
         const int a = i + 1 + t, c = j - t;
-        const float2 pa = P[a], pc = P[c];
+        const float2 pa = __ldcg(P + a), pc = __ldcg(P + c);
         P[a] = pc;
         P[c] = pa;
-        const int ta = tour[a], tc = tour[c];
+        const int ta = __ldcg(tour + a), tc = __ldcg(tour + c);
         tour[a] = tc;
         tour[c] = ta;
     }
     const int ehalf = (j - i - 1) >> 1;  // swap e positions i+1+t <-> j-1-t
     for (int t = gtid; t < ehalf; t += stride) {
         const int a = i + 1 + t, c = j - 1 - t;
-        const int ea = E[a], ec = E[c];
+        const int ea = __ldcg(E + a), ec = __ldcg(E + c);
         E[a] = ec;
         E[c] = ea;
     }
+    return true;
+}
+
+__global__ void __launch_bounds__(256) apply_kernel(float2* __restrict__ P, int* __restrict__ E, int* __restrict__ tour,
+                                                    const Slot* __restrict__ in, Slot* __restrict__ out,
+                                                    long long max_moves, int explicit_move, int ei, int ej)
+{
+    __shared__ Slot s_in;  // one read of the input state per block
+    if (threadIdx.x == 0) s_in = *in;
+    __syncthreads();
+    apply_phase(P, E, tour, &s_in, out, max_moves, explicit_move, ei, ej, blockIdx.x * blockDim.x + threadIdx.x,
+                gridDim.x * blockDim.x);
+}
+
+// ===========================================================================
+// Device-resident local search (§8(a) a4-a8 in ONE launch, world == 1): a
+// persistent cooperative grid alternates {sweep over all tiles, dynamically
+// scheduled; grid barrier; apply; grid barrier} until the local minimum, the
+// move cap or the per-launch iteration budget.  Slots ping-pong exactly as in
+// the multi-kernel path; the final parity is written to ctl[0].
+// ===========================================================================
+__device__ __forceinline__ void grid_sync(unsigned* bar, unsigned nblocks)
+{
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        volatile unsigned* vgen = bar + 1;
+        const unsigned gen = *vgen;
+        __threadfence();
+        if (atomicAdd(bar, 1u) == nblocks - 1) {
+            atomicExch(bar, 0u);
+            __threadfence();
+            atomicAdd(bar + 1, 1u);
+        } else {
+            while (*vgen == gen) __nanosleep(32);
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+template <int R>
+__global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2* __restrict__ P, int* __restrict__ E,
+                                                           int* __restrict__ tour, int n,
+                                                           const int2* __restrict__ tiles, int ntiles, int TJ,
+                                                           Slot* __restrict__ slots, int parity, long long max_moves,
+                                                           long long budget, unsigned* __restrict__ bar,
+                                                           int* __restrict__ ctl)
+{
+    extern __shared__ float4 smem[];
+    const TileSmem sm(smem, TJ);
+    __shared__ Slot s_in;
+    const int gtid = blockIdx.x * blockDim.x + threadIdx.x;
+    const int stride = gridDim.x * blockDim.x;
+    int p = parity;
+    for (long long it = 0; it < budget; it++) {
+        Slot* in = slots + p;
+        // one read of the settled state per block (not one per thread: a single hot address)
+        if (threadIdx.x == 0) s_in.done = *(volatile int*)&in->done;
+        __syncthreads();
+        if (s_in.done) break;  // uniform across the grid
+        // a4/a5: tiles are assigned round-robin (largest first); the grid is co-resident
+        for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+            sweep_tile<R, true>(P, E, n, tiles[t], TJ, in, sm);
+            __syncthreads();  // before the next tile overwrites the shared chunk
+        }
+        grid_sync(bar, gridDim.x);
+        if (threadIdx.x == 0) {
+            s_in.key = *(volatile unsigned long long*)&in->key;
+            s_in.last_key = in->last_key;
+            s_in.moves = *(volatile long long*)&in->moves;
+            s_in.length = *(volatile long long*)&in->length;
+            s_in.done = *(volatile int*)&in->done;
+        }
+        __syncthreads();
+        apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride);  // a7/a8
+        p ^= 1;
+        grid_sync(bar, gridDim.x);
+    }
+    if (gtid == 0) ctl[0] = p;
 }
 
 // ===========================================================================
@@ -359,6 +244,23 @@ __global__ void selftest_dist_kernel(long long smax, unsigned long long* bad, un
         }
     }
     if (nbad) atomicAdd(bad, nbad);
+}
+
+// Max relative error of sqrt_approx (MUFU.SQRT) over every float in [1, 2^31]
+// (the float squared distances the sqrt-sum filter takes; 0 maps to 0) and a
+// check that sqrt_approx(0) == 0.  Result: float bits of the max, in *out.
+__global__ void selftest_sqrt_kernel(unsigned* out, unsigned* zero_bad)
+{
+    const unsigned lo = 0x3F800000u, hi = 0x4F000000u;  // 1.0f .. 2^31
+    float worst = 0.f;
+    for (unsigned u = lo + blockIdx.x * blockDim.x + threadIdx.x; u <= hi; u += gridDim.x * blockDim.x) {
+        const float x = __uint_as_float(u);
+        const double ex = sqrt((double)x);
+        const float rel = (float)(fabs((double)sqrt_approx(x) - ex) / ex);
+        worst = fmaxf(worst, rel);
+    }
+    atomicMax(out, __float_as_uint(worst));
+    if (blockIdx.x == 0 && threadIdx.x == 0 && sqrt_approx(0.f) != 0.f) *zero_bad = 1;
 }
 
 __global__ void selftest_filter_kernel(unsigned long long* bad, unsigned long long* first)
@@ -408,19 +310,20 @@ cudaError_t launch_reset_key(Slot* slot, cudaStream_t st)
     return cudaGetLastError();
 }
 
-size_t sweep_smem_bytes(int TJ) { return (size_t)(TJ + 1) * sizeof(float4) + (size_t)(TJ + 1) * sizeof(float); }
+size_t sweep_smem_bytes(const Geometry& g) { return tile_smem_bytes(g.tj, g.ti()); }
+static const Geometry kMaxGeo{kRows, kMaxWarps, kMaxTJ};
 
 cudaError_t sweep_prepare()
 {
     return cudaFuncSetAttribute(sweep_kernel<kRows>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)sweep_smem_bytes(kMaxTJ));
+                                (int)sweep_smem_bytes(kMaxGeo));
 }
 
 cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
                          Slot* slot, int respect_done, cudaStream_t st)
 {
     if (ntiles <= 0) return cudaSuccess;
-    sweep_kernel<kRows><<<ntiles, 32 * g.warps, sweep_smem_bytes(g.tj), st>>>(P, E, n, tiles, g.tj, slot,
+    sweep_kernel<kRows><<<ntiles, 32 * g.warps, sweep_smem_bytes(g), st>>>(P, E, n, tiles, g.tj, slot,
                                                                                respect_done);
     g_launches += 1;
     return cudaGetLastError();
@@ -435,6 +338,76 @@ cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Sl
     apply_kernel<<<blocks, 256, 0, st>>>(P, E, tour, in, out, max_moves, explicit_move, ei, ej);
     g_launches += 1;
     return cudaGetLastError();
+}
+
+int local_search_grid(const Geometry& g, int ntiles)
+{
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, local_search_kernel<kRows>, 32 * g.warps,
+                                                      sweep_smem_bytes(g)) != cudaSuccess)
+        return 0;
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    int grid = per_sm * sms;
+    return grid < ntiles ? grid : ntiles;
+}
+
+cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
+                                Slot* slots, int parity, long long max_moves, long long budget, unsigned* bar,
+                                int* ctl, cudaStream_t st)
+{
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(local_search_kernel<kRows>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)sweep_smem_bytes(kMaxGeo));
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    int grid = local_search_grid(g, ntiles);
+    if (grid < 1) return cudaErrorInvalidConfiguration;
+    int TJ = g.tj;
+    void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &TJ, &slots, &parity, &max_moves, &budget, &bar, &ctl};
+    g_launches += 1;
+    return cudaLaunchCooperativeKernel((const void*)local_search_kernel<kRows>, dim3(grid), dim3(32 * g.warps), args,
+                                       sweep_smem_bytes(g), st);
+}
+
+cudaError_t run_selftest_sqrt(double* max_rel, int* zero_ok)
+{
+    unsigned* d = nullptr;
+    cudaError_t err = cudaMalloc(&d, 2 * sizeof(unsigned));
+    if (err != cudaSuccess) return err;
+    cudaMemset(d, 0, 2 * sizeof(unsigned));
+    selftest_sqrt_kernel<<<148 * 8, 256>>>(d, d + 1);
+    g_launches += 1;
+    unsigned h[2] = {0, 0};
+    err = cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    float f;
+    memcpy(&f, &h[0], sizeof(f));
+    *max_rel = f;
+    *zero_ok = h[1] == 0;
+    return err;
+}
+
+cudaError_t read_stats(long long* out4, int reset)
+{
+#ifdef TSP2OPT_STATS
+    unsigned long long h[4];
+    cudaError_t e = cudaMemcpyFromSymbol(h, g_stats, sizeof(h));
+    if (e != cudaSuccess) return e;
+    for (int k = 0; k < 4; k++) out4[k] = (long long)h[k];
+    if (reset) {
+        const unsigned long long z[4] = {0, 0, 0, 0};
+        e = cudaMemcpyToSymbol(g_stats, z, sizeof(z));
+    }
+    return e;
+#else
+    (void)reset;
+    for (int k = 0; k < 4; k++) out4[k] = -1;
+    return cudaSuccess;
+#endif
 }
 
 cudaError_t run_selftest(long long* out4)

@@ -1,0 +1,294 @@
+// tsp2opt_sweep.cuh -- the sweep of one (row block x column chunk) tile
+// (SURVEY.md §8(a) rows a4 + a5), shared by the per-sweep kernel and the
+// persistent local-search kernel of tsp2opt_kernels.cu.
+//
+// One CTA = one tile = rows [I0, I0 + 32*R*NW) x columns [J0, J0 + TJ) -- the
+// paper's problem division into "2 coordinate ranges" (L18 §IV.B; L20 Fig. 7,
+// Listing 2 "2 sets of coordinates needed, A for point i and B for point j").
+// Each lane owns R consecutive rows (R+1 cities in registers, packed FP32x2);
+// the warp walks the tile's columns, column city j being a shared-memory
+// broadcast.  Per column step the lane computes the R+1 squared distances of
+// its rows to column j+1 (diagonal reuse: s(i+1, j+1) of pair (i, j) is
+// s(i', j') of pair (i', j') = (i+1, j+1)) and tests every pair (i, j) with
+// the exact necessary condition of DESIGN.md §5.2:
+//     delta(i,j) <= B - 1   ==>   D(i,j) <= e_i + a1   or   D(i+1,j+1) <= e_j + a2
+// (a1 + a2 = B - 2) on squared distances (no sqrt).  Pairs that pass are
+// evaluated exactly (integer nint, the oracle's arithmetic) and accepted iff
+// delta < B; B is the lane's running bound, started from the global best.
+// Pairs are visited in increasing Fig. 3 cell order per lane, so a strict '<'
+// keeps the lowest cell among equal deltas (reading R5).
+//
+// PS (persistent) selects the global-load flavour: the per-sweep kernel reads
+// P and E through the read-only path (__ldg); the persistent kernel rewrites P
+// and E between sweeps, so it uses plain coherent loads (L1 is invalidated by
+// the gpu-scope fence of its grid barrier).
+#pragma once
+
+#include "tsp2opt_device.cuh"
+
+namespace tsp2opt {
+
+#ifdef TSP2OPT_STATS
+// Instrumented builds only: [0] warp column steps, [1] steps taking the exact
+// path, [2] candidate pairs evaluated exactly.
+__device__ unsigned long long g_stats[4];
+#endif
+
+template <bool PS, typename T>
+__device__ __forceinline__ T gld(const T* p)
+{
+    if constexpr (PS) return *p;
+    else return __ldg(p);
+}
+
+template <int R>
+struct Rows {
+    float2 xp[(R + 1) / 2];  // (x_r, x_{r+1}) packed pairs, biased floats, r = 0..R
+    float2 yp[(R + 1) / 2];
+};
+
+template <int R>
+__device__ __forceinline__ void column_sq(float (&s)[R + 1], const Rows<R>& rows, float4 c)
+{
+    const float2 ncx = make_float2(c.x, c.y), ncy = make_float2(c.z, c.w);
+#pragma unroll
+    for (int q = 0; q < (R + 1) / 2; q++) {
+        float2 v = sq2(rows.xp[q], rows.yp[q], ncx, ncy);
+        s[2 * q] = v.x;
+        s[2 * q + 1] = v.y;
+    }
+}
+
+template <int R>
+struct Bound {
+    int B;          // accept delta < B (lane-local running bound)
+    float a2f;      // column offset a2 = (B - 2) - a1
+    float srow[R];  // row thresholds: D(i_r, j) <= e_{i_r} + a1  <=>  s <= srow[r]
+};
+
+// Thresholds of the exact necessary condition for bound B:
+// delta <= B - 1 = c  ==>  D(i,j) <= e_i + a1  or  D(i+1,j+1) <= e_j + a2,
+// a1 = floor((c - 1) / 2), a2 = c - 1 - a1.
+template <int R>
+__device__ __forceinline__ void set_bound(Bound<R>& b, const int (&erow)[R], int B)
+{
+    b.B = B;
+    const int c = B - 1;
+    const int a1 = (c - 1) >> 1;
+    const int a2 = c - 1 - a1;
+    b.a2f = (float)a2;
+#pragma unroll
+    for (int r = 0; r < R; r++) b.srow[r] = sq_threshold((float)(erow[r] + a1));
+}
+
+// Shared memory of one tile: the column chunk (the paper's coordinate range
+// "B", L20 Listing 2) and the edges of the CTA's rows (range "A").
+struct TileSmem {
+    float4* colxy;  // [TJ + 1]: (-x, -x, -y, -y) of columns J0..J1 (biased floats)
+    float* cole;    // [TJ + 1]: e_j as float
+    float* rowe;    // [32 * R * warps]: e_i of the CTA's rows, as float
+    __device__ TileSmem(void* base, int TJ)
+        : colxy(reinterpret_cast<float4*>(base)),
+          cole(reinterpret_cast<float*>(colxy + TJ + 1)),
+          rowe(cole + TJ + 1)
+    {
+    }
+};
+
+// Same as set_bound, from the lane's row edges in shared memory (rare: the
+// bound dropped mid-tile).
+template <int R>
+__device__ __forceinline__ void reset_bound(Bound<R>& b, const float* my_rowe, int B)
+{
+    int erow[R];
+#pragma unroll
+    for (int r = 0; r < R; r++) erow[r] = (int)my_rowe[r];
+    set_bound<R>(b, erow, B);
+}
+
+// The fast test of one column step: does any pair (i_r, j), r < R, of this
+// lane pass the necessary condition?  Four independent predicate chains keep
+// the dependency depth short.
+template <int R, bool MASK>
+__device__ __forceinline__ bool step_any(const Bound<R>& b, const float (&cur)[R + 1], const float (&nxt)[R + 1],
+                                         float scol, int row0, int j)
+{
+    if (!MASK) {
+        float m = nxt[1];
+#pragma unroll
+        for (int r = 2; r <= R; r++) m = fminf(m, nxt[r]);
+        bool a0 = m <= scol, a1 = false, a2 = false, a3 = false;
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            const bool t = cur[r] <= b.srow[r];
+            if ((r & 3) == 0) a0 |= t;
+            else if ((r & 3) == 1) a1 |= t;
+            else if ((r & 3) == 2) a2 |= t;
+            else a3 |= t;
+        }
+        return (a0 | a1) | (a2 | a3);
+    } else {
+        bool any = false;
+#pragma unroll
+        for (int r = 0; r < R; r++) any |= ((cur[r] <= b.srow[r]) || (nxt[r + 1] <= scol)) && (row0 + r < j);
+        return any;
+    }
+}
+
+// Exact evaluation of this lane's candidate pairs of column step j (rare path;
+// only lanes with a candidate run it).  A second, tighter necessary condition
+// is applied first: nint(sqrt(s)) >= sqrt(s) - 1/2, so
+//     delta <= B - 1  ==>  sqrt(s1) + sqrt(s2) <= e_i + e_j + B,
+// evaluated with MUFU.SQRT on the float squared distances already in
+// registers; its error (< 0.04, the sqrt error is bounded
+// exhaustively by tsp2opt_selftest) is covered by a 0.5 slack.  Survivors are
+// evaluated with integer nint distances -- the oracle's arithmetic -- and
+// accepted iff delta < B, in increasing cell order.
+template <int R, bool MASK, bool PS>
+__device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1], const float (&nxt)[R + 1],
+                                           float scol, int row0, int j, float4 c0, float4 c1, float ej,
+                                           const float* my_rowe, const float2* P, unsigned long long& mykey)
+{
+    const float lim = ej + (float)b.B + 0.5f;
+    unsigned mask = 0;
+#pragma unroll
+    for (int r = 0; r < R; r++) {
+        bool cand = (cur[r] <= b.srow[r]) || (nxt[r + 1] <= scol);
+        if (MASK) cand = cand && (row0 + r < j);
+        if (cand) cand = sqrt_approx(cur[r]) + sqrt_approx(nxt[r + 1]) <= my_rowe[r] + lim;
+        mask |= (cand ? 1u : 0u) << r;
+    }
+#ifdef TSP2OPT_STATS
+    atomicAdd(&g_stats[2], (unsigned long long)__popc(mask));
+#endif
+    if (!mask) return;
+    const int xj = unbias(-c0.x), yj = unbias(-c0.z);
+    const int xj1 = unbias(-c1.x), yj1 = unbias(-c1.z);
+    const int ejn = (int)ej;
+    int B = b.B;
+    while (mask) {  // ascending r == ascending cell number
+        const int r = __ffs(mask) - 1;
+        mask &= mask - 1;
+        const float2 pi = gld<PS>(P + row0 + r), pi1 = gld<PS>(P + row0 + r + 1);
+        const int d = exact_dist_xy(unbias(pi.x), unbias(pi.y), xj, yj) +
+                      exact_dist_xy(unbias(pi1.x), unbias(pi1.y), xj1, yj1) - (int)my_rowe[r] - ejn;
+        if (d < B) {
+            B = d;
+            mykey = pack_key(d, row0 + r, j);
+        }
+    }
+    b.B = B;
+}
+
+template <int R, bool MASK, bool PS>
+__device__ __forceinline__ void column_step(const Rows<R>& rows, Bound<R>& b, const float (&cur)[R + 1],
+                                            float (&nxt)[R + 1], int row0, int j, int J0, const TileSmem& sm,
+                                            const float* my_rowe, const float2* P, unsigned long long& mykey)
+{
+    const float4 c1 = sm.colxy[j + 1 - J0];
+    column_sq<R>(nxt, rows, c1);
+    const float ej = sm.cole[j - J0];
+    const float scol = sq_threshold(ej + b.a2f);
+    const bool any = step_any<R, MASK>(b, cur, nxt, scol, row0, j);
+#ifdef TSP2OPT_STATS
+    if ((threadIdx.x & 31) == 0) atomicAdd(&g_stats[0], 1ULL);
+#endif
+    if (__builtin_expect(__any_sync(0xffffffffu, any), 0)) {
+#ifdef TSP2OPT_STATS
+        if ((threadIdx.x & 31) == 0) atomicAdd(&g_stats[1], 1ULL);
+#endif
+        const int B0 = b.B;
+        if (any) exact_step<R, MASK, PS>(b, cur, nxt, scol, row0, j, sm.colxy[j - J0], c1, ej, my_rowe, P, mykey);
+        // share the warp's best: a lane may accept delta <= (best of another lane)
+        const int wb = __reduce_min_sync(0xffffffffu, b.B);
+        const int nb = min(b.B, wb + 1);
+        if (nb < B0) reset_bound<R>(b, my_rowe, nb);
+    }
+}
+
+template <int R, bool MASK, bool PS>
+__device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0, int jstart, int J0, int J1,
+                                     const TileSmem& sm, const float* my_rowe, const float2* P,
+                                     unsigned long long& mykey)
+{
+    float sa[R + 1], sb[R + 1];
+    column_sq<R>(sa, rows, sm.colxy[jstart - J0]);
+    int j = jstart;
+    for (; j + 1 < J1; j += 2) {
+        column_step<R, MASK, PS>(rows, b, sa, sb, row0, j, J0, sm, my_rowe, P, mykey);
+        column_step<R, MASK, PS>(rows, b, sb, sa, row0, j + 1, J0, sm, my_rowe, P, mykey);
+    }
+    if (j < J1) column_step<R, MASK, PS>(rows, b, sa, sb, row0, j, J0, sm, my_rowe, P, mykey);
+}
+
+// Shared memory bytes of a tile with TJ columns and TI rows.
+__host__ __device__ inline size_t tile_smem_bytes(int TJ, int TI)
+{
+    return (size_t)(TJ + 1) * (sizeof(float4) + sizeof(float)) + (size_t)TI * sizeof(float);
+}
+
+// One tile.  All global loads of the tile (the lane's rows and row edges, the
+// CTA's share of the column chunk, the global best key) are issued before the
+// first use so their latencies overlap; then the column chunk and the row
+// edges are staged in shared memory, every warp walks the chunk, and the warp
+// minima are published with one atomicMin each (L16 Fig. 4 "Get best local
+// pair ... Get best global pair"; min is order-independent, so the result is
+// deterministic).  The caller synchronises the CTA before reusing `sm`.
+template <int R, bool PS>
+__device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n, int2 tile, int TJ, Slot* slot,
+                                           const TileSmem& sm)
+{
+    const int I0 = tile.x, J0 = tile.y;
+    const int J1 = min(J0 + TJ, n);  // columns j in [J0, J1), j <= n-1
+    const int ncol = J1 - J0;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int wrow0 = I0 + warp * 32 * R;
+    const int row0 = wrow0 + lane * R;
+    const int jstart = max(J0, wrow0 + 1);  // no pair of this warp has j <= wrow0
+    const bool active = jstart < J1;        // warp-uniform
+    float* my_rowe = sm.rowe + threadIdx.x * R;  // stride R (odd): conflict-free
+
+    Rows<R> rows;
+    int erow[R];
+    if (active) {
+#pragma unroll
+        for (int q = 0; q < (R + 1) / 2; q++) {
+            const float2 p0 = gld<PS>(P + row0 + 2 * q), p1 = gld<PS>(P + row0 + 2 * q + 1);
+            rows.xp[q] = make_float2(p0.x, p1.x);
+            rows.yp[q] = make_float2(p0.y, p1.y);
+        }
+#pragma unroll
+        for (int r = 0; r < R; r++) erow[r] = gld<PS>(E + row0 + r);
+    }
+    for (int c = threadIdx.x; c <= ncol; c += blockDim.x) {  // J1 <= n: P[n] = P[0] closes the tour
+        const float2 p = gld<PS>(P + J0 + c);
+        const int e = gld<PS>(E + J0 + c);
+        sm.colxy[c] = make_float4(-p.x, -p.x, -p.y, -p.y);
+        sm.cole[c] = (float)e;
+    }
+    // The slot key is the seed (0, cell 0) or a real pair of this sweep, so a
+    // pair of ours can only win with delta < 0 (key delta 0) or delta <= key delta.
+    const int dg = key_delta(*(volatile unsigned long long*)&slot->key);
+    if (active) {
+#pragma unroll
+        for (int r = 0; r < R; r++) my_rowe[r] = (float)erow[r];
+    }
+    __syncthreads();
+    if (!active) return;
+
+    unsigned long long mykey = kKeyNone;
+    Bound<R> b;
+    set_bound<R>(b, erow, dg == 0 ? 0 : dg + 1);
+    const bool masked = (wrow0 + 32 * R - 1) >= jstart;  // warp-uniform: some row >= some j
+    if (masked) walk<R, true, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
+    else walk<R, false, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
+
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const unsigned long long other = __shfl_xor_sync(0xffffffffu, mykey, o);
+        mykey = other < mykey ? other : mykey;
+    }
+    if (lane == 0 && mykey < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, mykey);
+}
+
+}  // namespace tsp2opt

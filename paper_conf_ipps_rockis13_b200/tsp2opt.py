@@ -13,7 +13,9 @@ import os
 
 import numpy as np
 
-from ._build import LIB
+from ._build import LIB as _DEFAULT_LIB
+
+LIB = os.environ.get("TSP2OPT_LIB", _DEFAULT_LIB)  # override: an alternative in-tree build (experiments)
 
 OK, MAXITER = 0, 1
 EINVAL, ERANGE, ENOTPERM, ESTATE, ECUDA, ENCCL, ENOMEM = -1, -2, -3, -4, -5, -6, -7
@@ -62,6 +64,8 @@ def _L():
             "tsp2opt_profile": ([P, I32], I32),
             "tsp2opt_profile_read": ([P, ctypes.POINTER(ctypes.c_double), pI64], I32),
             "tsp2opt_launch_count": ([], I64),
+            "tsp2opt_debug_stats": ([pI64, I32], I32),
+            "tsp2opt_selftest_sqrt": ([ctypes.POINTER(ctypes.c_double), pI32], I32),
             "tsp2opt_strerror": ([I32], ctypes.c_char_p),
             "tsp2opt_last_error": ([], ctypes.c_char_p),
         }
@@ -221,6 +225,13 @@ def profile_read(h):
     return ms.value, n.value
 
 
+def selftest_sqrt() -> dict:
+    """Max relative error of the sweep's MUFU.SQRT over every float in [1, 2^31]; sqrt(0) == 0."""
+    e, z = ctypes.c_double(), ctypes.c_int32()
+    _check(_L().tsp2opt_selftest_sqrt(ctypes.byref(e), ctypes.byref(z)), "tsp2opt_selftest_sqrt")
+    return dict(max_rel_err=e.value, zero_ok=bool(z.value))
+
+
 def launch_count() -> int:
     return int(_L().tsp2opt_launch_count())
 
@@ -290,3 +301,10 @@ class TSP2Opt:
 
     def profile_read(self):
         return profile_read(self.h)
+
+
+def debug_stats(reset: bool = True) -> dict:
+    """Sweep counters of an instrumented build (TSP2OPT_STATS); -1 in product builds."""
+    out = (ctypes.c_int64 * 4)()
+    _check(_L().tsp2opt_debug_stats(out, 1 if reset else 0), "tsp2opt_debug_stats")
+    return dict(warp_steps=out[0], slow_steps=out[1], exact_pairs=out[2])

@@ -26,6 +26,14 @@ def test_selftest_exhaustive_distance_and_filter(gpu):
     assert r["filter_violations"] == 0, f"squared-distance prefilter rejects a reachable (dx, dy): {r}"
 
 
+def test_selftest_sqrt_error_bound(gpu):
+    """The sqrt-sum prefilter's 0.5 slack needs a relative MUFU.SQRT
+    error <= 2^-21 on every float the filter can see."""
+    r = tsp2opt.selftest_sqrt()
+    assert r["zero_ok"]
+    assert 0 <= r["max_rel_err"] <= 2.0 ** -21, r
+
+
 SIZES = [3, 4, 5, 7, 16, 31, 32, 33, 100, 101, 479, 480, 481, 961, 1002, 1921, 2500]
 
 
@@ -209,3 +217,20 @@ def test_small_n_cases(gpu):
         res = g.local_search(t)
         ref = oracle.local_search(dup, t)
         assert np.array_equal(res["tour"], ref["tour"]) and res["length"] == ref["length"]
+
+
+@pytest.mark.parametrize("persistent", ["0", "1"])
+@pytest.mark.parametrize("kind,n,seed", [("uniform", 1002, 5), ("lattice", 3001, 6), ("uniform", 97, 7)])
+def test_local_search_parity_both_loops(gpu, monkeypatch, persistent, kind, n, seed):
+    """The persistent single-launch loop and the per-iteration kernel loop (used by
+    sharded handles) reach the oracle's local minimum identically."""
+    monkeypatch.setenv("TSP2OPT_PERSISTENT", persistent)
+    c, t = _inst(kind, n, seed)
+    ref = oracle.local_search(c, t)
+    with tsp2opt.TSP2Opt(c) as g:
+        res = g.local_search(t)
+        assert (res["iterations"], res["length"]) == (ref["iterations"], ref["length"])
+        assert np.array_equal(res["tour"], ref["tour"])
+        capped = g.local_search(t, max_iters=17)
+        want = oracle.local_search(c, t, max_iters=17)
+        assert capped["status"] == want["status"] and np.array_equal(capped["tour"], want["tour"])
