@@ -128,13 +128,52 @@ __device__ __forceinline__ float2 fma2(float2 a, float2 b, float2 c)
     return r;
 }
 
+// min over v[LO..HI) as a balanced tree of 3-input minima (FMNMX3): depth
+// log3 instead of the linear chain a fold would produce.
+template <int LO, int HI>
+__device__ __forceinline__ float tree_min(const float* v)
+{
+    static_assert(HI > LO, "empty range");
+    if constexpr (HI - LO == 1) {
+        return v[LO];
+    } else if constexpr (HI - LO == 2) {
+        return fminf(v[LO], v[LO + 1]);
+    } else if constexpr (HI - LO == 3) {
+        return fminf(fminf(v[LO], v[LO + 1]), v[LO + 2]);
+    } else {
+        constexpr int M1 = LO + (HI - LO) / 3, M2 = LO + 2 * (HI - LO) / 3;
+        return fminf(fminf(tree_min<LO, M1>(v), tree_min<M1, M2>(v)), tree_min<M2, HI>(v));
+    }
+}
+
+// 32-bit shared-memory addressing (keeps the fast loop free of generic->shared
+// conversions).
+__device__ __forceinline__ unsigned smem_addr(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ float4 lds4(unsigned a)
+{
+    float4 v;
+    asm("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ float2 lds2(unsigned a)
+{
+    float2 v;
+    asm("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(v.x), "=f"(v.y) : "r"(a));
+    return v;
+}
+
 // Squared distances of two row cities (packed) to one column city given as
 // negated biased coordinates (-x, -x) / (-y, -y):  s = dx*dx + dy*dy.
 __device__ __forceinline__ float2 sq2(float2 xr, float2 yr, float2 ncx, float2 ncy)
 {
+#ifdef TSP2OPT_SCALAR_SQ  // experiment: scalar FADD/FMUL/FFMA instead of the packed FP32x2 forms
+    const float dx0 = xr.x + ncx.x, dx1 = xr.y + ncx.y, dy0 = yr.x + ncy.x, dy1 = yr.y + ncy.y;
+    return make_float2(fmaf(dx0, dx0, dy0 * dy0), fmaf(dx1, dx1, dy1 * dy1));
+#else
     float2 dx = add2(xr, ncx);
     float2 dy = add2(yr, ncy);
     return fma2(dx, dx, mul2(dy, dy));
+#endif
 }
 
 // Per-rank / per-handle device state, ping-ponged between iterations: the

@@ -10,7 +10,9 @@
 
 namespace tsp2opt {
 
-constexpr int kRows = 15;     // R: rows per lane (R + 1 = 16 cities, 8 packed FP32x2 pairs)
+constexpr int kRowsLarge = 15;  // R for large n: 16 row cities per lane (8 packed FP32x2 pairs)
+constexpr int kRowsSmall = 7;   // R for small / medium n
+constexpr int kRows = kRowsLarge;  // the largest R (padding)
 constexpr int kMaxTJ = 1024;  // columns per tile, upper bound (shared memory sizing)
 constexpr int kMaxWarps = 4;  // warps per CTA, upper bound (__launch_bounds__(128))
 constexpr int kPad = 32 * kRows * kMaxWarps + kMaxTJ + 8;  // P/E/tour padding beyond n

@@ -10,6 +10,24 @@
 #include "tsp2opt_device.cuh"
 #include "tsp2opt_internal.h"
 #include "tsp2opt_sweep.cuh"
+#include "tsp2opt_sweep_xf.cuh"
+
+#include <type_traits>
+
+// Fast-path filter form of the sweep (DESIGN.md §5.2 / §5.2b): 1 = expanded
+// form (tsp2opt_sweep_xf.cuh), 0 = direct dx^2 + dy^2 form (default).
+#ifndef TSP2OPT_XF
+#define TSP2OPT_XF 0
+#endif
+#if TSP2OPT_XF
+#define TSP2OPT_TILE_SMEM TileSmemXF
+#define TSP2OPT_SWEEP_TILE sweep_tile_xf
+#define TSP2OPT_TILE_BYTES tile_smem_bytes_xf
+#else
+#define TSP2OPT_TILE_SMEM TileSmem
+#define TSP2OPT_SWEEP_TILE sweep_tile
+#define TSP2OPT_TILE_BYTES tile_smem_bytes
+#endif
 
 namespace tsp2opt {
 
@@ -77,9 +95,9 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* 
                                                      int respect_done)
 {
     extern __shared__ float4 smem[];
-    const TileSmem sm(smem, TJ);
+    const TSP2OPT_TILE_SMEM sm(smem, TJ);
     if (respect_done && *(volatile int*)&slot->done) return;  // converged: iteration is a no-op
-    sweep_tile<R, false>(P, E, n, tiles[blockIdx.x], TJ, slot, sm);
+    TSP2OPT_SWEEP_TILE<R, false>(P, E, n, tiles[blockIdx.x], TJ, slot, sm);
 }
 
 // ===========================================================================
@@ -197,7 +215,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
                                                            int* __restrict__ ctl)
 {
     extern __shared__ float4 smem[];
-    const TileSmem sm(smem, TJ);
+    const TSP2OPT_TILE_SMEM sm(smem, TJ);
     __shared__ Slot s_in;
     const int gtid = blockIdx.x * blockDim.x + threadIdx.x;
     const int stride = gridDim.x * blockDim.x;
@@ -210,7 +228,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
         if (s_in.done) break;  // uniform across the grid
         // a4/a5: tiles are assigned round-robin (largest first); the grid is co-resident
         for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
-            sweep_tile<R, true>(P, E, n, tiles[t], TJ, in, sm);
+            TSP2OPT_SWEEP_TILE<R, true>(P, E, n, tiles[t], TJ, in, sm);
             __syncthreads();  // before the next tile overwrites the shared chunk
         }
         grid_sync(bar, gridDim.x);
@@ -310,21 +328,46 @@ cudaError_t launch_reset_key(Slot* slot, cudaStream_t st)
     return cudaGetLastError();
 }
 
-size_t sweep_smem_bytes(const Geometry& g) { return tile_smem_bytes(g.tj, g.ti()); }
-static const Geometry kMaxGeo{kRows, kMaxWarps, kMaxTJ};
+size_t sweep_smem_bytes(const Geometry& g) { return TSP2OPT_TILE_BYTES(g.tj, g.ti()); }
+
+// The sweep is instantiated for R = 15 (large n: longest column steps) and
+// R = 7 (small / medium n: twice the warps per row block, lower latency per
+// tile); Geometry::rows selects one (choose_geometry in tsp2opt_api.cu).
+static_assert(kRowsLarge == 15 && kRowsSmall == 7, "instantiated row counts");
+template <typename F>
+static auto by_rows(int rows, F&& f)
+{
+    return rows == kRowsSmall ? f(std::integral_constant<int, kRowsSmall>{})
+                              : f(std::integral_constant<int, kRowsLarge>{});
+}
 
 cudaError_t sweep_prepare()
 {
-    return cudaFuncSetAttribute(sweep_kernel<kRows>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)sweep_smem_bytes(kMaxGeo));
+    for (int R : {kRowsSmall, kRowsLarge}) {
+        const Geometry gmax{R, kMaxWarps, kMaxTJ};
+        cudaError_t e = by_rows(R, [&](auto r) {
+            return cudaFuncSetAttribute(sweep_kernel<decltype(r)::value>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        (int)sweep_smem_bytes(gmax));
+        });
+        if (e != cudaSuccess) return e;
+        e = by_rows(R, [&](auto r) {
+            return cudaFuncSetAttribute(local_search_kernel<decltype(r)::value>,
+                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sweep_smem_bytes(gmax));
+        });
+        if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
 }
 
 cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
                          Slot* slot, int respect_done, cudaStream_t st)
 {
     if (ntiles <= 0) return cudaSuccess;
-    sweep_kernel<kRows><<<ntiles, 32 * g.warps, sweep_smem_bytes(g), st>>>(P, E, n, tiles, g.tj, slot,
-                                                                               respect_done);
+    by_rows(g.rows, [&](auto r) {
+        sweep_kernel<decltype(r)::value><<<ntiles, 32 * g.warps, sweep_smem_bytes(g), st>>>(P, E, n, tiles, g.tj,
+                                                                                            slot, respect_done);
+        return 0;
+    });
     g_launches += 1;
     return cudaGetLastError();
 }
@@ -343,9 +386,11 @@ cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Sl
 int local_search_grid(const Geometry& g, int ntiles)
 {
     int per_sm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, local_search_kernel<kRows>, 32 * g.warps,
-                                                      sweep_smem_bytes(g)) != cudaSuccess)
-        return 0;
+    cudaError_t e = by_rows(g.rows, [&](auto r) {
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, local_search_kernel<decltype(r)::value>,
+                                                             32 * g.warps, sweep_smem_bytes(g));
+    });
+    if (e != cudaSuccess) return 0;
     int dev = 0, sms = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
@@ -357,20 +402,15 @@ cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour,
                                 Slot* slots, int parity, long long max_moves, long long budget, unsigned* bar,
                                 int* ctl, cudaStream_t st)
 {
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(local_search_kernel<kRows>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)sweep_smem_bytes(kMaxGeo));
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
     int grid = local_search_grid(g, ntiles);
     if (grid < 1) return cudaErrorInvalidConfiguration;
     int TJ = g.tj;
     void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &TJ, &slots, &parity, &max_moves, &budget, &bar, &ctl};
     g_launches += 1;
-    return cudaLaunchCooperativeKernel((const void*)local_search_kernel<kRows>, dim3(grid), dim3(32 * g.warps), args,
-                                       sweep_smem_bytes(g), st);
+    return by_rows(g.rows, [&](auto r) {
+        return cudaLaunchCooperativeKernel((const void*)local_search_kernel<decltype(r)::value>, dim3(grid),
+                                           dim3(32 * g.warps), args, sweep_smem_bytes(g), st);
+    });
 }
 
 cudaError_t run_selftest_sqrt(double* max_rel, int* zero_ok)

@@ -84,13 +84,13 @@ __device__ __forceinline__ void set_bound(Bound<R>& b, const int (&erow)[R], int
 // Shared memory of one tile: the column chunk (the paper's coordinate range
 // "B", L20 Listing 2) and the edges of the CTA's rows (range "A").
 struct TileSmem {
-    float4* colxy;  // [TJ + 1]: (-x, -x, -y, -y) of columns J0..J1 (biased floats)
-    float* cole;    // [TJ + 1]: e_j as float
+    float4* colxy;  // [TJ + 2]: (-x, -x, -y, -y) of columns J0..J1 and one spare (biased floats)
+    float* cole;    // [TJ + 2]: e_j as float
     float* rowe;    // [32 * R * warps]: e_i of the CTA's rows, as float
     __device__ TileSmem(void* base, int TJ)
         : colxy(reinterpret_cast<float4*>(base)),
-          cole(reinterpret_cast<float*>(colxy + TJ + 1)),
-          rowe(cole + TJ + 1)
+          cole(reinterpret_cast<float*>(colxy + TJ + 2)),
+          rowe(cole + TJ + 2)
     {
     }
 };
@@ -224,7 +224,7 @@ __device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0,
 // Shared memory bytes of a tile with TJ columns and TI rows.
 __host__ __device__ inline size_t tile_smem_bytes(int TJ, int TI)
 {
-    return (size_t)(TJ + 1) * (sizeof(float4) + sizeof(float)) + (size_t)TI * sizeof(float);
+    return (size_t)(TJ + 2) * (sizeof(float4) + sizeof(float)) + (size_t)TI * sizeof(float);
 }
 
 // One tile.  All global loads of the tile (the lane's rows and row edges, the
@@ -260,7 +260,7 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
 #pragma unroll
         for (int r = 0; r < R; r++) erow[r] = gld<PS>(E + row0 + r);
     }
-    for (int c = threadIdx.x; c <= ncol; c += blockDim.x) {  // J1 <= n: P[n] = P[0] closes the tour
+    for (int c = threadIdx.x; c <= ncol + 1; c += blockDim.x) {  // J1 <= n: P[n] = P[0]; + 1 spare column
         const float2 p = gld<PS>(P + J0 + c);
         const int e = gld<PS>(E + J0 + c);
         sm.colxy[c] = make_float4(-p.x, -p.x, -p.y, -p.y);

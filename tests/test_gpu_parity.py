@@ -50,16 +50,19 @@ def test_best_move_parity_sizes(gpu, n, kind):
         assert g.best_move(th) == oracle.best_move(c, th)
 
 
+@pytest.mark.parametrize("rows", [7, 15])
 @pytest.mark.parametrize("warps,tj", [(1, 2), (1, 3), (1, 32), (2, 64), (4, 128), (4, 1024), (3, 7)])
-def test_best_move_parity_geometries(gpu, monkeypatch, warps, tj):
-    # tiny and odd tiles exercise masked diagonal tiles and ragged column tails
+def test_best_move_parity_geometries(gpu, monkeypatch, rows, warps, tj):
+    # tiny and odd tiles exercise masked diagonal tiles and ragged column tails,
+    # for both instantiated row counts R
+    monkeypatch.setenv("TSP2OPT_ROWS", str(rows))
     monkeypatch.setenv("TSP2OPT_WARPS", str(warps))
     monkeypatch.setenv("TSP2OPT_TJ", str(tj))
     for kind, n in (("uniform", 1002), ("lattice", 2000), ("uniform", 97)):
         c, t = _inst(kind, n, 5)
         with tsp2opt.TSP2Opt(c) as g:
             geo = g.geometry()
-            assert (geo["warps"], geo["tj"]) == (warps, tj)
+            assert (geo["rows"], geo["warps"], geo["tj"]) == (rows, warps, tj)
             assert geo["pairs"] == n * (n - 1) // 2
             assert g.best_move(t) == oracle.best_move(c, t)
 
