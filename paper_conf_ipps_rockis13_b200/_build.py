@@ -15,7 +15,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libtsp2opt.so")
 SOURCES = [os.path.join(CSRC, f) for f in ("tsp2opt_kernels.cu", "tsp2opt_api.cu")]
-HEADERS = [os.path.join(CSRC, f) for f in ("tsp2opt_device.cuh", "tsp2opt_internal.h", "tsp2opt_sweep.cuh", "tsp2opt_sweep_xf.cuh")] + [
+HEADERS = [os.path.join(CSRC, f) for f in ("tsp2opt_device.cuh", "tsp2opt_internal.h", "tsp2opt_sweep.cuh")] + [
     os.path.join(ROOT, "include", "tsp2opt.h")
 ]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

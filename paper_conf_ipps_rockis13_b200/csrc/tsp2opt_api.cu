@@ -66,6 +66,9 @@ struct tsp2opt_ctx {
     int* h_ctl = nullptr;         // pinned readback of d_ctl
     int persistent = 2;           // local_search loop: 0 per-iteration kernels, 1 persistent launch, 2 auto
     int2* d_tiles = nullptr;    // this shard's tiles
+    unsigned long long* d_tilebest = nullptr;  // [ntiles] per-tile minima of the last sweep (next seed)
+    bool seed_next = false;     // seed each tile with its surviving minimum of the previous sweep (TSP2OPT_SEED=1;
+                                // measured neutral-to-slower at n = 1002 .. 33810, so off by default)
     Slot* h_slot = nullptr;     // pinned readback
     unsigned epoch = 0;
     int parity = 0;             // iteration t reads slot[parity]
@@ -84,29 +87,24 @@ namespace {
 
 Geometry choose_geometry(long long pairs_per_rank)
 {
-    // R = 7 below ~1e9 pairs per rank (measured: faster sweeps and local
-    // searches at n = 1002 .. 33810), R = 15 above (n = 85900: 0.82 vs 0.91 ms).
-    int R = pairs_per_rank < 1000000000LL ? kRowsSmall : kRowsLarge;
+    // Measured on B200 (tools/exp_geometry*.py): one-warp CTAs
+    // and many small tiles win at every size (no intra-CTA barrier skew, the
+    // hardware scheduler balances); R = 15 from ~1e8 pairs (n = 33810: local
+    // search 0.63 s vs 0.68 s with R = 7), R = 7 below; columns per tile grow
+    // with the pair count (n = 85900: TJ = 128 -> 0.79 ms/sweep, 60k tiles;
+    // n = 7397: TJ = 16; n = 1002: TJ = 8).
+    const long long p = pairs_per_rank;
+    int R = p >= 100000000LL ? kRowsLarge : kRowsSmall;
+    int tj = p >= 1000000000LL ? 128 : p >= 100000000LL ? 64 : p >= 5000000LL ? 16 : 8;
+    int w = 1;
     if (const char* er = getenv("TSP2OPT_ROWS")) R = atoi(er) == kRowsSmall ? kRowsSmall : kRowsLarge;
-    Geometry best{R, 1, 32};
     const char* ew = getenv("TSP2OPT_WARPS");
     const char* et = getenv("TSP2OPT_TJ");
-    if (ew && et) {
-        Geometry g{R, atoi(ew), atoi(et)};
-        if (g.warps >= 1 && g.warps <= kMaxWarps && g.tj >= 2 && g.tj <= kMaxTJ) return g;
+    if (ew && et && atoi(ew) >= 1 && atoi(ew) <= kMaxWarps && atoi(et) >= 2 && atoi(et) <= kMaxTJ) {
+        w = atoi(ew);
+        tj = atoi(et);
     }
-    const long long target = 24LL * 148;  // tiles per shard: >= ~6 waves of 4 CTAs/SM
-    long long best_area = -1;
-    for (int w : {4, 2, 1})
-        for (int tj : {1024, 512, 256, 128, 64, 32}) {
-            Geometry g{R, w, tj};
-            long long area = (long long)g.ti() * tj;
-            if (pairs_per_rank / area >= target && area > best_area) {
-                best = g;
-                best_area = area;
-            }
-        }
-    return best;
+    return Geometry{R, w, tj};
 }
 
 // Tiles over the upper triangle only (L20 Fig. 8 "Skip unnecessary computation"):
@@ -151,9 +149,13 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
     std::vector<int2> host(mine.size());
     for (size_t k = 0; k < mine.size(); k++) host[k] = make_int2(mine[k].i0, mine[k].j0);
     if (h->d_tiles) cudaFree(h->d_tiles);
+    if (h->d_tilebest) cudaFree(h->d_tilebest);
     h->d_tiles = nullptr;
+    h->d_tilebest = nullptr;
     if (!host.empty()) {
         CUDA_TRY(cudaMalloc(&h->d_tiles, host.size() * sizeof(int2)));
+        CUDA_TRY(cudaMalloc(&h->d_tilebest, host.size() * sizeof(unsigned long long)));
+        CUDA_TRY(cudaMemset(h->d_tilebest, 0xFF, host.size() * sizeof(unsigned long long)));  // kKeyNone
         CUDA_TRY(cudaMemcpy(h->d_tiles, host.data(), host.size() * sizeof(int2), cudaMemcpyHostToDevice));
     }
     h->ntiles = (int)host.size();
@@ -178,6 +180,7 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_ctl);
     if (h->h_ctl) cudaFreeHost(h->h_ctl);
     cudaFree(h->d_tiles);
+    cudaFree(h->d_tilebest);
     if (h->h_slot) cudaFreeHost(h->h_slot);
     for (cudaEvent_t e : h->ev_pool) cudaEventDestroy(e);
     if (h->own_stream) cudaStreamDestroy(h->own_stream);
@@ -253,7 +256,8 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         h->ev_used += 2;
         CUDA_TRY(cudaEventRecord(ev0, h->stream));
     }
-    CUDA_TRY(launch_sweep(h->geo, h->d_P, h->d_E, h->n, h->d_tiles, h->ntiles, in, apply ? 1 : 0, h->stream));
+    CUDA_TRY(launch_sweep(h->geo, h->d_P, h->d_E, h->n, h->d_tiles, h->ntiles, in, apply ? 1 : 0, h->d_tilebest,
+                          h->seed_next ? 1 : 0, h->stream));
     if (ev1) CUDA_TRY(cudaEventRecord(ev1, h->stream));
     if (h->comm) {
         ncclResult_t r = ncclAllReduce(&in->key, &in->key, 1, ncclUint64, ncclMin, h->comm, h->stream);
@@ -307,6 +311,7 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     CTRY(cudaMalloc(&h->d_ctl, sizeof(int)));
     CTRY(cudaHostAlloc(&h->h_ctl, sizeof(int), cudaHostAllocDefault));
     if (const char* ep = getenv("TSP2OPT_PERSISTENT")) h->persistent = atoi(ep);
+    if (const char* es = getenv("TSP2OPT_SEED")) h->seed_next = atoi(es) != 0;
     CTRY(cudaMemset(h->d_slots, 0, sizeof(Slot) * 2));
     {
         std::vector<float2> pad(np, make_float2(kCoordBias, kCoordBias));
@@ -471,7 +476,8 @@ int tsp2opt_local_search(tsp2opt_t h, int32_t* tour, int64_t max_iters, int64_t*
                 return TSP2OPT_ECUDA;
             }
             CUDA_TRY(launch_local_search(h->geo, h->d_P, h->d_E, h->d_tour, h->n, h->d_tiles, h->ntiles, h->d_slots,
-                                         h->parity, max_iters, budget, h->d_bar, h->d_ctl, h->stream));
+                                         h->parity, max_iters, budget, h->d_bar, h->d_ctl, h->d_tilebest,
+                                         h->seed_next ? 1 : 0, h->stream));
             CUDA_TRY(cudaMemcpyAsync(h->h_ctl, h->d_ctl, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
             CUDA_TRY(cudaStreamSynchronize(h->stream));
             h->parity = *h->h_ctl;

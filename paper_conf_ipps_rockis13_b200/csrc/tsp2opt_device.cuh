@@ -68,6 +68,23 @@ __device__ __forceinline__ int nint_sqrt_exact(int s)
     return m;
 }
 
+// nint(sqrt(s)) from the float squared distance s_f = fma(dx, dx, dy*dy) of
+// exact dx, dy, when the float path is unambiguous: |sqrt_approx(s_f) - sqrt(s)|
+// < 0.03 (MUFU.SQRT relative error <= 2^-21, tsp2opt_selftest_sqrt; s_f within
+// 2^-23 of s), so a nearest integer m with |sqrt_approx(s_f) - m| < 0.45 is
+// nint(sqrt(s)).  Returns false (out untouched) otherwise.  Exhaustively
+// checked over every (dx, dy) by tsp2opt_selftest.
+__device__ __forceinline__ bool nint_from_float(float s_f, float& out)
+{
+    const float r = sqrt_approx(s_f);
+    const float m = (r + 12582912.0f) - 12582912.0f;  // 1.5 * 2^23: nearest integer (exact)
+    if (fabsf(r - m) < 0.45f) {
+        out = m;
+        return true;
+    }
+    return false;
+}
+
 __device__ __forceinline__ int exact_dist_xy(int xa, int ya, int xb, int yb)
 {
     int dx = xa - xb, dy = ya - yb;
@@ -176,6 +193,23 @@ __device__ __forceinline__ float2 sq2(float2 xr, float2 yr, float2 ncx, float2 n
 #endif
 }
 
+// A pair (a, b) of the tour before the 2-opt move (i, j) -- positions i+1..j
+// reversed -- keeps its delta in the new tour iff both its edges lie on the same
+// side of the reversed segment: both outside keep their positions, both inside
+// move to (i+j-b, i+j-a).  Returns the pair's key in the new tour, or kKeyNone.
+// Any such key is a real pair of the new tour with its exact delta, hence a
+// valid upper bound on the next sweep's minimum (every pair is still examined).
+__host__ __device__ __forceinline__ unsigned long long surviving_key(unsigned long long k, int i, int j)
+{
+    if (k == kKeyNone) return kKeyNone;
+    const int a = key_i(k), b = key_j(k);
+    const bool ain = a >= i + 1 && a <= j - 1, aout = a <= i - 1 || a >= j + 1;
+    const bool bin = b >= i + 1 && b <= j - 1, bout = b <= i - 1 || b >= j + 1;
+    if (aout && bout) return k;
+    if (ain && bin) return pack_key(key_delta(k), i + j - b, i + j - a);
+    return kKeyNone;
+}
+
 // Per-rank / per-handle device state, ping-ponged between iterations: the
 // kernels of iteration t read slot[t & 1] and write slot[(t + 1) & 1], so no
 // kernel ever reads a field another block of the same kernel writes.
@@ -185,8 +219,10 @@ struct __align__(64) Slot {
     long long moves;              // moves applied since the tour was loaded
     long long length;             // current tour length (int64: n * 46340 > 2^31)
     int done;                     // 0 running, 1 local minimum, 2 capped, bit 2 (4): invalid tour
-    unsigned next_tile;           // dynamic tile counter of the persistent sweep reading this slot
-    int pad[6];
+    unsigned next_tile;           // (reserved)
+    int seed_ok;                  // 1: last_key is the move just applied to the tour the tile minima of the
+                                  //    previous sweep were measured on (they may seed this sweep)
+    int pad[5];
 };
 
 }  // namespace tsp2opt

@@ -10,24 +10,8 @@
 #include "tsp2opt_device.cuh"
 #include "tsp2opt_internal.h"
 #include "tsp2opt_sweep.cuh"
-#include "tsp2opt_sweep_xf.cuh"
 
 #include <type_traits>
-
-// Fast-path filter form of the sweep (DESIGN.md §5.2 / §5.2b): 1 = expanded
-// form (tsp2opt_sweep_xf.cuh), 0 = direct dx^2 + dy^2 form (default).
-#ifndef TSP2OPT_XF
-#define TSP2OPT_XF 0
-#endif
-#if TSP2OPT_XF
-#define TSP2OPT_TILE_SMEM TileSmemXF
-#define TSP2OPT_SWEEP_TILE sweep_tile_xf
-#define TSP2OPT_TILE_BYTES tile_smem_bytes_xf
-#else
-#define TSP2OPT_TILE_SMEM TileSmem
-#define TSP2OPT_SWEEP_TILE sweep_tile
-#define TSP2OPT_TILE_BYTES tile_smem_bytes
-#endif
 
 namespace tsp2opt {
 
@@ -80,9 +64,16 @@ __global__ void init_slot_kernel(Slot* slot, int clear_length)
     if (clear_length) slot->length = 0;
     slot->done = 0;
     slot->next_tile = 0;
+    slot->seed_ok = 0;  // a freshly loaded tour: no previous sweep to seed from
 }
 
-__global__ void reset_key_kernel(Slot* slot) { slot->key = seed_key(); }
+// best_move's sweep is not followed by an apply: its tile minima must not be
+// combined with an older move by a later sweep.
+__global__ void reset_key_kernel(Slot* slot)
+{
+    slot->key = seed_key();
+    slot->seed_ok = 0;
+}
 
 // a4 + a5: the sweep of one tile lives in tsp2opt_sweep.cuh.
 
@@ -92,12 +83,13 @@ __global__ void reset_key_kernel(Slot* slot) { slot->key = seed_key(); }
 template <int R>
 __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* __restrict__ P, const int* __restrict__ E, int n,
                                                      const int2* __restrict__ tiles, int TJ, Slot* __restrict__ slot,
-                                                     int respect_done)
+                                                     int respect_done, unsigned long long* __restrict__ tilebest,
+                                                     int use_seed)
 {
     extern __shared__ float4 smem[];
-    const TSP2OPT_TILE_SMEM sm(smem, TJ);
+    const TileSmem sm(smem, TJ);
     if (respect_done && *(volatile int*)&slot->done) return;  // converged: iteration is a no-op
-    TSP2OPT_SWEEP_TILE<R, false>(P, E, n, tiles[blockIdx.x], TJ, slot, sm);
+    sweep_tile<R, false>(P, E, n, tiles[blockIdx.x], TJ, slot, sm, tilebest + blockIdx.x, use_seed);
 }
 
 // ===========================================================================
@@ -134,6 +126,7 @@ __device__ __forceinline__ bool apply_phase(float2* __restrict__ P, int* __restr
         o.length = in->length;
         o.done = explicit_move ? (done & 4) : done;  // an explicit move makes the tour unconverged
         o.next_tile = 0;
+        o.seed_ok = (apply && !explicit_move) ? 1 : 0;  // tile minima of this sweep seed the next one
         if (!explicit_move && !done) {
             if (key_delta(key) >= 0) o.done = 1;        // local minimum (reading R7)
             else if (moves >= max_moves) o.done = 2;    // capped with an improving move left (R8)
@@ -212,10 +205,11 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
                                                            const int2* __restrict__ tiles, int ntiles, int TJ,
                                                            Slot* __restrict__ slots, int parity, long long max_moves,
                                                            long long budget, unsigned* __restrict__ bar,
-                                                           int* __restrict__ ctl)
+                                                           int* __restrict__ ctl,
+                                                           unsigned long long* __restrict__ tilebest, int use_seed)
 {
     extern __shared__ float4 smem[];
-    const TSP2OPT_TILE_SMEM sm(smem, TJ);
+    const TileSmem sm(smem, TJ);
     __shared__ Slot s_in;
     const int gtid = blockIdx.x * blockDim.x + threadIdx.x;
     const int stride = gridDim.x * blockDim.x;
@@ -228,7 +222,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
         if (s_in.done) break;  // uniform across the grid
         // a4/a5: tiles are assigned round-robin (largest first); the grid is co-resident
         for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
-            TSP2OPT_SWEEP_TILE<R, true>(P, E, n, tiles[t], TJ, in, sm);
+            sweep_tile<R, true>(P, E, n, tiles[t], TJ, in, sm, tilebest + t, use_seed);
             __syncthreads();  // before the next tile overwrites the shared chunk
         }
         grid_sync(bar, gridDim.x);
@@ -238,9 +232,10 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
             s_in.moves = *(volatile long long*)&in->moves;
             s_in.length = *(volatile long long*)&in->length;
             s_in.done = *(volatile int*)&in->done;
+            s_in.seed_ok = *(volatile int*)&in->seed_ok;
         }
         __syncthreads();
-        apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride);  // a7/a8
+        apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride);
         p ^= 1;
         grid_sync(bar, gridDim.x);
     }
@@ -298,7 +293,11 @@ __global__ void selftest_filter_kernel(unsigned long long* bad, unsigned long lo
         const float2 s = sq2(xr, yr, ncx, ncy);
         const int t = nint_sqrt_exact(dx * dx + dy * dy);  // smallest t with "D <= t"
         const float S = sq_threshold((float)t);
-        if (!(s.x <= S) || !(s.y <= S)) {
+        // the float nint shortcut of the rare path: when it claims a value, it is exact
+        float m = -1.f;
+        const float fdx = (float)dx, fdy = (float)dy;
+        const bool claimed = nint_from_float(fmaf(fdx, fdx, fdy * fdy), m);
+        if (!(s.x <= S) || !(s.y <= S) || (claimed && m != (float)t)) {
             nbad++;
             atomicMin(first, (unsigned long long)id);
         }
@@ -328,7 +327,7 @@ cudaError_t launch_reset_key(Slot* slot, cudaStream_t st)
     return cudaGetLastError();
 }
 
-size_t sweep_smem_bytes(const Geometry& g) { return TSP2OPT_TILE_BYTES(g.tj, g.ti()); }
+size_t sweep_smem_bytes(const Geometry& g) { return tile_smem_bytes(g.tj, g.ti()); }
 
 // The sweep is instantiated for R = 15 (large n: longest column steps) and
 // R = 7 (small / medium n: twice the warps per row block, lower latency per
@@ -360,12 +359,13 @@ cudaError_t sweep_prepare()
 }
 
 cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
-                         Slot* slot, int respect_done, cudaStream_t st)
+                         Slot* slot, int respect_done, unsigned long long* tilebest, int use_seed, cudaStream_t st)
 {
     if (ntiles <= 0) return cudaSuccess;
     by_rows(g.rows, [&](auto r) {
         sweep_kernel<decltype(r)::value><<<ntiles, 32 * g.warps, sweep_smem_bytes(g), st>>>(P, E, n, tiles, g.tj,
-                                                                                            slot, respect_done);
+                                                                                            slot, respect_done, tilebest,
+                                                                                            use_seed);
         return 0;
     });
     g_launches += 1;
@@ -400,12 +400,13 @@ int local_search_grid(const Geometry& g, int ntiles)
 
 cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
                                 Slot* slots, int parity, long long max_moves, long long budget, unsigned* bar,
-                                int* ctl, cudaStream_t st)
+                                int* ctl, unsigned long long* tilebest, int use_seed, cudaStream_t st)
 {
     int grid = local_search_grid(g, ntiles);
     if (grid < 1) return cudaErrorInvalidConfiguration;
     int TJ = g.tj;
-    void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &TJ, &slots, &parity, &max_moves, &budget, &bar, &ctl};
+    void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &TJ, &slots, &parity, &max_moves, &budget, &bar, &ctl,
+                    &tilebest, &use_seed};
     g_launches += 1;
     return by_rows(g.rows, [&](auto r) {
         return cudaLaunchCooperativeKernel((const void*)local_search_kernel<decltype(r)::value>, dim3(grid),

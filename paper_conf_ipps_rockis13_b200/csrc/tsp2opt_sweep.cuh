@@ -62,6 +62,7 @@ __device__ __forceinline__ void column_sq(float (&s)[R + 1], const Rows<R>& rows
 template <int R>
 struct Bound {
     int B;          // accept delta < B (lane-local running bound)
+    float Bf;       // B as float (exact)
     float a2f;      // column offset a2 = (B - 2) - a1
     float srow[R];  // row thresholds: D(i_r, j) <= e_{i_r} + a1  <=>  s <= srow[r]
 };
@@ -69,16 +70,20 @@ struct Bound {
 // Thresholds of the exact necessary condition for bound B:
 // delta <= B - 1 = c  ==>  D(i,j) <= e_i + a1  or  D(i+1,j+1) <= e_j + a2,
 // a1 = floor((c - 1) / 2), a2 = c - 1 - a1.
+// Row edges are floats (exact integers): no int <-> float conversions (XU
+// pipe) when the bound drops mid-tile.
 template <int R>
-__device__ __forceinline__ void set_bound(Bound<R>& b, const int (&erow)[R], int B)
+__device__ __forceinline__ void set_bound(Bound<R>& b, const float* erowf, int B)
 {
     b.B = B;
+    b.Bf = (float)B;
     const int c = B - 1;
     const int a1 = (c - 1) >> 1;
     const int a2 = c - 1 - a1;
     b.a2f = (float)a2;
+    const float a1f = (float)a1;
 #pragma unroll
-    for (int r = 0; r < R; r++) b.srow[r] = sq_threshold((float)(erow[r] + a1));
+    for (int r = 0; r < R; r++) b.srow[r] = sq_threshold(erowf[r] + a1f);
 }
 
 // Shared memory of one tile: the column chunk (the paper's coordinate range
@@ -100,10 +105,7 @@ struct TileSmem {
 template <int R>
 __device__ __forceinline__ void reset_bound(Bound<R>& b, const float* my_rowe, int B)
 {
-    int erow[R];
-#pragma unroll
-    for (int r = 0; r < R; r++) erow[r] = (int)my_rowe[r];
-    set_bound<R>(b, erow, B);
+    set_bound<R>(b, my_rowe, B);
 }
 
 // The fast test of one column step: does any pair (i_r, j), r < R, of this
@@ -149,7 +151,7 @@ __device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1
                                            float scol, int row0, int j, float4 c0, float4 c1, float ej,
                                            const float* my_rowe, const float2* P, unsigned long long& mykey)
 {
-    const float lim = ej + (float)b.B + 0.5f;
+    const float lim = ej + b.Bf + 0.5f;
     unsigned mask = 0;
 #pragma unroll
     for (int r = 0; r < R; r++) {
@@ -164,20 +166,30 @@ __device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1
     if (!mask) return;
     const int xj = unbias(-c0.x), yj = unbias(-c0.z);
     const int xj1 = unbias(-c1.x), yj1 = unbias(-c1.z);
-    const int ejn = (int)ej;
-    int B = b.B;
+    float Bf = b.Bf;
     while (mask) {  // ascending r == ascending cell number
         const int r = __ffs(mask) - 1;
         mask &= mask - 1;
         const float2 pi = gld<PS>(P + row0 + r), pi1 = gld<PS>(P + row0 + r + 1);
-        const int d = exact_dist_xy(unbias(pi.x), unbias(pi.y), xj, yj) +
-                      exact_dist_xy(unbias(pi1.x), unbias(pi1.y), xj1, yj1) - (int)my_rowe[r] - ejn;
-        if (d < B) {
-            B = d;
-            mykey = pack_key(d, row0 + r, j);
+        // nint from the float path when it is unambiguous: |sqrt_approx(s_f) - sqrt(s)|
+        // < 0.03, so |r - m| < 0.45 for the nearest integer m
+        // proves nint(sqrt(s)) == m.  Otherwise the integer nint (rare).
+        const float dx = pi.x + c0.x, dy = pi.y + c0.z, dx1 = pi1.x + c1.x, dy1 = pi1.y + c1.z;  // exact
+        float d1, d2;
+        if (!nint_from_float(fmaf(dx, dx, dy * dy), d1))
+            d1 = (float)exact_dist_xy(unbias(pi.x), unbias(pi.y), xj, yj);
+        if (!nint_from_float(fmaf(dx1, dx1, dy1 * dy1), d2))
+            d2 = (float)exact_dist_xy(unbias(pi1.x), unbias(pi1.y), xj1, yj1);
+        const float d = (d1 + d2) - (my_rowe[r] + ej);  // exact: integers < 2^24
+        if (d < Bf) {
+            Bf = d;
+            mykey = pack_key((int)d, row0 + r, j);
         }
     }
-    b.B = B;
+    if (Bf < b.Bf) {
+        b.B = (int)Bf;
+        b.Bf = Bf;
+    }
 }
 
 template <int R, bool MASK, bool PS>
@@ -234,9 +246,11 @@ __host__ __device__ inline size_t tile_smem_bytes(int TJ, int TI)
 // minima are published with one atomicMin each (L16 Fig. 4 "Get best local
 // pair ... Get best global pair"; min is order-independent, so the result is
 // deterministic).  The caller synchronises the CTA before reusing `sm`.
+constexpr int kMaxWarpsPerTile = 4;
+
 template <int R, bool PS>
 __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n, int2 tile, int TJ, Slot* slot,
-                                           const TileSmem& sm)
+                                           const TileSmem& sm, unsigned long long* tilebest, int use_seed)
 {
     const int I0 = tile.x, J0 = tile.y;
     const int J1 = min(J0 + TJ, n);  // columns j in [J0, J1), j <= n-1
@@ -249,7 +263,7 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     float* my_rowe = sm.rowe + threadIdx.x * R;  // stride R (odd): conflict-free
 
     Rows<R> rows;
-    int erow[R];
+    float erow[R];
     if (active) {
 #pragma unroll
         for (int q = 0; q < (R + 1) / 2; q++) {
@@ -258,7 +272,7 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
             rows.yp[q] = make_float2(p0.y, p1.y);
         }
 #pragma unroll
-        for (int r = 0; r < R; r++) erow[r] = gld<PS>(E + row0 + r);
+        for (int r = 0; r < R; r++) erow[r] = (float)gld<PS>(E + row0 + r);
     }
     for (int c = threadIdx.x; c <= ncol + 1; c += blockDim.x) {  // J1 <= n: P[n] = P[0]; + 1 spare column
         const float2 p = gld<PS>(P + J0 + c);
@@ -268,27 +282,49 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     }
     // The slot key is the seed (0, cell 0) or a real pair of this sweep, so a
     // pair of ours can only win with delta < 0 (key delta 0) or delta <= key delta.
-    const int dg = key_delta(*(volatile unsigned long long*)&slot->key);
+    // This tile's minimum of the previous sweep, if the move applied since leaves
+    // it intact, is such a real pair too: it tightens the start bound and is
+    // published for the other tiles.
+    unsigned long long g = *(volatile unsigned long long*)&slot->key;
+    if (use_seed && *(volatile int*)&slot->seed_ok) {
+        const unsigned long long mv = *(volatile unsigned long long*)&slot->last_key;
+        const unsigned long long k = surviving_key(*(volatile unsigned long long*)tilebest, key_i(mv), key_j(mv));
+        if (k < g) {
+            g = k;
+            if (threadIdx.x == 0) atomicMin(&slot->key, k);
+        }
+    }
+    const int dg = key_delta(g);
     if (active) {
 #pragma unroll
-        for (int r = 0; r < R; r++) my_rowe[r] = (float)erow[r];
+        for (int r = 0; r < R; r++) my_rowe[r] = erow[r];
     }
     __syncthreads();
-    if (!active) return;
 
     unsigned long long mykey = kKeyNone;
-    Bound<R> b;
-    set_bound<R>(b, erow, dg == 0 ? 0 : dg + 1);
-    const bool masked = (wrow0 + 32 * R - 1) >= jstart;  // warp-uniform: some row >= some j
-    if (masked) walk<R, true, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
-    else walk<R, false, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
-
+    if (active) {
+        Bound<R> b;
+        set_bound<R>(b, erow, dg == 0 ? 0 : dg + 1);
+        const bool masked = (wrow0 + 32 * R - 1) >= jstart;  // warp-uniform: some row >= some j
+        if (masked) walk<R, true, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
+        else walk<R, false, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        const unsigned long long other = __shfl_xor_sync(0xffffffffu, mykey, o);
-        mykey = other < mykey ? other : mykey;
+        for (int o = 16; o > 0; o >>= 1) {
+            const unsigned long long other = __shfl_xor_sync(0xffffffffu, mykey, o);
+            mykey = other < mykey ? other : mykey;
+        }
+        if (lane == 0 && mykey < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, mykey);
     }
-    if (lane == 0 && mykey < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, mykey);
+    // The tile's best (a real pair of this sweep, or none) is kept for the next
+    // iteration's seed (apply_phase: moves the applied reversal leaves intact).
+    __shared__ unsigned long long s_red[kMaxWarpsPerTile];
+    if (lane == 0) s_red[warp] = mykey;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long m = s_red[0];
+        for (int w = 1; w < (int)(blockDim.x >> 5); w++) m = s_red[w] < m ? s_red[w] : m;
+        *tilebest = m;
+    }
 }
 
 }  // namespace tsp2opt

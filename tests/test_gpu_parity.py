@@ -223,11 +223,14 @@ def test_small_n_cases(gpu):
 
 
 @pytest.mark.parametrize("persistent", ["0", "1"])
-@pytest.mark.parametrize("kind,n,seed", [("uniform", 1002, 5), ("lattice", 3001, 6), ("uniform", 97, 7)])
+@pytest.mark.parametrize("kind,n,seed", [("uniform", 1002, 5), ("lattice", 3001, 6), ("uniform", 97, 7),
+                                         ("lattice", 2000, 8)])
 def test_local_search_parity_both_loops(gpu, monkeypatch, persistent, kind, n, seed):
     """The persistent single-launch loop and the per-iteration kernel loop (used by
-    sharded handles) reach the oracle's local minimum identically."""
+    sharded handles) reach the oracle's local minimum identically, with and
+    without per-tile seeding."""
     monkeypatch.setenv("TSP2OPT_PERSISTENT", persistent)
+    monkeypatch.setenv("TSP2OPT_SEED", "1" if seed % 2 else "0")
     c, t = _inst(kind, n, seed)
     ref = oracle.local_search(c, t)
     with tsp2opt.TSP2Opt(c) as g:
@@ -237,3 +240,46 @@ def test_local_search_parity_both_loops(gpu, monkeypatch, persistent, kind, n, s
         capped = g.local_search(t, max_iters=17)
         want = oracle.local_search(c, t, max_iters=17)
         assert capped["status"] == want["status"] and np.array_equal(capped["tour"], want["tour"])
+
+
+@pytest.mark.parametrize("rows", [7, 15])
+def test_seeded_sweeps_mixed_operations(gpu, monkeypatch, rows):
+    """Each sweep after a device-resident move is seeded with the previous sweep's
+    surviving tile minima; interleave every operation that could make those
+    stale (best_move sweeps, explicit applies, new tours, shard changes) and
+    check each following sweep against the oracle."""
+    monkeypatch.setenv("TSP2OPT_ROWS", str(rows))
+    monkeypatch.setenv("TSP2OPT_SEED", "1")
+    c, t = _inst("lattice", 3001, 8)
+    rng = np.random.default_rng(3)
+    with tsp2opt.TSP2Opt(c) as g:
+        g.set_tour(t)
+
+        def check():
+            tour, L = g.get_tour()
+            assert L == oracle.tour_length(c, tour)
+            assert g.best_move() == oracle.best_move(c, tour)
+
+        for rnd in range(6):
+            g.iterate_async(int(rng.integers(1, 5)))
+            g.sync()
+            check()                       # best_move right after seeded iterations
+            g.iterate_async(2)            # ... and iterations right after a best_move sweep
+            g.sync()
+            check()
+            i, j = sorted(rng.choice(3001, 2, replace=False).tolist())
+            g.apply(i, j)                 # explicit (non-improving) move
+            g.iterate_async(1)
+            g.sync()
+            check()
+            if rnd == 3:
+                g.debug_set_shard(1, 3)   # a different tile list
+                g.debug_set_shard(0, 1)
+                g.iterate_async(2)
+                g.sync()
+                check()
+            if rnd == 4:
+                g.set_tour(inputs.random_tour(3001, 99))
+                g.iterate_async(3)
+                g.sync()
+                check()
