@@ -206,6 +206,7 @@ def run_ours(args):
         ls = time_to_local_min(tsp2opt, args.ls_config)
 
     if rank == 0:
+        prof = ncu_profile_summary(args.config, args.tour)
         pk = peaks()
         sm_max = clocks.get("sm_max_mhz") or pk.get("sm_max_mhz") or 1965.0
         peak = PAIRS_PER_CLK_SM * N_SM * sm_max * 1e6 * world  # aggregate over ranks
@@ -230,9 +231,10 @@ def run_ours(args):
                        "n": n, "pairs_per_step": total_pairs, "l2": "flushed (256 MiB write) between timed steps",
                        "geometry": geo, "parallelism": f"tile-shard x{world}"},
             "roofline": {"bound": "alu", "achieved": achieved / 1e9, "peak": peak / 1e9, "unit": "Gpair/s",
-                         "frac": achieved / peak, "traffic": None,
+                         "frac": achieved / peak, "traffic": prof.get("traffic"),
                          "kernel": "sweep_kernel", "peak_def": f"{PAIRS_PER_CLK_SM} pairs/clk/SM x {N_SM} SMs x "
                          f"{sm_max:.0f} MHz (north_star: ~2 distance evaluations per pair; DESIGN.md §7)",
+                         "issue_util_ncu": prof.get("issue_util"), "ncu_profile": prof.get("path"),
                          "sweep_ms_avg": sweep_avg_ms, "sweep_share_of_step": sweep_avg_ms / (total_ms / args.steps)},
             "e2e": {"value": total_pairs * len(e2e_ms) / (e2e_total * 1e-3), "unit": UNIT,
                     "h2d_bytes_per_step": 4 * n, "d2h_bytes_per_step": 2 * 64,
@@ -249,6 +251,28 @@ def run_ours(args):
     g.close()
     if world > 1:
         dist.destroy_process_group()
+
+
+def ncu_profile_summary(cfg, tour):
+    """DRAM traffic per launch and issue utilisation of the sweep kernel from the
+    committed `ncu --set full` summary of this workload (profiles/, newest round)."""
+    import glob
+    paths = sorted(glob.glob(os.path.join(ROOT, "profiles", f"r*_sweep_{cfg}_{tour}_ncu.txt")))
+    if not paths:
+        return {}
+    vals = {}
+    for line in open(paths[-1]):
+        if line.startswith("ipc_per_sm"):
+            vals["ipc_per_sm"] = float(line.split()[3])
+        elif line.startswith(("dram_read", "dram_write")):
+            name, num, unit = (line.split() + ["byte"])[:3]
+            vals[name] = float(num) * {"Mbyte": 1e6, "Kbyte": 1e3, "byte": 1.0, "Gbyte": 1e9}.get(unit, 1.0)
+    out = {"path": os.path.relpath(paths[-1], ROOT)}
+    if "dram_read" in vals:
+        out["traffic"] = vals["dram_read"] + vals.get("dram_write", 0.0)
+    if "ipc_per_sm" in vals:
+        out["issue_util"] = vals["ipc_per_sm"] / 4.0
+    return out
 
 
 def time_to_local_min(tsp2opt, cfg_name):
