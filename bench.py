@@ -150,36 +150,48 @@ def run_ours(args):
         g.set_tour_device_async(d_tour.data_ptr())
         g.iterate_async(1)
 
-    for _ in range(args.warmup):
-        step()
-    s = g.sync()
-    first_move = s["last_move"]
+    def timed_steps(nsteps, sample_clocks):
+        """K device-timed steps (CUDA events on the library's stream, L2 flushed
+        between steps outside the events); the sweep kernel timed separately."""
+        for _ in range(args.warmup):
+            step()
+        s = g.sync()
+        first = s["last_move"]
+        sampler = ClockSampler(local) if sample_clocks else None
+        if sampler:
+            sampler.start()
+        starts = [torch.cuda.Event(enable_timing=True) for _ in range(nsteps)]
+        ends = [torch.cuda.Event(enable_timing=True) for _ in range(nsteps)]
+        g.profile(True)
+        launches0 = tsp2opt.launch_count()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        for k in range(nsteps):
+            l2_flush(flush)  # between timed steps, outside the events
+            starts[k].record(stream)
+            step()
+            ends[k].record(stream)
+        torch.cuda.synchronize()
+        nlaunch = tsp2opt.launch_count() - launches0
+        if world > 1:
+            dist.barrier()
+        clk = sampler.stop() if sampler else None
+        sms, sn = g.profile_read()
+        g.profile(False)
+        tot = sum(a.elapsed_time(b) for a, b in zip(starts, ends))
+        s = g.sync()
+        assert s["iterations"] == 1 and s["last_move"] == first, "steps must be identical"
+        return tot, sms / max(sn, 1), nlaunch, clk, first
 
-    sampler = ClockSampler(local)
-    sampler.start()
-    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    g.profile(True)
-    launches0 = tsp2opt.launch_count()
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    for k in range(args.steps):
-        l2_flush(flush)  # between timed steps, outside the events
-        starts[k].record(stream)
-        step()
-        ends[k].record(stream)
-    torch.cuda.synchronize()
-    launches = tsp2opt.launch_count() - launches0
-    if world > 1:
-        dist.barrier()
-    clocks = sampler.stop()
-    sweep_ms, sweep_n = g.profile_read()
-    g.profile(False)
-    step_ms = [a.elapsed_time(b) for a, b in zip(starts, ends)]
-    total_ms = sum(step_ms)
-    s = g.sync()
-    assert s["iterations"] == 1 and s["last_move"] == first_move, "steps must be identical"
+    # Headline: every pair tested individually (tile bounds off), DESIGN.md §7.
+    g.set_option(tsp2opt.OPT_TILE_BOUNDS, 0)
+    total_ms, sweep_avg_ms, launches, clocks, first_move = timed_steps(args.steps, True)
+    # Same workload with the exact tile-level bounds on (the library default).
+    g.set_option(tsp2opt.OPT_TILE_BOUNDS, 1)
+    tb_total_ms, tb_sweep_ms, _, _, tb_move = timed_steps(max(3, args.steps // 2), False)
+    assert tb_move == first_move
+    g.set_option(tsp2opt.OPT_TILE_BOUNDS, 0)
 
     # e2e: same metric through the public C ABI with HOST buffers each step
     # (H2D of the tour, device sweep + apply, D2H of the move and the state).
@@ -195,11 +207,13 @@ def run_ours(args):
             g.apply(i, j)
         e2e_ms.append((time.perf_counter() - t0) * 1e3)
     e2e_ms = e2e_ms[1:]
+    tb_steps = max(3, args.steps // 2)
 
-    t = torch.tensor([total_ms, sweep_ms / max(sweep_n, 1), sum(e2e_ms)], dtype=torch.float64, device="cuda")
+    t = torch.tensor([total_ms, sweep_avg_ms, sum(e2e_ms), tb_total_ms, tb_sweep_ms], dtype=torch.float64,
+                     device="cuda")
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    total_ms, sweep_avg_ms, e2e_total = t.tolist()
+    total_ms, sweep_avg_ms, e2e_total, tb_total_ms, tb_sweep_ms = t.tolist()
 
     ls = None
     if rank == 0 and world == 1 and not args.no_ls:
@@ -239,6 +253,10 @@ def run_ours(args):
             "e2e": {"value": total_pairs * len(e2e_ms) / (e2e_total * 1e-3), "unit": UNIT,
                     "h2d_bytes_per_step": 4 * n, "d2h_bytes_per_step": 2 * 64,
                     "api": "tsp2opt_best_move(host tour) + tsp2opt_apply"},
+            "tile_bounds": {"value": total_pairs * tb_steps / (tb_total_ms * 1e-3), "unit": UNIT,
+                            "ms_per_step": tb_total_ms / tb_steps, "sweep_ms_avg": tb_sweep_ms,
+                            "note": "same steps with the exact tile-level bounding-box bound on (library default); "
+                                    "pairs of a skipped tile are covered by one proof, not tested one by one"},
             "gpu_launches": launches,
             "clocks": clocks,
             "first_move": list(first_move),

@@ -126,6 +126,22 @@ int tsp2opt_local_search(tsp2opt_t h, int32_t *tour, int64_t max_iters, int64_t 
 /* Copy the current tour (host int32[n]) and its length out. */
 int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
 
+/* Execution options (none changes any result; all results stay bit-exact):
+ *  TSP2OPT_OPT_TILE_BOUNDS (default 1): skip a tile of the sweep when the
+ *      bounding boxes of its row and column cities prove that no pair can pass
+ *      the per-pair necessary condition; 0 tests every pair
+ *      individually (the pair-check throughput the bench reports).
+ *  TSP2OPT_OPT_SEED (default 0): start each tile from its own minimum of the
+ *      previous sweep when the applied move leaves that pair intact.
+ *  TSP2OPT_OPT_PERSISTENT (default 2): local_search loop, 0 = one sweep and one
+ *      apply kernel per iteration, 1 = one persistent cooperative launch,
+ *      2 = choose by size (world == 1 only).
+ * Returns TSP2OPT_EINVAL for an unknown option or value. */
+#define TSP2OPT_OPT_TILE_BOUNDS 1
+#define TSP2OPT_OPT_SEED 2
+#define TSP2OPT_OPT_PERSISTENT 3
+int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value);
+
 /* Diagnostics / test hooks ------------------------------------------------ */
 
 /* Restrict this handle's sweep to shard `rank` of `world` of the tile space

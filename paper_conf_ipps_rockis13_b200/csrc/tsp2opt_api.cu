@@ -69,6 +69,7 @@ struct tsp2opt_ctx {
     unsigned long long* d_tilebest = nullptr;  // [ntiles] per-tile minima of the last sweep (next seed)
     bool seed_next = false;     // seed each tile with its surviving minimum of the previous sweep (TSP2OPT_SEED=1;
                                 // measured neutral-to-slower at n = 1002 .. 33810, so off by default)
+    bool tile_bounds = true;    // tile-level bounding-box form of the filter (TSP2OPT_OPT_TILE_BOUNDS)
     Slot* h_slot = nullptr;     // pinned readback
     unsigned epoch = 0;
     int parity = 0;             // iteration t reads slot[parity]
@@ -240,6 +241,11 @@ int load_host_tour(tsp2opt_ctx* h, const int32_t* tour)
     return load_device_tour(h, h->d_tour_in);
 }
 
+int sweep_flags(const tsp2opt_ctx* h)
+{
+    return (h->seed_next ? kSweepSeed : 0) | (h->tile_bounds ? kSweepTileBounds : 0);
+}
+
 // One iteration: sweep (a4/a5) -> allreduce-min (a6) -> apply (a7/a8).
 int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
 {
@@ -257,7 +263,7 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         CUDA_TRY(cudaEventRecord(ev0, h->stream));
     }
     CUDA_TRY(launch_sweep(h->geo, h->d_P, h->d_E, h->n, h->d_tiles, h->ntiles, in, apply ? 1 : 0, h->d_tilebest,
-                          h->seed_next ? 1 : 0, h->stream));
+                          sweep_flags(h), h->stream));
     if (ev1) CUDA_TRY(cudaEventRecord(ev1, h->stream));
     if (h->comm) {
         ncclResult_t r = ncclAllReduce(&in->key, &in->key, 1, ncclUint64, ncclMin, h->comm, h->stream);
@@ -312,6 +318,7 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     CTRY(cudaHostAlloc(&h->h_ctl, sizeof(int), cudaHostAllocDefault));
     if (const char* ep = getenv("TSP2OPT_PERSISTENT")) h->persistent = atoi(ep);
     if (const char* es = getenv("TSP2OPT_SEED")) h->seed_next = atoi(es) != 0;
+    if (const char* eb = getenv("TSP2OPT_TILE_BOUNDS")) h->tile_bounds = atoi(eb) != 0;
     CTRY(cudaMemset(h->d_slots, 0, sizeof(Slot) * 2));
     {
         std::vector<float2> pad(np, make_float2(kCoordBias, kCoordBias));
@@ -477,7 +484,7 @@ int tsp2opt_local_search(tsp2opt_t h, int32_t* tour, int64_t max_iters, int64_t*
             }
             CUDA_TRY(launch_local_search(h->geo, h->d_P, h->d_E, h->d_tour, h->n, h->d_tiles, h->ntiles, h->d_slots,
                                          h->parity, max_iters, budget, h->d_bar, h->d_ctl, h->d_tilebest,
-                                         h->seed_next ? 1 : 0, h->stream));
+                                         sweep_flags(h), h->stream));
             CUDA_TRY(cudaMemcpyAsync(h->h_ctl, h->d_ctl, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
             CUDA_TRY(cudaStreamSynchronize(h->stream));
             h->parity = *h->h_ctl;
@@ -521,6 +528,21 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t* tour_out, int64_t* length)
     CUDA_TRY(cudaMemcpyAsync(tour_out, h->d_tour, sizeof(int32_t) * h->n, cudaMemcpyDeviceToHost, h->stream));
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     if (length) *length = h->h_slot->length;
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
+{
+    if (!h) return TSP2OPT_EINVAL;
+    switch (option) {
+    case TSP2OPT_OPT_TILE_BOUNDS: h->tile_bounds = value != 0; break;
+    case TSP2OPT_OPT_SEED: h->seed_next = value != 0; break;
+    case TSP2OPT_OPT_PERSISTENT:
+        if (value < 0 || value > 2) return TSP2OPT_EINVAL;
+        h->persistent = (int)value;
+        break;
+    default: return TSP2OPT_EINVAL;
+    }
     return TSP2OPT_OK;
 }
 

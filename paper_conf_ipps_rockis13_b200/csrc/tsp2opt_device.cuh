@@ -22,6 +22,10 @@ constexpr int kKeyJShift = 22;
 constexpr int kDeltaBias = 1 << 18;
 constexpr unsigned long long kKeyNone = ~0ULL;
 
+// sweep option bits (tsp2opt_set_option)
+constexpr int kSweepSeed = 1;        // seed each tile with its surviving minimum of the previous sweep
+constexpr int kSweepTileBounds = 2;  // skip tiles whose bounding boxes prove that no pair passes the filter
+
 __host__ __device__ __forceinline__ unsigned long long pack_key(int delta, int i, int j)
 {
     return ((unsigned long long)(unsigned)(delta + kDeltaBias) << kKeyDeltaShift) |

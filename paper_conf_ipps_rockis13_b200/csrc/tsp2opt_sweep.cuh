@@ -233,6 +233,62 @@ __device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0,
     if (j < J1) column_step<R, MASK, PS>(rows, b, sa, sb, row0, j, J0, sm, my_rowe, P, mykey);
 }
 
+// Tile-level form of the same exact necessary condition (a bound on all of the
+// tile's pairs at once).  Every squared distance the walk would compare is
+// between a city of the warp's row block (rows r = 0..R of every lane) and a
+// column city c in [cbeg, cend] of the staged chunk, so it is at least the
+// squared distance d2 between the two bounding boxes; every threshold it is
+// compared with is at most max(max_r srow[r], sq_threshold(max_j e_j + a2)).
+// If d2 exceeds that (with 2^-20 slack for the float roundings of d2 and of
+// the walk's own s_f >= s (1 - 2^-23)), no pair of the tile can pass the
+// per-pair filter and the walk is skipped.  Spatially coherent tours (the
+// later sweeps of a local search) skip most tiles; random tours skip none.
+template <int R>
+__device__ __forceinline__ bool tile_may_pass(const Rows<R>& rows, const Bound<R>& b, const TileSmem& sm, int cbeg,
+                                              int cend)
+{
+    float xlo = rows.xp[0].x, xhi = xlo, ylo = rows.yp[0].x, yhi = ylo;
+#pragma unroll
+    for (int q = 0; q < (R + 1) / 2; q++) {
+        xlo = fminf(xlo, fminf(rows.xp[q].x, rows.xp[q].y));
+        xhi = fmaxf(xhi, fmaxf(rows.xp[q].x, rows.xp[q].y));
+        ylo = fminf(ylo, fminf(rows.yp[q].x, rows.yp[q].y));
+        yhi = fmaxf(yhi, fmaxf(rows.yp[q].x, rows.yp[q].y));
+    }
+    float smax = b.srow[0];
+#pragma unroll
+    for (int r = 1; r < R; r++) smax = fmaxf(smax, b.srow[r]);
+    // column cities are staged negated: colxy = (-x, -x, -y, -y)
+    float cxlo = 3.0e38f, cxhi = -3.0e38f, cylo = 3.0e38f, cyhi = -3.0e38f, emax = -1.0f;
+    for (int c = cbeg + (int)(threadIdx.x & 31); c <= cend; c += 32) {
+        const float4 v = sm.colxy[c];
+        cxlo = fminf(cxlo, -v.x);
+        cxhi = fmaxf(cxhi, -v.x);
+        cylo = fminf(cylo, -v.z);
+        cyhi = fmaxf(cyhi, -v.z);
+        if (c < cend) emax = fmaxf(emax, sm.cole[c]);  // e_j of the step's own column j < J1
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        xlo = fminf(xlo, __shfl_xor_sync(0xffffffffu, xlo, o));
+        xhi = fmaxf(xhi, __shfl_xor_sync(0xffffffffu, xhi, o));
+        ylo = fminf(ylo, __shfl_xor_sync(0xffffffffu, ylo, o));
+        yhi = fmaxf(yhi, __shfl_xor_sync(0xffffffffu, yhi, o));
+        smax = fmaxf(smax, __shfl_xor_sync(0xffffffffu, smax, o));
+        cxlo = fminf(cxlo, __shfl_xor_sync(0xffffffffu, cxlo, o));
+        cxhi = fmaxf(cxhi, __shfl_xor_sync(0xffffffffu, cxhi, o));
+        cylo = fminf(cylo, __shfl_xor_sync(0xffffffffu, cylo, o));
+        cyhi = fmaxf(cyhi, __shfl_xor_sync(0xffffffffu, cyhi, o));
+        emax = fmaxf(emax, __shfl_xor_sync(0xffffffffu, emax, o));
+    }
+    const float thr = fmaxf(smax, sq_threshold(emax + b.a2f));
+    // box gaps: differences of biased floats are exact integers
+    const float gx = fmaxf(0.f, fmaxf(cxlo - xhi, xlo - cxhi));
+    const float gy = fmaxf(0.f, fmaxf(cylo - yhi, ylo - cyhi));
+    const float d2 = fmaf(gx, gx, gy * gy);
+    return d2 * 0.99999904632568359375f <= thr;  // (1 - 2^-20)
+}
+
 // Shared memory bytes of a tile with TJ columns and TI rows.
 __host__ __device__ inline size_t tile_smem_bytes(int TJ, int TI)
 {
@@ -250,7 +306,7 @@ constexpr int kMaxWarpsPerTile = 4;
 
 template <int R, bool PS>
 __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n, int2 tile, int TJ, Slot* slot,
-                                           const TileSmem& sm, unsigned long long* tilebest, int use_seed)
+                                           const TileSmem& sm, unsigned long long* tilebest, int flags)
 {
     const int I0 = tile.x, J0 = tile.y;
     const int J1 = min(J0 + TJ, n);  // columns j in [J0, J1), j <= n-1
@@ -286,7 +342,7 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     // it intact, is such a real pair too: it tightens the start bound and is
     // published for the other tiles.
     unsigned long long g = *(volatile unsigned long long*)&slot->key;
-    if (use_seed && *(volatile int*)&slot->seed_ok) {
+    if ((flags & kSweepSeed) && *(volatile int*)&slot->seed_ok) {
         const unsigned long long mv = *(volatile unsigned long long*)&slot->last_key;
         const unsigned long long k = surviving_key(*(volatile unsigned long long*)tilebest, key_i(mv), key_j(mv));
         if (k < g) {
@@ -306,8 +362,10 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
         Bound<R> b;
         set_bound<R>(b, erow, dg == 0 ? 0 : dg + 1);
         const bool masked = (wrow0 + 32 * R - 1) >= jstart;  // warp-uniform: some row >= some j
-        if (masked) walk<R, true, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
-        else walk<R, false, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
+        if (!(flags & kSweepTileBounds) || tile_may_pass<R>(rows, b, sm, jstart - J0, J1 - J0)) {
+            if (masked) walk<R, true, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
+            else walk<R, false, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
+        }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
             const unsigned long long other = __shfl_xor_sync(0xffffffffu, mykey, o);

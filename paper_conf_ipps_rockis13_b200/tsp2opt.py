@@ -58,6 +58,7 @@ def _L():
             "tsp2opt_local_search": ([P, P, I64, pI64, pI64], I32),
             "tsp2opt_get_tour": ([P, P, pI64], I32),
             "tsp2opt_debug_set_shard": ([P, I32, I32], I32),
+            "tsp2opt_set_option": ([P, I32, I64], I32),
             "tsp2opt_plan_shard": ([I32, I32, I32, pI32, pI32, pI32, P, I64, pI64, pI64], I32),
             "tsp2opt_get_geometry": ([P, pI32, pI32, pI32, pI64, pI64], I32),
             "tsp2opt_selftest": ([pI64, pI64, pI64, pI64], I32),
@@ -182,6 +183,13 @@ def get_tour(h, n: int):
     return t, L.value
 
 
+OPT_TILE_BOUNDS, OPT_SEED, OPT_PERSISTENT = 1, 2, 3
+
+
+def set_option(h, option: int, value: int) -> None:
+    _check(_L().tsp2opt_set_option(h, int(option), int(value)), "tsp2opt_set_option")
+
+
 def debug_set_shard(h, rank: int, world: int) -> None:
     _check(_L().tsp2opt_debug_set_shard(h, rank, world), "tsp2opt_debug_set_shard")
 
@@ -289,6 +297,9 @@ class TSP2Opt:
 
     def get_tour(self):
         return get_tour(self.h, self.n)
+
+    def set_option(self, option: int, value: int):
+        set_option(self.h, option, value)
 
     def debug_set_shard(self, rank, world):
         debug_set_shard(self.h, rank, world)

@@ -10,8 +10,12 @@ from paper_conf_ipps_rockis13_b200 import inputs, tsp2opt
 pytestmark = pytest.mark.gpu
 
 
+@pytest.mark.parametrize("bounds", ["0", "1"])
 @pytest.mark.parametrize("cfg", ["C3", "C4", "C5"])
-def test_full_size_first_sweep(gpu, cfg):
+def test_full_size_first_sweep(gpu, monkeypatch, cfg, bounds):
+    """bounds = 0 is the launch configuration bench.py times for `value` (every
+    pair tested individually); 1 is the library default (tile-level bounds)."""
+    monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", bounds)
     c, t = inputs.config_instance(cfg)
     with tsp2opt.TSP2Opt(c) as g:
         assert g.best_move(t) == oracle.best_move(c, t)

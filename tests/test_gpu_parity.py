@@ -50,11 +50,13 @@ def test_best_move_parity_sizes(gpu, n, kind):
         assert g.best_move(th) == oracle.best_move(c, th)
 
 
+@pytest.mark.parametrize("bounds", ["0", "1"])
 @pytest.mark.parametrize("rows", [7, 15])
 @pytest.mark.parametrize("warps,tj", [(1, 2), (1, 3), (1, 32), (2, 64), (4, 128), (4, 1024), (3, 7)])
-def test_best_move_parity_geometries(gpu, monkeypatch, rows, warps, tj):
+def test_best_move_parity_geometries(gpu, monkeypatch, rows, warps, tj, bounds):
     # tiny and odd tiles exercise masked diagonal tiles and ragged column tails,
-    # for both instantiated row counts R
+    # for both instantiated row counts R, with and without tile-level bounds
+    monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", bounds)
     monkeypatch.setenv("TSP2OPT_ROWS", str(rows))
     monkeypatch.setenv("TSP2OPT_WARPS", str(warps))
     monkeypatch.setenv("TSP2OPT_TJ", str(tj))
@@ -90,6 +92,7 @@ def test_local_search_parity(gpu, kind, n, seed):
     c, t = _inst(kind, n, seed)
     ref = oracle.local_search(c, t)
     with tsp2opt.TSP2Opt(c) as g:
+        g.set_option(tsp2opt.OPT_TILE_BOUNDS, seed % 2)  # both filter forms over the seeds
         res = g.local_search(t)
         assert res["status"] == tsp2opt.OK
         assert res["iterations"] == ref["iterations"]
