@@ -371,7 +371,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C5")
     ap.add_argument("--tour", default="random", choices=["random", "hilbert"])
-    ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert", help="configs timed to a local minimum (rank 0, N=1)")
+    ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert,C5:hilbert", help="configs timed to a local minimum (rank 0, N=1)")
     ap.add_argument("--no-ls", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)

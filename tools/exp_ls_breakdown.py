@@ -9,9 +9,9 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 os.environ.setdefault("TSP2OPT_PERSISTENT", "0")
 from paper_conf_ipps_rockis13_b200 import inputs, tsp2opt  # noqa: E402
 
-for seed in ("1", "0"):
+for seed in ("0",):
     os.environ["TSP2OPT_SEED"] = seed
-    for cfg, tk in (("C2", "random"), ("C3", "random"), ("C4", "hilbert")):
+    for cfg, tk in (("C2", "random"), ("C3", "random"), ("C4", "hilbert"), ("C5", "hilbert")):
         c, t = inputs.config_instance(cfg, tk)
         with tsp2opt.TSP2Opt(c) as g:
             g.local_search(t, max_iters=2)
