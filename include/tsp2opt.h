@@ -136,11 +136,19 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
  *  TSP2OPT_OPT_PERSISTENT (default 2): local_search loop, 0 = one sweep and one
  *      apply kernel per iteration, 1 = one persistent cooperative launch,
  *      2 = choose by size (world == 1 only).
+ *  TSP2OPT_OPT_TRACE (default 0): record the (i, j, delta) of the first `value`
+ *      moves applied by iterate_async / local_search since the tour was loaded
+ *      (read with tsp2opt_get_trace); 0 frees the buffer.
  * Returns TSP2OPT_EINVAL for an unknown option or value. */
 #define TSP2OPT_OPT_TILE_BOUNDS 1
 #define TSP2OPT_OPT_SEED 2
 #define TSP2OPT_OPT_PERSISTENT 3
+#define TSP2OPT_OPT_TRACE 4
 int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value);
+
+/* Recorded move trace: writes min(count, cap) rows of int32 (i, j, delta) into
+ * ijd (int32[3*cap]); *count = moves recorded (<= the trace capacity). */
+int tsp2opt_get_trace(tsp2opt_t h, int32_t *ijd, int64_t cap, int64_t *count);
 
 /* Diagnostics / test hooks ------------------------------------------------ */
 

@@ -70,6 +70,8 @@ struct tsp2opt_ctx {
     bool seed_next = false;     // seed each tile with its surviving minimum of the previous sweep (TSP2OPT_SEED=1;
                                 // measured neutral-to-slower at n = 1002 .. 33810, so off by default)
     bool tile_bounds = true;    // tile-level bounding-box form of the filter (TSP2OPT_OPT_TILE_BOUNDS)
+    unsigned long long* d_trace = nullptr;  // [trace_cap] keys of the applied moves (TSP2OPT_OPT_TRACE)
+    long long trace_cap = 0;
     Slot* h_slot = nullptr;     // pinned readback
     unsigned epoch = 0;
     int parity = 0;             // iteration t reads slot[parity]
@@ -96,7 +98,14 @@ Geometry choose_geometry(long long pairs_per_rank)
     // n = 7397: TJ = 16; n = 1002: TJ = 8).
     const long long p = pairs_per_rank;
     int R = p >= 100000000LL ? kRowsLarge : kRowsSmall;
-    int tj = p >= 1000000000LL ? 128 : p >= 100000000LL ? 64 : p >= 5000000LL ? 16 : 8;
+    // (beyond the measured range the tile count is capped near 1e6-1e7 so the
+    // host-side tile table stays small: n = 2^22 -> 18M tiles of 480 x 1024)
+    int tj = p >= 100000000000LL ? 1024
+             : p >= 10000000000LL ? 512
+             : p >= 1000000000LL  ? 128
+             : p >= 100000000LL   ? 64
+             : p >= 5000000LL     ? 16
+                                  : 8;
     int w = 1;
     if (const char* er = getenv("TSP2OPT_ROWS")) R = atoi(er) == kRowsSmall ? kRowsSmall : kRowsLarge;
     const char* ew = getenv("TSP2OPT_WARPS");
@@ -119,8 +128,11 @@ std::vector<Tile> build_tiles(int n, const Geometry& g)
         const int rows = std::min(I0 + TI, n - 1) - I0;
         for (int J0 = ((I0 + 1) / TJ) * TJ; J0 < n; J0 += TJ) {
             const int J1 = std::min(J0 + TJ, n);
-            long long p = 0;
-            for (int j = J0; j < J1; j++) p += std::max(0, std::min(j - I0, rows));
+            // sum over j in [J0, J1) of min(max(j - I0, 0), rows), in closed form
+            auto tri = [](long long m) { return m > 0 ? m * (m + 1) / 2 : 0; };  // 1 + 2 + ... + m
+            const long long a = std::max<long long>(J0, I0), b = std::min<long long>(J1, (long long)I0 + rows);
+            long long p = a < b ? tri(b - 1 - I0) - tri(a - 1 - I0) : 0;      // ramp part j - I0
+            p += (long long)rows * std::max<long long>(0, J1 - std::max<long long>(J0, (long long)I0 + rows));
             if (p > 0) t.push_back({I0, J0, p});
         }
     }
@@ -182,6 +194,7 @@ void free_ctx(tsp2opt_ctx* h)
     if (h->h_ctl) cudaFreeHost(h->h_ctl);
     cudaFree(h->d_tiles);
     cudaFree(h->d_tilebest);
+    cudaFree(h->d_trace);
     if (h->h_slot) cudaFreeHost(h->h_slot);
     for (cudaEvent_t e : h->ev_pool) cudaEventDestroy(e);
     if (h->own_stream) cudaStreamDestroy(h->own_stream);
@@ -271,7 +284,8 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
     }
     if (apply) {
         Slot* out = h->d_slots + (h->parity ^ 1);
-        CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, max_moves, 0, 0, 0, h->stream));
+        CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, max_moves, 0, 0, 0, h->d_trace,
+                              h->trace_cap, h->stream));
         h->parity ^= 1;
     }
     return TSP2OPT_OK;
@@ -427,7 +441,7 @@ int tsp2opt_apply(tsp2opt_t h, int32_t i, int32_t j)
     if (!h->has_tour) return TSP2OPT_ESTATE;
     Slot* in = h->d_slots + h->parity;
     Slot* out = h->d_slots + (h->parity ^ 1);
-    CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, 0, 1, i, j, h->stream));
+    CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, 0, 1, i, j, nullptr, 0, h->stream));
     h->parity ^= 1;
     return read_slot(h);
 }
@@ -484,7 +498,7 @@ int tsp2opt_local_search(tsp2opt_t h, int32_t* tour, int64_t max_iters, int64_t*
             }
             CUDA_TRY(launch_local_search(h->geo, h->d_P, h->d_E, h->d_tour, h->n, h->d_tiles, h->ntiles, h->d_slots,
                                          h->parity, max_iters, budget, h->d_bar, h->d_ctl, h->d_tilebest,
-                                         sweep_flags(h), h->stream));
+                                         sweep_flags(h), h->d_trace, h->trace_cap, h->stream));
             CUDA_TRY(cudaMemcpyAsync(h->h_ctl, h->d_ctl, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
             CUDA_TRY(cudaStreamSynchronize(h->stream));
             h->parity = *h->h_ctl;
@@ -537,11 +551,44 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
     switch (option) {
     case TSP2OPT_OPT_TILE_BOUNDS: h->tile_bounds = value != 0; break;
     case TSP2OPT_OPT_SEED: h->seed_next = value != 0; break;
+    case TSP2OPT_OPT_TRACE: {
+        if (value < 0) return TSP2OPT_EINVAL;
+        CUDA_TRY(cudaStreamSynchronize(h->stream));
+        cudaFree(h->d_trace);
+        h->d_trace = nullptr;
+        h->trace_cap = 0;
+        if (value > 0) {
+            CUDA_TRY(cudaMalloc(&h->d_trace, sizeof(unsigned long long) * (size_t)value));
+            h->trace_cap = value;
+        }
+        break;
+    }
     case TSP2OPT_OPT_PERSISTENT:
         if (value < 0 || value > 2) return TSP2OPT_EINVAL;
         h->persistent = (int)value;
         break;
     default: return TSP2OPT_EINVAL;
+    }
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_get_trace(tsp2opt_t h, int32_t* ijd, int64_t cap, int64_t* count)
+{
+    if (!h || !count || (cap > 0 && !ijd)) return TSP2OPT_EINVAL;
+    if (!h->has_tour) return TSP2OPT_ESTATE;
+    int rc = read_slot(h);
+    if (rc) return rc;
+    const long long k = std::min<long long>(h->h_slot->moves, h->trace_cap);
+    *count = k;
+    const long long m = std::min<long long>(k, cap);
+    if (m > 0) {
+        std::vector<unsigned long long> keys((size_t)m);
+        CUDA_TRY(cudaMemcpy(keys.data(), h->d_trace, sizeof(unsigned long long) * (size_t)m, cudaMemcpyDeviceToHost));
+        for (long long t = 0; t < m; t++) {
+            ijd[3 * t] = key_i(keys[t]);
+            ijd[3 * t + 1] = key_j(keys[t]);
+            ijd[3 * t + 2] = key_delta(keys[t]);
+        }
     }
     return TSP2OPT_OK;
 }

@@ -33,10 +33,12 @@ cudaError_t launch_reset_key(Slot* slot, cudaStream_t st);
 cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
                          Slot* slot, int respect_done, unsigned long long* tilebest, int flags, cudaStream_t st);
 cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Slot* out, long long max_moves,
-                         int explicit_move, int ei, int ej, cudaStream_t st);
+                         int explicit_move, int ei, int ej, unsigned long long* trace, long long trace_cap,
+                         cudaStream_t st);
 cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
                                 Slot* slots, int parity, long long max_moves, long long budget, unsigned* bar,
-                                int* ctl, unsigned long long* tilebest, int flags, cudaStream_t st);
+                                int* ctl, unsigned long long* tilebest, int flags, unsigned long long* trace,
+                                long long trace_cap, cudaStream_t st);
 cudaError_t read_stats(long long* out4, int reset);
 cudaError_t run_selftest_sqrt(double* max_rel, int* zero_ok);
 cudaError_t run_selftest(long long* out4);  // dist_bad, filter_bad, first bad s, first bad dx<<15|dy

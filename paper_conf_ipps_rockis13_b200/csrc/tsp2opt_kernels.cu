@@ -102,7 +102,8 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* 
 // Returns whether a move was applied (false: converged / capped / already done).
 __device__ __forceinline__ bool apply_phase(float2* __restrict__ P, int* __restrict__ E, int* __restrict__ tour,
                                             const Slot* __restrict__ in, Slot* __restrict__ out, long long max_moves,
-                                            int explicit_move, int ei, int ej, int gtid, int stride)
+                                            int explicit_move, int ei, int ej, int gtid, int stride,
+                                            unsigned long long* __restrict__ trace, long long trace_cap)
 {
     const unsigned long long key = in->key;
     const int done = in->done;
@@ -138,6 +139,7 @@ __device__ __forceinline__ bool apply_phase(float2* __restrict__ P, int* __restr
             o.moves = moves + 1;
             E[i] = ni;
             E[j] = nj;
+            if (trace && !explicit_move && moves < trace_cap) trace[moves] = key;  // move trace (tests)
         }
         *out = o;
     }
@@ -164,13 +166,14 @@ __device__ __forceinline__ bool apply_phase(float2* __restrict__ P, int* __restr
 
 __global__ void __launch_bounds__(256) apply_kernel(float2* __restrict__ P, int* __restrict__ E, int* __restrict__ tour,
                                                     const Slot* __restrict__ in, Slot* __restrict__ out,
-                                                    long long max_moves, int explicit_move, int ei, int ej)
+                                                    long long max_moves, int explicit_move, int ei, int ej,
+                                                    unsigned long long* __restrict__ trace, long long trace_cap)
 {
     __shared__ Slot s_in;  // one read of the input state per block
     if (threadIdx.x == 0) s_in = *in;
     __syncthreads();
     apply_phase(P, E, tour, &s_in, out, max_moves, explicit_move, ei, ej, blockIdx.x * blockDim.x + threadIdx.x,
-                gridDim.x * blockDim.x);
+                gridDim.x * blockDim.x, trace, trace_cap);
 }
 
 // ===========================================================================
@@ -206,7 +209,8 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
                                                            Slot* __restrict__ slots, int parity, long long max_moves,
                                                            long long budget, unsigned* __restrict__ bar,
                                                            int* __restrict__ ctl,
-                                                           unsigned long long* __restrict__ tilebest, int flags)
+                                                           unsigned long long* __restrict__ tilebest, int flags,
+                                                           unsigned long long* __restrict__ trace, long long trace_cap)
 {
     extern __shared__ float4 smem[];
     const TileSmem sm(smem, TJ);
@@ -235,7 +239,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
             s_in.seed_ok = *(volatile int*)&in->seed_ok;
         }
         __syncthreads();
-        apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride);
+        apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride, trace, trace_cap);
         p ^= 1;
         grid_sync(bar, gridDim.x);
     }
@@ -373,12 +377,14 @@ cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n
 }
 
 cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Slot* out, long long max_moves,
-                         int explicit_move, int ei, int ej, cudaStream_t st)
+                         int explicit_move, int ei, int ej, unsigned long long* trace, long long trace_cap,
+                         cudaStream_t st)
 {
     int blocks = (n / 2 + 255) / 256;
     if (blocks < 1) blocks = 1;
     if (blocks > 4 * 148) blocks = 4 * 148;
-    apply_kernel<<<blocks, 256, 0, st>>>(P, E, tour, in, out, max_moves, explicit_move, ei, ej);
+    apply_kernel<<<blocks, 256, 0, st>>>(P, E, tour, in, out, max_moves, explicit_move, ei, ej, trace,
+                                         trace_cap);
     g_launches += 1;
     return cudaGetLastError();
 }
@@ -400,13 +406,14 @@ int local_search_grid(const Geometry& g, int ntiles)
 
 cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
                                 Slot* slots, int parity, long long max_moves, long long budget, unsigned* bar,
-                                int* ctl, unsigned long long* tilebest, int flags, cudaStream_t st)
+                                int* ctl, unsigned long long* tilebest, int flags, unsigned long long* trace,
+                                long long trace_cap, cudaStream_t st)
 {
     int grid = local_search_grid(g, ntiles);
     if (grid < 1) return cudaErrorInvalidConfiguration;
     int TJ = g.tj;
     void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &TJ, &slots, &parity, &max_moves, &budget, &bar, &ctl,
-                    &tilebest, &flags};
+                    &tilebest, &flags, &trace, &trace_cap};
     g_launches += 1;
     return by_rows(g.rows, [&](auto r) {
         return cudaLaunchCooperativeKernel((const void*)local_search_kernel<decltype(r)::value>, dim3(grid),

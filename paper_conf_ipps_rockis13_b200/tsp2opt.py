@@ -59,6 +59,7 @@ def _L():
             "tsp2opt_get_tour": ([P, P, pI64], I32),
             "tsp2opt_debug_set_shard": ([P, I32, I32], I32),
             "tsp2opt_set_option": ([P, I32, I64], I32),
+            "tsp2opt_get_trace": ([P, P, I64, pI64], I32),
             "tsp2opt_plan_shard": ([I32, I32, I32, pI32, pI32, pI32, P, I64, pI64, pI64], I32),
             "tsp2opt_get_geometry": ([P, pI32, pI32, pI32, pI64, pI64], I32),
             "tsp2opt_selftest": ([pI64, pI64, pI64, pI64], I32),
@@ -183,11 +184,19 @@ def get_tour(h, n: int):
     return t, L.value
 
 
-OPT_TILE_BOUNDS, OPT_SEED, OPT_PERSISTENT = 1, 2, 3
+OPT_TILE_BOUNDS, OPT_SEED, OPT_PERSISTENT, OPT_TRACE = 1, 2, 3, 4
 
 
 def set_option(h, option: int, value: int) -> None:
     _check(_L().tsp2opt_set_option(h, int(option), int(value)), "tsp2opt_set_option")
+
+
+def get_trace(h, cap: int) -> np.ndarray:
+    """int32[count, 3] (i, j, delta) of the recorded moves (set_option(OPT_TRACE, cap) first)."""
+    out = np.zeros((max(cap, 1), 3), dtype=np.int32)
+    cnt = ctypes.c_int64()
+    _check(_L().tsp2opt_get_trace(h, _ptr(out), int(cap), ctypes.byref(cnt)), "tsp2opt_get_trace")
+    return out[: min(cnt.value, cap)].copy()
 
 
 def debug_set_shard(h, rank: int, world: int) -> None:
@@ -300,6 +309,9 @@ class TSP2Opt:
 
     def set_option(self, option: int, value: int):
         set_option(self.h, option, value)
+
+    def get_trace(self, cap: int):
+        return get_trace(self.h, cap)
 
     def debug_set_shard(self, rank, world):
         debug_set_shard(self.h, rank, world)

@@ -44,3 +44,31 @@ def test_C5_hilbert_start_sweep(gpu):
     th = inputs.hilbert_tour(c)
     with tsp2opt.TSP2Opt(c) as g:
         assert g.best_move(th) == oracle.best_move(c, th)
+
+
+@pytest.mark.parametrize("cfg,tk,nsamples", [("C3", "hilbert", 6), ("C4", "hilbert", 5), ("C5", "hilbert", 3)])
+def test_full_size_local_search_trace(gpu, cfg, tk, nsamples):
+    """Full local search at BASELINE.json sizes, in the default launch
+    configuration: the recorded move trace replayed on the CPU reproduces the
+    final tour and length; sampled iterations (first, last, evenly spaced) are
+    re-swept by the oracle from the replayed tour and must give the traced
+    move; the final tour carries the oracle's local-minimum certificate."""
+    c, t = inputs.config_instance(cfg, tk)
+    cap = 10 * len(t)
+    with tsp2opt.TSP2Opt(c) as g:
+        g.set_option(tsp2opt.OPT_TRACE, cap)
+        res = g.local_search(t)
+        trace = g.get_trace(cap)
+    k = res["iterations"]
+    assert res["status"] == tsp2opt.OK and len(trace) == k > 0
+    picks = set(np.linspace(0, k - 1, nsamples).astype(int).tolist())
+    tour = t.copy()
+    L = oracle.tour_length(c, tour)
+    for idx, (i, j, d) in enumerate(trace):
+        if idx in picks:
+            assert oracle.best_move(c, tour) == (int(i), int(j), int(d)), idx
+        assert d < 0
+        tour = oracle.apply(tour, int(i), int(j))
+        L += int(d)
+    assert np.array_equal(tour, res["tour"]) and L == res["length"] == oracle.tour_length(c, tour)
+    assert oracle.best_move(c, res["tour"]) == (0, 1, 0)  # local-minimum certificate
