@@ -63,6 +63,12 @@ def _load():
             lib.oracle_apply.restype = None
             lib.oracle_local_search.argtypes = [p, i64, p, i64, p, p, p, i64]
             lib.oracle_local_search.restype = ctypes.c_int
+            lib.oracle_double_bridge_cuts.argtypes = [i64, ctypes.c_uint64, i64, p, p, p]
+            lib.oracle_double_bridge_cuts.restype = None
+            lib.oracle_double_bridge.argtypes = [p, i64, i64, i64, i64, p]
+            lib.oracle_double_bridge.restype = None
+            lib.oracle_ils.argtypes = [p, i64, p, i64, ctypes.c_uint64, p, p]
+            lib.oracle_ils.restype = None
             lib.oracle_num_threads.argtypes = []
             lib.oracle_num_threads.restype = ctypes.c_int
             _lib = lib
@@ -154,6 +160,33 @@ def local_search(coords, tour, max_iters: int = -1, trace_cap: int = 0):
     it = int(out[1])
     return dict(tour=t, length=int(out[0]), iterations=it, status=int(st),
                 trace=tr[: min(it, trace_cap)].copy())
+
+
+def double_bridge_cuts(n: int, seed: int, it: int):
+    """(a, b, c) cut positions of ILS step `it` (reading R16)."""
+    out = np.zeros(3, dtype=np.int64)
+    _load().oracle_double_bridge_cuts(n, ctypes.c_uint64(seed & 0xFFFFFFFFFFFFFFFF), it,
+                                      _ptr(out[0:1]), _ptr(out[1:2]), _ptr(out[2:3]))
+    return int(out[0]), int(out[1]), int(out[2])
+
+
+def double_bridge(tour, a: int, b: int, c: int) -> np.ndarray:
+    t = np.ascontiguousarray(tour, dtype=np.int32)
+    out = np.empty_like(t)
+    _load().oracle_double_bridge(_ptr(t), t.size, a, b, c, _ptr(out))
+    return out
+
+
+def ils(coords, tour, iterations: int, seed: int):
+    """Iterated Local Search (L10 Algorithm 1; readings R14-R16).
+    Returns dict(tour, length, lengths) -- lengths[t] = best length after t steps."""
+    xy = _xy(coords)
+    t = np.array(tour, dtype=np.int32, copy=True)
+    out = np.zeros(1, dtype=np.int64)
+    lengths = np.zeros(iterations + 1, dtype=np.int64)
+    _load().oracle_ils(_ptr(xy), xy.shape[0], _ptr(t), int(iterations), ctypes.c_uint64(seed & 0xFFFFFFFFFFFFFFFF),
+                       _ptr(out), _ptr(lengths))
+    return dict(tour=t, length=int(out[0]), lengths=lengths)
 
 
 def num_threads() -> int:

@@ -218,6 +218,77 @@ int oracle_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64_t max
     return status;
 }
 
+/* ---------------------------------------------------------------------------
+ * Iterated Local Search (L10 Algorithm 1: s0 = GenerateInitialSolution();
+ * s* = 2optLocalSearch(s0); while not terminated: s' = Perturbation(s*);
+ * s*' = 2optLocalSearch(s'); s* = AcceptanceCriterion(s*, s*')), with the
+ * paper's choices (L18 §V): a random initial tour (the caller's), "a simple
+ * doublebridge move as a perturbation technique".  Readings (DESIGN.md §3,
+ * R14-R16): termination = a fixed number of iterations; acceptance = keep the
+ * new local minimum iff it is strictly shorter; the double bridge of the
+ * current tour t = A B C D (cut positions 1 <= a < b < c <= n-1, tour[0] in A)
+ * is A C B D, with segment lengths drawn from the counter-based splitmix64
+ * stream of `seed` (draw k of iteration it is output 3*it + k):
+ *   len_k = 1 + out % max(1, (n - 1) / 3),  a = len_0, b = a + len_1, c = b + len_2.
+ * ------------------------------------------------------------------------- */
+static uint64_t oracle_splitmix64_at(uint64_t seed, uint64_t k)
+{
+    /* output k (0-based) of splitmix64 seeded with `seed` (Steele, Lea, Flood) */
+    uint64_t z = seed + (k + 1) * 0x9E3779B97F4A7C15ULL;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+    return z ^ (z >> 31);
+}
+
+void oracle_double_bridge_cuts(int64_t n, uint64_t seed, int64_t it, int64_t *a, int64_t *b, int64_t *c)
+{
+    int64_t m = (n - 1) / 3;
+    if (m < 1) m = 1;
+    int64_t l0 = 1 + (int64_t)(oracle_splitmix64_at(seed, 3 * (uint64_t)it) % (uint64_t)m);
+    int64_t l1 = 1 + (int64_t)(oracle_splitmix64_at(seed, 3 * (uint64_t)it + 1) % (uint64_t)m);
+    int64_t l2 = 1 + (int64_t)(oracle_splitmix64_at(seed, 3 * (uint64_t)it + 2) % (uint64_t)m);
+    *a = l0;
+    *b = l0 + l1;
+    *c = l0 + l1 + l2;
+}
+
+/* out = A C B D for tour = A B C D with A = [0, a), B = [a, b), C = [b, c), D = [c, n) */
+void oracle_double_bridge(const int32_t *tour, int64_t n, int64_t a, int64_t b, int64_t c, int32_t *out)
+{
+    int64_t k = 0;
+    for (int64_t p = 0; p < a; p++) out[k++] = tour[p];
+    for (int64_t p = b; p < c; p++) out[k++] = tour[p];
+    for (int64_t p = a; p < b; p++) out[k++] = tour[p];
+    for (int64_t p = c; p < n; p++) out[k++] = tour[p];
+}
+
+/* Runs `iterations` ILS steps from `tour` (in: start tour; out: best tour).
+ * lengths (may be NULL) receives the current best length after each step
+ * (lengths[0] = the first local minimum, lengths[t+1] after step t). */
+void oracle_ils(const int32_t *xy, int64_t n, int32_t *tour, int64_t iterations, uint64_t seed,
+                int64_t *length, int64_t *lengths)
+{
+    int64_t L, it;
+    oracle_local_search(xy, n, tour, -1, &L, &it, NULL, 0);
+    if (lengths) lengths[0] = L;
+    int32_t *cand = (int32_t *)malloc(sizeof(int32_t) * n);
+    for (int64_t t = 0; t < iterations; t++) {
+        if (n >= 8) {
+            int64_t a, b, c, L2, it2;
+            oracle_double_bridge_cuts(n, seed, t, &a, &b, &c);
+            oracle_double_bridge(tour, n, a, b, c, cand);
+            oracle_local_search(xy, n, cand, -1, &L2, &it2, NULL, 0);
+            if (L2 < L) {
+                memcpy(tour, cand, sizeof(int32_t) * n);
+                L = L2;
+            }
+        }
+        if (lengths) lengths[t + 1] = L;
+    }
+    free(cand);
+    *length = L;
+}
+
 int oracle_num_threads(void)
 {
 #ifdef _OPENMP
