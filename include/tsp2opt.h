@@ -123,6 +123,19 @@ int tsp2opt_sync(tsp2opt_t h, int64_t *iterations, int64_t *length, int32_t *con
 int tsp2opt_local_search(tsp2opt_t h, int32_t *tour, int64_t max_iters, int64_t *length,
                          int64_t *iterations);
 
+/* Iterated Local Search (L10 Algorithm 1; L18 §V: random start tour, "a simple
+ * doublebridge move as a perturbation technique"), device-resident:
+ *   s* = local_search(tour); repeat `iterations` times:
+ *     s' = double_bridge(s*, cuts(seed, t)); s*' = local_search(s');
+ *     s* = s*' if length(s*') < length(s*)                  (readings R14-R16)
+ * cuts: splitmix64 output 3t+k of `seed` gives segment length
+ * l_k = 1 + out % max(1, (n-1)/3); a = l0, b = a + l1, c = b + l2; s' = A C B D
+ * for s* = A B C D cut at a < b < c (no perturbation when n < 8).
+ * tour: host int32[n], in = start tour, out = best tour; *length its length;
+ * lengths (NULL or int64[iterations+1]) = best length after each step. */
+int tsp2opt_ils(tsp2opt_t h, int32_t *tour, int64_t iterations, uint64_t seed, int64_t *length,
+                int64_t *lengths);
+
 /* Copy the current tour (host int32[n]) and its length out. */
 int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
 

@@ -71,6 +71,7 @@ struct tsp2opt_ctx {
                                 // measured neutral-to-slower at n = 1002 .. 33810, so off by default)
     bool tile_bounds = true;    // tile-level bounding-box form of the filter (TSP2OPT_OPT_TILE_BOUNDS)
     unsigned long long* d_trace = nullptr;  // [trace_cap] keys of the applied moves (TSP2OPT_OPT_TRACE)
+    int* d_best = nullptr;      // [n] best tour of an ILS run
     long long trace_cap = 0;
     Slot* h_slot = nullptr;     // pinned readback
     unsigned epoch = 0;
@@ -195,6 +196,7 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_tiles);
     cudaFree(h->d_tilebest);
     cudaFree(h->d_trace);
+    cudaFree(h->d_best);
     if (h->h_slot) cudaFreeHost(h->h_slot);
     for (cudaEvent_t e : h->ev_pool) cudaEventDestroy(e);
     if (h->own_stream) cudaStreamDestroy(h->own_stream);
@@ -289,6 +291,80 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         h->parity ^= 1;
     }
     return TSP2OPT_OK;
+}
+
+// Device-resident best-improvement loop on the loaded tour (a4-a8) until the
+// local minimum or max_iters moves; leaves the final state in h->h_slot.
+// Returns TSP2OPT_OK / TSP2OPT_MAXITER or a negative error.
+int run_local_search(tsp2opt_ctx* h, long long max_iters)
+{
+    int rc;
+    // Persistent single launch pays off while the per-iteration launch/sync
+    // overhead dominates the sweep (measured: faster up to n ~ 1e3, slower from
+    // n ~ 7e3 where the per-sweep kernels pack tiles better); TSP2OPT_PERSISTENT
+    // = 0 / 1 forces either loop, 2 (default) chooses by pair count.
+    const bool use_persistent =
+        !h->comm && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
+    if (use_persistent) {
+        // One persistent cooperative launch runs sweep -> apply to the local
+        // minimum; the per-launch iteration budget bounds a launch to roughly
+        // 2e12 pair checks (~0.5 s), after which the host relaunches.
+        const long long pairs = std::max(1LL, h->shard_pairs);
+        const long long budget = std::min(1LL << 20, std::max(16LL, 2000000000000LL / pairs));
+        for (long long launches = 0;; launches++) {
+            if (launches * budget > 1000LL * h->n + (1LL << 24)) {  // cannot happen: delta < 0 shortens the tour
+                g_last_error = "local search did not converge";
+                return TSP2OPT_ECUDA;
+            }
+            CUDA_TRY(launch_local_search(h->geo, h->d_P, h->d_E, h->d_tour, h->n, h->d_tiles, h->ntiles, h->d_slots,
+                                         h->parity, max_iters, budget, h->d_bar, h->d_ctl, h->d_tilebest,
+                                         sweep_flags(h), h->d_trace, h->trace_cap, h->stream));
+            CUDA_TRY(cudaMemcpyAsync(h->h_ctl, h->d_ctl, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+            CUDA_TRY(cudaStreamSynchronize(h->stream));
+            h->parity = *h->h_ctl;
+            rc = read_slot(h);
+            if (rc) return rc;
+            if (h->h_slot->done & 3) break;
+        }
+    } else {
+        // Multi-kernel loop (and sharded handles): batches of K iterations
+        // between host checks; an iteration after convergence is a no-op
+        // (sweep CTAs exit on the done flag).
+        long long k = 4;
+        for (;;) {
+            for (long long c = 0; c < k; c++) {
+                rc = enqueue_iteration(h, max_iters, true);
+                if (rc) return rc;
+            }
+            rc = read_slot(h);
+            if (rc) return rc;
+            if (h->h_slot->done & 3) break;
+            if (k < 64) k *= 2;
+        }
+    }
+    return (h->h_slot->done & 3) == 2 ? TSP2OPT_MAXITER : TSP2OPT_OK;
+}
+
+// ILS perturbation cuts (reading R16): splitmix64 output 3*it + k of `seed`
+// gives the k-th segment length 1 + out % max(1, (n-1)/3); a = l0, b = a + l1,
+// c = b + l2 (1 <= a < b < c <= n-1).
+uint64_t splitmix64_at(uint64_t seed, uint64_t k)
+{
+    uint64_t z = seed + (k + 1) * 0x9E3779B97F4A7C15ULL;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+    return z ^ (z >> 31);
+}
+
+void ils_cuts(long long n, uint64_t seed, long long it, long long* a, long long* b, long long* c)
+{
+    const unsigned long long m = (unsigned long long)std::max(1LL, (n - 1) / 3);
+    const long long l0 = 1 + (long long)(splitmix64_at(seed, 3ULL * it) % m);
+    const long long l1 = 1 + (long long)(splitmix64_at(seed, 3ULL * it + 1) % m);
+    const long long l2 = 1 + (long long)(splitmix64_at(seed, 3ULL * it + 2) % m);
+    *a = l0;
+    *b = l0 + l1;
+    *c = l0 + l1 + l2;
 }
 
 int create_common(const int32_t* xy, int32_t n, int rank, int world, const void* nccl_id, tsp2opt_t* out)
@@ -479,58 +555,56 @@ int tsp2opt_local_search(tsp2opt_t h, int32_t* tour, int64_t max_iters, int64_t*
     if (!h || !tour || !length || !iterations || max_iters < 0) return TSP2OPT_EINVAL;
     int rc = load_host_tour(h, tour);
     if (rc) return rc;
-    // Persistent single launch pays off while the per-iteration launch/sync
-    // overhead dominates the sweep (measured: faster up to n ~ 1e3, slower from
-    // n ~ 7e3 where the per-sweep kernels pack tiles better); TSP2OPT_PERSISTENT
-    // = 0 / 1 forces either loop, 2 (default) chooses by pair count.
-    const bool use_persistent =
-        !h->comm && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
-    if (use_persistent) {
-        // One persistent cooperative launch runs sweep -> apply to the local
-        // minimum; the per-launch iteration budget bounds a launch to roughly
-        // 2e12 pair checks (~0.5 s), after which the host relaunches.
-        const long long pairs = std::max(1LL, h->shard_pairs);
-        const long long budget = std::min(1LL << 20, std::max(16LL, 2000000000000LL / pairs));
-        for (long long launches = 0;; launches++) {
-            if (launches * budget > 1000LL * h->n + (1LL << 24)) {  // cannot happen: delta < 0 shortens the tour
-                g_last_error = "local search did not converge";
-                return TSP2OPT_ECUDA;
-            }
-            CUDA_TRY(launch_local_search(h->geo, h->d_P, h->d_E, h->d_tour, h->n, h->d_tiles, h->ntiles, h->d_slots,
-                                         h->parity, max_iters, budget, h->d_bar, h->d_ctl, h->d_tilebest,
-                                         sweep_flags(h), h->d_trace, h->trace_cap, h->stream));
-            CUDA_TRY(cudaMemcpyAsync(h->h_ctl, h->d_ctl, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
-            CUDA_TRY(cudaStreamSynchronize(h->stream));
-            h->parity = *h->h_ctl;
-            rc = read_slot(h);
-            if (rc) return rc;
-            if (h->h_slot->done & 3) break;
-        }
-        CUDA_TRY(cudaMemcpyAsync(tour, h->d_tour, sizeof(int32_t) * h->n, cudaMemcpyDeviceToHost, h->stream));
-        CUDA_TRY(cudaStreamSynchronize(h->stream));
-        *length = h->h_slot->length;
-        *iterations = h->h_slot->moves;
-        return (h->h_slot->done & 3) == 2 ? TSP2OPT_MAXITER : TSP2OPT_OK;
-    }
-    // Multi-kernel loop (sharded handles): batches of K iterations between host
-    // checks; an iteration after convergence is a no-op (sweep CTAs exit on the
-    // done flag).
-    long long k = 4;
-    for (;;) {
-        for (long long c = 0; c < k; c++) {
-            rc = enqueue_iteration(h, max_iters, true);
-            if (rc) return rc;
-        }
-        rc = read_slot(h);
-        if (rc) return rc;
-        if (h->h_slot->done & 3) break;
-        if (k < 64) k *= 2;
-    }
+    rc = run_local_search(h, max_iters);
+    if (rc < 0) return rc;
     CUDA_TRY(cudaMemcpyAsync(tour, h->d_tour, sizeof(int32_t) * h->n, cudaMemcpyDeviceToHost, h->stream));
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     *length = h->h_slot->length;
     *iterations = h->h_slot->moves;
-    return (h->h_slot->done & 3) == 2 ? TSP2OPT_MAXITER : TSP2OPT_OK;
+    return rc;
+}
+
+int tsp2opt_ils(tsp2opt_t h, int32_t* tour, int64_t iterations, uint64_t seed, int64_t* length, int64_t* lengths)
+{
+    if (!h || !tour || !length || iterations < 0) return TSP2OPT_EINVAL;
+    int rc = load_host_tour(h, tour);
+    if (rc) return rc;
+    if (!h->d_best) CUDA_TRY(cudaMalloc(&h->d_best, sizeof(int) * (size_t)h->n));
+    // s* = 2optLocalSearch(s0)
+    rc = run_local_search(h, TSP2OPT_MAX_ITERS_UNBOUNDED);
+    if (rc < 0) return rc;
+    long long best = h->h_slot->length;
+    CUDA_TRY(cudaMemcpyAsync(h->d_best, h->d_tour, sizeof(int) * (size_t)h->n, cudaMemcpyDeviceToDevice, h->stream));
+    if (lengths) lengths[0] = best;
+    for (long long t = 0; t < iterations; t++) {
+        if (h->n >= 8) {
+            // s' = Perturbation(s*): double bridge of the best tour (device gather),
+            // s*' = 2optLocalSearch(s'), accept iff strictly shorter (R14-R16)
+            long long a, b, c;
+            ils_cuts(h->n, seed, t, &a, &b, &c);
+            CUDA_TRY(launch_double_bridge(h->d_best, h->d_tour_in, h->n, (int)a, (int)b, (int)c, h->stream));
+            rc = load_device_tour(h, h->d_tour_in);
+            if (rc) return rc;
+            rc = run_local_search(h, TSP2OPT_MAX_ITERS_UNBOUNDED);
+            if (rc < 0) return rc;
+            if (h->h_slot->length < best) {
+                best = h->h_slot->length;
+                CUDA_TRY(cudaMemcpyAsync(h->d_best, h->d_tour, sizeof(int) * (size_t)h->n, cudaMemcpyDeviceToDevice,
+                                         h->stream));
+            }
+        }
+        if (lengths) lengths[t + 1] = best;
+    }
+    // leave the handle holding the best tour
+    CUDA_TRY(cudaMemcpyAsync(h->d_tour_in, h->d_best, sizeof(int) * (size_t)h->n, cudaMemcpyDeviceToDevice,
+                             h->stream));
+    rc = load_device_tour(h, h->d_tour_in);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(tour, h->d_best, sizeof(int32_t) * h->n, cudaMemcpyDeviceToHost, h->stream));
+    rc = read_slot(h);
+    if (rc) return rc;
+    *length = best;
+    return TSP2OPT_OK;
 }
 
 int tsp2opt_get_tour(tsp2opt_t h, int32_t* tour_out, int64_t* length)

@@ -69,6 +69,20 @@ __global__ void init_slot_kernel(Slot* slot, int clear_length)
 
 // best_move's sweep is not followed by an apply: its tile minima must not be
 // combined with an older move by a later sweep.
+// ILS perturbation (L18 §V "a simple doublebridge move"): out = A C B D for
+// in = A B C D, A = [0, a), B = [a, b), C = [b, c), D = [c, n); one thread per
+// output position.
+__global__ void double_bridge_kernel(const int* __restrict__ in, int* __restrict__ out, int n, int a, int b, int c)
+{
+    const int k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= n) return;
+    int src;
+    if (k < a || k >= c) src = k;                 // A and D stay
+    else if (k < a + (c - b)) src = b + (k - a);  // C moves forward
+    else src = a + (k - a - (c - b));             // B moves back
+    out[k] = in[src];
+}
+
 __global__ void reset_key_kernel(Slot* slot)
 {
     slot->key = seed_key();
@@ -321,6 +335,13 @@ cudaError_t launch_load_tour(const int* coords, const int* tour_src, int* tour_d
     init_slot_kernel<<<1, 1, 0, st>>>(slot, 1);
     load_tour_kernel<<<(n + 255) / 256, 256, 0, st>>>(coords, tour_src, tour_dst, P, E, n, slot, stamp, epoch);
     g_launches += 2;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_double_bridge(const int* in, int* out, int n, int a, int b, int c, cudaStream_t st)
+{
+    double_bridge_kernel<<<(n + 255) / 256, 256, 0, st>>>(in, out, n, a, b, c);
+    g_launches += 1;
     return cudaGetLastError();
 }
 

@@ -60,6 +60,7 @@ def _L():
             "tsp2opt_debug_set_shard": ([P, I32, I32], I32),
             "tsp2opt_set_option": ([P, I32, I64], I32),
             "tsp2opt_get_trace": ([P, P, I64, pI64], I32),
+            "tsp2opt_ils": ([P, P, I64, ctypes.c_uint64, pI64, P], I32),
             "tsp2opt_plan_shard": ([I32, I32, I32, pI32, pI32, pI32, P, I64, pI64, pI64], I32),
             "tsp2opt_get_geometry": ([P, pI32, pI32, pI32, pI64, pI64], I32),
             "tsp2opt_selftest": ([pI64, pI64, pI64, pI64], I32),
@@ -174,6 +175,16 @@ def local_search(h, tour, max_iters: int | None = None):
     mi = MAX_ITERS_UNBOUNDED if max_iters is None else int(max_iters)
     st = _check(_L().tsp2opt_local_search(h, _ptr(t), mi, ctypes.byref(L), ctypes.byref(it)), "tsp2opt_local_search")
     return dict(tour=t, length=L.value, iterations=it.value, status=st)
+
+
+def ils(h, tour, iterations: int, seed: int):
+    """Iterated Local Search (Algorithm 1): dict(tour, length, lengths)."""
+    t = np.array(tour, dtype=np.int32, copy=True)
+    L = ctypes.c_int64()
+    lengths = np.zeros(int(iterations) + 1, dtype=np.int64)
+    _check(_L().tsp2opt_ils(h, _ptr(t), int(iterations), ctypes.c_uint64(seed & 0xFFFFFFFFFFFFFFFF), ctypes.byref(L),
+                            _ptr(lengths)), "tsp2opt_ils")
+    return dict(tour=t, length=L.value, lengths=lengths)
 
 
 def get_tour(h, n: int):
@@ -306,6 +317,9 @@ class TSP2Opt:
 
     def get_tour(self):
         return get_tour(self.h, self.n)
+
+    def ils(self, tour, iterations: int, seed: int):
+        return ils(self.h, tour, iterations, seed)
 
     def set_option(self, option: int, value: int):
         set_option(self.h, option, value)

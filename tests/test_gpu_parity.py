@@ -286,3 +286,18 @@ def test_seeded_sweeps_mixed_operations(gpu, monkeypatch, rows):
                 g.iterate_async(3)
                 g.sync()
                 check()
+
+
+@pytest.mark.parametrize("kind,n,iters,seed", [("uniform", 8, 20, 1), ("uniform", 100, 60, 2), ("lattice", 100, 40, 3),
+                                               ("uniform", 200, 30, 4), ("uniform", 1002, 8, 5), ("lattice", 1002, 8, 6)])
+def test_ils_parity(gpu, kind, n, iters, seed):
+    """Iterated Local Search (L10 Algorithm 1, double-bridge perturbation):
+    the best length after every step, the final tour and length match the oracle."""
+    c, t = _inst(kind, n, seed)
+    ref = oracle.ils(c, t, iters, seed=1000 + seed)
+    with tsp2opt.TSP2Opt(c) as g:
+        res = g.ils(t, iters, 1000 + seed)
+        assert res["lengths"].tolist() == ref["lengths"].tolist()
+        assert res["length"] == ref["length"] and np.array_equal(res["tour"], ref["tour"])
+        tour, L = g.get_tour()  # the handle holds the best tour afterwards
+        assert np.array_equal(tour, ref["tour"]) and L == ref["length"]
