@@ -215,9 +215,10 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms, sweep_avg_ms, e2e_total, tb_total_ms, tb_sweep_ms = t.tolist()
 
-    ls = None
+    ls = ils = None
     if rank == 0 and world == 1 and not args.no_ls:
         ls = time_to_local_min(tsp2opt, args.ls_config)
+        ils = time_ils(tsp2opt, args.ils_config) if args.ils_config else None
 
     if rank == 0:
         prof = ncu_profile_summary(args.config, args.tour)
@@ -263,6 +264,8 @@ def run_ours(args):
         }
         if ls:
             line["time_to_local_minimum"] = ls
+        if ils:
+            line["ils"] = ils
         if world == 1 and not args.no_cpu:
             line["cpu_baseline"] = cpu_baseline(args, coords, tour, total_pairs)
         print(json.dumps(line), flush=True)
@@ -308,6 +311,24 @@ def time_to_local_min(tsp2opt, cfg_name):
         out.append({"config": name, "n": n, "start": tk or inputs.CONFIGS[name]["tour"], "seconds": dt,
                     "iterations": r["iterations"], "length": r["length"],
                     "pair_checks_per_s": (r["iterations"] + 1) * n * (n - 1) / 2 / dt})
+    return out
+
+
+def time_ils(tsp2opt, spec):
+    """Iterated Local Search (Algorithm 1) throughput: `cfg:iterations` entries."""
+    out = []
+    for item in spec.split(","):
+        name, _, iters = item.partition(":")
+        iters = int(iters or 50)
+        coords, tour = inputs.config_instance(name)
+        with tsp2opt.TSP2Opt(coords) as g:
+            g.ils(tour, 1, 7)  # warm-up
+            t0 = time.perf_counter()
+            r = g.ils(tour, iters, 2013)
+            dt = time.perf_counter() - t0
+        out.append({"config": name, "n": len(tour), "ils_iterations": iters, "seconds": dt,
+                    "ils_iterations_per_s": iters / dt, "first_local_min": int(r["lengths"][0]),
+                    "best_length": r["length"], "seed": 2013})
     return out
 
 
@@ -372,6 +393,7 @@ def main():
     ap.add_argument("--config", default="C5")
     ap.add_argument("--tour", default="random", choices=["random", "hilbert"])
     ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert,C5:hilbert", help="configs timed to a local minimum (rank 0, N=1)")
+    ap.add_argument("--ils-config", default="C1:200,C2:50", help="Iterated Local Search runs cfg:iterations")
     ap.add_argument("--no-ls", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
