@@ -215,10 +215,11 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms, sweep_avg_ms, e2e_total, tb_total_ms, tb_sweep_ms = t.tolist()
 
-    ls = ils = None
+    ls = ils = batch = None
     if rank == 0 and world == 1 and not args.no_ls:
         ls = time_to_local_min(tsp2opt, args.ls_config)
         ils = time_ils(tsp2opt, args.ils_config) if args.ils_config else None
+        batch = time_batch(tsp2opt, args.batch_config, not args.no_cpu) if args.batch_config else None
 
     if rank == 0:
         prof = ncu_profile_summary(args.config, args.tour)
@@ -266,6 +267,8 @@ def run_ours(args):
             line["time_to_local_minimum"] = ls
         if ils:
             line["ils"] = ils
+        if batch:
+            line["batch_local_search"] = batch
         if world == 1 and not args.no_cpu:
             line["cpu_baseline"] = cpu_baseline(args, coords, tour, total_pairs)
         print(json.dumps(line), flush=True)
@@ -332,6 +335,60 @@ def time_ils(tsp2opt, spec):
     return out
 
 
+def time_batch(tsp2opt, spec, with_oracle=True):
+    """Batched small-instance local search: `n:batch`
+    entries; B independent uniform instances (seeds 1..B, random starts) solved
+    to their local minima, one CTA each.  Device-resident (CUDA events around
+    tsp2opt_batch_local_search_async) and end to end through the host API."""
+    import torch
+
+    out = []
+    for item in spec.split(","):
+        n, _, B = item.partition(":")
+        n, B = int(n), int(B or 4736)
+        cs = np.stack([inputs.make_coords("uniform", n, 1 + b) for b in range(B)]).astype(np.int32)
+        ts = np.stack([inputs.random_tour(n, 1 + b) for b in range(B)]).astype(np.int32)
+        dc, d0 = torch.from_numpy(cs).cuda(), torch.from_numpy(ts).cuda()
+        dl = torch.zeros(B, dtype=torch.int64, device="cuda")
+        di = torch.zeros(B, dtype=torch.int64, device="cuda")
+        st = torch.cuda.current_stream()
+        dev = []
+        for rep in range(4):
+            dt_ = d0.clone()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            e0.record()
+            tsp2opt.batch_local_search_async(dc.data_ptr(), n, B, dt_.data_ptr(), dl.data_ptr(), di.data_ptr(),
+                                             stream=st.cuda_stream)
+            e1.record()
+            torch.cuda.synchronize()
+            if rep:
+                dev.append(e0.elapsed_time(e1) * 1e-3)
+        dev_s = float(np.median(dev))
+        moves = int(di.sum())
+        t0 = time.perf_counter()
+        r = tsp2opt.batch_local_search(cs, ts)
+        host_s = time.perf_counter() - t0
+        ok = bool((r["lengths"] == dl.cpu().numpy()).all())
+        item_out = {"n": n, "instances": B, "coords": "uniform seeds 1..B", "start": "random",
+                    "device_s": dev_s, "instances_per_s": B / dev_s,
+                    "pairs_per_s": (moves + B) * n * (n - 1) / 2 / dev_s, "mean_moves": moves / B,
+                    "e2e_s": host_s, "e2e_instances_per_s": B / host_s, "e2e_h2d_bytes": int(cs.nbytes + ts.nbytes),
+                    "e2e_d2h_bytes": int(ts.nbytes + 16 * B), "e2e_matches_device": ok, "gpu_launches": 1}
+        if with_oracle:
+            import oracle
+
+            k, t1 = 0, time.perf_counter()
+            while k < B and time.perf_counter() - t1 < 3.0:
+                oracle.local_search(cs[k], ts[k])
+                k += 1
+            osec = time.perf_counter() - t1
+            item_out["cpu_oracle"] = {"instances_per_s": k / osec, "sample": f"{k} instances one after another",
+                                      "cores": oracle.num_threads()}
+        out.append(item_out)
+    return out
+
+
 # ----------------------------------------------------------------------------- oracle timing
 def cpu_baseline(args, coords, tour, total_pairs):
     import oracle
@@ -394,6 +451,7 @@ def main():
     ap.add_argument("--tour", default="random", choices=["random", "hilbert"])
     ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert,C5:hilbert", help="configs timed to a local minimum (rank 0, N=1)")
     ap.add_argument("--ils-config", default="C1:200,C2:50", help="Iterated Local Search runs cfg:iterations")
+    ap.add_argument("--batch-config", default="100:4736,1002:592", help="batched local search n:instances")
     ap.add_argument("--no-ls", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)

@@ -136,6 +136,27 @@ int tsp2opt_local_search(tsp2opt_t h, int32_t *tour, int64_t max_iters, int64_t 
 int tsp2opt_ils(tsp2opt_t h, int32_t *tour, int64_t iterations, uint64_t seed, int64_t *length,
                 int64_t *lengths);
 
+/* Batched local search of `batch` independent instances of the same size n
+ * (3 <= n <= 4096), one CTA per instance, everything in shared memory
+ * (the paper's small-n case, L18 §V "smaller than 200").
+ * Stateless (no handle; uses the current CUDA device).  coords_xy: host
+ * int32[batch * 2n] (instance b at offset 2n*b); tours: host int32[batch * n],
+ * in = start tours, out = local minima (or after max_iters moves);
+ * lengths / iterations: int64[batch].  Same result per instance as
+ * tsp2opt_local_search.  Errors as tsp2opt_create / set_tour; nothing is
+ * written on error. */
+int tsp2opt_batch_local_search(const int32_t *coords_xy, int32_t n, int32_t batch, int32_t *tours,
+                               int64_t max_iters, int64_t *lengths, int64_t *iterations);
+
+/* The same on DEVICE buffers (same layouts), enqueued on `stream`
+ * (cudaStream_t, NULL = legacy default stream); returns after the launch.
+ * Contents are validated on the device: an instance whose tour is not a
+ * permutation or whose coordinates leave [0, 2^15) gets lengths[b] =
+ * iterations[b] = -1 and its tour is left unchanged.  The caller owns all
+ * buffers and synchronises the stream before reading them. */
+int tsp2opt_batch_local_search_async(const int32_t *d_coords_xy, int32_t n, int32_t batch, int32_t *d_tours,
+                                     int64_t max_iters, int64_t *d_lengths, int64_t *d_iterations, void *stream);
+
 /* Copy the current tour (host int32[n]) and its length out. */
 int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
 

@@ -564,6 +564,64 @@ int tsp2opt_local_search(tsp2opt_t h, int32_t* tour, int64_t max_iters, int64_t*
     return rc;
 }
 
+int tsp2opt_batch_local_search(const int32_t* coords_xy, int32_t n, int32_t batch, int32_t* tours,
+                               int64_t max_iters, int64_t* lengths, int64_t* iterations)
+{
+    if (!coords_xy || !tours || !lengths || !iterations || batch < 1 || max_iters < 0) return TSP2OPT_EINVAL;
+    if (n < 3 || n > kBatchMaxN) return TSP2OPT_EINVAL;
+    for (long long b = 0; b < batch; b++) {
+        int rc = validate_coords(coords_xy + 2 * n * b, n);
+        if (rc) return rc;
+        rc = validate_tour(tours + (long long)n * b, n);
+        if (rc) return rc;
+    }
+    int* d_xy = nullptr;
+    int* d_t = nullptr;
+    long long* d_out = nullptr;
+    auto cleanup = [&]() {
+        cudaFree(d_xy);
+        cudaFree(d_t);
+        cudaFree(d_out);
+    };
+    auto fail = [&](cudaError_t e, const char* what) {
+        cleanup();
+        return cuda_fail(e, what);
+    };
+    const size_t nxy = sizeof(int) * 2 * (size_t)n * batch, nt = sizeof(int) * (size_t)n * batch;
+    cudaError_t e;
+    if ((e = cudaMalloc(&d_xy, nxy)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMalloc(&d_t, nt)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMalloc(&d_out, sizeof(long long) * 2 * (size_t)batch)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMemcpy(d_xy, coords_xy, nxy, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "H2D");
+    if ((e = cudaMemcpy(d_t, tours, nt, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "H2D");
+    if ((e = launch_batch_local_search(d_xy, d_t, n, batch, max_iters, d_out, d_out + batch, nullptr)) != cudaSuccess)
+        return fail(e, "batch_ls_kernel");
+    if ((e = cudaMemcpy(tours, d_t, nt, cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
+    std::vector<long long> out(2 * (size_t)batch);
+    if ((e = cudaMemcpy(out.data(), d_out, sizeof(long long) * out.size(), cudaMemcpyDeviceToHost)) != cudaSuccess)
+        return fail(e, "D2H");
+    cleanup();
+    for (int b = 0; b < batch; b++)
+        if (out[b] < 0) return TSP2OPT_ENOTPERM;  // unreachable: validated above
+    for (int b = 0; b < batch; b++) {
+        lengths[b] = out[b];
+        iterations[b] = out[batch + b];
+    }
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_batch_local_search_async(const int32_t* d_coords_xy, int32_t n, int32_t batch, int32_t* d_tours,
+                                     int64_t max_iters, int64_t* d_lengths, int64_t* d_iterations, void* stream)
+{
+    if (!d_coords_xy || !d_tours || !d_lengths || !d_iterations || batch < 1 || max_iters < 0) return TSP2OPT_EINVAL;
+    if (n < 3 || n > kBatchMaxN) return TSP2OPT_EINVAL;
+    const cudaError_t e = launch_batch_local_search(d_coords_xy, d_tours, n, batch, max_iters,
+                                                    reinterpret_cast<long long*>(d_lengths),
+                                                    reinterpret_cast<long long*>(d_iterations),
+                                                    static_cast<cudaStream_t>(stream));
+    return e == cudaSuccess ? TSP2OPT_OK : cuda_fail(e, "batch_ls_kernel");
+}
+
 int tsp2opt_ils(tsp2opt_t h, int32_t* tour, int64_t iterations, uint64_t seed, int64_t* length, int64_t* lengths)
 {
     if (!h || !tour || !length || iterations < 0) return TSP2OPT_EINVAL;

@@ -25,6 +25,11 @@ struct Geometry {
 };
 
 long long launch_count();
+void count_launch(int k = 1);
+constexpr int kBatchMaxN = 4096;  // batched local search: one instance per CTA, all in shared memory
+size_t batch_smem_bytes(int n);
+cudaError_t launch_batch_local_search(const int* coords, int* tours, int n, int batch, long long max_iters,
+                                      long long* lengths, long long* iters, cudaStream_t st);
 size_t sweep_smem_bytes(const Geometry& g);
 cudaError_t sweep_prepare();
 cudaError_t launch_load_tour(const int* coords, const int* tour_src, int* tour_dst, float2* P, int* E, int n,

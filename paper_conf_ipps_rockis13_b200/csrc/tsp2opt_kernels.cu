@@ -328,6 +328,7 @@ __global__ void selftest_filter_kernel(unsigned long long* bad, unsigned long lo
 // ===========================================================================
 static std::atomic<long long> g_launches{0};
 long long launch_count() { return g_launches.load(); }
+void count_launch(int k) { g_launches += k; }
 
 cudaError_t launch_load_tour(const int* coords, const int* tour_src, int* tour_dst, float2* P, int* E, int n,
                              Slot* slot, unsigned* stamp, unsigned epoch, cudaStream_t st)

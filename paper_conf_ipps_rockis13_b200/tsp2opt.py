@@ -61,6 +61,8 @@ def _L():
             "tsp2opt_set_option": ([P, I32, I64], I32),
             "tsp2opt_get_trace": ([P, P, I64, pI64], I32),
             "tsp2opt_ils": ([P, P, I64, ctypes.c_uint64, pI64, P], I32),
+            "tsp2opt_batch_local_search": ([P, I32, I32, P, I64, P, P], I32),
+            "tsp2opt_batch_local_search_async": ([P, I32, I32, P, I64, P, P, P], I32),
             "tsp2opt_plan_shard": ([I32, I32, I32, pI32, pI32, pI32, P, I64, pI64, pI64], I32),
             "tsp2opt_get_geometry": ([P, pI32, pI32, pI32, pI64, pI64], I32),
             "tsp2opt_selftest": ([pI64, pI64, pI64, pI64], I32),
@@ -175,6 +177,28 @@ def local_search(h, tour, max_iters: int | None = None):
     mi = MAX_ITERS_UNBOUNDED if max_iters is None else int(max_iters)
     st = _check(_L().tsp2opt_local_search(h, _ptr(t), mi, ctypes.byref(L), ctypes.byref(it)), "tsp2opt_local_search")
     return dict(tour=t, length=L.value, iterations=it.value, status=st)
+
+
+def batch_local_search(coords, tours, max_iters: int | None = None):
+    """coords int32[B, n, 2], tours int32[B, n] -> dict(tours, lengths, iterations) (one CTA per instance)."""
+    xy = _i32(coords)
+    B, n = xy.shape[0], xy.shape[1]
+    t = np.array(tours, dtype=np.int32, copy=True).reshape(B, n)
+    L = np.zeros(B, dtype=np.int64)
+    it = np.zeros(B, dtype=np.int64)
+    mi = MAX_ITERS_UNBOUNDED if max_iters is None else int(max_iters)
+    _check(_L().tsp2opt_batch_local_search(_ptr(xy), n, B, _ptr(t), mi, _ptr(L), _ptr(it)),
+           "tsp2opt_batch_local_search")
+    return dict(tours=t, lengths=L, iterations=it)
+
+
+def batch_local_search_async(d_coords: int, n: int, batch: int, d_tours: int, d_lengths: int, d_iters: int,
+                             max_iters: int | None = None, stream: int = 0):
+    """Device-pointer form (raw addresses, e.g. torch tensor.data_ptr()); see include/tsp2opt.h."""
+    mi = MAX_ITERS_UNBOUNDED if max_iters is None else int(max_iters)
+    _check(_L().tsp2opt_batch_local_search_async(ctypes.c_void_p(d_coords), n, batch, ctypes.c_void_p(d_tours), mi,
+                                                 ctypes.c_void_p(d_lengths), ctypes.c_void_p(d_iters),
+                                                 ctypes.c_void_p(stream)), "tsp2opt_batch_local_search_async")
 
 
 def ils(h, tour, iterations: int, seed: int):

@@ -57,6 +57,21 @@ def test_argument_validation_without_gpu():
     assert lib.tsp2opt_best_move(None, None, None, None, None) == tsp2opt.EINVAL
     assert lib.tsp2opt_apply(None, 0, 1) == tsp2opt.EINVAL
     assert lib.tsp2opt_local_search(None, None, 0, None, None) == tsp2opt.EINVAL
+    # batched entry: sizes, ranges and permutations are checked before any device work
+    L = np.zeros(2, np.int64)
+    xy2 = np.zeros((2, 10, 2), np.int32)
+    t2 = np.tile(np.arange(10, dtype=np.int32), (2, 1))
+    bls = lib.tsp2opt_batch_local_search
+    assert bls(None, 10, 2, t2.ctypes.data, 5, L.ctypes.data, L.ctypes.data) == tsp2opt.EINVAL
+    for n, b in ((2, 2), (4097, 1), (10, 0)):
+        assert bls(xy2.ctypes.data, n, b, t2.ctypes.data, 5, L.ctypes.data, L.ctypes.data) == tsp2opt.EINVAL
+    assert bls(xy2.ctypes.data, 10, 2, t2.ctypes.data, -1, L.ctypes.data, L.ctypes.data) == tsp2opt.EINVAL
+    badxy = xy2.copy()
+    badxy[1, 3, 0] = 1 << 15
+    assert bls(badxy.ctypes.data, 10, 2, t2.ctypes.data, 5, L.ctypes.data, L.ctypes.data) == tsp2opt.ERANGE
+    badt = t2.copy()
+    badt[1, 4] = 5
+    assert bls(xy2.ctypes.data, 10, 2, badt.ctypes.data, 5, L.ctypes.data, L.ctypes.data) == tsp2opt.ENOTPERM
     assert lib.tsp2opt_strerror(tsp2opt.ENOTPERM) == b"tour is not a permutation of 0..n-1"
 
 
