@@ -69,6 +69,8 @@ def _load():
             lib.oracle_double_bridge.restype = None
             lib.oracle_ils.argtypes = [p, i64, p, i64, ctypes.c_uint64, p, p]
             lib.oracle_ils.restype = None
+            lib.oracle_mf_tour.argtypes = [p, i64, p]
+            lib.oracle_mf_tour.restype = ctypes.c_int
             lib.oracle_num_threads.argtypes = []
             lib.oracle_num_threads.restype = ctypes.c_int
             _lib = lib
@@ -187,6 +189,15 @@ def ils(coords, tour, iterations: int, seed: int):
     _load().oracle_ils(_ptr(xy), xy.shape[0], _ptr(t), int(iterations), ctypes.c_uint64(seed & 0xFFFFFFFFFFFFFFFF),
                        _ptr(out), _ptr(lengths))
     return dict(tour=t, length=int(out[0]), lengths=lengths)
+
+
+def mf_tour(coords) -> np.ndarray:
+    """Multiple Fragment (greedy) start tour (L22 §V; reading R17), n <= 20000."""
+    xy = _xy(coords)
+    t = np.zeros(xy.shape[0], dtype=np.int32)
+    if _load().oracle_mf_tour(_ptr(xy), xy.shape[0], _ptr(t)) != 0:
+        raise ValueError("oracle_mf_tour: n out of range [3, 20000] or out of memory")
+    return t
 
 
 def num_threads() -> int:

@@ -289,6 +289,86 @@ void oracle_ils(const int32_t *xy, int64_t n, int32_t *tour, int64_t iterations,
     *length = L;
 }
 
+/* ---------------------------------------------------------------------------
+ * Multiple Fragment (greedy) start tour.  L22 §V: "an initial solution based
+ * on the Multiple Fragment(Greedy) heuristic[18]"; the paper gives no more
+ * than the name, so reading R17 fixes the textbook definition:
+ * take the edges {u, v} in increasing order of (d(u,v), min(u,v), max(u,v))
+ * and keep an edge iff both ends have degree < 2 and it does not close a
+ * cycle; the n-1 kept edges form a Hamiltonian path, closed by the edge
+ * between its two ends.  Tour: start at city 0, step to its lower-id
+ * neighbour, then follow the cycle.  Plain version: all C(n,2) edges, one
+ * sort, union-find -- O(n^2 log n) time and 8 C(n,2) bytes, for n <= 20000.
+ * Returns 0, or -1 if n is out of range or memory runs out.
+ * ------------------------------------------------------------------------- */
+static int cmp_u64(const void *a, const void *b)
+{
+    uint64_t x = *(const uint64_t *)a, y = *(const uint64_t *)b;
+    return x < y ? -1 : x > y;
+}
+
+static int64_t uf_find(int64_t *parent, int64_t x)
+{
+    while (parent[x] != x) {
+        parent[x] = parent[parent[x]];
+        x = parent[x];
+    }
+    return x;
+}
+
+int oracle_mf_tour(const int32_t *xy, int64_t n, int32_t *tour)
+{
+    if (n < 3 || n > 20000) return -1;
+    const int64_t m = n * (n - 1) / 2;
+    uint64_t *key = (uint64_t *)malloc(sizeof(uint64_t) * m);
+    int64_t *parent = (int64_t *)malloc(sizeof(int64_t) * n);
+    int64_t *adj = (int64_t *)malloc(sizeof(int64_t) * 2 * n);
+    int32_t *deg = (int32_t *)calloc(n, sizeof(int32_t));
+    if (!key || !parent || !adj || !deg) {
+        free(key), free(parent), free(adj), free(deg);
+        return -1;
+    }
+    int64_t e = 0;
+    for (int64_t v = 1; v < n; v++)
+        for (int64_t u = 0; u < v; u++) {
+            const uint64_t d = (uint64_t)oracle_dist(xy[2 * u], xy[2 * u + 1], xy[2 * v], xy[2 * v + 1]);
+            key[e++] = d << 44 | (uint64_t)u << 22 | (uint64_t)v;  /* d < 2^17, u < v < 2^22 */
+        }
+    qsort(key, m, sizeof(uint64_t), cmp_u64);
+    for (int64_t k = 0; k < n; k++) parent[k] = k;
+    int64_t kept = 0;
+    for (int64_t t = 0; t < m && kept < n - 1; t++) {
+        const int64_t u = (int64_t)(key[t] >> 22 & 0x3FFFFF), v = (int64_t)(key[t] & 0x3FFFFF);
+        if (deg[u] >= 2 || deg[v] >= 2) continue;
+        const int64_t ru = uf_find(parent, u), rv = uf_find(parent, v);
+        if (ru == rv) continue; /* would close a cycle */
+        parent[ru] = rv;
+        adj[2 * u + deg[u]++] = v;
+        adj[2 * v + deg[v]++] = u;
+        kept++;
+    }
+    /* close the Hamiltonian path: its two ends are the cities of degree 1 */
+    int64_t a = -1, b = -1;
+    for (int64_t k = 0; k < n; k++)
+        if (deg[k] < 2) {
+            if (a < 0) a = k;
+            else b = k;
+        }
+    adj[2 * a + deg[a]++] = b;
+    adj[2 * b + deg[b]++] = a;
+    /* walk: 0, then its lower-id neighbour */
+    int64_t prev = 0, cur = adj[0] < adj[1] ? adj[0] : adj[1];
+    tour[0] = 0;
+    for (int64_t k = 1; k < n; k++) {
+        tour[k] = (int32_t)cur;
+        const int64_t next = adj[2 * cur] == prev ? adj[2 * cur + 1] : adj[2 * cur];
+        prev = cur;
+        cur = next;
+    }
+    free(key), free(parent), free(adj), free(deg);
+    return 0;
+}
+
 int oracle_num_threads(void)
 {
 #ifdef _OPENMP
