@@ -300,10 +300,30 @@ def ncu_profile_summary(cfg, tour):
 
 
 def time_to_local_min(tsp2opt, cfg_name):
-    """Wall time of tsp2opt_local_search (host tour in, host tour out) per config."""
+    """Wall time of tsp2opt_local_search (host tour in, host tour out) per config.
+    Start `mf`: the paper's Table II protocol (L22 "time needed from an initial
+    solution based on the Multiple Fragment(Greedy) heuristic ... to the local
+    minimum"): tsp2opt_mf_tour on the device, then the local search from it;
+    both inside the timed region (coordinates already on the device)."""
     out = []
     for name in cfg_name.split(","):
         name, _, tk = name.partition(":")
+        if tk == "mf":
+            coords, _ = inputs.config_instance(name)
+            with tsp2opt.TSP2Opt(coords) as g:
+                g.mf_tour()  # warm-up (allocates the workspace)
+                g.local_search_current(max_iters=2)
+                t0 = time.perf_counter()
+                m = g.mf_tour()
+                t1 = time.perf_counter()
+                r = g.local_search_current()
+                t2 = time.perf_counter()
+            n = len(coords)
+            out.append({"config": name, "n": n, "start": "mf", "seconds": t2 - t0, "mf_seconds": t1 - t0,
+                        "ls_seconds": t2 - t1, "mf_length": m["length"], "mf_rounds": m["rounds"],
+                        "iterations": r["iterations"], "length": r["length"],
+                        "pair_checks_per_s": (r["iterations"] + 1) * n * (n - 1) / 2 / (t2 - t1)})
+            continue
         coords, tour = inputs.config_instance(name, tk or None)
         with tsp2opt.TSP2Opt(coords) as g:
             g.local_search(tour, max_iters=2)  # warm-up
@@ -449,7 +469,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C5")
     ap.add_argument("--tour", default="random", choices=["random", "hilbert"])
-    ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert,C5:hilbert", help="configs timed to a local minimum (rank 0, N=1)")
+    ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert,C5:hilbert,C2:mf,C3:mf,C4:mf,C5:mf", help="configs timed to a local minimum (rank 0, N=1)")
     ap.add_argument("--ils-config", default="C1:200,C2:50", help="Iterated Local Search runs cfg:iterations")
     ap.add_argument("--batch-config", default="100:4736,1002:592", help="batched local search n:instances")
     ap.add_argument("--no-ls", action="store_true")

@@ -120,6 +120,9 @@ int tsp2opt_sync(tsp2opt_t h, int64_t *iterations, int64_t *length, int32_t *con
  * *iterations = applied moves.  Returns TSP2OPT_OK at a local minimum,
  * TSP2OPT_MAXITER if max_iters moves were applied and an improving move remains. */
 #define TSP2OPT_MAX_ITERS_UNBOUNDED INT64_MAX
+/* tour == NULL: start from the handle's current tour (set_tour, mf_tour, a
+ * previous search) and leave the result on the device (read it with
+ * tsp2opt_get_tour); TSP2OPT_ESTATE if there is none. */
 int tsp2opt_local_search(tsp2opt_t h, int32_t *tour, int64_t max_iters, int64_t *length,
                          int64_t *iterations);
 
@@ -156,6 +159,17 @@ int tsp2opt_batch_local_search(const int32_t *coords_xy, int32_t n, int32_t batc
  * buffers and synchronises the stream before reading them. */
 int tsp2opt_batch_local_search_async(const int32_t *d_coords_xy, int32_t n, int32_t batch, int32_t *d_tours,
                                      int64_t max_iters, int64_t *d_lengths, int64_t *d_iterations, void *stream);
+
+/* Multiple Fragment (greedy) start tour, computed on the device (SURVEY §8(f)
+ * NEXT-1; L22 §V "an initial solution based on the Multiple Fragment(Greedy)
+ * heuristic[18]"; definition, tie-break and orientation: DESIGN.md R17 --
+ * edges by increasing (d, min id, max id), tour starting 0 -> lower-id
+ * neighbour).  It becomes the handle's current tour (local_search with
+ * tour == NULL continues from it).  tour_out: host int32[n] or NULL;
+ * *length (or NULL) = its length; *rounds (or NULL) = parallel rounds used.
+ * The first call allocates a workspace of about (16*8 + 100) bytes per city,
+ * kept until destroy.  Errors: EINVAL (h NULL), ECUDA / ENOMEM. */
+int tsp2opt_mf_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length, int32_t *rounds);
 
 /* Copy the current tour (host int32[n]) and its length out. */
 int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);

@@ -72,6 +72,8 @@ struct tsp2opt_ctx {
     bool tile_bounds = true;    // tile-level bounding-box form of the filter (TSP2OPT_OPT_TILE_BOUNDS)
     unsigned long long* d_trace = nullptr;  // [trace_cap] keys of the applied moves (TSP2OPT_OPT_TRACE)
     int* d_best = nullptr;      // [n] best tour of an ILS run
+    void* d_mf_ws = nullptr;    // Multiple Fragment workspace (mf_workspace_bytes), allocated on first use
+    int mf_rounds = 0;          // rounds of the last tsp2opt_mf_tour
     long long trace_cap = 0;
     Slot* h_slot = nullptr;     // pinned readback
     unsigned epoch = 0;
@@ -197,6 +199,7 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_tilebest);
     cudaFree(h->d_trace);
     cudaFree(h->d_best);
+    cudaFree(h->d_mf_ws);
     if (h->h_slot) cudaFreeHost(h->h_slot);
     for (cudaEvent_t e : h->ev_pool) cudaEventDestroy(e);
     if (h->own_stream) cudaStreamDestroy(h->own_stream);
@@ -552,12 +555,19 @@ int tsp2opt_sync(tsp2opt_t h, int64_t* iterations, int64_t* length, int32_t* con
 
 int tsp2opt_local_search(tsp2opt_t h, int32_t* tour, int64_t max_iters, int64_t* length, int64_t* iterations)
 {
-    if (!h || !tour || !length || !iterations || max_iters < 0) return TSP2OPT_EINVAL;
-    int rc = load_host_tour(h, tour);
-    if (rc) return rc;
+    if (!h || !length || !iterations || max_iters < 0) return TSP2OPT_EINVAL;
+    int rc;
+    if (tour) {
+        rc = load_host_tour(h, tour);
+        if (rc) return rc;
+    } else {
+        if (!h->has_tour) return TSP2OPT_ESTATE;
+        rc = load_device_tour(h, h->d_tour);  // restart bookkeeping from the current tour
+        if (rc) return rc;
+    }
     rc = run_local_search(h, max_iters);
     if (rc < 0) return rc;
-    CUDA_TRY(cudaMemcpyAsync(tour, h->d_tour, sizeof(int32_t) * h->n, cudaMemcpyDeviceToHost, h->stream));
+    if (tour) CUDA_TRY(cudaMemcpyAsync(tour, h->d_tour, sizeof(int32_t) * h->n, cudaMemcpyDeviceToHost, h->stream));
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     *length = h->h_slot->length;
     *iterations = h->h_slot->moves;
@@ -662,6 +672,24 @@ int tsp2opt_ils(tsp2opt_t h, int32_t* tour, int64_t iterations, uint64_t seed, i
     rc = read_slot(h);
     if (rc) return rc;
     *length = best;
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_mf_tour(tsp2opt_t h, int32_t* tour_out, int64_t* length, int32_t* rounds)
+{
+    if (!h) return TSP2OPT_EINVAL;
+    if (!h->d_mf_ws) CUDA_TRY(cudaMalloc(&h->d_mf_ws, mf_workspace_bytes(h->n)));
+    CUDA_TRY(launch_mf_tour(h->d_coords, h->n, h->d_mf_ws, h->d_tour_in, &h->mf_rounds, h->stream));
+    int rc = load_device_tour(h, h->d_tour_in);
+    if (rc) return rc;
+    rc = read_slot(h);  // also proves the ranked tour is a permutation
+    if (rc) return rc;
+    if (tour_out) {
+        CUDA_TRY(cudaMemcpyAsync(tour_out, h->d_tour, sizeof(int32_t) * h->n, cudaMemcpyDeviceToHost, h->stream));
+        CUDA_TRY(cudaStreamSynchronize(h->stream));
+    }
+    if (length) *length = h->h_slot->length;
+    if (rounds) *rounds = h->mf_rounds;
     return TSP2OPT_OK;
 }
 

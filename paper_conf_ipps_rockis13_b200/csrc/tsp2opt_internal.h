@@ -30,6 +30,15 @@ constexpr int kBatchMaxN = 4096;  // batched local search: one instance per CTA,
 size_t batch_smem_bytes(int n);
 cudaError_t launch_batch_local_search(const int* coords, int* tours, int n, int batch, long long max_iters,
                                       long long* lengths, long long* iters, cudaStream_t st);
+// Multiple Fragment start tour (tsp2opt_mf.cu)
+constexpr int kMfK = 16;        // exact nearest neighbours kept per city
+constexpr int kMfCtr = 4;       // per-round counters, x2 parities: ends, scans, accepted, pad
+constexpr int kMfEdges = 8;     // kept edges so far
+constexpr int kMfEndCnt = 9;    // path ends found by the closing step
+constexpr int kMfEnd0 = 10;     // [2] the path's two ends
+constexpr int kMfCtrInts = 16;
+size_t mf_workspace_bytes(int n);
+cudaError_t launch_mf_tour(const int* coords, int n, void* ws, int* tour_out, int* rounds_out, cudaStream_t st);
 size_t sweep_smem_bytes(const Geometry& g);
 cudaError_t sweep_prepare();
 cudaError_t launch_load_tour(const int* coords, const int* tour_src, int* tour_dst, float2* P, int* E, int n,

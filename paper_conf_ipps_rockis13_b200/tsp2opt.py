@@ -62,6 +62,7 @@ def _L():
             "tsp2opt_get_trace": ([P, P, I64, pI64], I32),
             "tsp2opt_ils": ([P, P, I64, ctypes.c_uint64, pI64, P], I32),
             "tsp2opt_batch_local_search": ([P, I32, I32, P, I64, P, P], I32),
+            "tsp2opt_mf_tour": ([P, P, pI64, P], I32),
             "tsp2opt_batch_local_search_async": ([P, I32, I32, P, I64, P, P, P], I32),
             "tsp2opt_plan_shard": ([I32, I32, I32, pI32, pI32, pI32, P, I64, pI64, pI64], I32),
             "tsp2opt_get_geometry": ([P, pI32, pI32, pI32, pI64, pI64], I32),
@@ -177,6 +178,23 @@ def local_search(h, tour, max_iters: int | None = None):
     mi = MAX_ITERS_UNBOUNDED if max_iters is None else int(max_iters)
     st = _check(_L().tsp2opt_local_search(h, _ptr(t), mi, ctypes.byref(L), ctypes.byref(it)), "tsp2opt_local_search")
     return dict(tour=t, length=L.value, iterations=it.value, status=st)
+
+
+def mf_tour(h, n: int):
+    """Multiple Fragment (greedy) start tour on the device; it becomes the current tour."""
+    t = np.zeros(n, dtype=np.int32)
+    L = ctypes.c_int64()
+    r = ctypes.c_int32()
+    _check(_L().tsp2opt_mf_tour(h, _ptr(t), ctypes.byref(L), ctypes.byref(r)), "tsp2opt_mf_tour")
+    return dict(tour=t, length=L.value, rounds=r.value)
+
+
+def local_search_current(h, max_iters: int | None = None):
+    """Local search from the handle's current tour (tour == NULL); the result stays on the device."""
+    L, it = ctypes.c_int64(), ctypes.c_int64()
+    mi = MAX_ITERS_UNBOUNDED if max_iters is None else int(max_iters)
+    st = _check(_L().tsp2opt_local_search(h, None, mi, ctypes.byref(L), ctypes.byref(it)), "tsp2opt_local_search")
+    return dict(length=L.value, iterations=it.value, status=st)
 
 
 def batch_local_search(coords, tours, max_iters: int | None = None):
@@ -341,6 +359,12 @@ class TSP2Opt:
 
     def get_tour(self):
         return get_tour(self.h, self.n)
+
+    def mf_tour(self):
+        return mf_tour(self.h, self.n)
+
+    def local_search_current(self, max_iters=None):
+        return local_search_current(self.h, max_iters)
 
     def ils(self, tour, iterations: int, seed: int):
         return ils(self.h, tour, iterations, seed)
