@@ -175,10 +175,12 @@ int tsp2opt_mf_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length, int32_t *ro
 int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
 
 /* Execution options (none changes any result; all results stay bit-exact):
- *  TSP2OPT_OPT_TILE_BOUNDS (default 1): skip a tile of the sweep when the
+ *  TSP2OPT_OPT_TILE_BOUNDS (default 2 from 1e8 pairs per rank, else 1): 1 = skip a tile of the sweep when the
  *      bounding boxes of its row and column cities prove that no pair can pass
- *      the per-pair necessary condition; 0 tests every pair
- *      individually (the pair-check throughput the bench reports).
+ *      the per-pair necessary condition; 2 = the same, plus a
+ *      pre-sweep cull (per-block boxes, one test per tile with delta < 0 as the
+ *      condition) so the sweep launches over the kept tiles only; 0 tests every
+ *      pair individually (the pair-check throughput the bench reports).
  *  TSP2OPT_OPT_SEED (default 0): start each tile from its own minimum of the
  *      previous sweep when the applied move leaves that pair intact.
  *  TSP2OPT_OPT_PERSISTENT (default 2): local_search loop, 0 = one sweep and one
@@ -242,7 +244,8 @@ int tsp2opt_selftest_sqrt(double *max_rel_err, int32_t *zero_ok);
 
 /* Sweep counters of an instrumented build (-DTSP2OPT_STATS): out4[0] warp column
  * steps, [1] steps that took the exact path, [2] candidate pairs evaluated
- * exactly; -1 in product builds.  reset != 0 zeroes them afterwards. */
+ * exactly, [3] warp tiles walked (not skipped by the tile bound); -1 in
+ * product builds.  reset != 0 zeroes them afterwards. */
 int tsp2opt_debug_stats(int64_t *out4, int32_t reset);
 
 /* Number of this library's kernel launches since load (for gpu_launches). */

@@ -69,7 +69,20 @@ struct tsp2opt_ctx {
     unsigned long long* d_tilebest = nullptr;  // [ntiles] per-tile minima of the last sweep (next seed)
     bool seed_next = false;     // seed each tile with its surviving minimum of the previous sweep (TSP2OPT_SEED=1;
                                 // measured neutral-to-slower at n = 1002 .. 33810, so off by default)
-    bool tile_bounds = true;    // tile-level bounding-box form of the filter (TSP2OPT_OPT_TILE_BOUNDS)
+    int tile_bounds = 1;        // TSP2OPT_OPT_TILE_BOUNDS: 0 off, 1 per-tile bound inside the sweep, 2 also the
+                                // pre-sweep cull (box + cull kernels; the sweep runs over the kept tiles only)
+    Box* d_rbox = nullptr;      // culled sweep: per row-block / column-chunk summaries
+    Box* d_cbox = nullptr;
+    // The culled sweep has its own tiling (narrower column chunks: a finer cull
+    // and more, shorter work items for the few tiles a coherent tour keeps).
+    Geometry cgeo{};
+    std::vector<Tile> all_ctiles;
+    int2* d_ctiles = nullptr;   // this shard's cull tiles
+    unsigned long long* d_ctilebest = nullptr;  // their per-tile minima (seeds)
+    int* d_list = nullptr;      // kept cull-tile indices [nctiles]
+    int nctiles = 0;
+    int list_grid = 0;          // CTAs of the culled sweep (co-resident)
+    int last_tiling = -1;       // tiling of the previous sweep (0 dense, 1 cull): seeds are per tiling
     unsigned long long* d_trace = nullptr;  // [trace_cap] keys of the applied moves (TSP2OPT_OPT_TRACE)
     int* d_best = nullptr;      // [n] best tour of an ILS run
     void* d_mf_ws = nullptr;    // Multiple Fragment workspace (mf_workspace_bytes), allocated on first use
@@ -158,23 +171,39 @@ std::vector<Tile> shard_tiles(const std::vector<Tile>& all, int rank, int world,
     return mine;
 }
 
-int upload_shard(tsp2opt_ctx* h, int rank, int world)
+// Upload this rank's share of one tiling: tile origins and per-tile seeds.
+int upload_tiling(const std::vector<Tile>& all, int rank, int world, int2** d_tiles,
+                  unsigned long long** d_best, int* ntiles, long long* pairs)
 {
-    long long pairs = 0;
-    std::vector<Tile> mine = shard_tiles(h->all_tiles, rank, world, &pairs);
+    std::vector<Tile> mine = shard_tiles(all, rank, world, pairs);
     std::vector<int2> host(mine.size());
     for (size_t k = 0; k < mine.size(); k++) host[k] = make_int2(mine[k].i0, mine[k].j0);
-    if (h->d_tiles) cudaFree(h->d_tiles);
-    if (h->d_tilebest) cudaFree(h->d_tilebest);
-    h->d_tiles = nullptr;
-    h->d_tilebest = nullptr;
+    cudaFree(*d_tiles);
+    cudaFree(*d_best);
+    *d_tiles = nullptr;
+    *d_best = nullptr;
     if (!host.empty()) {
-        CUDA_TRY(cudaMalloc(&h->d_tiles, host.size() * sizeof(int2)));
-        CUDA_TRY(cudaMalloc(&h->d_tilebest, host.size() * sizeof(unsigned long long)));
-        CUDA_TRY(cudaMemset(h->d_tilebest, 0xFF, host.size() * sizeof(unsigned long long)));  // kKeyNone
-        CUDA_TRY(cudaMemcpy(h->d_tiles, host.data(), host.size() * sizeof(int2), cudaMemcpyHostToDevice));
+        CUDA_TRY(cudaMalloc(d_tiles, host.size() * sizeof(int2)));
+        CUDA_TRY(cudaMalloc(d_best, host.size() * sizeof(unsigned long long)));
+        CUDA_TRY(cudaMemset(*d_best, 0xFF, host.size() * sizeof(unsigned long long)));  // kKeyNone
+        CUDA_TRY(cudaMemcpy(*d_tiles, host.data(), host.size() * sizeof(int2), cudaMemcpyHostToDevice));
     }
-    h->ntiles = (int)host.size();
+    *ntiles = (int)host.size();
+    return TSP2OPT_OK;
+}
+
+int upload_shard(tsp2opt_ctx* h, int rank, int world)
+{
+    long long pairs = 0, cpairs = 0;
+    int rc = upload_tiling(h->all_tiles, rank, world, &h->d_tiles, &h->d_tilebest, &h->ntiles, &pairs);
+    if (rc) return rc;
+    rc = upload_tiling(h->all_ctiles, rank, world, &h->d_ctiles, &h->d_ctilebest, &h->nctiles, &cpairs);
+    if (rc) return rc;
+    cudaFree(h->d_list);
+    h->d_list = nullptr;
+    if (h->nctiles > 0) CUDA_TRY(cudaMalloc(&h->d_list, sizeof(int) * (size_t)h->nctiles));
+    h->list_grid = sweep_list_grid(h->cgeo, h->nctiles);
+    h->last_tiling = -1;
     h->shard_pairs = pairs;
     h->shard_rank = rank;
     h->shard_world = world;
@@ -197,6 +226,11 @@ void free_ctx(tsp2opt_ctx* h)
     if (h->h_ctl) cudaFreeHost(h->h_ctl);
     cudaFree(h->d_tiles);
     cudaFree(h->d_tilebest);
+    cudaFree(h->d_ctiles);
+    cudaFree(h->d_ctilebest);
+    cudaFree(h->d_list);
+    cudaFree(h->d_rbox);
+    cudaFree(h->d_cbox);
     cudaFree(h->d_trace);
     cudaFree(h->d_best);
     cudaFree(h->d_mf_ws);
@@ -261,7 +295,7 @@ int load_host_tour(tsp2opt_ctx* h, const int32_t* tour)
 
 int sweep_flags(const tsp2opt_ctx* h)
 {
-    return (h->seed_next ? kSweepSeed : 0) | (h->tile_bounds ? kSweepTileBounds : 0);
+    return (h->seed_next ? kSweepSeed : 0) | (h->tile_bounds != 0 ? kSweepTileBounds : 0);
 }
 
 // One iteration: sweep (a4/a5) -> allreduce-min (a6) -> apply (a7/a8).
@@ -280,8 +314,20 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         h->ev_used += 2;
         CUDA_TRY(cudaEventRecord(ev0, h->stream));
     }
-    CUDA_TRY(launch_sweep(h->geo, h->d_P, h->d_E, h->n, h->d_tiles, h->ntiles, in, apply ? 1 : 0, h->d_tilebest,
-                          sweep_flags(h), h->stream));
+    const int tiling = h->tile_bounds == 2 ? 1 : 0;
+    if (h->seed_next && h->last_tiling != tiling) {
+        // per-tile seeds are kept per tiling: the other tiling's minima are stale
+        if (tiling) CUDA_TRY(cudaMemsetAsync(h->d_ctilebest, 0xFF, sizeof(unsigned long long) * h->nctiles, h->stream));
+        else CUDA_TRY(cudaMemsetAsync(h->d_tilebest, 0xFF, sizeof(unsigned long long) * h->ntiles, h->stream));
+    }
+    h->last_tiling = tiling;
+    if (tiling) {  // cull first, then sweep the kept tiles only
+        CUDA_TRY(launch_cull_sweep(h->cgeo, h->d_P, h->d_E, h->n, h->d_ctiles, h->nctiles, h->list_grid, h->d_rbox,
+                                   h->d_cbox, h->d_list, in, apply ? 1 : 0, h->d_ctilebest, sweep_flags(h), h->stream));
+    } else {
+        CUDA_TRY(launch_sweep(h->geo, h->d_P, h->d_E, h->n, h->d_tiles, h->ntiles, in, apply ? 1 : 0, h->d_tilebest,
+                              sweep_flags(h), h->stream));
+    }
     if (ev1) CUDA_TRY(cudaEventRecord(ev1, h->stream));
     if (h->comm) {
         ncclResult_t r = ncclAllReduce(&in->key, &in->key, 1, ncclUint64, ncclMin, h->comm, h->stream);
@@ -411,7 +457,7 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     CTRY(cudaHostAlloc(&h->h_ctl, sizeof(int), cudaHostAllocDefault));
     if (const char* ep = getenv("TSP2OPT_PERSISTENT")) h->persistent = atoi(ep);
     if (const char* es = getenv("TSP2OPT_SEED")) h->seed_next = atoi(es) != 0;
-    if (const char* eb = getenv("TSP2OPT_TILE_BOUNDS")) h->tile_bounds = atoi(eb) != 0;
+
     CTRY(cudaMemset(h->d_slots, 0, sizeof(Slot) * 2));
     {
         std::vector<float2> pad(np, make_float2(kCoordBias, kCoordBias));
@@ -421,7 +467,24 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     CTRY(sweep_prepare());
     const long long total_pairs = (long long)n * (n - 1) / 2;
     h->geo = choose_geometry(total_pairs / world);
+    // Pre-sweep cull from ~1e8 pairs per rank (measured, local search from MF: n = 85900 129 vs
+    // 221 us per iteration, n = 33810 80 vs 89 us; n = 7397 38 vs 29 us, where the extra
+    // launches cost more than the skipped tiles).
+    h->tile_bounds = total_pairs / world >= 100000000LL ? 2 : 1;
+    if (const char* eb = getenv("TSP2OPT_TILE_BOUNDS")) h->tile_bounds = std::min(2, std::max(0, atoi(eb)));
     h->all_tiles = build_tiles(n, h->geo);
+    // Culled-sweep tiling: R = 7 rows per lane and narrow column chunks (measured,
+    // local search from MF).
+    h->cgeo = Geometry{kRowsSmall, 1, total_pairs / world >= 1000000000LL ? 64 : 32};
+    if (const char* er = getenv("TSP2OPT_CULL_ROWS")) h->cgeo.rows = atoi(er) == kRowsSmall ? kRowsSmall : kRowsLarge;
+    if (const char* ec = getenv("TSP2OPT_CULL_TJ"))
+        if (atoi(ec) >= 2 && atoi(ec) <= kMaxTJ) h->cgeo.tj = atoi(ec);
+    h->all_ctiles = build_tiles(n, h->cgeo);
+    {
+        const int nrb = (n - 1 + h->cgeo.ti() - 1) / h->cgeo.ti(), ncc = (n + h->cgeo.tj - 1) / h->cgeo.tj;
+        CTRY(cudaMalloc(&h->d_rbox, sizeof(Box) * (size_t)nrb));
+        CTRY(cudaMalloc(&h->d_cbox, sizeof(Box) * (size_t)ncc));
+    }
     rc = upload_shard(h, rank, world);
     if (rc) return fail(rc);
     if (world > 1) {
@@ -709,7 +772,10 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
 {
     if (!h) return TSP2OPT_EINVAL;
     switch (option) {
-    case TSP2OPT_OPT_TILE_BOUNDS: h->tile_bounds = value != 0; break;
+    case TSP2OPT_OPT_TILE_BOUNDS:
+        if (value < 0 || value > 2) return TSP2OPT_EINVAL;
+        h->tile_bounds = (int)value;
+        break;
     case TSP2OPT_OPT_SEED: h->seed_next = value != 0; break;
     case TSP2OPT_OPT_TRACE: {
         if (value < 0) return TSP2OPT_EINVAL;

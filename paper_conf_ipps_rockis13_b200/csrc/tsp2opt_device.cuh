@@ -26,6 +26,14 @@ constexpr unsigned long long kKeyNone = ~0ULL;
 constexpr int kSweepSeed = 1;        // seed each tile with its surviving minimum of the previous sweep
 constexpr int kSweepTileBounds = 2;  // skip tiles whose bounding boxes prove that no pair passes the filter
 
+// Bounding box of a run of route positions (unbiased integer coordinates) and
+// the largest tour edge leaving it: the summaries the tile cull compares.
+struct __align__(32) Box {
+    int xlo, xhi, ylo, yhi;
+    int emax;
+    int pad[3];
+};
+
 __host__ __device__ __forceinline__ unsigned long long pack_key(int delta, int i, int j)
 {
     return ((unsigned long long)(unsigned)(delta + kDeltaBias) << kKeyDeltaShift) |
@@ -223,10 +231,11 @@ struct __align__(64) Slot {
     long long moves;              // moves applied since the tour was loaded
     long long length;             // current tour length (int64: n * 46340 > 2^31)
     int done;                     // 0 running, 1 local minimum, 2 capped, bit 2 (4): invalid tour
-    unsigned next_tile;           // (reserved)
+    unsigned next_tile;           // culled sweep: next entry of the kept-tile list to claim
     int seed_ok;                  // 1: last_key is the move just applied to the tour the tile minima of the
                                   //    previous sweep were measured on (they may seed this sweep)
-    int pad[5];
+    unsigned ncull;               // culled sweep: number of kept tiles in the list
+    int pad[4];
 };
 
 }  // namespace tsp2opt

@@ -64,6 +64,7 @@ __global__ void init_slot_kernel(Slot* slot, int clear_length)
     if (clear_length) slot->length = 0;
     slot->done = 0;
     slot->next_tile = 0;
+    slot->ncull = 0;
     slot->seed_ok = 0;  // a freshly loaded tour: no previous sweep to seed from
 }
 
@@ -107,6 +108,149 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* 
 }
 
 // ===========================================================================
+// Culled sweep (TSP2OPT_OPT_TILE_BOUNDS = 2): the tile-level bound of
+// tile_may_pass, evaluated for every tile BEFORE the sweep from per-block
+// summaries, so the sweep launches only over the tiles that survive.  A
+// spatially coherent tour (the later sweeps of a local search) keeps a few
+// percent of the tiles; visiting the others only to skip them cost most of a
+// sweep (60k one-warp CTAs at n = 85900).
+//
+// Exactness: a pair with delta < 0 has D(i,j) <= e_i - 1 or
+// D(i+1,j+1) <= e_j - 1 (otherwise delta >= 0); D(a,b) <= t <=> s <= t^2 + t.
+// Every city a pair of the tile touches (i, i+1 in the row block, j, j+1 in
+// the column chunk) lies in the block's / chunk's box, so s >= gap^2 of the
+// two boxes, and every edge it compares is <= max(emax_rows, emax_cols).  If
+// gap^2 > T^2 + T with T = max emax - 1, no pair of the tile has delta < 0,
+// and pairs with delta >= 0 never change the sweep's result (it is the min
+// over improving pairs, else the seed (0, 1, 0); reading R7).  Integer
+// arithmetic, no rounding.
+// ===========================================================================
+// One warp per summary: row block b = positions [b*TI, min(b*TI + TI, n-1))
+// (cities up to the block end + 1), column chunk c = [c*TJ, min(c*TJ + TJ, n))
+// (cities up to + 1; P[n] = P[0]).
+__global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, const int* __restrict__ E, int n,
+                                                  int TI, int nrb, int TJ, int ncc, Box* __restrict__ rbox,
+                                                  Box* __restrict__ cbox, Slot* __restrict__ slot,
+                                                  int respect_done)
+{
+    // the cull and the list sweep that follow start from zeroed counters (a
+    // best_move sweep leaves them set on the slot the next iteration reads)
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        slot->ncull = 0;
+        slot->next_tile = 0;
+    }
+    if (respect_done && *(volatile const int*)&slot->done) return;
+    const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+    int k0, ke;
+    Box* out;
+    if (w < nrb) {
+        k0 = w * TI;
+        ke = min(k0 + TI, n - 1);
+        out = rbox + w;
+    } else if (w < nrb + ncc) {
+        k0 = (w - nrb) * TJ;
+        ke = min(k0 + TJ, n);
+        out = cbox + (w - nrb);
+    } else {
+        return;  // whole warps only
+    }
+    int xlo = 1 << 30, xhi = -1, ylo = 1 << 30, yhi = -1, emax = 0;
+    // up to kBoxIters positions per lane, all loads issued before the first use
+    constexpr int kBoxIters = (32 * kRowsLarge * kMaxWarps + 1 + 31) / 32;
+#pragma unroll
+    for (int it = 0; it < kBoxIters; it++) {
+        const int k = k0 + lane + 32 * it;
+        if (k <= ke) {
+            const float2 p = P[k];
+            const int x = unbias(p.x), y = unbias(p.y);
+            xlo = min(xlo, x);
+            xhi = max(xhi, x);
+            ylo = min(ylo, y);
+            yhi = max(yhi, y);
+            if (k < ke) emax = max(emax, E[k]);
+        }
+    }
+    const unsigned full = 0xffffffffu;
+    xlo = __reduce_min_sync(full, xlo);
+    xhi = __reduce_max_sync(full, xhi);
+    ylo = __reduce_min_sync(full, ylo);
+    yhi = __reduce_max_sync(full, yhi);
+    emax = __reduce_max_sync(full, emax);
+    if (lane == 0) {
+        Box b;
+        b.xlo = xlo;
+        b.xhi = xhi;
+        b.ylo = ylo;
+        b.yhi = yhi;
+        b.emax = emax;
+        b.pad[0] = b.pad[1] = b.pad[2] = 0;
+        *out = b;
+    }
+}
+
+// One thread per tile of the shard: keep the tile iff its boxes allow a pair
+// with delta < 0; kept tile indices are appended to list[] (warp-aggregated
+// atomic on slot->ncull).  With seeding, a culled tile's minimum is "none".
+__global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tiles, int ntiles, int TI, int TJ,
+                                                   const Box* __restrict__ rbox, const Box* __restrict__ cbox,
+                                                   Slot* __restrict__ slot, int* __restrict__ list,
+                                                   unsigned long long* __restrict__ tilebest, int flags,
+                                                   int respect_done)
+{
+    if (respect_done && *(volatile int*)&slot->done) return;  // grid-uniform
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    bool keep = false;
+    if (t < ntiles) {
+        const int2 tl = tiles[t];
+        const Box r = rbox[tl.x / TI], c = cbox[tl.y / TJ];
+        const long long gx = max(0, max(c.xlo - r.xhi, r.xlo - c.xhi));
+        const long long gy = max(0, max(c.ylo - r.yhi, r.ylo - c.yhi));
+        const long long T = (long long)max(r.emax, c.emax) - 1;
+        keep = T >= 0 && gx * gx + gy * gy <= T * T + T;
+        if (!keep && (flags & kSweepSeed)) tilebest[t] = kKeyNone;
+    }
+    const unsigned m = __ballot_sync(0xffffffffu, keep);
+    if (m) {
+        const int lane = threadIdx.x & 31, leader = __ffs(m) - 1;
+        unsigned base = 0;
+        if (lane == leader) base = atomicAdd(&slot->ncull, (unsigned)__popc(m));
+        base = __shfl_sync(0xffffffffu, base, leader);
+        if (keep) list[base + __popc(m & ((1u << lane) - 1u))] = t;
+    }
+}
+
+// The sweep over the culled list: a grid of co-resident CTAs takes list
+// entries one at a time from slot->next_tile (dynamic scheduling: the kept
+// tiles of a coherent tour cluster along the diagonal, per-tile claims keep
+// the CTAs balanced) until the list is done.
+template <int R>
+__global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const float2* __restrict__ P,
+                                                                      const int* __restrict__ E, int n,
+                                                                      const int2* __restrict__ tiles,
+                                                                      const int* __restrict__ list, int TJ,
+                                                                      Slot* __restrict__ slot, int respect_done,
+                                                                      unsigned long long* __restrict__ tilebest,
+                                                                      int flags)
+{
+    extern __shared__ float4 smem[];
+    const TileSmem sm(smem, TJ);
+    __shared__ int s_t;
+    if (respect_done && *(volatile int*)&slot->done) return;
+    const unsigned count = *(volatile unsigned*)&slot->ncull;
+    for (;;) {
+        if (threadIdx.x == 0) {
+            const unsigned k = atomicAdd(&slot->next_tile, 1u);
+            s_t = k < count ? list[k] : -1;
+        }
+        __syncthreads();
+        const int t = s_t;
+        if (t < 0) break;
+        sweep_tile<R, false>(P, E, n, tiles[t], TJ, slot, sm, tilebest + t, flags);
+        __syncthreads();  // before the next tile overwrites the shared chunk (and s_t)
+    }
+}
+
+// ===========================================================================
 // a7 + a8: apply the best move of slot_in (or an explicit (i, j)) and write
 // the next iteration's state into slot_out.  Reverses P and tour on [i+1, j]
 // and e on [i+1, j-1]; the two new edges are exact distances of the
@@ -141,6 +285,7 @@ __device__ __forceinline__ bool apply_phase(float2* __restrict__ P, int* __restr
         o.length = in->length;
         o.done = explicit_move ? (done & 4) : done;  // an explicit move makes the tour unconverged
         o.next_tile = 0;
+        o.ncull = 0;
         o.seed_ok = (apply && !explicit_move) ? 1 : 0;  // tile minima of this sweep seed the next one
         if (!explicit_move && !done) {
             if (key_delta(key) >= 0) o.done = 1;        // local minimum (reading R7)
@@ -376,6 +521,11 @@ cudaError_t sweep_prepare()
         });
         if (e != cudaSuccess) return e;
         e = by_rows(R, [&](auto r) {
+            return cudaFuncSetAttribute(sweep_list_kernel<decltype(r)::value>,
+                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sweep_smem_bytes(gmax));
+        });
+        if (e != cudaSuccess) return e;
+        e = by_rows(R, [&](auto r) {
             return cudaFuncSetAttribute(local_search_kernel<decltype(r)::value>,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sweep_smem_bytes(gmax));
         });
@@ -395,6 +545,40 @@ cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n
         return 0;
     });
     g_launches += 1;
+    return cudaGetLastError();
+}
+
+int sweep_list_grid(const Geometry& g, int ntiles)
+{
+    int per_sm = 0;
+    cudaError_t e = by_rows(g.rows, [&](auto r) {
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sweep_list_kernel<decltype(r)::value>,
+                                                             32 * g.warps, sweep_smem_bytes(g));
+    });
+    if (e != cudaSuccess) return 0;
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int grid = per_sm * sms;
+    return grid < ntiles ? grid : ntiles;
+}
+
+cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles,
+                              int ntiles, int grid, Box* rbox, Box* cbox, int* list, Slot* slot, int respect_done,
+                              unsigned long long* tilebest, int flags, cudaStream_t st)
+{
+    if (ntiles <= 0 || grid <= 0) return cudaSuccess;
+    const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
+    const int warps = nrb + ncc;
+    box_kernel<<<(warps + 7) / 8, 256, 0, st>>>(P, E, n, TI, nrb, g.tj, ncc, rbox, cbox, slot, respect_done);
+    cull_kernel<<<(ntiles + 255) / 256, 256, 0, st>>>(tiles, ntiles, TI, g.tj, rbox, cbox, slot, list, tilebest,
+                                                      flags, respect_done);
+    by_rows(g.rows, [&](auto r) {
+        sweep_list_kernel<decltype(r)::value><<<grid, 32 * g.warps, sweep_smem_bytes(g), st>>>(
+            P, E, n, tiles, list, g.tj, slot, respect_done, tilebest, flags);
+        return 0;
+    });
+    g_launches += 3;
     return cudaGetLastError();
 }
 

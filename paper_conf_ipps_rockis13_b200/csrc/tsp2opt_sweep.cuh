@@ -30,7 +30,8 @@ namespace tsp2opt {
 
 #ifdef TSP2OPT_STATS
 // Instrumented builds only: [0] warp column steps, [1] steps taking the exact
-// path, [2] candidate pairs evaluated exactly.
+// path, [2] candidate pairs evaluated exactly, [3] warp tiles walked (not
+// skipped by the tile bound).
 __device__ unsigned long long g_stats[4];
 #endif
 
@@ -363,6 +364,9 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
         set_bound<R>(b, erow, dg == 0 ? 0 : dg + 1);
         const bool masked = (wrow0 + 32 * R - 1) >= jstart;  // warp-uniform: some row >= some j
         if (!(flags & kSweepTileBounds) || tile_may_pass<R>(rows, b, sm, jstart - J0, J1 - J0)) {
+#ifdef TSP2OPT_STATS
+            if (lane == 0) atomicAdd(&g_stats[3], 1ULL);
+#endif
             if (masked) walk<R, true, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
             else walk<R, false, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
         }

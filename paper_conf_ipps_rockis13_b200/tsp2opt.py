@@ -392,4 +392,4 @@ def debug_stats(reset: bool = True) -> dict:
     """Sweep counters of an instrumented build (TSP2OPT_STATS); -1 in product builds."""
     out = (ctypes.c_int64 * 4)()
     _check(_L().tsp2opt_debug_stats(out, 1 if reset else 0), "tsp2opt_debug_stats")
-    return dict(warp_steps=out[0], slow_steps=out[1], exact_pairs=out[2])
+    return dict(warp_steps=out[0], slow_steps=out[1], exact_pairs=out[2], tiles_walked=out[3])

@@ -10,11 +10,12 @@ from paper_conf_ipps_rockis13_b200 import inputs, tsp2opt
 pytestmark = pytest.mark.gpu
 
 
-@pytest.mark.parametrize("bounds", ["0", "1"])
+@pytest.mark.parametrize("bounds", ["0", "1", "2"])
 @pytest.mark.parametrize("cfg", ["C3", "C4", "C5"])
 def test_full_size_first_sweep(gpu, monkeypatch, cfg, bounds):
     """bounds = 0 is the launch configuration bench.py times for `value` (every
-    pair tested individually); 1 is the library default (tile-level bounds)."""
+    pair tested individually); 1 the in-sweep tile bounds; 2 (library default)
+    adds the pre-sweep tile cull."""
     monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", bounds)
     c, t = inputs.config_instance(cfg)
     with tsp2opt.TSP2Opt(c) as g:
@@ -46,16 +47,19 @@ def test_C5_hilbert_start_sweep(gpu):
         assert g.best_move(th) == oracle.best_move(c, th)
 
 
-@pytest.mark.parametrize("cfg,tk,nsamples", [("C3", "hilbert", 6), ("C4", "hilbert", 5), ("C5", "hilbert", 3)])
+@pytest.mark.parametrize("cfg,tk,nsamples", [("C3", "hilbert", 6), ("C4", "hilbert", 5), ("C5", "hilbert", 3),
+                                             ("C5", "mf", 3)])
 def test_full_size_local_search_trace(gpu, cfg, tk, nsamples):
     """Full local search at BASELINE.json sizes, in the default launch
     configuration: the recorded move trace replayed on the CPU reproduces the
     final tour and length; sampled iterations (first, last, evenly spaced) are
     re-swept by the oracle from the replayed tour and must give the traced
     move; the final tour carries the oracle's local-minimum certificate."""
-    c, t = inputs.config_instance(cfg, tk)
+    c, t = inputs.config_instance(cfg, "random" if tk == "mf" else tk)
     cap = 10 * len(t)
     with tsp2opt.TSP2Opt(c) as g:
+        if tk == "mf":  # the Multiple Fragment start (its own parity: tests/test_gpu_mf.py)
+            t = g.mf_tour()["tour"]
         g.set_option(tsp2opt.OPT_TRACE, cap)
         res = g.local_search(t)
         trace = g.get_trace(cap)

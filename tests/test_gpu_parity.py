@@ -50,7 +50,7 @@ def test_best_move_parity_sizes(gpu, n, kind):
         assert g.best_move(th) == oracle.best_move(c, th)
 
 
-@pytest.mark.parametrize("bounds", ["0", "1"])
+@pytest.mark.parametrize("bounds", ["0", "1", "2"])
 @pytest.mark.parametrize("rows", [7, 15])
 @pytest.mark.parametrize("warps,tj", [(1, 2), (1, 3), (1, 32), (2, 64), (4, 128), (4, 1024), (3, 7)])
 def test_best_move_parity_geometries(gpu, monkeypatch, rows, warps, tj, bounds):
@@ -92,7 +92,7 @@ def test_local_search_parity(gpu, kind, n, seed):
     c, t = _inst(kind, n, seed)
     ref = oracle.local_search(c, t)
     with tsp2opt.TSP2Opt(c) as g:
-        g.set_option(tsp2opt.OPT_TILE_BOUNDS, seed % 2)  # both filter forms over the seeds
+        g.set_option(tsp2opt.OPT_TILE_BOUNDS, seed % 3)  # every filter form over the seeds
         res = g.local_search(t)
         assert res["status"] == tsp2opt.OK
         assert res["iterations"] == ref["iterations"]
@@ -245,14 +245,16 @@ def test_local_search_parity_both_loops(gpu, monkeypatch, persistent, kind, n, s
         assert capped["status"] == want["status"] and np.array_equal(capped["tour"], want["tour"])
 
 
+@pytest.mark.parametrize("bounds", ["1", "2"])
 @pytest.mark.parametrize("rows", [7, 15])
-def test_seeded_sweeps_mixed_operations(gpu, monkeypatch, rows):
+def test_seeded_sweeps_mixed_operations(gpu, monkeypatch, rows, bounds):
     """Each sweep after a device-resident move is seeded with the previous sweep's
     surviving tile minima; interleave every operation that could make those
     stale (best_move sweeps, explicit applies, new tours, shard changes) and
     check each following sweep against the oracle."""
     monkeypatch.setenv("TSP2OPT_ROWS", str(rows))
     monkeypatch.setenv("TSP2OPT_SEED", "1")
+    monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", bounds)  # 2: culled tiles must reset their seeds
     c, t = _inst("lattice", 3001, 8)
     rng = np.random.default_rng(3)
     with tsp2opt.TSP2Opt(c) as g:
