@@ -59,6 +59,15 @@ constexpr float kCoordBias = 8388608.0f;  // 2^23
 __host__ __device__ __forceinline__ float bias_coord(int x) { return (float)(x + (1 << 23)); }
 __device__ __forceinline__ int unbias(float f) { return __float_as_int(f) - 0x4B000000; }
 
+// Programmatic dependent launch (sm_90+): a kernel launched with the PDL
+// attribute may be dispatched while its predecessor drains; pdl_wait() blocks
+// until the predecessor grid has completed and its writes are visible (a no-op
+// without the attribute), pdl_trigger() lets the successor be dispatched.  The
+// iteration kernels call both first thing, before any global access, so the
+// only overlap is launch latency and CTA dispatch -- never data.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 __device__ __forceinline__ float sqrt_approx(float x)
 {
     float r;

@@ -103,6 +103,8 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* 
 {
     extern __shared__ float4 smem[];
     const TileSmem sm(smem, TJ);
+    pdl_trigger();
+    pdl_wait();
     if (respect_done && *(volatile int*)&slot->done) return;  // converged: iteration is a no-op
     sweep_tile<R, false>(P, E, n, tiles[blockIdx.x], TJ, slot, sm, tilebest + blockIdx.x, flags);
 }
@@ -133,6 +135,8 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
                                                   Box* __restrict__ cbox, Slot* __restrict__ slot,
                                                   int respect_done)
 {
+    pdl_trigger();
+    pdl_wait();
     // the cull and the list sweep that follow start from zeroed counters (a
     // best_move sweep leaves them set on the slot the next iteration reads)
     if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -197,6 +201,8 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
                                                    unsigned long long* __restrict__ tilebest, int flags,
                                                    int respect_done)
 {
+    pdl_trigger();
+    pdl_wait();
     if (respect_done && *(volatile int*)&slot->done) return;  // grid-uniform
     const int t = blockIdx.x * blockDim.x + threadIdx.x;
     bool keep = false;
@@ -235,6 +241,8 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const flo
     extern __shared__ float4 smem[];
     const TileSmem sm(smem, TJ);
     __shared__ int s_t;
+    pdl_trigger();
+    pdl_wait();
     if (respect_done && *(volatile int*)&slot->done) return;
     const unsigned count = *(volatile unsigned*)&slot->ncull;
     for (;;) {
@@ -329,6 +337,8 @@ __global__ void __launch_bounds__(256) apply_kernel(float2* __restrict__ P, int*
                                                     unsigned long long* __restrict__ trace, long long trace_cap)
 {
     __shared__ Slot s_in;  // one read of the input state per block
+    pdl_trigger();
+    pdl_wait();
     if (threadIdx.x == 0) s_in = *in;
     __syncthreads();
     apply_phase(P, E, tour, &s_in, out, max_moves, explicit_move, ei, ej, blockIdx.x * blockDim.x + threadIdx.x,
@@ -472,6 +482,33 @@ __global__ void selftest_filter_kernel(unsigned long long* bad, unsigned long lo
 // Host-side launchers
 // ===========================================================================
 static std::atomic<long long> g_launches{0};
+
+// Launch with the programmatic-dependent-launch attribute (TSP2OPT_PDL=0
+// turns it off: plain stream order).
+static bool pdl_enabled()
+{
+    static const bool on = [] {
+        const char* e = getenv("TSP2OPT_PDL");
+        return !(e && atoi(e) == 0);
+    }();
+    return on;
+}
+template <typename... KArgs, typename... Args>
+static cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                             Args... args)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl_enabled() ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
 long long launch_count() { return g_launches.load(); }
 void count_launch(int k) { g_launches += k; }
 
@@ -539,10 +576,8 @@ cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n
 {
     if (ntiles <= 0) return cudaSuccess;
     by_rows(g.rows, [&](auto r) {
-        sweep_kernel<decltype(r)::value><<<ntiles, 32 * g.warps, sweep_smem_bytes(g), st>>>(P, E, n, tiles, g.tj,
-                                                                                            slot, respect_done, tilebest,
-                                                                                            flags);
-        return 0;
+        return launch_pdl(sweep_kernel<decltype(r)::value>, dim3(ntiles), dim3(32 * g.warps), sweep_smem_bytes(g),
+                          st, P, E, n, tiles, g.tj, slot, respect_done, tilebest, flags);
     });
     g_launches += 1;
     return cudaGetLastError();
@@ -570,16 +605,18 @@ cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, 
     if (ntiles <= 0 || grid <= 0) return cudaSuccess;
     const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
     const int warps = nrb + ncc;
-    box_kernel<<<(warps + 7) / 8, 256, 0, st>>>(P, E, n, TI, nrb, g.tj, ncc, rbox, cbox, slot, respect_done);
-    cull_kernel<<<(ntiles + 255) / 256, 256, 0, st>>>(tiles, ntiles, TI, g.tj, rbox, cbox, slot, list, tilebest,
-                                                      flags, respect_done);
-    by_rows(g.rows, [&](auto r) {
-        sweep_list_kernel<decltype(r)::value><<<grid, 32 * g.warps, sweep_smem_bytes(g), st>>>(
-            P, E, n, tiles, list, g.tj, slot, respect_done, tilebest, flags);
-        return 0;
+    cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, n, TI, nrb, g.tj, ncc, rbox,
+                               cbox, slot, respect_done);
+    if (e != cudaSuccess) return e;
+    e = launch_pdl(cull_kernel, dim3((ntiles + 255) / 256), dim3(256), 0, st, tiles, ntiles, TI, g.tj, rbox, cbox, slot,
+                   list, tilebest, flags, respect_done);
+    if (e != cudaSuccess) return e;
+    e = by_rows(g.rows, [&](auto r) {
+        return launch_pdl(sweep_list_kernel<decltype(r)::value>, dim3(grid), dim3(32 * g.warps), sweep_smem_bytes(g),
+                          st, P, E, n, tiles, list, g.tj, slot, respect_done, tilebest, flags);
     });
     g_launches += 3;
-    return cudaGetLastError();
+    return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Slot* out, long long max_moves,
@@ -589,8 +626,9 @@ cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Sl
     int blocks = (n / 2 + 255) / 256;
     if (blocks < 1) blocks = 1;
     if (blocks > 4 * 148) blocks = 4 * 148;
-    apply_kernel<<<blocks, 256, 0, st>>>(P, E, tour, in, out, max_moves, explicit_move, ei, ej, trace,
-                                         trace_cap);
+    cudaError_t e = launch_pdl(apply_kernel, dim3(blocks), dim3(256), 0, st, P, E, tour, in, out, max_moves,
+                               explicit_move, ei, ej, trace, trace_cap);
+    if (e != cudaSuccess) return e;
     g_launches += 1;
     return cudaGetLastError();
 }
