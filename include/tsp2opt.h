@@ -160,6 +160,28 @@ int tsp2opt_batch_local_search(const int32_t *coords_xy, int32_t n, int32_t batc
 int tsp2opt_batch_local_search_async(const int32_t *d_coords_xy, int32_t n, int32_t batch, int32_t *d_tours,
                                      int64_t max_iters, int64_t *d_lengths, int64_t *d_iterations, void *stream);
 
+/* Batched Iterated Local Search: `batch` independent replicas of L10
+ * Algorithm 1 ("batched multi-replica runs for n < 200";
+ * L18 §V: the paper's GPU ILS gave no speedup below 200 cities), one CTA per
+ * replica, everything in shared memory (3 <= n <= 4096).  Replica b runs
+ * exactly what tsp2opt_ils(h_b, tour_b, iterations, seeds[b]) runs (same
+ * double-bridge cuts and acceptance, readings R14-R16) on its own instance.
+ * coords_xy: host int32[batch * 2n] (replica b at offset 2n*b; repeat one
+ * instance for multi-start runs); tours: host int32[batch * n], in = start
+ * tours, out = best tours; seeds: uint64[batch]; lengths: int64[batch] best
+ * lengths; history (or NULL): int64[batch * (iterations + 1)], the best length
+ * after each step.  Errors as tsp2opt_batch_local_search; nothing is written
+ * on error. */
+int tsp2opt_batch_ils(const int32_t *coords_xy, int32_t n, int32_t batch, int32_t *tours, int64_t iterations,
+                      const uint64_t *seeds, int64_t *lengths, int64_t *history);
+
+/* The same on DEVICE buffers, enqueued on `stream`; an invalid replica (not a
+ * permutation, coordinate out of range) gets lengths[b] = -1 and keeps its
+ * tour.  The caller synchronises the stream before reading. */
+int tsp2opt_batch_ils_async(const int32_t *d_coords_xy, int32_t n, int32_t batch, int32_t *d_tours,
+                            int64_t iterations, const uint64_t *d_seeds, int64_t *d_lengths, int64_t *d_history,
+                            void *stream);
+
 /* Multiple Fragment (greedy) start tour, computed on the device (SURVEY §8(f)
  * NEXT-1; L22 §V "an initial solution based on the Multiple Fragment(Greedy)
  * heuristic[18]"; definition, tie-break and orientation: DESIGN.md R17 --

@@ -394,28 +394,6 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
     return (h->h_slot->done & 3) == 2 ? TSP2OPT_MAXITER : TSP2OPT_OK;
 }
 
-// ILS perturbation cuts (reading R16): splitmix64 output 3*it + k of `seed`
-// gives the k-th segment length 1 + out % max(1, (n-1)/3); a = l0, b = a + l1,
-// c = b + l2 (1 <= a < b < c <= n-1).
-uint64_t splitmix64_at(uint64_t seed, uint64_t k)
-{
-    uint64_t z = seed + (k + 1) * 0x9E3779B97F4A7C15ULL;
-    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
-    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
-    return z ^ (z >> 31);
-}
-
-void ils_cuts(long long n, uint64_t seed, long long it, long long* a, long long* b, long long* c)
-{
-    const unsigned long long m = (unsigned long long)std::max(1LL, (n - 1) / 3);
-    const long long l0 = 1 + (long long)(splitmix64_at(seed, 3ULL * it) % m);
-    const long long l1 = 1 + (long long)(splitmix64_at(seed, 3ULL * it + 1) % m);
-    const long long l2 = 1 + (long long)(splitmix64_at(seed, 3ULL * it + 2) % m);
-    *a = l0;
-    *b = l0 + l1;
-    *c = l0 + l1 + l2;
-}
-
 int create_common(const int32_t* xy, int32_t n, int rank, int world, const void* nccl_id, tsp2opt_t* out)
 {
     if (!out) return TSP2OPT_EINVAL;
@@ -693,6 +671,68 @@ int tsp2opt_batch_local_search_async(const int32_t* d_coords_xy, int32_t n, int3
                                                     reinterpret_cast<long long*>(d_iterations),
                                                     static_cast<cudaStream_t>(stream));
     return e == cudaSuccess ? TSP2OPT_OK : cuda_fail(e, "batch_ls_kernel");
+}
+
+int tsp2opt_batch_ils(const int32_t* coords_xy, int32_t n, int32_t batch, int32_t* tours, int64_t iterations,
+                      const uint64_t* seeds, int64_t* lengths, int64_t* history)
+{
+    if (!coords_xy || !tours || !seeds || !lengths || batch < 1 || iterations < 0) return TSP2OPT_EINVAL;
+    if (n < 3 || n > kBatchMaxN) return TSP2OPT_EINVAL;
+    for (long long b = 0; b < batch; b++) {
+        int rc = validate_coords(coords_xy + 2 * n * b, n);
+        if (rc) return rc;
+        rc = validate_tour(tours + (long long)n * b, n);
+        if (rc) return rc;
+    }
+    const size_t nxy = sizeof(int) * 2 * (size_t)n * batch, nt = sizeof(int) * (size_t)n * batch;
+    const size_t nh = history ? sizeof(long long) * (size_t)(iterations + 1) * batch : 0;
+    int* d_xy = nullptr;
+    int* d_t = nullptr;
+    unsigned long long* d_seed = nullptr;
+    long long* d_len = nullptr;
+    long long* d_hist = nullptr;
+    auto cleanup = [&]() {
+        cudaFree(d_xy);
+        cudaFree(d_t);
+        cudaFree(d_seed);
+        cudaFree(d_len);
+        cudaFree(d_hist);
+    };
+    auto fail = [&](cudaError_t e, const char* what) {
+        cleanup();
+        return cuda_fail(e, what);
+    };
+    cudaError_t e;
+    if ((e = cudaMalloc(&d_xy, nxy)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMalloc(&d_t, nt)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMalloc(&d_seed, sizeof(uint64_t) * batch)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMalloc(&d_len, sizeof(long long) * batch)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if (nh && (e = cudaMalloc(&d_hist, nh)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMemcpy(d_xy, coords_xy, nxy, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "H2D");
+    if ((e = cudaMemcpy(d_t, tours, nt, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "H2D");
+    if ((e = cudaMemcpy(d_seed, seeds, sizeof(uint64_t) * batch, cudaMemcpyHostToDevice)) != cudaSuccess)
+        return fail(e, "H2D");
+    if ((e = launch_batch_ils(d_xy, d_t, n, batch, iterations, d_seed, d_len, d_hist, nullptr)) != cudaSuccess)
+        return fail(e, "batch_ils_kernel");
+    if ((e = cudaMemcpy(tours, d_t, nt, cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
+    if ((e = cudaMemcpy(lengths, d_len, sizeof(long long) * batch, cudaMemcpyDeviceToHost)) != cudaSuccess)
+        return fail(e, "D2H");
+    if (nh && (e = cudaMemcpy(history, d_hist, nh, cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
+    cleanup();
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_batch_ils_async(const int32_t* d_coords_xy, int32_t n, int32_t batch, int32_t* d_tours,
+                            int64_t iterations, const uint64_t* d_seeds, int64_t* d_lengths, int64_t* d_history,
+                            void* stream)
+{
+    if (!d_coords_xy || !d_tours || !d_seeds || !d_lengths || batch < 1 || iterations < 0) return TSP2OPT_EINVAL;
+    if (n < 3 || n > kBatchMaxN) return TSP2OPT_EINVAL;
+    const cudaError_t e = launch_batch_ils(d_coords_xy, d_tours, n, batch, iterations,
+                                           reinterpret_cast<const unsigned long long*>(d_seeds),
+                                           reinterpret_cast<long long*>(d_lengths),
+                                           reinterpret_cast<long long*>(d_history), static_cast<cudaStream_t>(stream));
+    return e == cudaSuccess ? TSP2OPT_OK : cuda_fail(e, "batch_ils_kernel");
 }
 
 int tsp2opt_ils(tsp2opt_t h, int32_t* tour, int64_t iterations, uint64_t seed, int64_t* length, int64_t* lengths)

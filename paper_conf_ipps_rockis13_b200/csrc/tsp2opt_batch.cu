@@ -32,60 +32,24 @@ constexpr int kBatchPackedMaxN = 256;  // measured: packed wins at n = 100, ties
 // per distance, and the float delta (three roundings <= 0.008 each) exceeds the
 // exact one by at most 1.074.  delta <= B therefore implies df <= B + 1.25.
 constexpr float kBatchSlack = 1.25f;
+constexpr long long kNoMoveCap = 0x7FFFFFFFFFFFFFFFLL;
 
+// Shared state of one CTA's local search.
+struct BlockLs {
+    unsigned long long red[2][kBatchMaxThreads / 32];
+    long long len;  // current tour length
+    int bad;
+    int best[2];    // per-sweep shared bound (ping-pong)
+};
+
+// Best-improvement local search of the CTA's instance, in shared memory:
+// P[n+1] / E[n+1] / tour[n] hold a loaded tour and ls.len its length.  Runs
+// to the local minimum or max_iters moves; returns the moves applied.  All
+// threads of the CTA call it; it ends with a __syncthreads.
 template <bool PACKED>
-__global__ void __launch_bounds__(kBatchMaxThreads) batch_ls_kernel(const int* __restrict__ coords,
-                                                                    int* __restrict__ tours, int n,
-                                                                    long long max_iters,
-                                                                    long long* __restrict__ lengths,
-                                                                    long long* __restrict__ iters)
+__device__ __forceinline__ long long block_local_search(float2* P, float* E, int* tour, int n, long long max_iters, BlockLs& ls)
 {
-    extern __shared__ float2 bsm[];
-    float2* P = bsm;                                  // [n + 1] route-ordered, biased; P[n] = P[0]
-    float* E = reinterpret_cast<float*>(P + n + 1);  // [n + 1] e_k = d(k, k+1) (exact integers); E[n] pad
-    int* tour = reinterpret_cast<int*>(E + n + 1);    // [n]
-    __shared__ unsigned long long red[2][kBatchMaxThreads / 32];
-    __shared__ long long s_len;
-    __shared__ int s_bad;
-    __shared__ int s_best[2];
-    const int b = blockIdx.x, T = blockDim.x, nw = T >> 5, lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const int* xy = coords + 2LL * n * b;
-    int* gt = tours + (long long)n * b;
-    int* stamp = reinterpret_cast<int*>(E);
-
-    // load + validate (range, permutation via stamps)
-    for (int k = threadIdx.x; k <= n; k += T) stamp[k] = 0;
-    if (threadIdx.x == 0) {
-        s_bad = 0;
-        s_len = 0;
-    }
-    __syncthreads();
-    for (int k = threadIdx.x; k < n; k += T) {
-        const int c = gt[k];
-        if (c < 0 || c >= n || atomicAdd(&stamp[c], 1) != 0) {
-            s_bad = 1;
-            continue;
-        }
-        const int x = xy[2 * c], y = xy[2 * c + 1];
-        if ((unsigned)x >= (1u << 15) || (unsigned)y >= (1u << 15)) s_bad = 1;
-        tour[k] = c;
-        P[k] = make_float2(bias_coord(x), bias_coord(y));
-    }
-    __syncthreads();
-    if (s_bad) {
-        if (threadIdx.x == 0) lengths[b] = iters[b] = -1;
-        return;
-    }
-    if (threadIdx.x == 0) P[n] = P[0];
-    __syncthreads();
-    long long part = 0;
-    for (int k = threadIdx.x; k <= n; k += T) {
-        const int e = k < n ? exact_dist_biased(P[k], P[k + 1]) : 0;
-        E[k] = (float)e;
-        part += e;
-    }
-    atomicAdd((unsigned long long*)&s_len, (unsigned long long)part);
-
+    const int T = blockDim.x, nw = T >> 5, lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     // packed layout: this warp's windows and its lane's first entry
     int pk0 = 0, pk1 = 0, pi0 = 0, plim0 = 0;
     if (PACKED) {
@@ -101,7 +65,7 @@ __global__ void __launch_bounds__(kBatchMaxThreads) batch_ls_kernel(const int* _
         }
         pi0 = q;
     }
-    if (threadIdx.x == 0) s_best[0] = s_best[1] = 0;
+    if (threadIdx.x == 0) ls.best[0] = ls.best[1] = 0;
     __syncthreads();
 
     long long moves = 0;
@@ -137,8 +101,8 @@ __global__ void __launch_bounds__(kBatchMaxThreads) batch_ls_kernel(const int* _
                 if (++since >= 8) {  // share the best delta with the block (see below)
                     since = 0;
                     const int Bw = __reduce_min_sync(0xffffffffu, key_delta(key));
-                    const int Bs = *(volatile int*)&s_best[par];
-                    if (Bw < Bs && lane == 0) atomicMin(&s_best[par], Bw);
+                    const int Bs = *(volatile int*)&ls.best[par];
+                    if (Bw < Bs && lane == 0) atomicMin(&ls.best[par], Bw);
                     if (lane != 31) Bl = (float)min(Bw, Bs) + kBatchSlack;
                 }
                 i += 31;
@@ -182,8 +146,8 @@ __global__ void __launch_bounds__(kBatchMaxThreads) batch_ls_kernel(const int* _
                 // bounds the sweep's min): publish after a hit, poll every 4th diagonal
                 if (hit || (r & 3) == 3) {
                     const int Bw = __reduce_min_sync(0xffffffffu, key_delta(key));
-                    const int Bs = *(volatile int*)&s_best[par];
-                    if (Bw < Bs && lane == 0) atomicMin(&s_best[par], Bw);
+                    const int Bs = *(volatile int*)&ls.best[par];
+                    if (Bw < Bs && lane == 0) atomicMin(&ls.best[par], Bw);
                     if (lane != 31) Bl = (float)min(Bw, Bs) + kBatchSlack;
                 }
             }
@@ -193,11 +157,11 @@ __global__ void __launch_bounds__(kBatchMaxThreads) batch_ls_kernel(const int* _
             const unsigned long long v = __shfl_xor_sync(0xffffffffu, key, o);
             key = v < key ? v : key;
         }
-        if (lane == 0) red[par][w] = key;
-        __syncthreads();  // all scans done: P/E may now change; red[par] complete
-        unsigned long long best = red[par][0];
-        for (int t = 1; t < nw; t++) best = red[par][t] < best ? red[par][t] : best;
-        if (threadIdx.x == 0) s_best[par ^ 1] = 0;  // the next sweep's bound (read after the closing barrier)
+        if (lane == 0) ls.red[par][w] = key;
+        __syncthreads();  // all scans done: P/E may now change; ls.red[par] complete
+        unsigned long long best = ls.red[par][0];
+        for (int t = 1; t < nw; t++) best = ls.red[par][t] < best ? ls.red[par][t] : best;
+        if (threadIdx.x == 0) ls.best[par ^ 1] = 0;  // the next sweep's bound (read after the closing barrier)
         if (key_delta(best) >= 0 || moves >= max_iters) break;
         // reverse positions i+1..j of P and tour, edges on [i+1, j-1]; thread 0
         // owns the swap of (i+1, j), so it reads the old endpoints before writing
@@ -206,7 +170,7 @@ __global__ void __launch_bounds__(kBatchMaxThreads) batch_ls_kernel(const int* _
             const float2 pi = P[bi], pj = P[bj], pi1 = P[bi + 1], pj1 = P[bj + 1];
             E[bi] = (float)exact_dist_biased(pi, pj);
             E[bj] = (float)exact_dist_biased(pi1, pj1);
-            s_len += key_delta(best);
+            ls.len += key_delta(best);
         }
         for (int t = threadIdx.x; t < (bj - bi) / 2; t += T) {
             const int a = bi + 1 + t, c = bj - t;
@@ -226,14 +190,165 @@ __global__ void __launch_bounds__(kBatchMaxThreads) batch_ls_kernel(const int* _
         moves++;
         __syncthreads();
     }
-    for (int k = threadIdx.x; k < n; k += T) gt[k] = tour[k];
+    return moves;
+}
+
+// Load instance b (coordinates -> biased P, validated tour) into shared
+// memory and compute its edges and length.  Returns false (and reports
+// lengths[b] = iters[b] = -1) if the tour is not a permutation or a
+// coordinate is out of range.
+__device__ __forceinline__ bool block_load(const int* xy, const int* gt, int n, float2* P, float* E, int* tour, BlockLs& ls)
+{
+    const int T = blockDim.x;
+    int* stamp = reinterpret_cast<int*>(E);
+    for (int k = threadIdx.x; k <= n; k += T) stamp[k] = 0;
     if (threadIdx.x == 0) {
-        lengths[b] = s_len;
+        ls.bad = 0;
+        ls.len = 0;
+        ls.best[0] = ls.best[1] = 0;
+    }
+    __syncthreads();
+    for (int k = threadIdx.x; k < n; k += T) {
+        const int c = gt[k];
+        if (c < 0 || c >= n || atomicAdd(&stamp[c], 1) != 0) {
+            ls.bad = 1;
+            continue;
+        }
+        const int x = xy[2 * c], y = xy[2 * c + 1];
+        if ((unsigned)x >= (1u << 15) || (unsigned)y >= (1u << 15)) ls.bad = 1;
+        tour[k] = c;
+        P[k] = make_float2(bias_coord(x), bias_coord(y));
+    }
+    __syncthreads();
+    if (ls.bad) return false;  // uniform
+    if (threadIdx.x == 0) P[n] = P[0];
+    __syncthreads();
+    long long part = 0;
+    for (int k = threadIdx.x; k <= n; k += T) {
+        const int e = k < n ? exact_dist_biased(P[k], P[k + 1]) : 0;
+        E[k] = (float)e;
+        part += e;
+    }
+    atomicAdd((unsigned long long*)&ls.len, (unsigned long long)part);
+    __syncthreads();
+    return true;
+}
+
+template <bool PACKED>
+__global__ void __launch_bounds__(kBatchMaxThreads) batch_ls_kernel(const int* __restrict__ coords,
+                                                                    int* __restrict__ tours, int n,
+                                                                    long long max_iters,
+                                                                    long long* __restrict__ lengths,
+                                                                    long long* __restrict__ iters)
+{
+    extern __shared__ float2 bsm[];
+    float2* P = bsm;                                  // [n + 1] route-ordered, biased; P[n] = P[0]
+    float* E = reinterpret_cast<float*>(P + n + 1);  // [n + 1] e_k = d(k, k+1) (exact integers); E[n] pad
+    int* tour = reinterpret_cast<int*>(E + n + 1);    // [n]
+    __shared__ BlockLs ls;
+    const int b = blockIdx.x;
+    int* gt = tours + (long long)n * b;
+    if (!block_load(coords + 2LL * n * b, gt, n, P, E, tour, ls)) {
+        if (threadIdx.x == 0) lengths[b] = iters[b] = -1;
+        return;
+    }
+    const long long moves = block_local_search<PACKED>(P, E, tour, n, max_iters, ls);
+    for (int k = threadIdx.x; k < n; k += blockDim.x) gt[k] = tour[k];
+    if (threadIdx.x == 0) {
+        lengths[b] = ls.len;
         iters[b] = moves;
     }
 }
 
+// Batched Iterated Local Search (L10 Algorithm 1; SURVEY §8(f) NEXT-2
+// "batched multi-replica runs for n < 200"): one CTA per replica runs the
+// whole of Algorithm 1 in shared memory -- s* = LS(s0); `iterations` times
+// {s' = double_bridge(s*, cuts(seeds[b], t)); s*' = LS(s'); s* = s*' iff
+// strictly shorter} (readings R14-R16, the same cuts as tsp2opt_ils).
+// history (or NULL): int64[batch * (iterations + 1)], the best length after
+// each step.  The replica's coordinates are kept in shared memory by city id
+// for the re-gather after each perturbation.
+template <bool PACKED>
+__global__ void __launch_bounds__(kBatchMaxThreads) batch_ils_kernel(const int* __restrict__ coords,
+                                                                     int* __restrict__ tours, int n,
+                                                                     long long iterations,
+                                                                     const unsigned long long* __restrict__ seeds,
+                                                                     long long* __restrict__ lengths,
+                                                                     long long* __restrict__ history)
+{
+    extern __shared__ float2 bsm[];
+    float2* P = bsm;                                  // [n + 1]
+    float* E = reinterpret_cast<float*>(P + n + 1);  // [n + 1]
+    int* tour = reinterpret_cast<int*>(E + n + 1);    // [n] current tour
+    int* best = tour + n;                             // [n] s*
+    float2* C = reinterpret_cast<float2*>((reinterpret_cast<uintptr_t>(best + n) + 7) & ~uintptr_t(7));  // [n] by city id
+    __shared__ BlockLs ls;
+    __shared__ long long s_best_len;
+    const int b = blockIdx.x, T = blockDim.x;
+    const int* xy = coords + 2LL * n * b;
+    int* gt = tours + (long long)n * b;
+    long long* hist = history ? history + (iterations + 1) * b : nullptr;
+    if (!block_load(xy, gt, n, P, E, tour, ls)) {
+        if (threadIdx.x == 0) lengths[b] = -1;
+        return;
+    }
+    for (int c = threadIdx.x; c < n; c += T) C[c] = make_float2(bias_coord(xy[2 * c]), bias_coord(xy[2 * c + 1]));
+    block_local_search<PACKED>(P, E, tour, n, kNoMoveCap, ls);
+    for (int k = threadIdx.x; k < n; k += T) best[k] = tour[k];
+    if (threadIdx.x == 0) {
+        s_best_len = ls.len;
+        if (hist) hist[0] = ls.len;
+    }
+    __syncthreads();
+    const unsigned long long seed = seeds[b];
+    for (long long t = 0; t < iterations; t++) {
+        if (n >= 8) {
+            long long a, bb, c;
+            ils_cuts(n, seed, t, &a, &bb, &c);
+            // s' = A C B D of s* = A B C D, gathered with its coordinates and edges
+            for (int k = threadIdx.x; k < n; k += T) {
+                int src;
+                if (k < a || k >= c) src = k;
+                else if (k < a + (c - bb)) src = (int)(bb + (k - a));
+                else src = (int)(a + (k - a - (c - bb)));
+                const int city = best[src];
+                tour[k] = city;
+                P[k] = C[city];
+            }
+            if (threadIdx.x == 0) ls.len = 0;
+            __syncthreads();
+            if (threadIdx.x == 0) P[n] = P[0];
+            __syncthreads();
+            long long part = 0;
+            for (int k = threadIdx.x; k < n; k += T) {
+                const int e = exact_dist_biased(P[k], P[k + 1]);
+                E[k] = (float)e;
+                part += e;
+            }
+            if (threadIdx.x == 0) ls.best[0] = ls.best[1] = 0;
+            atomicAdd((unsigned long long*)&ls.len, (unsigned long long)part);
+            __syncthreads();
+            block_local_search<PACKED>(P, E, tour, n, kNoMoveCap, ls);
+            if (ls.len < s_best_len) {  // uniform: ls.len settled before the closing barrier
+                for (int k = threadIdx.x; k < n; k += T) best[k] = tour[k];
+                __syncthreads();  // everyone has read s_best_len before it changes
+                if (threadIdx.x == 0) s_best_len = ls.len;
+            }
+        }
+        if (threadIdx.x == 0 && hist) hist[t + 1] = s_best_len;
+        __syncthreads();
+    }
+    for (int k = threadIdx.x; k < n; k += T) gt[k] = best[k];
+    if (threadIdx.x == 0) lengths[b] = s_best_len;
+}
+
 size_t batch_smem_bytes(int n) { return (size_t)(n + 1) * (sizeof(float2) + sizeof(float)) + (size_t)n * sizeof(int); }
+
+// + best tour, up to 8 B of alignment, coordinates by city id
+size_t batch_ils_smem_bytes(int n)
+{
+    return batch_smem_bytes(n) + (size_t)n * sizeof(int) + 8 + (size_t)n * sizeof(float2);
+}
 
 // Packed windows waste no lanes on short diagonals; per-diagonal windows need
 // no wrap logic.  TSP2OPT_BATCH_PACKED=0/1 overrides the size rule.
@@ -261,6 +376,19 @@ cudaError_t launch_batch_local_search(const int* coords, int* tours, int n, int 
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     kern<<<batch, batch_threads(n), smem, st>>>(coords, tours, n, max_iters, lengths, iters);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_batch_ils(const int* coords, int* tours, int n, int batch, long long iterations,
+                             const unsigned long long* seeds, long long* lengths, long long* history, cudaStream_t st)
+{
+    const size_t smem = batch_ils_smem_bytes(n);
+    const bool packed = batch_packed(n);
+    auto kern = packed ? batch_ils_kernel<true> : batch_ils_kernel<false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    kern<<<batch, batch_threads(n), smem, st>>>(coords, tours, n, iterations, seeds, lengths, history);
     count_launch();
     return cudaGetLastError();
 }

@@ -214,6 +214,32 @@ __device__ __forceinline__ float2 sq2(float2 xr, float2 yr, float2 ncx, float2 n
 #endif
 }
 
+// ILS perturbation cuts (reading R16; L18 §V "a simple doublebridge move"):
+// splitmix64 output 3*it + k of `seed` gives the k-th segment length
+// 1 + out % max(1, (n-1)/3); a = l0, b = a + l1, c = b + l2
+// (1 <= a < b < c <= n-1).  Used on the host (tsp2opt_ils) and on the device
+// (batched ILS); the oracle implements the same counter-based generator on
+// its own.
+__host__ __device__ __forceinline__ uint64_t splitmix64_at(uint64_t seed, uint64_t k)
+{
+    uint64_t z = seed + (k + 1) * 0x9E3779B97F4A7C15ULL;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+    return z ^ (z >> 31);
+}
+
+__host__ __device__ __forceinline__ void ils_cuts(long long n, uint64_t seed, long long it, long long* a,
+                                                  long long* b, long long* c)
+{
+    const unsigned long long m = (unsigned long long)((n - 1) / 3 > 1 ? (n - 1) / 3 : 1);  // max(1, (n-1)/3)
+    const long long l0 = 1 + (long long)(splitmix64_at(seed, 3ULL * it) % m);
+    const long long l1 = 1 + (long long)(splitmix64_at(seed, 3ULL * it + 1) % m);
+    const long long l2 = 1 + (long long)(splitmix64_at(seed, 3ULL * it + 2) % m);
+    *a = l0;
+    *b = l0 + l1;
+    *c = l0 + l1 + l2;
+}
+
 // A pair (a, b) of the tour before the 2-opt move (i, j) -- positions i+1..j
 // reversed -- keeps its delta in the new tour iff both its edges lie on the same
 // side of the reversed segment: both outside keep their positions, both inside

@@ -30,6 +30,8 @@ constexpr int kBatchMaxN = 4096;  // batched local search: one instance per CTA,
 size_t batch_smem_bytes(int n);
 cudaError_t launch_batch_local_search(const int* coords, int* tours, int n, int batch, long long max_iters,
                                       long long* lengths, long long* iters, cudaStream_t st);
+cudaError_t launch_batch_ils(const int* coords, int* tours, int n, int batch, long long iterations,
+                             const unsigned long long* seeds, long long* lengths, long long* history, cudaStream_t st);
 // Multiple Fragment start tour (tsp2opt_mf.cu)
 constexpr int kMfK = 16;        // exact nearest neighbours kept per city
 constexpr int kMfCtr = 4;       // per-round counters, x2 parities: ends, scans, accepted, pad

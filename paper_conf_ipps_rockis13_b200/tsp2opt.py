@@ -64,6 +64,8 @@ def _L():
             "tsp2opt_batch_local_search": ([P, I32, I32, P, I64, P, P], I32),
             "tsp2opt_mf_tour": ([P, P, pI64, P], I32),
             "tsp2opt_batch_local_search_async": ([P, I32, I32, P, I64, P, P, P], I32),
+            "tsp2opt_batch_ils": ([P, I32, I32, P, I64, P, P, P], I32),
+            "tsp2opt_batch_ils_async": ([P, I32, I32, P, I64, P, P, P, P], I32),
             "tsp2opt_plan_shard": ([I32, I32, I32, pI32, pI32, pI32, P, I64, pI64, pI64], I32),
             "tsp2opt_get_geometry": ([P, pI32, pI32, pI32, pI64, pI64], I32),
             "tsp2opt_selftest": ([pI64, pI64, pI64, pI64], I32),
@@ -217,6 +219,32 @@ def batch_local_search_async(d_coords: int, n: int, batch: int, d_tours: int, d_
     _check(_L().tsp2opt_batch_local_search_async(ctypes.c_void_p(d_coords), n, batch, ctypes.c_void_p(d_tours), mi,
                                                  ctypes.c_void_p(d_lengths), ctypes.c_void_p(d_iters),
                                                  ctypes.c_void_p(stream)), "tsp2opt_batch_local_search_async")
+
+
+def batch_ils(coords, tours, iterations: int, seeds, history: bool = True):
+    """Batched Iterated Local Search, one replica per CTA: coords int32[B, n, 2],
+    tours int32[B, n], seeds uint64[B] -> dict(tours, lengths[, history int64[B, iterations+1]])."""
+    xy = _i32(coords)
+    B, n = xy.shape[0], xy.shape[1]
+    t = np.array(tours, dtype=np.int32, copy=True).reshape(B, n)
+    sd = np.ascontiguousarray(np.asarray(seeds, dtype=np.uint64).reshape(B))
+    L = np.zeros(B, dtype=np.int64)
+    hist = np.zeros((B, int(iterations) + 1), dtype=np.int64) if history else None
+    _check(_L().tsp2opt_batch_ils(_ptr(xy), n, B, _ptr(t), int(iterations), _ptr(sd), _ptr(L),
+                                  _ptr(hist) if history else None), "tsp2opt_batch_ils")
+    out = dict(tours=t, lengths=L)
+    if history:
+        out["history"] = hist
+    return out
+
+
+def batch_ils_async(d_coords: int, n: int, batch: int, d_tours: int, iterations: int, d_seeds: int, d_lengths: int,
+                    d_history: int = 0, stream: int = 0):
+    """Device-pointer form (raw addresses); see include/tsp2opt.h."""
+    _check(_L().tsp2opt_batch_ils_async(ctypes.c_void_p(d_coords), n, batch, ctypes.c_void_p(d_tours),
+                                        int(iterations), ctypes.c_void_p(d_seeds), ctypes.c_void_p(d_lengths),
+                                        ctypes.c_void_p(d_history or None), ctypes.c_void_p(stream)),
+           "tsp2opt_batch_ils_async")
 
 
 def ils(h, tour, iterations: int, seed: int):

@@ -131,10 +131,15 @@ def test_max_iters_parity(gpu):
             assert res["length"] == ref["length"] and np.array_equal(res["tour"], ref["tour"])
 
 
+@pytest.mark.parametrize("bounds", ["1", "2"])
 @pytest.mark.parametrize("world", [2, 3, 8])
-def test_simulated_shards_min_equals_full(gpu, world):
+def test_simulated_shards_min_equals_full(gpu, monkeypatch, world, bounds):
+    """Every shard's sweep, then the min over shards == the unsharded sweep ==
+    the oracle; with the culled sweep (bounds 2) the tours are spatially
+    coherent (Hilbert order) so most tiles of every shard are culled."""
+    monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", bounds)
     for kind, n in (("uniform", 1002), ("lattice", 7397)):
-        c, t = _inst(kind, n, 2)
+        c, t = _inst(kind, n, 2, "hilbert" if bounds == "2" else "random")
         with tsp2opt.TSP2Opt(c) as g:
             full = g.best_move(t)
             keys, pairs = [], 0
