@@ -220,6 +220,7 @@ def run_ours(args):
         ls = time_to_local_min(tsp2opt, args.ls_config)
         ils = time_ils(tsp2opt, args.ils_config) if args.ils_config else None
         batch = time_batch(tsp2opt, args.batch_config, not args.no_cpu) if args.batch_config else None
+        batch_ils = time_batch_ils(tsp2opt, args.batch_ils_config, not args.no_cpu) if args.batch_ils_config else None
 
     if rank == 0:
         prof = ncu_profile_summary(args.config, args.tour)
@@ -269,6 +270,8 @@ def run_ours(args):
             line["ils"] = ils
         if batch:
             line["batch_local_search"] = batch
+        if batch_ils:
+            line["batch_ils"] = batch_ils
         if world == 1 and not args.no_cpu:
             line["cpu_baseline"] = cpu_baseline(args, coords, tour, total_pairs)
         print(json.dumps(line), flush=True)
@@ -409,6 +412,65 @@ def time_batch(tsp2opt, spec, with_oracle=True):
     return out
 
 
+def time_batch_ils(tsp2opt, spec, with_oracle=True):
+    """Batched Iterated Local Search (Algorithm 1):
+    `cfg:replicas:steps` entries; multi-start on ONE instance of config cfg
+    (replica b: random start tour seed 1000+b, perturbation seed 2013+b), one
+    CTA per replica.  Device-resident (CUDA events around
+    tsp2opt_batch_ils_async) and end to end through the host API."""
+    import torch
+
+    out = []
+    for item in spec.split(","):
+        name, R, T = item.split(":")
+        R, T = int(R), int(T)
+        c, _ = inputs.config_instance(name)
+        n = len(c)
+        cs = np.repeat(np.asarray(c, dtype=np.int32)[None], R, axis=0)
+        ts = np.stack([inputs.make_tour("random", c, 1000 + b) for b in range(R)]).astype(np.int32)
+        seeds = np.arange(2013, 2013 + R, dtype=np.uint64)
+        dc, d0 = torch.from_numpy(cs).cuda(), torch.from_numpy(ts).cuda()
+        ds = torch.from_numpy(seeds.view(np.int64)).cuda()
+        dl = torch.zeros(R, dtype=torch.int64, device="cuda")
+        st = torch.cuda.current_stream()
+        dev = []
+        for rep in range(3):
+            dt_ = d0.clone()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            e0.record()
+            tsp2opt.batch_ils_async(dc.data_ptr(), n, R, dt_.data_ptr(), T, ds.data_ptr(), dl.data_ptr(),
+                                    stream=st.cuda_stream)
+            e1.record()
+            torch.cuda.synchronize()
+            if rep:
+                dev.append(e0.elapsed_time(e1) * 1e-3)
+        dev_s = float(np.median(dev))
+        t0 = time.perf_counter()
+        r = tsp2opt.batch_ils(cs, ts, T, seeds, history=False)
+        host_s = time.perf_counter() - t0
+        L = dl.cpu().numpy()
+        item_out = {"config": name, "n": n, "replicas": R, "ils_steps": T, "device_s": dev_s,
+                    "ils_steps_per_s": R * T / dev_s, "best_length": int(L.min()), "mean_length": float(L.mean()),
+                    "e2e_s": host_s, "e2e_ils_steps_per_s": R * T / host_s,
+                    "e2e_h2d_bytes": int(cs.nbytes + ts.nbytes + seeds.nbytes), "e2e_d2h_bytes": int(ts.nbytes + 8 * R),
+                    "e2e_matches_device": bool((r["lengths"] == L).all()), "gpu_launches": 1}
+        if with_oracle:
+            import oracle
+
+            k, t1 = 0, time.perf_counter()
+            steps = max(1, T // 10)
+            while k < R and time.perf_counter() - t1 < 3.0:
+                oracle.ils(c, ts[k], steps, int(seeds[k]))
+                k += 1
+            osec = time.perf_counter() - t1
+            item_out["cpu_oracle"] = {"ils_steps_per_s": k * steps / osec,
+                                      "sample": f"{k} replicas x {steps} ILS steps one after another (each "
+                                                f"includes its first local search)", "cores": oracle.num_threads()}
+        out.append(item_out)
+    return out
+
+
 # ----------------------------------------------------------------------------- oracle timing
 def cpu_baseline(args, coords, tour, total_pairs):
     import oracle
@@ -472,6 +534,7 @@ def main():
     ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert,C5:hilbert,C2:mf,C3:mf,C4:mf,C5:mf", help="configs timed to a local minimum (rank 0, N=1)")
     ap.add_argument("--ils-config", default="C1:200,C2:50", help="Iterated Local Search runs cfg:iterations")
     ap.add_argument("--batch-config", default="100:4736,1002:592", help="batched local search n:instances")
+    ap.add_argument("--batch-ils-config", default="C1:4736:100", help="batched ILS cfg:replicas:steps")
     ap.add_argument("--no-ls", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
