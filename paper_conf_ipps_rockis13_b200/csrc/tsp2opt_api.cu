@@ -79,7 +79,7 @@ struct tsp2opt_ctx {
     std::vector<Tile> all_ctiles;
     int2* d_ctiles = nullptr;   // this shard's cull tiles
     unsigned long long* d_ctilebest = nullptr;  // their per-tile minima (seeds)
-    int* d_list = nullptr;      // kept cull-tile indices [nctiles]
+    int4* d_list = nullptr;     // kept cull tiles (I0, J0, index) [nctiles]
     int nctiles = 0;
     int list_grid = 0;          // CTAs of the culled sweep (co-resident)
     int last_tiling = -1;       // tiling of the previous sweep (0 dense, 1 cull): seeds are per tiling
@@ -201,7 +201,7 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
     if (rc) return rc;
     cudaFree(h->d_list);
     h->d_list = nullptr;
-    if (h->nctiles > 0) CUDA_TRY(cudaMalloc(&h->d_list, sizeof(int) * (size_t)h->nctiles));
+    if (h->nctiles > 0) CUDA_TRY(cudaMalloc(&h->d_list, sizeof(int4) * (size_t)h->nctiles));
     h->list_grid = sweep_list_grid(h->cgeo, h->nctiles);
     h->last_tiling = -1;
     h->shard_pairs = pairs;

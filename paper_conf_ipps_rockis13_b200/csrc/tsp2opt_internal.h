@@ -53,7 +53,7 @@ cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n
 // into list / slot->ncull, then the sweep over the list with `grid` CTAs.
 int sweep_list_grid(const Geometry& g, int ntiles);
 cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles,
-                              int ntiles, int grid, Box* rbox, Box* cbox, int* list, Slot* slot, int respect_done,
+                              int ntiles, int grid, Box* rbox, Box* cbox, int4* list, Slot* slot, int respect_done,
                               unsigned long long* tilebest, int flags, cudaStream_t st);
 cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Slot* out, long long max_moves,
                          int explicit_move, int ei, int ej, unsigned long long* trace, long long trace_cap,

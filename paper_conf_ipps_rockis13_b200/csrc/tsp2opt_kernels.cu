@@ -193,11 +193,11 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
 }
 
 // One thread per tile of the shard: keep the tile iff its boxes allow a pair
-// with delta < 0; kept tile indices are appended to list[] (warp-aggregated
+// with delta < 0; kept tiles (I0, J0, index) are appended to list[] (warp-aggregated
 // atomic on slot->ncull).  With seeding, a culled tile's minimum is "none".
 __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tiles, int ntiles, int TI, int TJ,
                                                    const Box* __restrict__ rbox, const Box* __restrict__ cbox,
-                                                   Slot* __restrict__ slot, int* __restrict__ list,
+                                                   Slot* __restrict__ slot, int4* __restrict__ list,
                                                    unsigned long long* __restrict__ tilebest, int flags,
                                                    int respect_done)
 {
@@ -206,8 +206,9 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
     if (respect_done && *(volatile int*)&slot->done) return;  // grid-uniform
     const int t = blockIdx.x * blockDim.x + threadIdx.x;
     bool keep = false;
+    int2 tl = make_int2(0, 0);
     if (t < ntiles) {
-        const int2 tl = tiles[t];
+        tl = tiles[t];
         const Box r = rbox[tl.x / TI], c = cbox[tl.y / TJ];
         const long long gx = max(0, max(c.xlo - r.xhi, r.xlo - c.xhi));
         const long long gy = max(0, max(c.ylo - r.yhi, r.ylo - c.yhi));
@@ -221,39 +222,41 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
         unsigned base = 0;
         if (lane == leader) base = atomicAdd(&slot->ncull, (unsigned)__popc(m));
         base = __shfl_sync(0xffffffffu, base, leader);
-        if (keep) list[base + __popc(m & ((1u << lane) - 1u))] = t;
+        if (keep) list[base + __popc(m & ((1u << lane) - 1u))] = make_int4(tl.x, tl.y, t, 0);
     }
 }
 
 // The sweep over the culled list: a grid of co-resident CTAs takes list
-// entries one at a time from slot->next_tile (dynamic scheduling: the kept
-// tiles of a coherent tour cluster along the diagonal, per-tile claims keep
-// the CTAs balanced) until the list is done.
+// entries one at a time -- entry blockIdx.x first, then claims from
+// slot->next_tile (dynamic scheduling: the kept tiles of a coherent tour
+// cluster along the diagonal, per-tile claims keep the CTAs balanced) until
+// the list is done.
 template <int R>
 __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const float2* __restrict__ P,
                                                                       const int* __restrict__ E, int n,
                                                                       const int2* __restrict__ tiles,
-                                                                      const int* __restrict__ list, int TJ,
+                                                                      const int4* __restrict__ list, int TJ,
                                                                       Slot* __restrict__ slot, int respect_done,
                                                                       unsigned long long* __restrict__ tilebest,
                                                                       int flags)
 {
     extern __shared__ float4 smem[];
     const TileSmem sm(smem, TJ);
-    __shared__ int s_t;
+    __shared__ int4 s_t;
     pdl_trigger();
     pdl_wait();
     if (respect_done && *(volatile int*)&slot->done) return;
     const unsigned count = *(volatile unsigned*)&slot->ncull;
+    // first entry static (entry blockIdx.x: no burst of 3k atomics on one
+    // address at kernel start), then dynamic claims past the first wave
+    unsigned k = blockIdx.x;
     for (;;) {
-        if (threadIdx.x == 0) {
-            const unsigned k = atomicAdd(&slot->next_tile, 1u);
-            s_t = k < count ? list[k] : -1;
-        }
+        if (threadIdx.x == 0) s_t = k < count ? list[k] : make_int4(0, 0, -1, 0);
         __syncthreads();
-        const int t = s_t;
-        if (t < 0) break;
-        sweep_tile<R, false>(P, E, n, tiles[t], TJ, slot, sm, tilebest + t, flags);
+        const int4 e = s_t;
+        if (e.z < 0) break;
+        sweep_tile<R, false>(P, E, n, make_int2(e.x, e.y), TJ, slot, sm, tilebest + e.z, flags);
+        if (threadIdx.x == 0) k = gridDim.x + atomicAdd(&slot->next_tile, 1u);
         __syncthreads();  // before the next tile overwrites the shared chunk (and s_t)
     }
 }
@@ -599,7 +602,7 @@ int sweep_list_grid(const Geometry& g, int ntiles)
 }
 
 cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles,
-                              int ntiles, int grid, Box* rbox, Box* cbox, int* list, Slot* slot, int respect_done,
+                              int ntiles, int grid, Box* rbox, Box* cbox, int4* list, Slot* slot, int respect_done,
                               unsigned long long* tilebest, int flags, cudaStream_t st)
 {
     if (ntiles <= 0 || grid <= 0) return cudaSuccess;

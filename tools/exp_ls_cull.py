@@ -21,7 +21,7 @@ for cfg, tk in CASES:
         dt = time.perf_counter() - t0
         st = tsp2opt.debug_stats(True)
         sweeps = r["iterations"] + 1
-        st.update(cfg=cfg, start=tk, geo=geo, s=round(dt, 4), iters=r["iterations"],
+        st.update(cfg=cfg, start=tk, geo=geo, walked_per_sweep=round(st["tiles_walked"] / (r["iterations"] + 1)), s=round(dt, 4), iters=r["iterations"],
                   walked_frac=round(st["tiles_walked"] / (sweeps * geo["tiles"] * geo["warps"]), 5),
                   steps_per_sweep=round(st["warp_steps"] / sweeps), pairs_per_sweep=geo["pairs"])
         print(json.dumps(st), flush=True)
