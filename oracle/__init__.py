@@ -6,7 +6,7 @@ reference legs may import this package.  It wraps oracle/tsp2opt_oracle.c
 the CUDA path in paper_conf_ipps_rockis13_b200/.
 
 Functions mirror the C file; each cites the passage it follows there.
-Parity pins: tests/test_oracle.py.  `parity unpinned`: none.
+Parity pins: tests/test_oracle*.py (pruned neighbourhood: tests/test_oracle_pruned.py).  `parity unpinned`: none.
 """
 from __future__ import annotations
 
@@ -71,6 +71,14 @@ def _load():
             lib.oracle_ils.restype = None
             lib.oracle_mf_tour.argtypes = [p, i64, p]
             lib.oracle_mf_tour.restype = ctypes.c_int
+            lib.oracle_knn.argtypes = [p, i64, i64, p]
+            lib.oracle_knn.restype = None
+            lib.oracle_pruned_best_move_plain.argtypes = [p, i64, p, p, i64, p, p, p]
+            lib.oracle_pruned_best_move_plain.restype = None
+            lib.oracle_pruned_best_move.argtypes = [p, i64, p, p, i64, p, p, p]
+            lib.oracle_pruned_best_move.restype = None
+            lib.oracle_pruned_local_search.argtypes = [p, i64, p, i64, i64, ctypes.c_int, p, p, p, i64]
+            lib.oracle_pruned_local_search.restype = ctypes.c_int
             lib.oracle_num_threads.argtypes = []
             lib.oracle_num_threads.restype = ctypes.c_int
             _lib = lib
@@ -198,6 +206,52 @@ def mf_tour(coords) -> np.ndarray:
     if _load().oracle_mf_tour(_ptr(xy), xy.shape[0], _ptr(t)) != 0:
         raise ValueError("oracle_mf_tour: n out of range [3, 20000] or out of memory")
     return t
+
+
+def _check_k(K: int) -> int:
+    if int(K) < 1:
+        raise ValueError("K must be >= 1")
+    return int(K)
+
+
+def knn(coords, K: int) -> np.ndarray:
+    """N_K: int32[n, K] -- the K nearest cities of every city by (d, id), -1 pad
+    (reading R18; L26 §VII "neighborhood pruning")."""
+    xy = _xy(coords)
+    K = _check_k(K)
+    out = np.zeros((xy.shape[0], K), dtype=np.int32)
+    _load().oracle_knn(_ptr(xy), xy.shape[0], K, _ptr(out))
+    return out
+
+
+def pruned_best_move(coords, tour, K: int, plain: bool = False, nbr=None):
+    """(i, j, delta): best move of the K-nearest-neighbour pruned neighbourhood
+    M_K (reading R18); plain=True scans all pairs with the membership test,
+    else the O(nK) enumeration from the candidate lists."""
+    xy = _xy(coords)
+    K = _check_k(K)
+    t = np.ascontiguousarray(tour, dtype=np.int32)
+    nb = knn(xy, K) if nbr is None else np.ascontiguousarray(nbr, dtype=np.int32)
+    out = np.zeros(3, dtype=np.int64)
+    fn = _load().oracle_pruned_best_move_plain if plain else _load().oracle_pruned_best_move
+    fn(_ptr(xy), xy.shape[0], _ptr(t), _ptr(nb), K, _ptr(out[0:1]), _ptr(out[1:2]), _ptr(out[2:3]))
+    return int(out[0]), int(out[1]), int(out[2])
+
+
+def pruned_local_search(coords, tour, K: int, max_iters: int = -1, trace_cap: int = 0, plain: bool = False):
+    """Best-improvement local search over M_K; same return dict as local_search."""
+    xy = _xy(coords)
+    K = _check_k(K)
+    t = np.array(tour, dtype=np.int32, copy=True)
+    out = np.zeros(2, dtype=np.int64)
+    tr = np.zeros((max(trace_cap, 1), 3), dtype=np.int64)
+    st = _load().oracle_pruned_local_search(
+        _ptr(xy), xy.shape[0], _ptr(t), K, int(max_iters), 1 if plain else 0,
+        _ptr(out[0:1]), _ptr(out[1:2]), _ptr(tr) if trace_cap > 0 else None, int(trace_cap),
+    )
+    it = int(out[1])
+    return dict(tour=t, length=int(out[0]), iterations=it, status=int(st),
+                trace=tr[: min(it, trace_cap)].copy())
 
 
 def num_threads() -> int:

@@ -27,6 +27,11 @@
  *   oracle_local_search -- delta == full recomputation after every move,
  *                        local-minimum certificate, convex-position hull order,
  *                        brute-force global optimum is a 2-opt local minimum.
+ *   oracle_knn, oracle_pruned_* (tests/test_oracle_pruned.py) -- K nearest by
+ *                        a Python sort of (nint, id); best pruned move by brute
+ *                        force over explicitly built neighbours whose CREATED
+ *                        edges (edge-set difference) meet E_K; K >= n-1 equals
+ *                        the full oracle; list enumeration == plain scan.
  */
 #include <math.h>
 #include <stdint.h>
@@ -376,4 +381,155 @@ int oracle_num_threads(void)
 #else
     return 1;
 #endif
+}
+
+/* ---------------------------------------------------------------------------
+ * Neighbourhood-pruned best-improvement 2-opt.
+ * L18 §V: "Possibly limiting the neighborhood would also bring an improvement
+ * in efficiency"; L26 §VII: "simple ideas such as neighborhood pruning can be
+ * applied at the cost of the quality of the solution".  The paper names the
+ * idea only; reading R18 fixes the textbook K-nearest-neighbour
+ * candidate rule:
+ *   N_K(a)  = the K cities c != a with the smallest (d(a,c), c);
+ *   E_K     = { {a,c} : c in N_K(a) or a in N_K(c) };
+ *   M_K     = the 2-opt pairs (i, j), 0 <= i < j <= n-1 of the closed tour,
+ *             with {t[i], t[j]} in E_K or {t[i+1], t[j+1]} in E_K
+ *             (a move is kept iff one of the two edges it creates joins
+ *             candidate neighbours).
+ * The best move is the lowest (delta, Fig. 3 cell) over the pairs of M_K with
+ * delta < 0, else (0, 1, 0) (reading R7).  K >= n-1 gives the full
+ * neighbourhood (every pair), i.e. oracle_best_move.
+ * ------------------------------------------------------------------------- */
+
+/* N_K by plain selection: for every city, keep the K smallest (d, id) of all
+ * other cities by insertion into a sorted list.  nbr[a*K + r] = r-th nearest,
+ * -1 where n-1 < K. */
+void oracle_knn(const int32_t *xy, int64_t n, int64_t K, int32_t *nbr)
+{
+#pragma omp parallel for schedule(dynamic, 64)
+    for (int64_t a = 0; a < n; a++) {
+        int64_t *bd = (int64_t *)malloc(sizeof(int64_t) * K);
+        int32_t *bc = (int32_t *)malloc(sizeof(int32_t) * K);
+        int64_t cnt = 0;
+        for (int64_t c = 0; c < n; c++) {
+            if (c == a) continue;
+            int64_t d = oracle_dist(xy[2 * a], xy[2 * a + 1], xy[2 * c], xy[2 * c + 1]);
+            if (cnt == K && d >= bd[K - 1]) continue; /* ids ascend: (d, c) > the K-th */
+            int64_t r = cnt < K ? cnt++ : K - 1;
+            while (r > 0 && bd[r - 1] > d) { /* equal d: the earlier (lower) id stays first */
+                bd[r] = bd[r - 1];
+                bc[r] = bc[r - 1];
+                r--;
+            }
+            bd[r] = d;
+            bc[r] = (int32_t)c;
+        }
+        for (int64_t r = 0; r < K; r++) nbr[a * K + r] = r < cnt ? bc[r] : -1;
+        free(bd);
+        free(bc);
+    }
+}
+
+/* {a, c} in E_K */
+static int in_candidate_edges(const int32_t *nbr, int64_t K, int64_t a, int64_t c)
+{
+    for (int64_t r = 0; r < K; r++)
+        if (nbr[a * K + r] == c || nbr[c * K + r] == a) return 1;
+    return 0;
+}
+
+/* Plain form: every pair of the full sweep in Fig. 3 order, kept iff in M_K. */
+void oracle_pruned_best_move_plain(const int32_t *xy, int64_t n, const int32_t *tour, const int32_t *nbr,
+                                   int64_t K, int64_t *bi, int64_t *bj, int64_t *bdelta)
+{
+    int64_t best_d = 0, best_i = 0, best_j = 1;
+#pragma omp parallel
+    {
+        int64_t td = 0, ti = 0, tj = 1;
+#pragma omp for schedule(dynamic, 16) nowait
+        for (int64_t j = 1; j < n; j++) {
+            for (int64_t i = 0; i < j; i++) {
+                if (!in_candidate_edges(nbr, K, tour[i], tour[j]) &&
+                    !in_candidate_edges(nbr, K, tour[i + 1], tour[(j + 1) % n]))
+                    continue;
+                int64_t d = oracle_delta(xy, n, tour, i, j);
+                if (d < td || (d == td && oracle_cell(i, j) < oracle_cell(ti, tj))) {
+                    td = d; ti = i; tj = j;
+                }
+            }
+        }
+#pragma omp critical
+        {
+            if (td < best_d || (td == best_d && oracle_cell(ti, tj) < oracle_cell(best_i, best_j))) {
+                best_d = td; best_i = ti; best_j = tj;
+            }
+        }
+    }
+    *bi = best_i; *bj = best_j; *bdelta = best_d;
+}
+
+/* The same set M_K enumerated from the candidate lists, O(nK) per sweep: for
+ * every candidate edge {a, c} (a at position p, c at position q, u < v the two
+ * positions), the two moves that create it are
+ *   (u, v)        -- {t[i], t[j]} = {a, c}, and
+ *   (u-1, v-1)    -- {t[i+1], t[j+1]} = {a, c}; for u = 0 position 0 is
+ *                    position n of the closed tour, giving (v-1, n-1).
+ * Pinned to oracle_pruned_best_move_plain (tests/test_oracle_pruned.py). */
+void oracle_pruned_best_move(const int32_t *xy, int64_t n, const int32_t *tour, const int32_t *nbr, int64_t K,
+                             int64_t *bi, int64_t *bj, int64_t *bdelta)
+{
+    int64_t best_d = 0, best_i = 0, best_j = 1;
+    int64_t *pos = (int64_t *)malloc(sizeof(int64_t) * n);
+    for (int64_t k = 0; k < n; k++) pos[tour[k]] = k;
+    for (int64_t p = 0; p < n; p++) {
+        const int64_t a = tour[p];
+        for (int64_t r = 0; r < K; r++) {
+            const int64_t c = nbr[a * K + r];
+            if (c < 0) continue;
+            const int64_t q = pos[c];
+            const int64_t u = p < q ? p : q, v = p < q ? q : p;
+            const int64_t cand[2][2] = {{u, v}, {u >= 1 ? u - 1 : v - 1, u >= 1 ? v - 1 : n - 1}};
+            for (int m = 0; m < 2; m++) {
+                const int64_t i = cand[m][0], j = cand[m][1];
+                const int64_t d = oracle_delta(xy, n, tour, i, j);
+                if (d < best_d || (d == best_d && oracle_cell(i, j) < oracle_cell(best_i, best_j))) {
+                    best_d = d; best_i = i; best_j = j;
+                }
+            }
+        }
+    }
+    free(pos);
+    *bi = best_i; *bj = best_j; *bdelta = best_d;
+}
+
+/* Best-improvement local search over M_K (same loop, status and trace
+ * conventions as oracle_local_search).  plain != 0 uses the plain sweep. */
+int oracle_pruned_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64_t K, int64_t max_iters, int plain,
+                               int64_t *length, int64_t *iterations, int64_t *trace, int64_t trace_cap)
+{
+    int32_t *nbr = (int32_t *)malloc(sizeof(int32_t) * n * K);
+    oracle_knn(xy, n, K, nbr);
+    int64_t L = oracle_tour_length(xy, n, tour);
+    int64_t it = 0;
+    int status = 0;
+    for (;;) {
+        int64_t i, j, d;
+        if (plain) oracle_pruned_best_move_plain(xy, n, tour, nbr, K, &i, &j, &d);
+        else oracle_pruned_best_move(xy, n, tour, nbr, K, &i, &j, &d);
+        if (d >= 0) break;
+        if (max_iters >= 0 && it >= max_iters) { /* reading R8 */
+            status = 1;
+            break;
+        }
+        oracle_apply(tour, i, j);
+        L += d;
+        if (trace && it < trace_cap) {
+            trace[3 * it] = i; trace[3 * it + 1] = j; trace[3 * it + 2] = d;
+        }
+        it++;
+    }
+    free(nbr);
+    *length = L;
+    *iterations = it;
+    return status;
 }
