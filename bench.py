@@ -215,9 +215,10 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms, sweep_avg_ms, e2e_total, tb_total_ms, tb_sweep_ms = t.tolist()
 
-    ls = ils = batch = None
+    ls = ils = batch = pruned = None
     if rank == 0 and world == 1 and not args.no_ls:
         ls = time_to_local_min(tsp2opt, args.ls_config)
+        pruned = time_pruned(tsp2opt, args.pruned_config) if args.pruned_config else None
         ils = time_ils(tsp2opt, args.ils_config) if args.ils_config else None
         batch = time_batch(tsp2opt, args.batch_config, not args.no_cpu) if args.batch_config else None
         batch_ils = time_batch_ils(tsp2opt, args.batch_ils_config, not args.no_cpu) if args.batch_ils_config else None
@@ -268,6 +269,8 @@ def run_ours(args):
             line["time_to_local_minimum"] = ls
         if ils:
             line["ils"] = ils
+        if pruned:
+            line["pruned_local_search"] = pruned
         if batch:
             line["batch_local_search"] = batch
         if batch_ils:
@@ -337,6 +340,48 @@ def time_to_local_min(tsp2opt, cfg_name):
         out.append({"config": name, "n": n, "start": tk or inputs.CONFIGS[name]["tour"], "seconds": dt,
                     "iterations": r["iterations"], "length": r["length"],
                     "pair_checks_per_s": (r["iterations"] + 1) * n * (n - 1) / 2 / dt})
+    return out
+
+
+def time_pruned(tsp2opt, spec):
+    """Neighbourhood-pruned 2-opt (TSP2OPT_OPT_NEIGHBOURS = K; SURVEY §8(f)
+    NEXT-4, L26 §VII "neighborhood pruning ... at the cost of the quality";
+    reading R18) from the Multiple Fragment start, `cfg:K` entries: MF tour,
+    the local search over M_K, then the full neighbourhood continued from the
+    pruned minimum to a full 2-opt local minimum (polish); all on the device,
+    wall time of each call.  The pruned sweep kernel is timed by the library's
+    CUDA events around every sweep launch."""
+    out = []
+    for item in spec.split(","):
+        if not item:
+            continue
+        name, K = item.split(":")
+        K = int(K)
+        coords, _ = inputs.config_instance(name)
+        n = len(coords)
+        with tsp2opt.TSP2Opt(coords) as g:
+            g.mf_tour()  # warm-up: MF workspace, candidate lists, kernels
+            g.set_option(tsp2opt.OPT_NEIGHBOURS, K)
+            g.local_search_current(max_iters=2)
+            g.set_option(tsp2opt.OPT_NEIGHBOURS, 0)
+            t0 = time.perf_counter()
+            m = g.mf_tour()
+            t1 = time.perf_counter()
+            g.set_option(tsp2opt.OPT_NEIGHBOURS, K)
+            g.profile(True)
+            r = g.local_search_current()
+            t2 = time.perf_counter()
+            sweep_ms, sweeps = g.profile_read()
+            g.profile(False)
+            g.set_option(tsp2opt.OPT_NEIGHBOURS, 0)
+            f = g.local_search_current()
+            t3 = time.perf_counter()
+        out.append({"config": name, "n": n, "K": K, "start": "mf", "mf_seconds": t1 - t0, "mf_length": m["length"],
+                    "pruned_seconds": t2 - t1, "pruned_iterations": r["iterations"], "pruned_length": r["length"],
+                    "pruned_sweep_us_avg": 1e3 * sweep_ms / max(1, sweeps), "pruned_sweeps": sweeps,
+                    "candidates_per_sweep": 2 * K * n,
+                    "polish_seconds": t3 - t2, "polish_iterations": f["iterations"], "length": f["length"],
+                    "seconds": t3 - t0})
     return out
 
 
@@ -533,6 +578,7 @@ def main():
     ap.add_argument("--tour", default="random", choices=["random", "hilbert"])
     ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert,C5:hilbert,C2:mf,C3:mf,C4:mf,C5:mf", help="configs timed to a local minimum (rank 0, N=1)")
     ap.add_argument("--ils-config", default="C1:200,C2:50", help="Iterated Local Search runs cfg:iterations")
+    ap.add_argument("--pruned-config", default="C3:8,C4:8,C5:8,C5:16", help="pruned 2-opt from MF, cfg:K")
     ap.add_argument("--batch-config", default="100:4736,1002:592", help="batched local search n:instances")
     ap.add_argument("--batch-ils-config", default="C1:4736:100", help="batched ILS cfg:replicas:steps")
     ap.add_argument("--no-ls", action="store_true")

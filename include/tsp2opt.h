@@ -196,7 +196,7 @@ int tsp2opt_mf_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length, int32_t *ro
 /* Copy the current tour (host int32[n]) and its length out. */
 int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
 
-/* Execution options (none changes any result; all results stay bit-exact):
+/* Execution options (none but TSP2OPT_OPT_NEIGHBOURS changes any result; all results stay bit-exact):
  *  TSP2OPT_OPT_TILE_BOUNDS (default 2 from 1e8 pairs per rank, else 1): 1 = skip a tile of the sweep when the
  *      bounding boxes of its row and column cities prove that no pair can pass
  *      the per-pair necessary condition; 2 = the same, plus a
@@ -211,11 +211,24 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
  *  TSP2OPT_OPT_TRACE (default 0): record the (i, j, delta) of the first `value`
  *      moves applied by iterate_async / local_search since the tour was loaded
  *      (read with tsp2opt_get_trace); 0 frees the buffer.
+ *  TSP2OPT_OPT_NEIGHBOURS (default 0, at most TSP2OPT_MAX_NEIGHBOURS): K > 0
+ *      switches best_move / local_search / ils of this handle to the
+ *      neighbourhood-pruned 2-opt (L18 §V "limiting
+ *      the neighborhood", L26 §VII "neighborhood pruning ... at the cost of the
+ *      quality of the solution"; reading R18): only the moves that
+ *      create an edge {a, c} with c among the K nearest cities of a by (d, id)
+ *      or a among those of c; best = lowest (delta, Fig. 3 cell) over them,
+ *      else (0, 1, 0).  O(nK) per sweep instead of C(n,2); the result equals
+ *      oracle_pruned_best_move, not the full sweep's.  The exact candidate
+ *      lists are built on the device on first use (8 * 16 * n bytes).
+ *      0 restores the full neighbourhood.  tsp2opt_ils needs K = 0 (EINVAL).
  * Returns TSP2OPT_EINVAL for an unknown option or value. */
 #define TSP2OPT_OPT_TILE_BOUNDS 1
 #define TSP2OPT_OPT_SEED 2
 #define TSP2OPT_OPT_PERSISTENT 3
 #define TSP2OPT_OPT_TRACE 4
+#define TSP2OPT_OPT_NEIGHBOURS 5
+#define TSP2OPT_MAX_NEIGHBOURS 16
 int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value);
 
 /* Recorded move trace: writes min(count, cap) rows of int32 (i, j, delta) into

@@ -481,20 +481,31 @@ void oracle_pruned_best_move(const int32_t *xy, int64_t n, const int32_t *tour, 
     int64_t best_d = 0, best_i = 0, best_j = 1;
     int64_t *pos = (int64_t *)malloc(sizeof(int64_t) * n);
     for (int64_t k = 0; k < n; k++) pos[tour[k]] = k;
-    for (int64_t p = 0; p < n; p++) {
-        const int64_t a = tour[p];
-        for (int64_t r = 0; r < K; r++) {
-            const int64_t c = nbr[a * K + r];
-            if (c < 0) continue;
-            const int64_t q = pos[c];
-            const int64_t u = p < q ? p : q, v = p < q ? q : p;
-            const int64_t cand[2][2] = {{u, v}, {u >= 1 ? u - 1 : v - 1, u >= 1 ? v - 1 : n - 1}};
-            for (int m = 0; m < 2; m++) {
-                const int64_t i = cand[m][0], j = cand[m][1];
-                const int64_t d = oracle_delta(xy, n, tour, i, j);
-                if (d < best_d || (d == best_d && oracle_cell(i, j) < oracle_cell(best_i, best_j))) {
-                    best_d = d; best_i = i; best_j = j;
+#pragma omp parallel
+    {
+        int64_t td = 0, ti = 0, tj = 1;
+#pragma omp for schedule(static) nowait
+        for (int64_t p = 0; p < n; p++) {
+            const int64_t a = tour[p];
+            for (int64_t r = 0; r < K; r++) {
+                const int64_t c = nbr[a * K + r];
+                if (c < 0) continue;
+                const int64_t q = pos[c];
+                const int64_t u = p < q ? p : q, v = p < q ? q : p;
+                const int64_t cand[2][2] = {{u, v}, {u >= 1 ? u - 1 : v - 1, u >= 1 ? v - 1 : n - 1}};
+                for (int m = 0; m < 2; m++) {
+                    const int64_t i = cand[m][0], j = cand[m][1];
+                    const int64_t d = oracle_delta(xy, n, tour, i, j);
+                    if (d < td || (d == td && oracle_cell(i, j) < oracle_cell(ti, tj))) {
+                        td = d; ti = i; tj = j;
+                    }
                 }
+            }
+        }
+#pragma omp critical
+        {
+            if (td < best_d || (td == best_d && oracle_cell(ti, tj) < oracle_cell(best_i, best_j))) {
+                best_d = td; best_i = ti; best_j = tj;
             }
         }
     }

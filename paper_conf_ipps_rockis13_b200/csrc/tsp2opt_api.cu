@@ -18,6 +18,7 @@
 #include "tsp2opt_internal.h"
 
 using namespace tsp2opt;
+static_assert(kMaxNeighbours == TSP2OPT_MAX_NEIGHBOURS, "candidate list width");
 
 namespace {
 
@@ -87,6 +88,9 @@ struct tsp2opt_ctx {
     int* d_best = nullptr;      // [n] best tour of an ILS run
     void* d_mf_ws = nullptr;    // Multiple Fragment workspace (mf_workspace_bytes), allocated on first use
     int mf_rounds = 0;          // rounds of the last tsp2opt_mf_tour
+    int nbr_k = 0;              // TSP2OPT_OPT_NEIGHBOURS: 0 full neighbourhood, K > 0 the pruned M_K (reading R18)
+    unsigned long long* d_knn = nullptr;  // [n * kMaxNeighbours] exact nearest-neighbour keys (d << 22 | c)
+    int* d_pos = nullptr;       // [n] inverse permutation pos[tour[k]] = k (pruned sweep only)
     long long trace_cap = 0;
     Slot* h_slot = nullptr;     // pinned readback
     unsigned epoch = 0;
@@ -234,6 +238,8 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_trace);
     cudaFree(h->d_best);
     cudaFree(h->d_mf_ws);
+    cudaFree(h->d_knn);
+    cudaFree(h->d_pos);
     if (h->h_slot) cudaFreeHost(h->h_slot);
     for (cudaEvent_t e : h->ev_pool) cudaEventDestroy(e);
     if (h->own_stream) cudaStreamDestroy(h->own_stream);
@@ -281,6 +287,7 @@ int load_device_tour(tsp2opt_ctx* h, const int32_t* d_src)
     }
     CUDA_TRY(launch_load_tour(h->d_coords, d_src, h->d_tour, h->d_P, h->d_E, h->n, h->d_slots + 0, h->d_stamp,
                               h->epoch, h->stream));
+    if (h->nbr_k > 0) CUDA_TRY(launch_pos(h->d_tour, h->d_pos, h->n, h->stream));
     h->has_tour = true;
     return TSP2OPT_OK;
 }
@@ -314,14 +321,19 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         h->ev_used += 2;
         CUDA_TRY(cudaEventRecord(ev0, h->stream));
     }
-    const int tiling = h->tile_bounds == 2 ? 1 : 0;
-    if (h->seed_next && h->last_tiling != tiling) {
+    const int tiling = h->nbr_k > 0 ? 2 : h->tile_bounds == 2 ? 1 : 0;
+    if (h->seed_next && h->last_tiling != tiling && tiling < 2) {
         // per-tile seeds are kept per tiling: the other tiling's minima are stale
         if (tiling) CUDA_TRY(cudaMemsetAsync(h->d_ctilebest, 0xFF, sizeof(unsigned long long) * h->nctiles, h->stream));
         else CUDA_TRY(cudaMemsetAsync(h->d_tilebest, 0xFF, sizeof(unsigned long long) * h->ntiles, h->stream));
     }
     h->last_tiling = tiling;
-    if (tiling) {  // cull first, then sweep the kept tiles only
+    if (tiling == 2) {  // pruned neighbourhood M_K: this shard's positions, O(nK)
+        const int p0 = (int)((long long)h->n * h->shard_rank / h->shard_world);
+        const int p1 = (int)((long long)h->n * (h->shard_rank + 1) / h->shard_world);
+        CUDA_TRY(launch_pruned_sweep(h->d_P, h->d_E, h->d_tour, h->d_pos, h->d_knn, h->nbr_k, h->n, p0, p1, in,
+                                     apply ? 1 : 0, h->stream));
+    } else if (tiling) {  // cull first, then sweep the kept tiles only
         CUDA_TRY(launch_cull_sweep(h->cgeo, h->d_P, h->d_E, h->n, h->d_ctiles, h->nctiles, h->list_grid, h->d_rbox,
                                    h->d_cbox, h->d_list, in, apply ? 1 : 0, h->d_ctilebest, sweep_flags(h), h->stream));
     } else {
@@ -336,7 +348,7 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
     if (apply) {
         Slot* out = h->d_slots + (h->parity ^ 1);
         CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, max_moves, 0, 0, 0, h->d_trace,
-                              h->trace_cap, h->stream));
+                              h->trace_cap, h->nbr_k > 0 ? h->d_pos : nullptr, h->stream));
         h->parity ^= 1;
     }
     return TSP2OPT_OK;
@@ -353,7 +365,7 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
     // n ~ 7e3 where the per-sweep kernels pack tiles better); TSP2OPT_PERSISTENT
     // = 0 / 1 forces either loop, 2 (default) chooses by pair count.
     const bool use_persistent =
-        !h->comm && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
+        !h->comm && h->nbr_k == 0 && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
     if (use_persistent) {
         // One persistent cooperative launch runs sweep -> apply to the local
         // minimum; the per-launch iteration budget bounds a launch to roughly
@@ -561,7 +573,8 @@ int tsp2opt_apply(tsp2opt_t h, int32_t i, int32_t j)
     if (!h->has_tour) return TSP2OPT_ESTATE;
     Slot* in = h->d_slots + h->parity;
     Slot* out = h->d_slots + (h->parity ^ 1);
-    CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, 0, 1, i, j, nullptr, 0, h->stream));
+    CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, 0, 1, i, j, nullptr, 0,
+                          h->nbr_k > 0 ? h->d_pos : nullptr, h->stream));
     h->parity ^= 1;
     return read_slot(h);
 }
@@ -738,6 +751,10 @@ int tsp2opt_batch_ils_async(const int32_t* d_coords_xy, int32_t n, int32_t batch
 int tsp2opt_ils(tsp2opt_t h, int32_t* tour, int64_t iterations, uint64_t seed, int64_t* length, int64_t* lengths)
 {
     if (!h || !tour || !length || iterations < 0) return TSP2OPT_EINVAL;
+    if (h->nbr_k > 0) {  // ILS is defined (and pinned) on the full neighbourhood only
+        g_last_error = "tsp2opt_ils: set TSP2OPT_OPT_NEIGHBOURS to 0 first";
+        return TSP2OPT_EINVAL;
+    }
     int rc = load_host_tour(h, tour);
     if (rc) return rc;
     if (!h->d_best) CUDA_TRY(cudaMalloc(&h->d_best, sizeof(int) * (size_t)h->n));
@@ -833,6 +850,25 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
         if (value < 0 || value > 2) return TSP2OPT_EINVAL;
         h->persistent = (int)value;
         break;
+    case TSP2OPT_OPT_NEIGHBOURS: {
+        if (value < 0 || value > kMaxNeighbours) return TSP2OPT_EINVAL;
+        if (value > 0) {
+            if (!h->d_knn) {  // exact candidate lists, once per handle (coordinates never change)
+                unsigned long long* knn = nullptr;
+                CUDA_TRY(cudaMalloc(&knn, sizeof(unsigned long long) * kMaxNeighbours * (size_t)h->n));
+                h->d_knn = knn;
+                CUDA_TRY(launch_knn(h->d_coords, h->n, h->d_knn, h->stream));
+            }
+            if (!h->d_pos) CUDA_TRY(cudaMalloc(&h->d_pos, sizeof(int) * (size_t)h->n));
+            if (h->has_tour) CUDA_TRY(launch_pos(h->d_tour, h->d_pos, h->n, h->stream));
+        }
+        // the pending key may be a pair of the other neighbourhood: restart it from the seed
+        if (h->has_tour) CUDA_TRY(launch_reset_key(h->d_slots + h->parity, h->stream));
+        CUDA_TRY(cudaStreamSynchronize(h->stream));
+        h->nbr_k = (int)value;
+        h->last_tiling = -1;  // per-tile seeds of a dense sweep are stale after pruned moves
+        break;
+    }
     default: return TSP2OPT_EINVAL;
     }
     return TSP2OPT_OK;

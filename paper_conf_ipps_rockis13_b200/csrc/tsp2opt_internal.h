@@ -3,6 +3,7 @@
 #pragma once
 
 #include <atomic>
+#include <algorithm>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -26,6 +27,26 @@ struct Geometry {
 
 long long launch_count();
 void count_launch(int k = 1);
+
+// Launch with the programmatic-dependent-launch attribute (TSP2OPT_PDL=0 turns
+// it off: plain stream order).  DESIGN.md §5.3.
+bool pdl_enabled();
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_kernel_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                                     Args... args)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl_enabled() ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
 constexpr int kBatchMaxN = 4096;  // batched local search: one instance per CTA, all in shared memory
 size_t batch_smem_bytes(int n);
 cudaError_t launch_batch_local_search(const int* coords, int* tours, int n, int batch, long long max_iters,
@@ -41,6 +62,14 @@ constexpr int kMfEnd0 = 10;     // [2] the path's two ends
 constexpr int kMfCtrInts = 16;
 size_t mf_workspace_bytes(int n);
 cudaError_t launch_mf_tour(const int* coords, int n, void* ws, int* tour_out, int* rounds_out, cudaStream_t st);
+// Exact kMfK nearest neighbours of every city, keys (d << 22 | c) ascending by (d, c), ~0 pad
+cudaError_t launch_knn(const int* coords, int n, unsigned long long* knn, cudaStream_t st);
+// Neighbourhood-pruned sweep (tsp2opt_pruned.cu; reading R18): candidates of positions [p0, p1)
+constexpr int kMaxNeighbours = kMfK;
+cudaError_t launch_pruned_sweep(const float2* P, const int* E, const int* tour, const int* pos,
+                                const unsigned long long* knn, int K, int n, int p0, int p1, Slot* slot,
+                                int respect_done, cudaStream_t st);
+cudaError_t launch_pos(const int* tour, int* pos, int n, cudaStream_t st);
 size_t sweep_smem_bytes(const Geometry& g);
 cudaError_t sweep_prepare();
 cudaError_t launch_load_tour(const int* coords, const int* tour_src, int* tour_dst, float2* P, int* E, int n,
@@ -57,7 +86,7 @@ cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, 
                               unsigned long long* tilebest, int flags, cudaStream_t st);
 cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Slot* out, long long max_moves,
                          int explicit_move, int ei, int ej, unsigned long long* trace, long long trace_cap,
-                         cudaStream_t st);
+                         int* pos, cudaStream_t st);
 cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
                                 Slot* slots, int parity, long long max_moves, long long budget, unsigned* bar,
                                 int* ctl, unsigned long long* tilebest, int flags, unsigned long long* trace,

@@ -272,7 +272,8 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const flo
 __device__ __forceinline__ bool apply_phase(float2* __restrict__ P, int* __restrict__ E, int* __restrict__ tour,
                                             const Slot* __restrict__ in, Slot* __restrict__ out, long long max_moves,
                                             int explicit_move, int ei, int ej, int gtid, int stride,
-                                            unsigned long long* __restrict__ trace, long long trace_cap)
+                                            unsigned long long* __restrict__ trace, long long trace_cap,
+                                            int* __restrict__ pos)
 {
     const unsigned long long key = in->key;
     const int done = in->done;
@@ -323,6 +324,10 @@ __device__ __forceinline__ bool apply_phase(float2* __restrict__ P, int* __restr
         const int ta = __ldcg(tour + a), tc = __ldcg(tour + c);
         tour[a] = tc;
         tour[c] = ta;
+        if (pos) {  // pruned sweep: keep the inverse permutation current
+            pos[tc] = a;
+            pos[ta] = c;
+        }
     }
     const int ehalf = (j - i - 1) >> 1;  // swap e positions i+1+t <-> j-1-t
     for (int t = gtid; t < ehalf; t += stride) {
@@ -337,7 +342,8 @@ __device__ __forceinline__ bool apply_phase(float2* __restrict__ P, int* __restr
 __global__ void __launch_bounds__(256) apply_kernel(float2* __restrict__ P, int* __restrict__ E, int* __restrict__ tour,
                                                     const Slot* __restrict__ in, Slot* __restrict__ out,
                                                     long long max_moves, int explicit_move, int ei, int ej,
-                                                    unsigned long long* __restrict__ trace, long long trace_cap)
+                                                    unsigned long long* __restrict__ trace, long long trace_cap,
+                                            int* __restrict__ pos)
 {
     __shared__ Slot s_in;  // one read of the input state per block
     pdl_trigger();
@@ -345,7 +351,7 @@ __global__ void __launch_bounds__(256) apply_kernel(float2* __restrict__ P, int*
     if (threadIdx.x == 0) s_in = *in;
     __syncthreads();
     apply_phase(P, E, tour, &s_in, out, max_moves, explicit_move, ei, ej, blockIdx.x * blockDim.x + threadIdx.x,
-                gridDim.x * blockDim.x, trace, trace_cap);
+                gridDim.x * blockDim.x, trace, trace_cap, pos);
 }
 
 // ===========================================================================
@@ -382,7 +388,8 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
                                                            long long budget, unsigned* __restrict__ bar,
                                                            int* __restrict__ ctl,
                                                            unsigned long long* __restrict__ tilebest, int flags,
-                                                           unsigned long long* __restrict__ trace, long long trace_cap)
+                                                           unsigned long long* __restrict__ trace, long long trace_cap,
+                                            int* __restrict__ pos)
 {
     extern __shared__ float4 smem[];
     const TileSmem sm(smem, TJ);
@@ -411,7 +418,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
             s_in.seed_ok = *(volatile int*)&in->seed_ok;
         }
         __syncthreads();
-        apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride, trace, trace_cap);
+        apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride, trace, trace_cap, nullptr);
         p ^= 1;
         grid_sync(bar, gridDim.x);
     }
@@ -486,9 +493,7 @@ __global__ void selftest_filter_kernel(unsigned long long* bad, unsigned long lo
 // ===========================================================================
 static std::atomic<long long> g_launches{0};
 
-// Launch with the programmatic-dependent-launch attribute (TSP2OPT_PDL=0
-// turns it off: plain stream order).
-static bool pdl_enabled()
+bool pdl_enabled()
 {
     static const bool on = [] {
         const char* e = getenv("TSP2OPT_PDL");
@@ -500,17 +505,7 @@ template <typename... KArgs, typename... Args>
 static cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
                              Args... args)
 {
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = grid;
-    cfg.blockDim = block;
-    cfg.dynamicSmemBytes = smem;
-    cfg.stream = st;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    attr[0].val.programmaticStreamSerializationAllowed = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = pdl_enabled() ? 1 : 0;
-    return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+    return launch_kernel_pdl(kernel, grid, block, smem, st, args...);
 }
 long long launch_count() { return g_launches.load(); }
 void count_launch(int k) { g_launches += k; }
@@ -624,13 +619,13 @@ cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, 
 
 cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Slot* out, long long max_moves,
                          int explicit_move, int ei, int ej, unsigned long long* trace, long long trace_cap,
-                         cudaStream_t st)
+                         int* pos, cudaStream_t st)
 {
     int blocks = (n / 2 + 255) / 256;
     if (blocks < 1) blocks = 1;
     if (blocks > 4 * 148) blocks = 4 * 148;
     cudaError_t e = launch_pdl(apply_kernel, dim3(blocks), dim3(256), 0, st, P, E, tour, in, out, max_moves,
-                               explicit_move, ei, ej, trace, trace_cap);
+                               explicit_move, ei, ej, trace, trace_cap, pos);
     if (e != cudaSuccess) return e;
     g_launches += 1;
     return cudaGetLastError();

@@ -284,6 +284,13 @@ struct MfLayout {
 
 size_t mf_workspace_bytes(int n) { return MfLayout(n).total; }
 
+cudaError_t launch_knn(const int* coords, int n, unsigned long long* knn, cudaStream_t st)
+{
+    knn_kernel<<<blocks(n, kKnnThreads), kKnnThreads, 0, st>>>(coords, n, knn);
+    count_launch(1);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_mf_tour(const int* coords, int n, void* ws, int* tour_out, int* rounds_out, cudaStream_t st)
 {
     const MfLayout L(n);

@@ -265,7 +265,8 @@ def get_tour(h, n: int):
     return t, L.value
 
 
-OPT_TILE_BOUNDS, OPT_SEED, OPT_PERSISTENT, OPT_TRACE = 1, 2, 3, 4
+OPT_TILE_BOUNDS, OPT_SEED, OPT_PERSISTENT, OPT_TRACE, OPT_NEIGHBOURS = 1, 2, 3, 4, 5
+MAX_NEIGHBOURS = 16  # TSP2OPT_MAX_NEIGHBOURS
 
 
 def set_option(h, option: int, value: int) -> None:
