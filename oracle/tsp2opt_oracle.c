@@ -32,6 +32,11 @@
  *                        force over explicitly built neighbours whose CREATED
  *                        edges (edge-set difference) meet E_K; K >= n-1 equals
  *                        the full oracle; list enumeration == plain scan.
+ *   oracle25_* (tests/test_oracle_25opt.py) -- 2.5-opt: brute force over
+ *                        neighbours built from the move's wording with list
+ *                        operations on city ids; the neighbourhood as a set of
+ *                        cycles == 2-opt neighbours + node insertions; the
+ *                        sweep == the per-move definition; global optima.
  */
 #include <math.h>
 #include <stdint.h>
@@ -540,6 +545,138 @@ int oracle_pruned_local_search(const int32_t *xy, int64_t n, int32_t *tour, int6
         it++;
     }
     free(nbr);
+    *length = L;
+    *iterations = it;
+    return status;
+}
+
+/* ---------------------------------------------------------------------------
+ * 2.5-opt (2h-opt): best-improvement 2-opt plus node insertion (SURVEY.md
+ * §8(f) NEXT-4).  L26 §VII: "Our future work is to efficiently implement more
+ * complex local search algorithms such as 2.5-opt"; the paper gives no
+ * definition, so reading R19 takes the textbook 2h-opt
+ * neighbourhood over the same pairs 0 <= i < j <= n-1 of the closed tour as
+ * the 2-opt sweep (reading R1), three moves per pair:
+ *   type 0  the 2-opt move (reverse positions i+1..j);
+ *   type 1  (j >= i+2) move city t[i+1] between t[j] and t[j+1]:
+ *           delta = d(t_i, t_{i+2}) - e_i - e_{i+1} + d(t_j, t_{i+1}) + d(t_{i+1}, t_{j+1}) - e_j;
+ *   type 2  (j >= i+2) move city t[j] between t[i] and t[i+1]:
+ *           delta = d(t_{j-1}, t_{j+1}) - e_{j-1} - e_j + d(t_i, t_j) + d(t_j, t_{i+1}) - e_i.
+ * Best = the lowest (delta, Fig. 3 cell, type) with delta < 0, else
+ * (0, 1, type 0, delta 0).  Positions i+1..j are the only ones that move:
+ * type 1 rotates them left by one, type 2 right by one, so t[0] never moves
+ * (reading R6) and every city but t[0] can be inserted into every edge that
+ * does not touch it.
+ * ------------------------------------------------------------------------- */
+int64_t oracle25_delta(const int32_t *xy, int64_t n, const int32_t *tour, int64_t i, int64_t j, int type)
+{
+    if (type == 0) return oracle_delta(xy, n, tour, i, j);
+    if (j < i + 2) return INT64_MAX; /* not a move */
+    if (type == 1)
+        return dpos(xy, tour, n, i, i + 2) - dpos(xy, tour, n, i, i + 1) - dpos(xy, tour, n, i + 1, i + 2)
+             + dpos(xy, tour, n, j, i + 1) + dpos(xy, tour, n, i + 1, j + 1) - dpos(xy, tour, n, j, j + 1);
+    return dpos(xy, tour, n, j - 1, j + 1) - dpos(xy, tour, n, j - 1, j) - dpos(xy, tour, n, j, j + 1)
+         + dpos(xy, tour, n, i, j) + dpos(xy, tour, n, j, i + 1) - dpos(xy, tour, n, i, i + 1);
+}
+
+/* One exhaustive 2.5-opt sweep.  Same terms as oracle25_delta, computed once
+ * per sweep: route-ordered coordinates, edges e_k and removal gains
+ * g_k = d(t_{k-1}, t_{k+1}) - e_{k-1} - e_k; per pair the three distances
+ * d(i,j), d(i+1,j+1), d(i+1,j).  Pinned to oracle25_delta and to a brute
+ * force over explicitly built neighbours (tests/test_oracle_25opt.py). */
+void oracle25_best_move(const int32_t *xy, int64_t n, const int32_t *tour,
+                        int64_t *bi, int64_t *bj, int64_t *btype, int64_t *bdelta)
+{
+    int64_t best_d = 0, best_i = 0, best_j = 1, best_t = 0;
+    int64_t *px = (int64_t *)malloc(sizeof(int64_t) * (n + 1));
+    int64_t *py = (int64_t *)malloc(sizeof(int64_t) * (n + 1));
+    int64_t *e = (int64_t *)malloc(sizeof(int64_t) * n);
+    int64_t *g = (int64_t *)malloc(sizeof(int64_t) * n);
+    for (int64_t k = 0; k <= n; k++) {
+        int64_t c = tour[k % n];
+        px[k] = xy[2 * c];
+        py[k] = xy[2 * c + 1];
+    }
+    for (int64_t k = 0; k < n; k++) e[k] = oracle_dist(px[k], py[k], px[k + 1], py[k + 1]);
+    for (int64_t k = 0; k < n; k++) {
+        int64_t km = (k + n - 1) % n;
+        g[k] = oracle_dist(px[km], py[km], px[k + 1], py[k + 1]) - e[km] - e[k];
+    }
+#pragma omp parallel
+    {
+        int64_t td = 0, ti = 0, tj = 1, tt = 0;
+#pragma omp for schedule(dynamic, 16) nowait
+        for (int64_t j = 1; j < n; j++) {
+            for (int64_t i = 0; i < j; i++) {
+                const int64_t dij = oracle_dist(px[i], py[i], px[j], py[j]);
+                const int64_t di1j1 = oracle_dist(px[i + 1], py[i + 1], px[j + 1], py[j + 1]);
+                int64_t d[3] = {dij + di1j1 - e[i] - e[j], INT64_MAX, INT64_MAX};
+                if (j >= i + 2) {
+                    const int64_t di1j = oracle_dist(px[i + 1], py[i + 1], px[j], py[j]);
+                    d[1] = g[i + 1] + di1j + di1j1 - e[j];
+                    d[2] = g[j] + dij + di1j - e[i];
+                }
+                for (int t = 0; t < 3; t++) {
+                    /* visiting (cell, type) in increasing order: strict '<' keeps the lowest */
+                    if (d[t] < td || (d[t] == td && (oracle_cell(i, j) < oracle_cell(ti, tj) ||
+                                                     (oracle_cell(i, j) == oracle_cell(ti, tj) && t < tt)))) {
+                        td = d[t]; ti = i; tj = j; tt = t;
+                    }
+                }
+            }
+        }
+#pragma omp critical
+        {
+            if (td < best_d || (td == best_d && (oracle_cell(ti, tj) < oracle_cell(best_i, best_j) ||
+                                                 (oracle_cell(ti, tj) == oracle_cell(best_i, best_j) && tt < best_t)))) {
+                best_d = td; best_i = ti; best_j = tj; best_t = tt;
+            }
+        }
+    }
+    free(px); free(py); free(e); free(g);
+    *bi = best_i; *bj = best_j; *btype = best_t; *bdelta = best_d;
+}
+
+/* Apply move (i, j, type): type 0 reverses positions i+1..j; type 1 moves
+ * t[i+1] to position j (positions i+2..j shift left); type 2 moves t[j] to
+ * position i+1 (positions i+1..j-1 shift right). */
+void oracle25_apply(int32_t *tour, int64_t i, int64_t j, int type)
+{
+    if (type == 0) {
+        oracle_apply(tour, i, j);
+    } else if (type == 1) {
+        int32_t c = tour[i + 1];
+        for (int64_t k = i + 1; k < j; k++) tour[k] = tour[k + 1];
+        tour[j] = c;
+    } else {
+        int32_t c = tour[j];
+        for (int64_t k = j; k > i + 1; k--) tour[k] = tour[k - 1];
+        tour[i + 1] = c;
+    }
+}
+
+/* Best-improvement 2.5-opt local search; trace rows (i, j, delta, type). */
+int oracle25_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64_t max_iters,
+                          int64_t *length, int64_t *iterations, int64_t *trace, int64_t trace_cap)
+{
+    int64_t L = oracle_tour_length(xy, n, tour);
+    int64_t it = 0;
+    int status = 0;
+    for (;;) {
+        int64_t i, j, t, d;
+        oracle25_best_move(xy, n, tour, &i, &j, &t, &d);
+        if (d >= 0) break;
+        if (max_iters >= 0 && it >= max_iters) { /* reading R8 */
+            status = 1;
+            break;
+        }
+        oracle25_apply(tour, i, j, (int)t);
+        L += d;
+        if (trace && it < trace_cap) {
+            trace[4 * it] = i; trace[4 * it + 1] = j; trace[4 * it + 2] = d; trace[4 * it + 3] = t;
+        }
+        it++;
+    }
     *length = L;
     *iterations = it;
     return status;
