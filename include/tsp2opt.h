@@ -222,6 +222,19 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
  *      oracle_pruned_best_move, not the full sweep's.  The exact candidate
  *      lists are built on the device on first use (8 * 16 * n bytes).
  *      0 restores the full neighbourhood.  tsp2opt_ils needs K = 0 (EINVAL).
+ *  TSP2OPT_OPT_NODE_INSERTION (default 0): 1 switches best_move / apply /
+ *      iterate_async / local_search to best-improvement 2.5-opt (SURVEY.md
+ *      §8(f) NEXT-4; L26 §VII "more complex local search algorithms such as
+ *      2.5-opt"; reading R19): per pair 0 <= i < j <= n-1 three
+ *      moves -- type 0 the 2-opt move, type 1 (j >= i+2) city t[i+1] into the
+ *      edge (t[j], t[j+1]), type 2 (j >= i+2) city t[j] into the edge
+ *      (t[i], t[i+1]); best = lowest (delta, Fig. 3 cell, type), else
+ *      (0, 1, 0).  best_move reports (i, j, delta) and its type is the lowest
+ *      reaching delta at (i, j) (tsp2opt_best_move_typed reports it).  Type 1
+ *      rotates positions i+1..j left by one, type 2 right by one; t[0] never
+ *      moves.  Results equal oracle25_*.  Not with TSP2OPT_OPT_NEIGHBOURS > 0
+ *      (EINVAL) or tsp2opt_ils; the sweep uses R = 7 rows per lane and the
+ *      per-tile bound (no pre-sweep cull, no persistent loop).
  * Returns TSP2OPT_EINVAL for an unknown option or value. */
 #define TSP2OPT_OPT_TILE_BOUNDS 1
 #define TSP2OPT_OPT_SEED 2
@@ -229,6 +242,7 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
 #define TSP2OPT_OPT_TRACE 4
 #define TSP2OPT_OPT_NEIGHBOURS 5
 #define TSP2OPT_MAX_NEIGHBOURS 16
+#define TSP2OPT_OPT_NODE_INSERTION 6
 int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value);
 
 /* Recorded move trace: writes min(count, cap) rows of int32 (i, j, delta) into
@@ -236,6 +250,17 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value);
 int tsp2opt_get_trace(tsp2opt_t h, int32_t *ijd, int64_t cap, int64_t *count);
 
 /* Diagnostics / test hooks ------------------------------------------------ */
+
+/* 2.5-opt companions of best_move / apply / get_trace (TSP2OPT_OPT_NODE_INSERTION;
+ * reading R19).  best_move_typed also reports the move type (always 0 for
+ * 2-opt handles).  apply_typed applies move (i, j, type): type 0 is
+ * tsp2opt_apply; types 1 and 2 need the 2.5-opt mode and 0 <= i, i+2 <= j < n
+ * (else EINVAL).  get_trace_typed writes rows of int32 (i, j, delta, type)
+ * into ijdt (int32[4*cap]); *count as tsp2opt_get_trace. */
+int tsp2opt_best_move_typed(tsp2opt_t h, const int32_t *tour, int32_t *i, int32_t *j, int32_t *type,
+                            int32_t *delta);
+int tsp2opt_apply_typed(tsp2opt_t h, int32_t i, int32_t j, int32_t type);
+int tsp2opt_get_trace_typed(tsp2opt_t h, int32_t *ijdt, int64_t cap, int64_t *count);
 
 /* Restrict this handle's sweep to shard `rank` of `world` of the tile space
  * WITHOUT any collective (world = 1 restores the full sweep).  Used to check on

@@ -91,6 +91,10 @@ struct tsp2opt_ctx {
     int nbr_k = 0;              // TSP2OPT_OPT_NEIGHBOURS: 0 full neighbourhood, K > 0 the pruned M_K (reading R18)
     unsigned long long* d_knn = nullptr;  // [n * kMaxNeighbours] exact nearest-neighbour keys (d << 22 | c)
     int* d_pos = nullptr;       // [n] inverse permutation pos[tour[k]] = k (pruned sweep only)
+    int or25 = 0;               // TSP2OPT_OPT_NODE_INSERTION: 1 = 2.5-opt (2-opt plus node insertion, reading R19)
+    int* d_G = nullptr;         // [n + 1 + pad] removal gains g_k (2.5-opt only)
+    unsigned* d_bar25 = nullptr;  // [2] grid barrier of the 2.5-opt apply
+    int* d_ttype = nullptr;     // [trace_cap] move types of the traced moves (2.5-opt)
     long long trace_cap = 0;
     Slot* h_slot = nullptr;     // pinned readback
     unsigned epoch = 0;
@@ -240,6 +244,9 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_mf_ws);
     cudaFree(h->d_knn);
     cudaFree(h->d_pos);
+    cudaFree(h->d_G);
+    cudaFree(h->d_bar25);
+    cudaFree(h->d_ttype);
     if (h->h_slot) cudaFreeHost(h->h_slot);
     for (cudaEvent_t e : h->ev_pool) cudaEventDestroy(e);
     if (h->own_stream) cudaStreamDestroy(h->own_stream);
@@ -288,6 +295,7 @@ int load_device_tour(tsp2opt_ctx* h, const int32_t* d_src)
     CUDA_TRY(launch_load_tour(h->d_coords, d_src, h->d_tour, h->d_P, h->d_E, h->n, h->d_slots + 0, h->d_stamp,
                               h->epoch, h->stream));
     if (h->nbr_k > 0) CUDA_TRY(launch_pos(h->d_tour, h->d_pos, h->n, h->stream));
+    if (h->or25) CUDA_TRY(launch_gain(h->d_P, h->d_G, h->n, 0, h->n - 1, h->stream));
     h->has_tour = true;
     return TSP2OPT_OK;
 }
@@ -321,14 +329,17 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         h->ev_used += 2;
         CUDA_TRY(cudaEventRecord(ev0, h->stream));
     }
-    const int tiling = h->nbr_k > 0 ? 2 : h->tile_bounds == 2 ? 1 : 0;
+    const int tiling = h->or25 ? 3 : h->nbr_k > 0 ? 2 : h->tile_bounds == 2 ? 1 : 0;
     if (h->seed_next && h->last_tiling != tiling && tiling < 2) {
         // per-tile seeds are kept per tiling: the other tiling's minima are stale
         if (tiling) CUDA_TRY(cudaMemsetAsync(h->d_ctilebest, 0xFF, sizeof(unsigned long long) * h->nctiles, h->stream));
         else CUDA_TRY(cudaMemsetAsync(h->d_tilebest, 0xFF, sizeof(unsigned long long) * h->ntiles, h->stream));
     }
     h->last_tiling = tiling;
-    if (tiling == 2) {  // pruned neighbourhood M_K: this shard's positions, O(nK)
+    if (tiling == 3) {  // 2.5-opt: dense tiling (R = 7), per-tile bound unless TILE_BOUNDS = 0
+        CUDA_TRY(launch_sweep25(h->geo, h->d_P, h->d_E, h->d_G, h->n, h->d_tiles, h->ntiles, in, apply ? 1 : 0,
+                                h->tile_bounds != 0 ? kSweepTileBounds : 0, h->stream));
+    } else if (tiling == 2) {  // pruned neighbourhood M_K: this shard's positions, O(nK)
         const int p0 = (int)((long long)h->n * h->shard_rank / h->shard_world);
         const int p1 = (int)((long long)h->n * (h->shard_rank + 1) / h->shard_world);
         CUDA_TRY(launch_pruned_sweep(h->d_P, h->d_E, h->d_tour, h->d_pos, h->d_knn, h->nbr_k, h->n, p0, p1, in,
@@ -345,7 +356,12 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         ncclResult_t r = ncclAllReduce(&in->key, &in->key, 1, ncclUint64, ncclMin, h->comm, h->stream);
         if (r != ncclSuccess) return nccl_fail(r, "ncclAllReduce");
     }
-    if (apply) {
+    if (apply && h->or25) {
+        Slot* out = h->d_slots + (h->parity ^ 1);
+        CUDA_TRY(launch_apply25(h->d_P, h->d_E, h->d_G, h->d_tour, h->n, in, out, max_moves, 0, 0, 0, 0, h->d_trace,
+                                h->d_ttype, h->trace_cap, h->d_bar25, h->stream));
+        h->parity ^= 1;
+    } else if (apply) {
         Slot* out = h->d_slots + (h->parity ^ 1);
         CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, max_moves, 0, 0, 0, h->d_trace,
                               h->trace_cap, h->nbr_k > 0 ? h->d_pos : nullptr, h->stream));
@@ -365,7 +381,7 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
     // n ~ 7e3 where the per-sweep kernels pack tiles better); TSP2OPT_PERSISTENT
     // = 0 / 1 forces either loop, 2 (default) chooses by pair count.
     const bool use_persistent =
-        !h->comm && h->nbr_k == 0 && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
+        !h->comm && h->nbr_k == 0 && !h->or25 && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
     if (use_persistent) {
         // One persistent cooperative launch runs sweep -> apply to the local
         // minimum; the per-launch iteration budget bounds a launch to roughly
@@ -455,6 +471,7 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     }
     CTRY(cudaMemcpy(h->d_coords, xy, sizeof(int) * 2 * (size_t)n, cudaMemcpyHostToDevice));
     CTRY(sweep_prepare());
+    CTRY(sweep25_prepare());
     const long long total_pairs = (long long)n * (n - 1) / 2;
     h->geo = choose_geometry(total_pairs / world);
     // Pre-sweep cull from ~1e8 pairs per rank (measured, local search from MF: n = 85900 129 vs
@@ -573,8 +590,12 @@ int tsp2opt_apply(tsp2opt_t h, int32_t i, int32_t j)
     if (!h->has_tour) return TSP2OPT_ESTATE;
     Slot* in = h->d_slots + h->parity;
     Slot* out = h->d_slots + (h->parity ^ 1);
-    CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, 0, 1, i, j, nullptr, 0,
-                          h->nbr_k > 0 ? h->d_pos : nullptr, h->stream));
+    if (h->or25)
+        CUDA_TRY(launch_apply25(h->d_P, h->d_E, h->d_G, h->d_tour, h->n, in, out, 0, 1, i, j, 0, nullptr, nullptr, 0,
+                                h->d_bar25, h->stream));
+    else
+        CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, 0, 1, i, j, nullptr, 0,
+                              h->nbr_k > 0 ? h->d_pos : nullptr, h->stream));
     h->parity ^= 1;
     return read_slot(h);
 }
@@ -751,8 +772,8 @@ int tsp2opt_batch_ils_async(const int32_t* d_coords_xy, int32_t n, int32_t batch
 int tsp2opt_ils(tsp2opt_t h, int32_t* tour, int64_t iterations, uint64_t seed, int64_t* length, int64_t* lengths)
 {
     if (!h || !tour || !length || iterations < 0) return TSP2OPT_EINVAL;
-    if (h->nbr_k > 0) {  // ILS is defined (and pinned) on the full neighbourhood only
-        g_last_error = "tsp2opt_ils: set TSP2OPT_OPT_NEIGHBOURS to 0 first";
+    if (h->nbr_k > 0 || h->or25) {  // ILS is defined (and pinned) on the full 2-opt neighbourhood only
+        g_last_error = "tsp2opt_ils: set TSP2OPT_OPT_NEIGHBOURS and TSP2OPT_OPT_NODE_INSERTION to 0 first";
         return TSP2OPT_EINVAL;
     }
     int rc = load_host_tour(h, tour);
@@ -838,10 +859,14 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
         if (value < 0) return TSP2OPT_EINVAL;
         CUDA_TRY(cudaStreamSynchronize(h->stream));
         cudaFree(h->d_trace);
+        cudaFree(h->d_ttype);
         h->d_trace = nullptr;
+        h->d_ttype = nullptr;
         h->trace_cap = 0;
         if (value > 0) {
             CUDA_TRY(cudaMalloc(&h->d_trace, sizeof(unsigned long long) * (size_t)value));
+            CUDA_TRY(cudaMalloc(&h->d_ttype, sizeof(int) * (size_t)value));
+            CUDA_TRY(cudaMemset(h->d_ttype, 0, sizeof(int) * (size_t)value));
             h->trace_cap = value;
         }
         break;
@@ -850,8 +875,37 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
         if (value < 0 || value > 2) return TSP2OPT_EINVAL;
         h->persistent = (int)value;
         break;
+    case TSP2OPT_OPT_NODE_INSERTION: {
+        if (value < 0 || value > 1 || (value && h->nbr_k > 0)) return TSP2OPT_EINVAL;
+        CUDA_TRY(cudaStreamSynchronize(h->stream));
+        if (value && !h->d_G) {
+            const size_t np = (size_t)h->n + 1 + kPad;
+            CUDA_TRY(cudaMalloc(&h->d_G, sizeof(int) * np));
+            CUDA_TRY(cudaMemset(h->d_G, 0, sizeof(int) * np));
+            CUDA_TRY(cudaMalloc(&h->d_bar25, sizeof(unsigned) * 2));
+            CUDA_TRY(cudaMemset(h->d_bar25, 0, sizeof(unsigned) * 2));
+        }
+            // the 2.5-opt sweep is instantiated for R = 7 only; the 2-opt geometry comes back with value 0
+        const long long total_pairs = (long long)h->n * (h->n - 1) / 2;
+        Geometry g = choose_geometry(total_pairs / h->world);
+        if (value) g.rows = kRowsSmall;
+        if (g.rows != h->geo.rows || g.tj != h->geo.tj || g.warps != h->geo.warps) {
+            h->geo = g;
+            h->all_tiles = build_tiles(h->n, h->geo);
+            int rc = upload_shard(h, h->shard_rank, h->shard_world);
+            if (rc) return rc;
+        }
+        h->or25 = (int)value;
+        if (h->has_tour) {
+            if (value) CUDA_TRY(launch_gain(h->d_P, h->d_G, h->n, 0, h->n - 1, h->stream));
+            CUDA_TRY(launch_reset_key(h->d_slots + h->parity, h->stream));
+        }
+        h->last_tiling = -1;
+        CUDA_TRY(cudaStreamSynchronize(h->stream));
+        break;
+    }
     case TSP2OPT_OPT_NEIGHBOURS: {
-        if (value < 0 || value > kMaxNeighbours) return TSP2OPT_EINVAL;
+        if (value < 0 || value > kMaxNeighbours || (value && h->or25)) return TSP2OPT_EINVAL;
         if (value > 0) {
             if (!h->d_knn) {  // exact candidate lists, once per handle (coordinates never change)
                 unsigned long long* knn = nullptr;
@@ -893,6 +947,66 @@ int tsp2opt_get_trace(tsp2opt_t h, int32_t* ijd, int64_t cap, int64_t* count)
         }
     }
     return TSP2OPT_OK;
+}
+
+int tsp2opt_get_trace_typed(tsp2opt_t h, int32_t* ijdt, int64_t cap, int64_t* count)
+{
+    if (!h || !count || (cap > 0 && !ijdt)) return TSP2OPT_EINVAL;
+    if (!h->has_tour) return TSP2OPT_ESTATE;
+    int rc = read_slot(h);
+    if (rc) return rc;
+    const long long k = std::min<long long>(h->h_slot->moves, h->trace_cap);
+    *count = k;
+    const long long m = std::min<long long>(k, cap);
+    if (m > 0) {
+        std::vector<unsigned long long> keys((size_t)m);
+        std::vector<int> types((size_t)m);
+        CUDA_TRY(cudaMemcpy(keys.data(), h->d_trace, sizeof(unsigned long long) * (size_t)m, cudaMemcpyDeviceToHost));
+        CUDA_TRY(cudaMemcpy(types.data(), h->d_ttype, sizeof(int) * (size_t)m, cudaMemcpyDeviceToHost));
+        for (long long t = 0; t < m; t++) {
+            ijdt[4 * t] = key_i(keys[t]);
+            ijdt[4 * t + 1] = key_j(keys[t]);
+            ijdt[4 * t + 2] = key_delta(keys[t]);
+            ijdt[4 * t + 3] = h->or25 ? types[t] : 0;
+        }
+    }
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_best_move_typed(tsp2opt_t h, const int32_t* tour, int32_t* i, int32_t* j, int32_t* type, int32_t* delta)
+{
+    if (!h || !i || !j || !type || !delta) return TSP2OPT_EINVAL;
+    if (tour) {
+        int rc = load_host_tour(h, tour);
+        if (rc) return rc;
+    }
+    if (!h->has_tour) return TSP2OPT_ESTATE;
+    CUDA_TRY(launch_reset_key(h->d_slots + h->parity, h->stream));
+    int rc = enqueue_iteration(h, 0, false);
+    if (rc) return rc;
+    if (h->or25) CUDA_TRY(launch_decide25(h->d_P, h->d_E, h->d_G, h->d_slots + h->parity, h->stream));
+    rc = read_slot(h);
+    if (rc) return rc;
+    const unsigned long long k = h->h_slot->key;
+    *i = key_i(k);
+    *j = key_j(k);
+    *delta = key_delta(k);
+    *type = h->or25 ? h->h_slot->mtype : 0;
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_apply_typed(tsp2opt_t h, int32_t i, int32_t j, int32_t type)
+{
+    if (!h || type < 0 || type > 2) return TSP2OPT_EINVAL;
+    if (type == 0) return tsp2opt_apply(h, i, j);
+    if (!h->or25 || !(0 <= i && i + 2 <= j && j < h->n)) return TSP2OPT_EINVAL;
+    if (!h->has_tour) return TSP2OPT_ESTATE;
+    Slot* in = h->d_slots + h->parity;
+    Slot* out = h->d_slots + (h->parity ^ 1);
+    CUDA_TRY(launch_apply25(h->d_P, h->d_E, h->d_G, h->d_tour, h->n, in, out, 0, 1, i, j, type, nullptr, nullptr, 0,
+                            h->d_bar25, h->stream));
+    h->parity ^= 1;
+    return read_slot(h);
 }
 
 int tsp2opt_debug_set_shard(tsp2opt_t h, int32_t rank, int32_t world)

@@ -270,7 +270,29 @@ struct __align__(64) Slot {
     int seed_ok;                  // 1: last_key is the move just applied to the tour the tile minima of the
                                   //    previous sweep were measured on (they may seed this sweep)
     unsigned ncull;               // culled sweep: number of kept tiles in the list
-    int pad[4];
+    int mtype;                    // 2.5-opt: type of the move last applied / decided (reading R19)
+    int pad[3];
 };
+
+// Software grid barrier for co-resident grids (cooperative launches): arrive
+// on bar[0], the last block resets it and advances the generation bar[1].
+__device__ __forceinline__ void grid_sync(unsigned* bar, unsigned nblocks)
+{
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        volatile unsigned* vgen = bar + 1;
+        const unsigned gen = *vgen;
+        __threadfence();
+        if (atomicAdd(bar, 1u) == nblocks - 1) {
+            atomicExch(bar, 0u);
+            __threadfence();
+            atomicAdd(bar + 1, 1u);
+        } else {
+            while (*vgen == gen) __nanosleep(32);
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
 
 }  // namespace tsp2opt

@@ -70,6 +70,17 @@ cudaError_t launch_pruned_sweep(const float2* P, const int* E, const int* tour, 
                                 const unsigned long long* knn, int K, int n, int p0, int p1, Slot* slot,
                                 int respect_done, cudaStream_t st);
 cudaError_t launch_pos(const int* tour, int* pos, int n, cudaStream_t st);
+// 2.5-opt (tsp2opt_sweep25.cu; reading R19): sweep over the dense tiling with R = kRowsSmall,
+// per-position removal gains G, cooperative apply resolving the move type.
+size_t sweep25_smem_bytes(const Geometry& g);
+cudaError_t sweep25_prepare();
+cudaError_t launch_sweep25(const Geometry& g, const float2* P, const int* E, const int* G, int n, const int2* tiles,
+                           int ntiles, Slot* slot, int respect_done, int flags, cudaStream_t st);
+cudaError_t launch_gain(const float2* P, int* G, int n, int lo, int hi, cudaStream_t st);
+cudaError_t launch_decide25(const float2* P, const int* E, const int* G, Slot* slot, cudaStream_t st);
+cudaError_t launch_apply25(float2* P, int* E, int* G, int* tour, int n, const Slot* in, Slot* out,
+                           long long max_moves, int explicit_move, int ei, int ej, int etype,
+                           unsigned long long* trace, int* ttype, long long trace_cap, unsigned* bar, cudaStream_t st);
 size_t sweep_smem_bytes(const Geometry& g);
 cudaError_t sweep_prepare();
 cudaError_t launch_load_tour(const int* coords, const int* tour_src, int* tour_dst, float2* P, int* E, int n,

@@ -66,6 +66,7 @@ __global__ void init_slot_kernel(Slot* slot, int clear_length)
     slot->next_tile = 0;
     slot->ncull = 0;
     slot->seed_ok = 0;  // a freshly loaded tour: no previous sweep to seed from
+    slot->mtype = 0;
 }
 
 // best_move's sweep is not followed by an apply: its tile minima must not be
@@ -298,6 +299,7 @@ __device__ __forceinline__ bool apply_phase(float2* __restrict__ P, int* __restr
         o.done = explicit_move ? (done & 4) : done;  // an explicit move makes the tour unconverged
         o.next_tile = 0;
         o.ncull = 0;
+        o.mtype = 0;
         o.seed_ok = (apply && !explicit_move) ? 1 : 0;  // tile minima of this sweep seed the next one
         if (!explicit_move && !done) {
             if (key_delta(key) >= 0) o.done = 1;        // local minimum (reading R7)
@@ -361,24 +363,7 @@ __global__ void __launch_bounds__(256) apply_kernel(float2* __restrict__ P, int*
 // move cap or the per-launch iteration budget.  Slots ping-pong exactly as in
 // the multi-kernel path; the final parity is written to ctl[0].
 // ===========================================================================
-__device__ __forceinline__ void grid_sync(unsigned* bar, unsigned nblocks)
-{
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        volatile unsigned* vgen = bar + 1;
-        const unsigned gen = *vgen;
-        __threadfence();
-        if (atomicAdd(bar, 1u) == nblocks - 1) {
-            atomicExch(bar, 0u);
-            __threadfence();
-            atomicAdd(bar + 1, 1u);
-        } else {
-            while (*vgen == gen) __nanosleep(32);
-        }
-        __threadfence();
-    }
-    __syncthreads();
-}
+// grid_sync: tsp2opt_device.cuh
 
 template <int R>
 __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2* __restrict__ P, int* __restrict__ E,
@@ -388,8 +373,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
                                                            long long budget, unsigned* __restrict__ bar,
                                                            int* __restrict__ ctl,
                                                            unsigned long long* __restrict__ tilebest, int flags,
-                                                           unsigned long long* __restrict__ trace, long long trace_cap,
-                                            int* __restrict__ pos)
+                                                           unsigned long long* __restrict__ trace, long long trace_cap)
 {
     extern __shared__ float4 smem[];
     const TileSmem sm(smem, TJ);

@@ -60,6 +60,9 @@ def _L():
             "tsp2opt_debug_set_shard": ([P, I32, I32], I32),
             "tsp2opt_set_option": ([P, I32, I64], I32),
             "tsp2opt_get_trace": ([P, P, I64, pI64], I32),
+            "tsp2opt_get_trace_typed": ([P, P, I64, pI64], I32),
+            "tsp2opt_best_move_typed": ([P, P, pI32, pI32, pI32, pI32], I32),
+            "tsp2opt_apply_typed": ([P, I32, I32, I32], I32),
             "tsp2opt_ils": ([P, P, I64, ctypes.c_uint64, pI64, P], I32),
             "tsp2opt_batch_local_search": ([P, I32, I32, P, I64, P, P], I32),
             "tsp2opt_mf_tour": ([P, P, pI64, P], I32),
@@ -159,6 +162,23 @@ def best_move(h, tour=None):
 
 def apply(h, i: int, j: int) -> None:
     _check(_L().tsp2opt_apply(h, int(i), int(j)), "tsp2opt_apply")
+
+
+def best_move_typed(h, tour=None):
+    """(i, j, type, delta): the best move with its type (2.5-opt handles; type 0 otherwise)."""
+    i, j, t, d = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+    if tour is None:
+        tp = None
+    else:
+        tt = _i32(tour)
+        tp = _ptr(tt)
+    _check(_L().tsp2opt_best_move_typed(h, tp, ctypes.byref(i), ctypes.byref(j), ctypes.byref(t), ctypes.byref(d)),
+           "tsp2opt_best_move_typed")
+    return i.value, j.value, t.value, d.value
+
+
+def apply_typed(h, i: int, j: int, typ: int) -> None:
+    _check(_L().tsp2opt_apply_typed(h, int(i), int(j), int(typ)), "tsp2opt_apply_typed")
 
 
 def iterate_async(h, count: int) -> None:
@@ -265,7 +285,7 @@ def get_tour(h, n: int):
     return t, L.value
 
 
-OPT_TILE_BOUNDS, OPT_SEED, OPT_PERSISTENT, OPT_TRACE, OPT_NEIGHBOURS = 1, 2, 3, 4, 5
+OPT_TILE_BOUNDS, OPT_SEED, OPT_PERSISTENT, OPT_TRACE, OPT_NEIGHBOURS, OPT_NODE_INSERTION = 1, 2, 3, 4, 5, 6
 MAX_NEIGHBOURS = 16  # TSP2OPT_MAX_NEIGHBOURS
 
 
@@ -278,6 +298,14 @@ def get_trace(h, cap: int) -> np.ndarray:
     out = np.zeros((max(cap, 1), 3), dtype=np.int32)
     cnt = ctypes.c_int64()
     _check(_L().tsp2opt_get_trace(h, _ptr(out), int(cap), ctypes.byref(cnt)), "tsp2opt_get_trace")
+    return out[: min(cnt.value, cap)].copy()
+
+
+def get_trace_typed(h, cap: int) -> np.ndarray:
+    """int32[count, 4] (i, j, delta, type) of the recorded moves."""
+    out = np.zeros((max(cap, 1), 4), dtype=np.int32)
+    cnt = ctypes.c_int64()
+    _check(_L().tsp2opt_get_trace_typed(h, _ptr(out), int(cap), ctypes.byref(cnt)), "tsp2opt_get_trace_typed")
     return out[: min(cnt.value, cap)].copy()
 
 
@@ -376,6 +404,15 @@ class TSP2Opt:
 
     def apply(self, i, j):
         apply(self.h, i, j)
+
+    def best_move_typed(self, tour=None):
+        return best_move_typed(self.h, tour)
+
+    def apply_typed(self, i, j, typ):
+        apply_typed(self.h, i, j, typ)
+
+    def get_trace_typed(self, cap: int):
+        return get_trace_typed(self.h, cap)
 
     def iterate_async(self, count: int):
         iterate_async(self.h, count)
