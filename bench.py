@@ -215,10 +215,11 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms, sweep_avg_ms, e2e_total, tb_total_ms, tb_sweep_ms = t.tolist()
 
-    ls = ils = batch = pruned = None
+    ls = ils = batch = pruned = or25 = None
     if rank == 0 and world == 1 and not args.no_ls:
         ls = time_to_local_min(tsp2opt, args.ls_config)
         pruned = time_pruned(tsp2opt, args.pruned_config) if args.pruned_config else None
+        or25 = time_25opt(tsp2opt, args.or25_config) if args.or25_config else None
         ils = time_ils(tsp2opt, args.ils_config) if args.ils_config else None
         batch = time_batch(tsp2opt, args.batch_config, not args.no_cpu) if args.batch_config else None
         batch_ils = time_batch_ils(tsp2opt, args.batch_ils_config, not args.no_cpu) if args.batch_ils_config else None
@@ -271,6 +272,8 @@ def run_ours(args):
             line["ils"] = ils
         if pruned:
             line["pruned_local_search"] = pruned
+        if or25:
+            line["local_search_25opt"] = or25
         if batch:
             line["batch_local_search"] = batch
         if batch_ils:
@@ -382,6 +385,37 @@ def time_pruned(tsp2opt, spec):
                     "candidates_per_sweep": 2 * K * n,
                     "polish_seconds": t3 - t2, "polish_iterations": f["iterations"], "length": f["length"],
                     "seconds": t3 - t0})
+    return out
+
+
+def time_25opt(tsp2opt, spec):
+    """Best-improvement 2.5-opt (TSP2OPT_OPT_NODE_INSERTION; SURVEY §8(f) NEXT-4,
+    L26 §VII "2.5-opt"; reading R19) from the Multiple Fragment start, wall time
+    of the MF tour and of the local search (device-resident, as the `mf` entries
+    of time_to_local_minimum); the 2.5-opt sweep kernel is timed by the
+    library's CUDA events."""
+    out = []
+    for name in spec.split(","):
+        if not name:
+            continue
+        coords, _ = inputs.config_instance(name)
+        n = len(coords)
+        with tsp2opt.TSP2Opt(coords) as g:
+            g.set_option(tsp2opt.OPT_NODE_INSERTION, 1)
+            g.mf_tour()  # warm-up
+            g.local_search_current(max_iters=2)
+            t0 = time.perf_counter()
+            m = g.mf_tour()
+            t1 = time.perf_counter()
+            g.profile(True)
+            r = g.local_search_current()
+            t2 = time.perf_counter()
+            sweep_ms, sweeps = g.profile_read()
+            g.profile(False)
+        out.append({"config": name, "n": n, "start": "mf", "moves": "2-opt + node insertion", "seconds": t2 - t0,
+                    "mf_seconds": t1 - t0, "ls_seconds": t2 - t1, "mf_length": m["length"],
+                    "iterations": r["iterations"], "length": r["length"],
+                    "sweep_us_avg": 1e3 * sweep_ms / max(1, sweeps), "sweeps": sweeps})
     return out
 
 
@@ -579,6 +613,7 @@ def main():
     ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert,C5:hilbert,C2:mf,C3:mf,C4:mf,C5:mf", help="configs timed to a local minimum (rank 0, N=1)")
     ap.add_argument("--ils-config", default="C1:200,C2:50", help="Iterated Local Search runs cfg:iterations")
     ap.add_argument("--pruned-config", default="C3:8,C4:8,C5:8,C5:16", help="pruned 2-opt from MF, cfg:K")
+    ap.add_argument("--or25-config", default="C3,C4,C5", help="2.5-opt local search from MF, configs")
     ap.add_argument("--batch-config", default="100:4736,1002:592", help="batched local search n:instances")
     ap.add_argument("--batch-ils-config", default="C1:4736:100", help="batched ILS cfg:replicas:steps")
     ap.add_argument("--no-ls", action="store_true")

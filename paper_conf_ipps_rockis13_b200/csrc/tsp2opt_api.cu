@@ -83,6 +83,7 @@ struct tsp2opt_ctx {
     int4* d_list = nullptr;     // kept cull tiles (I0, J0, index) [nctiles]
     int nctiles = 0;
     int list_grid = 0;          // CTAs of the culled sweep (co-resident)
+    int list25_grid = 0;        // CTAs of the 2.5-opt culled sweep
     int last_tiling = -1;       // tiling of the previous sweep (0 dense, 1 cull): seeds are per tiling
     unsigned long long* d_trace = nullptr;  // [trace_cap] keys of the applied moves (TSP2OPT_OPT_TRACE)
     int* d_best = nullptr;      // [n] best tour of an ILS run
@@ -211,6 +212,7 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
     h->d_list = nullptr;
     if (h->nctiles > 0) CUDA_TRY(cudaMalloc(&h->d_list, sizeof(int4) * (size_t)h->nctiles));
     h->list_grid = sweep_list_grid(h->cgeo, h->nctiles);
+    h->list25_grid = sweep25_list_grid(h->cgeo, h->nctiles);
     h->last_tiling = -1;
     h->shard_pairs = pairs;
     h->shard_rank = rank;
@@ -336,7 +338,12 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         else CUDA_TRY(cudaMemsetAsync(h->d_tilebest, 0xFF, sizeof(unsigned long long) * h->ntiles, h->stream));
     }
     h->last_tiling = tiling;
-    if (tiling == 3) {  // 2.5-opt: dense tiling (R = 7), per-tile bound unless TILE_BOUNDS = 0
+    if (tiling == 3 && h->tile_bounds == 2) {  // 2.5-opt, culled: box + cull (with gains) + list sweep
+        CUDA_TRY(launch_box_cull(h->cgeo, h->d_P, h->d_E, h->d_G, h->n, h->d_ctiles, h->nctiles, h->d_rbox, h->d_cbox,
+                                 h->d_list, in, apply ? 1 : 0, h->stream));
+        CUDA_TRY(launch_sweep25_list(h->cgeo, h->d_P, h->d_E, h->d_G, h->n, h->d_list, h->list25_grid, in,
+                                     apply ? 1 : 0, h->stream));
+    } else if (tiling == 3) {  // 2.5-opt: dense tiling (R = 7), per-tile bound unless TILE_BOUNDS = 0
         CUDA_TRY(launch_sweep25(h->geo, h->d_P, h->d_E, h->d_G, h->n, h->d_tiles, h->ntiles, in, apply ? 1 : 0,
                                 h->tile_bounds != 0 ? kSweepTileBounds : 0, h->stream));
     } else if (tiling == 2) {  // pruned neighbourhood M_K: this shard's positions, O(nK)

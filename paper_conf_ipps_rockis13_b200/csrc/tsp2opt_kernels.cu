@@ -131,10 +131,14 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* 
 // One warp per summary: row block b = positions [b*TI, min(b*TI + TI, n-1))
 // (cities up to the block end + 1), column chunk c = [c*TJ, min(c*TJ + TJ, n))
 // (cities up to + 1; P[n] = P[0]).
-__global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, const int* __restrict__ E, int n,
-                                                  int TI, int nrb, int TJ, int ncc, Box* __restrict__ rbox,
-                                                  Box* __restrict__ cbox, Slot* __restrict__ slot,
-                                                  int respect_done)
+// With G (2.5-opt, reading R19) the box also carries gneg = max(-g_k) over its
+// positions: a node-insertion move with delta < 0 needs D(i+1, j) <= -1 - g
+// for g = g_{i+1} or g_j (tsp2opt_sweep25.cu), so the cull threshold becomes
+// max(emax, gneg) - 1 of the two boxes.
+__global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, const int* __restrict__ E,
+                                                  const int* __restrict__ G, int n, int TI, int nrb, int TJ, int ncc,
+                                                  Box* __restrict__ rbox, Box* __restrict__ cbox,
+                                                  Slot* __restrict__ slot, int respect_done)
 {
     pdl_trigger();
     pdl_wait();
@@ -159,7 +163,7 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
     } else {
         return;  // whole warps only
     }
-    int xlo = 1 << 30, xhi = -1, ylo = 1 << 30, yhi = -1, emax = 0;
+    int xlo = 1 << 30, xhi = -1, ylo = 1 << 30, yhi = -1, emax = 0, gneg = 0;
     // up to kBoxIters positions per lane, all loads issued before the first use
     constexpr int kBoxIters = (32 * kRowsLarge * kMaxWarps + 1 + 31) / 32;
 #pragma unroll
@@ -173,6 +177,7 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
             ylo = min(ylo, y);
             yhi = max(yhi, y);
             if (k < ke) emax = max(emax, E[k]);
+            if (G) gneg = max(gneg, -G[k == n ? 0 : k]);
         }
     }
     const unsigned full = 0xffffffffu;
@@ -181,6 +186,7 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
     ylo = __reduce_min_sync(full, ylo);
     yhi = __reduce_max_sync(full, yhi);
     emax = __reduce_max_sync(full, emax);
+    gneg = __reduce_max_sync(full, gneg);
     if (lane == 0) {
         Box b;
         b.xlo = xlo;
@@ -188,7 +194,8 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
         b.ylo = ylo;
         b.yhi = yhi;
         b.emax = emax;
-        b.pad[0] = b.pad[1] = b.pad[2] = 0;
+        b.pad[0] = gneg;  // 0 without G
+        b.pad[1] = b.pad[2] = 0;
         *out = b;
     }
 }
@@ -213,7 +220,7 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
         const Box r = rbox[tl.x / TI], c = cbox[tl.y / TJ];
         const long long gx = max(0, max(c.xlo - r.xhi, r.xlo - c.xhi));
         const long long gy = max(0, max(c.ylo - r.yhi, r.ylo - c.yhi));
-        const long long T = (long long)max(r.emax, c.emax) - 1;
+        const long long T = (long long)max(max(r.emax, c.emax), max(r.pad[0], c.pad[0])) - 1;  // pad[0]: gneg
         keep = T >= 0 && gx * gx + gy * gy <= T * T + T;
         if (!keep && (flags & kSweepSeed)) tilebest[t] = kKeyNone;
     }
@@ -565,6 +572,20 @@ cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n
     return cudaGetLastError();
 }
 
+cudaError_t launch_box_cull(const Geometry& g, const float2* P, const int* E, const int* G, int n, const int2* tiles,
+                            int ntiles, Box* rbox, Box* cbox, int4* list, Slot* slot, int respect_done, cudaStream_t st)
+{
+    const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
+    const int warps = nrb + ncc;
+    cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, G, n, TI, nrb, g.tj, ncc,
+                               rbox, cbox, slot, respect_done);
+    if (e != cudaSuccess) return e;
+    e = launch_pdl(cull_kernel, dim3((ntiles + 255) / 256), dim3(256), 0, st, tiles, ntiles, TI, g.tj, rbox, cbox, slot,
+                   list, (unsigned long long*)nullptr, 0, respect_done);
+    g_launches += 2;
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
+
 int sweep_list_grid(const Geometry& g, int ntiles)
 {
     int per_sm = 0;
@@ -587,8 +608,8 @@ cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, 
     if (ntiles <= 0 || grid <= 0) return cudaSuccess;
     const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
     const int warps = nrb + ncc;
-    cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, n, TI, nrb, g.tj, ncc, rbox,
-                               cbox, slot, respect_done);
+    cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, (const int*)nullptr, n, TI,
+                               nrb, g.tj, ncc, rbox, cbox, slot, respect_done);
     if (e != cudaSuccess) return e;
     e = launch_pdl(cull_kernel, dim3((ntiles + 255) / 256), dim3(256), 0, st, tiles, ntiles, TI, g.tj, rbox, cbox, slot,
                    list, tilebest, flags, respect_done);

@@ -280,19 +280,14 @@ __device__ __forceinline__ void reverse_range(float2* P, int* tour, int lo, int 
 
 }  // namespace
 
-// a4 + a5 of the 2.5-opt sweep: one (row block x column chunk) tile per CTA.
-__global__ void __launch_bounds__(128, 4) sweep25_kernel(const float2* __restrict__ P, const int* __restrict__ E,
-                                                         const int* __restrict__ G, int n,
-                                                         const int2* __restrict__ tiles, int TJ,
-                                                         Slot* __restrict__ slot, int respect_done, int flags)
+// a4 + a5 of the 2.5-opt sweep over one (row block x column chunk) tile.
+// The caller synchronises the CTA before the shared chunk is reused.
+__device__ __forceinline__ void sweep25_tile(const float2* __restrict__ P, const int* __restrict__ E,
+                                             const int* __restrict__ G, int n, int2 tile, int TJ,
+                                             Slot* __restrict__ slot, void* smem, int flags)
 {
-    extern __shared__ float4 smem25[];
-    pdl_trigger();
-    pdl_wait();
-    if (respect_done && *(volatile int*)&slot->done) return;  // converged: iteration is a no-op
     const int TI = 32 * R25 * (int)(blockDim.x >> 5);
-    const Tile25Smem sm(smem25, TJ, TI);
-    const int2 tile = tiles[blockIdx.x];
+    const Tile25Smem sm(smem, TJ, TI);
     const int I0 = tile.x, J0 = tile.y;
     const int J1 = min(J0 + TJ, n);
     const int ncol = J1 - J0;
@@ -350,6 +345,43 @@ __global__ void __launch_bounds__(128, 4) sweep25_kernel(const float2* __restric
         mykey = other < mykey ? other : mykey;
     }
     if (lane == 0 && mykey < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, mykey);
+}
+
+__global__ void __launch_bounds__(128, 4) sweep25_kernel(const float2* __restrict__ P, const int* __restrict__ E,
+                                                         const int* __restrict__ G, int n,
+                                                         const int2* __restrict__ tiles, int TJ,
+                                                         Slot* __restrict__ slot, int respect_done, int flags)
+{
+    extern __shared__ float4 smem25[];
+    pdl_trigger();
+    pdl_wait();
+    if (respect_done && *(volatile int*)&slot->done) return;  // converged: iteration is a no-op
+    sweep25_tile(P, E, G, n, tiles[blockIdx.x], TJ, slot, smem25, flags);
+}
+
+// The 2.5-opt sweep over the culled list (as sweep_list_kernel: first entry
+// static, then dynamic claims on slot->next_tile).
+__global__ void __launch_bounds__(128, 4) sweep25_list_kernel(const float2* __restrict__ P,
+                                                              const int* __restrict__ E, const int* __restrict__ G,
+                                                              int n, const int4* __restrict__ list, int TJ,
+                                                              Slot* __restrict__ slot, int respect_done)
+{
+    extern __shared__ float4 smem25[];
+    __shared__ int4 s_t;
+    pdl_trigger();
+    pdl_wait();
+    if (respect_done && *(volatile int*)&slot->done) return;
+    const unsigned count = *(volatile unsigned*)&slot->ncull;
+    unsigned k = blockIdx.x;
+    for (;;) {
+        if (threadIdx.x == 0) s_t = k < count ? list[k] : make_int4(0, 0, -1, 0);
+        __syncthreads();
+        const int4 e = s_t;
+        if (e.z < 0) break;
+        sweep25_tile(P, E, G, n, make_int2(e.x, e.y), TJ, slot, smem25, kSweepTileBounds);
+        if (threadIdx.x == 0) k = gridDim.x + atomicAdd(&slot->next_tile, 1u);
+        __syncthreads();
+    }
 }
 
 // g_k for positions [lo, hi] (after a tour load / when the mode is switched on)
@@ -459,8 +491,34 @@ size_t sweep25_smem_bytes(const Geometry& g)
 
 cudaError_t sweep25_prepare()
 {
-    return cudaFuncSetAttribute(sweep25_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)sweep25_smem_bytes(Geometry{R25, kMaxWarps, kMaxTJ}));
+    const int bytes = (int)sweep25_smem_bytes(Geometry{R25, kMaxWarps, kMaxTJ});
+    cudaError_t e = cudaFuncSetAttribute(sweep25_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e != cudaSuccess) return e;
+    return cudaFuncSetAttribute(sweep25_list_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+}
+
+int sweep25_list_grid(const Geometry& g, int ntiles)
+{
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sweep25_list_kernel, 32 * g.warps,
+                                                      sweep25_smem_bytes(g)) != cudaSuccess)
+        return 0;
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    return std::min(per_sm * sms, ntiles);
+}
+
+cudaError_t launch_sweep25_list(const Geometry& g, const float2* P, const int* E, const int* G, int n,
+                                const int4* list, int grid, Slot* slot, int respect_done, cudaStream_t st)
+{
+    if (grid <= 0) return cudaSuccess;
+    if (g.rows != R25) return cudaErrorInvalidValue;
+    cudaError_t e = launch_kernel_pdl(sweep25_list_kernel, dim3(grid), dim3(32 * g.warps), sweep25_smem_bytes(g), st,
+                                      P, E, G, n, list, g.tj, slot, respect_done);
+    if (e != cudaSuccess) return e;
+    count_launch(1);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_sweep25(const Geometry& g, const float2* P, const int* E, const int* G, int n, const int2* tiles,

@@ -30,7 +30,7 @@ def test_best_move25_parity(gpu, n, kind):
             assert g.best_move(t) == (i, j, d)
 
 
-@pytest.mark.parametrize("bounds", ["0", "1"])
+@pytest.mark.parametrize("bounds", ["0", "1", "2"])
 @pytest.mark.parametrize("warps,tj", [(1, 2), (1, 3), (1, 32), (2, 64), (4, 128), (3, 7)])
 def test_best_move25_geometries(gpu, monkeypatch, warps, tj, bounds):
     monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", bounds)
@@ -62,6 +62,26 @@ def test_local_search25_trace(gpu, kind, n, seed):
     assert np.array_equal(res["tour"], want["tour"])
     assert np.array_equal(np.asarray(trace, dtype=np.int64), want["trace"])
     assert set(np.unique(want["trace"][:, 3]).tolist()) == {0, 1, 2}  # every move type occurs
+
+
+@pytest.mark.parametrize("cull_tj", ["2", "3", "32", "64"])
+@pytest.mark.parametrize("kind,n,seed", [("uniform", 1002, 5), ("lattice", 2000, 6)])
+def test_local_search25_culled(gpu, monkeypatch, cull_tj, kind, n, seed):
+    """The pre-sweep cull with the gain term (box + cull + list sweep), forced at
+    small n, with narrow and ragged column chunks."""
+    monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", "2")
+    monkeypatch.setenv("TSP2OPT_CULL_TJ", cull_tj)
+    c = inputs.make_coords(kind, n, seed)
+    t = inputs.random_tour(n, seed)
+    want = oracle.local_search25(c, t, trace_cap=10 * n)
+    with _handle(c) as g:
+        g.set_option(tsp2opt.OPT_TRACE, 10 * n)
+        res = g.local_search(t)
+        trace = g.get_trace_typed(10 * n)
+        assert g.best_move_typed(inputs.hilbert_tour(c)) == oracle.best_move25(c, inputs.hilbert_tour(c))
+    assert (res["iterations"], res["length"]) == (want["iterations"], want["length"])
+    assert np.array_equal(res["tour"], want["tour"])
+    assert np.array_equal(np.asarray(trace, dtype=np.int64), want["trace"])
 
 
 def test_local_search25_ties_and_degenerate(gpu):
