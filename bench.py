@@ -215,7 +215,7 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms, sweep_avg_ms, e2e_total, tb_total_ms, tb_sweep_ms = t.tolist()
 
-    ls = ils = batch = pruned = or25 = None
+    ls = ils = batch = batch_ils = pruned = or25 = None
     if rank == 0 and world == 1 and not args.no_ls:
         ls = time_to_local_min(tsp2opt, args.ls_config)
         pruned = time_pruned(tsp2opt, args.pruned_config) if args.pruned_config else None
