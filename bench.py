@@ -218,8 +218,8 @@ def run_ours(args):
     ls = ils = batch = batch_ils = pruned = or25 = None
     if rank == 0 and world == 1 and not args.no_ls:
         ls = time_to_local_min(tsp2opt, args.ls_config)
-        pruned = time_pruned(tsp2opt, args.pruned_config) if args.pruned_config else None
-        or25 = time_25opt(tsp2opt, args.or25_config) if args.or25_config else None
+        pruned = time_pruned(tsp2opt, args.pruned_config, not args.no_cpu) if args.pruned_config else None
+        or25 = time_25opt(tsp2opt, args.or25_config, not args.no_cpu) if args.or25_config else None
         ils = time_ils(tsp2opt, args.ils_config) if args.ils_config else None
         batch = time_batch(tsp2opt, args.batch_config, not args.no_cpu) if args.batch_config else None
         batch_ils = time_batch_ils(tsp2opt, args.batch_ils_config, not args.no_cpu) if args.batch_ils_config else None
@@ -346,7 +346,7 @@ def time_to_local_min(tsp2opt, cfg_name):
     return out
 
 
-def time_pruned(tsp2opt, spec):
+def time_pruned(tsp2opt, spec, with_oracle=True):
     """Neighbourhood-pruned 2-opt (TSP2OPT_OPT_NEIGHBOURS = K; SURVEY §8(f)
     NEXT-4, L26 §VII "neighborhood pruning ... at the cost of the quality";
     reading R18) from the Multiple Fragment start, `cfg:K` entries: MF tour,
@@ -379,16 +379,27 @@ def time_pruned(tsp2opt, spec):
             g.set_option(tsp2opt.OPT_NEIGHBOURS, 0)
             f = g.local_search_current()
             t3 = time.perf_counter()
-        out.append({"config": name, "n": n, "K": K, "start": "mf", "mf_seconds": t1 - t0, "mf_length": m["length"],
-                    "pruned_seconds": t2 - t1, "pruned_iterations": r["iterations"], "pruned_length": r["length"],
-                    "pruned_sweep_us_avg": 1e3 * sweep_ms / max(1, sweeps), "pruned_sweeps": sweeps,
-                    "candidates_per_sweep": 2 * K * n,
-                    "polish_seconds": t3 - t2, "polish_iterations": f["iterations"], "length": f["length"],
-                    "seconds": t3 - t0})
+        entry = {"config": name, "n": n, "K": K, "start": "mf", "mf_seconds": t1 - t0, "mf_length": m["length"],
+                 "pruned_seconds": t2 - t1, "pruned_iterations": r["iterations"], "pruned_length": r["length"],
+                 "pruned_sweep_us_avg": 1e3 * sweep_ms / max(1, sweeps), "pruned_sweeps": sweeps,
+                 "candidates_per_sweep": 2 * K * n,
+                 "polish_seconds": t3 - t2, "polish_iterations": f["iterations"], "length": f["length"],
+                 "seconds": t3 - t0}
+        if with_oracle and n <= 20000:  # the oracle's MF tour is O(n^2 log n): the small configs only
+            import oracle
+            mt = oracle.mf_tour(coords)
+            o0 = time.perf_counter()
+            o = oracle.pruned_local_search(coords, mt, K)
+            o1 = time.perf_counter()
+            entry["cpu_oracle"] = {"seconds": o1 - o0, "iterations": o["iterations"], "length": o["length"],
+                                   "matches_gpu": bool(o["iterations"] == r["iterations"] and o["length"] == r["length"]),
+                                   "cores": oracle.num_threads(), "kind": "oracle",
+                                   "sample": "the whole pruned local search from the oracle's own MF tour"}
+        out.append(entry)
     return out
 
 
-def time_25opt(tsp2opt, spec):
+def time_25opt(tsp2opt, spec, with_oracle=True):
     """Best-improvement 2.5-opt (TSP2OPT_OPT_NODE_INSERTION; SURVEY §8(f) NEXT-4,
     L26 §VII "2.5-opt"; reading R19) from the Multiple Fragment start, wall time
     of the MF tour and of the local search (device-resident, as the `mf` entries
@@ -412,10 +423,23 @@ def time_25opt(tsp2opt, spec):
             t2 = time.perf_counter()
             sweep_ms, sweeps = g.profile_read()
             g.profile(False)
-        out.append({"config": name, "n": n, "start": "mf", "moves": "2-opt + node insertion", "seconds": t2 - t0,
-                    "mf_seconds": t1 - t0, "ls_seconds": t2 - t1, "mf_length": m["length"],
-                    "iterations": r["iterations"], "length": r["length"],
-                    "sweep_us_avg": 1e3 * sweep_ms / max(1, sweeps), "sweeps": sweeps})
+        entry = {"config": name, "n": n, "start": "mf", "moves": "2-opt + node insertion", "seconds": t2 - t0,
+                 "mf_seconds": t1 - t0, "ls_seconds": t2 - t1, "mf_length": m["length"],
+                 "iterations": r["iterations"], "length": r["length"],
+                 "sweep_us_avg": 1e3 * sweep_ms / max(1, sweeps), "sweeps": sweeps}
+        if with_oracle and n <= 20000:
+            import oracle
+            mt = oracle.mf_tour(coords)
+            reps = 10
+            o0 = time.perf_counter()
+            for _ in range(reps):
+                oracle.best_move25(coords, mt)
+            per = (time.perf_counter() - o0) / reps
+            entry["cpu_oracle"] = {"sweep_seconds": per, "est_ls_seconds": per * (r["iterations"] + 1),
+                                   "cores": oracle.num_threads(), "kind": "oracle",
+                                   "sample": f"{reps} oracle 2.5-opt sweeps of the MF tour; the local search "
+                                             "estimate is per-sweep time x (moves + 1)"}
+        out.append(entry)
     return out
 
 
