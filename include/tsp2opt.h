@@ -197,12 +197,16 @@ int tsp2opt_mf_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length, int32_t *ro
 int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
 
 /* Execution options (none but TSP2OPT_OPT_NEIGHBOURS changes any result; all results stay bit-exact):
- *  TSP2OPT_OPT_TILE_BOUNDS (default 2 from 1e8 pairs per rank, else 1): 1 = skip a tile of the sweep when the
+ *  TSP2OPT_OPT_TILE_BOUNDS (default 3 from 1e8 pairs per rank, else 1): 1 = skip a tile of the sweep when the
  *      bounding boxes of its row and column cities prove that no pair can pass
  *      the per-pair necessary condition; 2 = the same, plus a
  *      pre-sweep cull (per-block boxes, one test per tile with delta < 0 as the
  *      condition) so the sweep launches over the kept tiles only; 0 tests every
- *      pair individually (the pair-check throughput the bench reports).
+ *      pair individually (the pair-check throughput the bench reports); 3 = the
+ *      culled sweep made incremental: each tile keeps its own minimum over its
+ *      improving pairs, and after a move only the tiles with a row or column
+ *      position in the move's [i, j] are culled / re-swept, the rest keep their
+ *      minimum.
  *  TSP2OPT_OPT_SEED (default 0): start each tile from its own minimum of the
  *      previous sweep when the applied move leaves that pair intact.
  *  TSP2OPT_OPT_PERSISTENT (default 2): local_search loop, 0 = one sweep and one

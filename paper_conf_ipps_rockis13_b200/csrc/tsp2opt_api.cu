@@ -85,6 +85,7 @@ struct tsp2opt_ctx {
     int list_grid = 0;          // CTAs of the culled sweep (co-resident)
     int list25_grid = 0;        // CTAs of the 2.5-opt culled sweep
     int last_tiling = -1;       // tiling of the previous sweep (0 dense, 1 cull): seeds are per tiling
+    bool inc_valid = false;     // the stored per-tile minima are those of an incremental sweep of the current tiling
     unsigned long long* d_trace = nullptr;  // [trace_cap] keys of the applied moves (TSP2OPT_OPT_TRACE)
     int* d_best = nullptr;      // [n] best tour of an ILS run
     void* d_mf_ws = nullptr;    // Multiple Fragment workspace (mf_workspace_bytes), allocated on first use
@@ -214,6 +215,7 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
     h->list_grid = sweep_list_grid(h->cgeo, h->nctiles);
     h->list25_grid = sweep25_list_grid(h->cgeo, h->nctiles);
     h->last_tiling = -1;
+    h->inc_valid = false;
     h->shard_pairs = pairs;
     h->shard_rank = rank;
     h->shard_world = world;
@@ -312,7 +314,8 @@ int load_host_tour(tsp2opt_ctx* h, const int32_t* tour)
 
 int sweep_flags(const tsp2opt_ctx* h)
 {
-    return (h->seed_next ? kSweepSeed : 0) | (h->tile_bounds != 0 ? kSweepTileBounds : 0);
+    return (h->seed_next ? kSweepSeed : 0) | (h->tile_bounds != 0 ? kSweepTileBounds : 0) |
+           (h->tile_bounds == 3 ? kSweepIncremental : 0);
 }
 
 // One iteration: sweep (a4/a5) -> allreduce-min (a6) -> apply (a7/a8).
@@ -331,14 +334,21 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         h->ev_used += 2;
         CUDA_TRY(cudaEventRecord(ev0, h->stream));
     }
-    const int tiling = h->or25 ? 3 : h->nbr_k > 0 ? 2 : h->tile_bounds == 2 ? 1 : 0;
+    const int tiling = h->or25 ? 3 : h->nbr_k > 0 ? 2 : h->tile_bounds >= 2 ? 1 : 0;
     if (h->seed_next && h->last_tiling != tiling && tiling < 2) {
         // per-tile seeds are kept per tiling: the other tiling's minima are stale
         if (tiling) CUDA_TRY(cudaMemsetAsync(h->d_ctilebest, 0xFF, sizeof(unsigned long long) * h->nctiles, h->stream));
         else CUDA_TRY(cudaMemsetAsync(h->d_tilebest, 0xFF, sizeof(unsigned long long) * h->ntiles, h->stream));
     }
+    int flags = sweep_flags(h);
+    if (flags & kSweepIncremental) {
+        if (tiling != 1 || !h->inc_valid || h->last_tiling != tiling) flags |= kSweepFull;
+        h->inc_valid = tiling == 1;
+    } else {
+        h->inc_valid = false;
+    }
     h->last_tiling = tiling;
-    if (tiling == 3 && h->tile_bounds == 2) {  // 2.5-opt, culled: box + cull (with gains) + list sweep
+    if (tiling == 3 && h->tile_bounds >= 2) {  // 2.5-opt, culled: box + cull (with gains) + list sweep
         CUDA_TRY(launch_box_cull(h->cgeo, h->d_P, h->d_E, h->d_G, h->n, h->d_ctiles, h->nctiles, h->d_rbox, h->d_cbox,
                                  h->d_list, in, apply ? 1 : 0, h->stream));
         CUDA_TRY(launch_sweep25_list(h->cgeo, h->d_P, h->d_E, h->d_G, h->n, h->d_list, h->list25_grid, in,
@@ -353,7 +363,7 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
                                      apply ? 1 : 0, h->stream));
     } else if (tiling) {  // cull first, then sweep the kept tiles only
         CUDA_TRY(launch_cull_sweep(h->cgeo, h->d_P, h->d_E, h->n, h->d_ctiles, h->nctiles, h->list_grid, h->d_rbox,
-                                   h->d_cbox, h->d_list, in, apply ? 1 : 0, h->d_ctilebest, sweep_flags(h), h->stream));
+                                   h->d_cbox, h->d_list, in, apply ? 1 : 0, h->d_ctilebest, flags, h->stream));
     } else {
         CUDA_TRY(launch_sweep(h->geo, h->d_P, h->d_E, h->n, h->d_tiles, h->ntiles, in, apply ? 1 : 0, h->d_tilebest,
                               sweep_flags(h), h->stream));
@@ -390,6 +400,7 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
     const bool use_persistent =
         !h->comm && h->nbr_k == 0 && !h->or25 && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
     if (use_persistent) {
+        h->inc_valid = false;
         // One persistent cooperative launch runs sweep -> apply to the local
         // minimum; the per-launch iteration budget bounds a launch to roughly
         // 2e12 pair checks (~0.5 s), after which the host relaunches.
@@ -481,11 +492,12 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     CTRY(sweep25_prepare());
     const long long total_pairs = (long long)n * (n - 1) / 2;
     h->geo = choose_geometry(total_pairs / world);
-    // Pre-sweep cull from ~1e8 pairs per rank (measured, local search from MF: n = 85900 129 vs
-    // 221 us per iteration, n = 33810 80 vs 89 us; n = 7397 38 vs 29 us, where the extra
-    // launches cost more than the skipped tiles).
-    h->tile_bounds = total_pairs / world >= 100000000LL ? 2 : 1;
-    if (const char* eb = getenv("TSP2OPT_TILE_BOUNDS")) h->tile_bounds = std::min(2, std::max(0, atoi(eb)));
+    // Pre-sweep cull, incremental, from ~1e8 pairs per rank (measured, local search from MF:
+    // n = 85900 39 vs 65 (cull) vs 212 (in-sweep bound) us per iteration, n = 33810 26 vs 36 vs
+    // 79 us; n = 7397 23 vs 25 vs 18 us, where the extra launches cost more than the skipped
+    // tiles; profiles/r01_ls_incremental.jsonl).
+    h->tile_bounds = total_pairs / world >= 100000000LL ? 3 : 1;
+    if (const char* eb = getenv("TSP2OPT_TILE_BOUNDS")) h->tile_bounds = std::min(3, std::max(0, atoi(eb)));
     h->all_tiles = build_tiles(n, h->geo);
     // Culled-sweep tiling: R = 7 rows per lane and narrow column chunks (measured,
     // local search from MF).
@@ -856,9 +868,10 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t* tour_out, int64_t* length)
 int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
 {
     if (!h) return TSP2OPT_EINVAL;
+    h->inc_valid = false;  // any option change: the next incremental sweep starts from scratch
     switch (option) {
     case TSP2OPT_OPT_TILE_BOUNDS:
-        if (value < 0 || value > 2) return TSP2OPT_EINVAL;
+        if (value < 0 || value > 3) return TSP2OPT_EINVAL;
         h->tile_bounds = (int)value;
         break;
     case TSP2OPT_OPT_SEED: h->seed_next = value != 0; break;

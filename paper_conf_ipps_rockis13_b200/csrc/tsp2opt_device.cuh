@@ -25,6 +25,10 @@ constexpr unsigned long long kKeyNone = ~0ULL;
 // sweep option bits (tsp2opt_set_option)
 constexpr int kSweepSeed = 1;        // seed each tile with its surviving minimum of the previous sweep
 constexpr int kSweepTileBounds = 2;  // skip tiles whose bounding boxes prove that no pair passes the filter
+constexpr int kSweepLocal = 4;       // tile-local bound (start at delta < 0, ignore the global key): the tile's
+                                     // minimum is then exact on its own and can be reused while the tile is clean
+constexpr int kSweepIncremental = 8; // culled sweep: only tiles the last applied move touched are re-swept
+constexpr int kSweepFull = 16;       // incremental sweep whose stored minima are not valid yet: re-sweep all
 
 // Bounding box of a run of route positions (unbiased integer coordinates) and
 // the largest tour edge leaving it: the summaries the tile cull compares.

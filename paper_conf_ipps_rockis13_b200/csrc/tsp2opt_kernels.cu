@@ -138,10 +138,18 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* 
 __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, const int* __restrict__ E,
                                                   const int* __restrict__ G, int n, int TI, int nrb, int TJ, int ncc,
                                                   Box* __restrict__ rbox, Box* __restrict__ cbox,
-                                                  Slot* __restrict__ slot, int respect_done)
+                                                  Slot* __restrict__ slot, int respect_done, int incremental)
 {
     pdl_trigger();
     pdl_wait();
+    // incremental: only the summaries of blocks the last applied move touched
+    // (P changed on [i+1, j], E on [i, j]) are recomputed; the others stand
+    int dlo = 0, dhi = n;
+    if (incremental && *(volatile const int*)&slot->seed_ok) {
+        const unsigned long long mv = *(volatile const unsigned long long*)&slot->last_key;
+        dlo = key_i(mv);
+        dhi = key_j(mv);
+    }
     // the cull and the list sweep that follow start from zeroed counters (a
     // best_move sweep leaves them set on the slot the next iteration reads)
     if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -163,6 +171,7 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
     } else {
         return;  // whole warps only
     }
+    if (ke < dlo || k0 > dhi) return;  // clean: its summary stands (whole warp)
     int xlo = 1 << 30, xhi = -1, ylo = 1 << 30, yhi = -1, emax = 0, gneg = 0;
     // up to kBoxIters positions per lane, all loads issued before the first use
     constexpr int kBoxIters = (32 * kRowsLarge * kMaxWarps + 1 + 31) / 32;
@@ -202,12 +211,13 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
 
 // One thread per tile of the shard: keep the tile iff its boxes allow a pair
 // with delta < 0; kept tiles (I0, J0, index) are appended to list[] (warp-aggregated
-// atomic on slot->ncull).  With seeding, a culled tile's minimum is "none".
+// atomic on slot->ncull).  With seeding or the incremental sweep, a culled
+// tile's minimum is "none".
 __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tiles, int ntiles, int TI, int TJ,
                                                    const Box* __restrict__ rbox, const Box* __restrict__ cbox,
                                                    Slot* __restrict__ slot, int4* __restrict__ list,
                                                    unsigned long long* __restrict__ tilebest, int flags,
-                                                   int respect_done)
+                                                   int respect_done, int n)
 {
     pdl_trigger();
     pdl_wait();
@@ -215,14 +225,44 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
     const int t = blockIdx.x * blockDim.x + threadIdx.x;
     bool keep = false;
     int2 tl = make_int2(0, 0);
-    if (t < ntiles) {
+    // kSweepIncremental: a tile whose pairs (a, b) all have a, b outside the
+    // last applied move's [i, j] is clean -- positions a, a+1, b, b+1 kept
+    // their cities and e_a, e_b their lengths, so every delta and the tile's
+    // stored minimum stand.  Otherwise (or without a valid last move) it is
+    // culled (minimum: none) or listed for the sweep.
+    int dlo = 0, dhi = n;
+    if ((flags & kSweepIncremental) && !(flags & kSweepFull) && *(volatile int*)&slot->seed_ok) {
+        const unsigned long long mv = *(volatile unsigned long long*)&slot->last_key;
+        dlo = key_i(mv);
+        dhi = key_j(mv);
+    }
+    bool live = t < ntiles;
+    unsigned long long clean_min = kKeyNone;
+    if (live) {
         tl = tiles[t];
+        live = (tl.x <= dhi && tl.x + TI >= dlo) || (tl.y <= dhi && tl.y + TJ >= dlo);  // dirty
+        if (!live) clean_min = tilebest[t];  // a clean tile's stored minimum stands
+    }
+    if (flags & kSweepIncremental) {
+        // the clean tiles' share of the sweep's minimum (the re-swept tiles add
+        // theirs from the list sweep); one atomic per block at most
+        __shared__ unsigned long long s_min[8];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) clean_min = min(clean_min, __shfl_xor_sync(0xffffffffu, clean_min, o));
+        if ((threadIdx.x & 31) == 0) s_min[threadIdx.x >> 5] = clean_min;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            for (int w = 1; w < (int)(blockDim.x >> 5); w++) clean_min = min(clean_min, s_min[w]);
+            if (clean_min < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, clean_min);
+        }
+    }
+    if (live) {
         const Box r = rbox[tl.x / TI], c = cbox[tl.y / TJ];
         const long long gx = max(0, max(c.xlo - r.xhi, r.xlo - c.xhi));
         const long long gy = max(0, max(c.ylo - r.yhi, r.ylo - c.yhi));
         const long long T = (long long)max(max(r.emax, c.emax), max(r.pad[0], c.pad[0])) - 1;  // pad[0]: gneg
         keep = T >= 0 && gx * gx + gy * gy <= T * T + T;
-        if (!keep && (flags & kSweepSeed)) tilebest[t] = kKeyNone;
+        if (!keep && (flags & (kSweepSeed | kSweepIncremental))) tilebest[t] = kKeyNone;
     }
     const unsigned m = __ballot_sync(0xffffffffu, keep);
     if (m) {
@@ -578,10 +618,10 @@ cudaError_t launch_box_cull(const Geometry& g, const float2* P, const int* E, co
     const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
     const int warps = nrb + ncc;
     cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, G, n, TI, nrb, g.tj, ncc,
-                               rbox, cbox, slot, respect_done);
+                               rbox, cbox, slot, respect_done, 0);
     if (e != cudaSuccess) return e;
     e = launch_pdl(cull_kernel, dim3((ntiles + 255) / 256), dim3(256), 0, st, tiles, ntiles, TI, g.tj, rbox, cbox, slot,
-                   list, (unsigned long long*)nullptr, 0, respect_done);
+                   list, (unsigned long long*)nullptr, 0, respect_done, n);
     g_launches += 2;
     return e != cudaSuccess ? e : cudaGetLastError();
 }
@@ -608,17 +648,20 @@ cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, 
     if (ntiles <= 0 || grid <= 0) return cudaSuccess;
     const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
     const int warps = nrb + ncc;
+    const bool inc = (flags & kSweepIncremental) != 0;
     cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, (const int*)nullptr, n, TI,
-                               nrb, g.tj, ncc, rbox, cbox, slot, respect_done);
+                               nrb, g.tj, ncc, rbox, cbox, slot, respect_done, inc && !(flags & kSweepFull) ? 1 : 0);
     if (e != cudaSuccess) return e;
     e = launch_pdl(cull_kernel, dim3((ntiles + 255) / 256), dim3(256), 0, st, tiles, ntiles, TI, g.tj, rbox, cbox, slot,
-                   list, tilebest, flags, respect_done);
+                   list, tilebest, flags, respect_done, n);
     if (e != cudaSuccess) return e;
+    if (inc) flags = (flags | kSweepLocal) & ~kSweepSeed;  // tile-local minima, reusable while clean
     e = by_rows(g.rows, [&](auto r) {
         return launch_pdl(sweep_list_kernel<decltype(r)::value>, dim3(grid), dim3(32 * g.warps), sweep_smem_bytes(g),
                           st, P, E, n, tiles, list, g.tj, slot, respect_done, tilebest, flags);
     });
     g_launches += 3;
+    if (e != cudaSuccess) return e;
     return e != cudaSuccess ? e : cudaGetLastError();
 }
 

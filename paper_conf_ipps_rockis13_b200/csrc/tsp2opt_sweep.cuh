@@ -342,8 +342,10 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     // This tile's minimum of the previous sweep, if the move applied since leaves
     // it intact, is such a real pair too: it tightens the start bound and is
     // published for the other tiles.
-    unsigned long long g = *(volatile unsigned long long*)&slot->key;
-    if ((flags & kSweepSeed) && *(volatile int*)&slot->seed_ok) {
+    // kSweepLocal: the tile's own minimum over its improving pairs, independent
+    // of every other tile (reused by the incremental sweep while the tile is clean)
+    unsigned long long g = (flags & kSweepLocal) ? seed_key() : *(volatile unsigned long long*)&slot->key;
+    if (!(flags & kSweepLocal) && (flags & kSweepSeed) && *(volatile int*)&slot->seed_ok) {
         const unsigned long long mv = *(volatile unsigned long long*)&slot->last_key;
         const unsigned long long k = surviving_key(*(volatile unsigned long long*)tilebest, key_i(mv), key_j(mv));
         if (k < g) {

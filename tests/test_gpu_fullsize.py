@@ -10,7 +10,7 @@ from paper_conf_ipps_rockis13_b200 import inputs, tsp2opt
 pytestmark = pytest.mark.gpu
 
 
-@pytest.mark.parametrize("bounds", ["0", "1", "2"])
+@pytest.mark.parametrize("bounds", ["0", "1", "2", "3"])
 @pytest.mark.parametrize("cfg", ["C3", "C4", "C5"])
 def test_full_size_first_sweep(gpu, monkeypatch, cfg, bounds):
     """bounds = 0 is the launch configuration bench.py times for `value` (every

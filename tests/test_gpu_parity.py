@@ -50,7 +50,7 @@ def test_best_move_parity_sizes(gpu, n, kind):
         assert g.best_move(th) == oracle.best_move(c, th)
 
 
-@pytest.mark.parametrize("bounds", ["0", "1", "2"])
+@pytest.mark.parametrize("bounds", ["0", "1", "2", "3"])
 @pytest.mark.parametrize("rows", [7, 15])
 @pytest.mark.parametrize("warps,tj", [(1, 2), (1, 3), (1, 32), (2, 64), (4, 128), (4, 1024), (3, 7)])
 def test_best_move_parity_geometries(gpu, monkeypatch, rows, warps, tj, bounds):
@@ -92,7 +92,7 @@ def test_local_search_parity(gpu, kind, n, seed):
     c, t = _inst(kind, n, seed)
     ref = oracle.local_search(c, t)
     with tsp2opt.TSP2Opt(c) as g:
-        g.set_option(tsp2opt.OPT_TILE_BOUNDS, seed % 3)  # every filter form over the seeds
+        g.set_option(tsp2opt.OPT_TILE_BOUNDS, seed % 4)  # every filter form over the seeds
         res = g.local_search(t)
         assert res["status"] == tsp2opt.OK
         assert res["iterations"] == ref["iterations"]
@@ -131,7 +131,7 @@ def test_max_iters_parity(gpu):
             assert res["length"] == ref["length"] and np.array_equal(res["tour"], ref["tour"])
 
 
-@pytest.mark.parametrize("bounds", ["1", "2"])
+@pytest.mark.parametrize("bounds", ["1", "2", "3"])
 @pytest.mark.parametrize("world", [2, 3, 8])
 def test_simulated_shards_min_equals_full(gpu, monkeypatch, world, bounds):
     """Every shard's sweep, then the min over shards == the unsharded sweep ==
@@ -139,7 +139,7 @@ def test_simulated_shards_min_equals_full(gpu, monkeypatch, world, bounds):
     coherent (Hilbert order) so most tiles of every shard are culled."""
     monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", bounds)
     for kind, n in (("uniform", 1002), ("lattice", 7397)):
-        c, t = _inst(kind, n, 2, "hilbert" if bounds == "2" else "random")
+        c, t = _inst(kind, n, 2, "hilbert" if bounds in ("2", "3") else "random")
         with tsp2opt.TSP2Opt(c) as g:
             full = g.best_move(t)
             keys, pairs = [], 0
@@ -250,7 +250,7 @@ def test_local_search_parity_both_loops(gpu, monkeypatch, persistent, kind, n, s
         assert capped["status"] == want["status"] and np.array_equal(capped["tour"], want["tour"])
 
 
-@pytest.mark.parametrize("bounds", ["1", "2"])
+@pytest.mark.parametrize("bounds", ["1", "2", "3"])
 @pytest.mark.parametrize("rows", [7, 15])
 def test_seeded_sweeps_mixed_operations(gpu, monkeypatch, rows, bounds):
     """Each sweep after a device-resident move is seeded with the previous sweep's
@@ -260,6 +260,7 @@ def test_seeded_sweeps_mixed_operations(gpu, monkeypatch, rows, bounds):
     monkeypatch.setenv("TSP2OPT_ROWS", str(rows))
     monkeypatch.setenv("TSP2OPT_SEED", "1")
     monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", bounds)  # 2: culled tiles must reset their seeds
+    monkeypatch.setenv("TSP2OPT_CULL_ROWS", str(rows))  # 3: stored tile minima across every state change
     c, t = _inst("lattice", 3001, 8)
     rng = np.random.default_rng(3)
     with tsp2opt.TSP2Opt(c) as g:
@@ -308,3 +309,24 @@ def test_ils_parity(gpu, kind, n, iters, seed):
         assert res["length"] == ref["length"] and np.array_equal(res["tour"], ref["tour"])
         tour, L = g.get_tour()  # the handle holds the best tour afterwards
         assert np.array_equal(tour, ref["tour"]) and L == ref["length"]
+
+
+@pytest.mark.parametrize("cull_tj", ["2", "3", "32", "64"])
+@pytest.mark.parametrize("rows", [7, 15])
+@pytest.mark.parametrize("kind,n,seed,start", [("uniform", 2000, 11, "random"), ("lattice", 3001, 12, "hilbert")])
+def test_incremental_culled_local_search(gpu, monkeypatch, cull_tj, rows, kind, n, seed, start):
+    """TSP2OPT_OPT_TILE_BOUNDS = 3: after each move only the tiles with a row or
+    column position in the move's [i, j] are culled / re-swept and the others
+    keep their stored minimum; the whole move trace must equal the oracle's."""
+    monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", "3")
+    monkeypatch.setenv("TSP2OPT_CULL_TJ", cull_tj)
+    monkeypatch.setenv("TSP2OPT_CULL_ROWS", str(rows))
+    c, t = _inst(kind, n, seed, start)
+    ref = oracle.local_search(c, t, trace_cap=10 * n)
+    with tsp2opt.TSP2Opt(c) as g:
+        g.set_option(tsp2opt.OPT_TRACE, 10 * n)
+        res = g.local_search(t)
+        trace = g.get_trace(10 * n)
+    assert (res["iterations"], res["length"]) == (ref["iterations"], ref["length"])
+    assert np.array_equal(res["tour"], ref["tour"])
+    assert np.array_equal(np.asarray(trace, dtype=np.int64), ref["trace"])
