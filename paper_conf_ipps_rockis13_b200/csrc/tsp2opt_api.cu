@@ -341,18 +341,22 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         else CUDA_TRY(cudaMemsetAsync(h->d_tilebest, 0xFF, sizeof(unsigned long long) * h->ntiles, h->stream));
     }
     int flags = sweep_flags(h);
-    if (flags & kSweepIncremental) {
-        if (tiling != 1 || !h->inc_valid || h->last_tiling != tiling) flags |= kSweepFull;
-        h->inc_valid = tiling == 1;
+    // A lone sweep (best_move: no apply follows) takes the global bound -- faster on
+    // incoherent tours; its minima are not reusable, so the next incremental sweep is full.
+    if (!apply) flags &= ~kSweepIncremental;
+    if (flags & kSweepIncremental) {  // the culled tilings (2-opt and 2.5-opt) keep per-tile minima
+        const bool culled = tiling == 1 || tiling == 3;
+        if (!culled || !h->inc_valid || h->last_tiling != tiling) flags |= kSweepFull;
+        h->inc_valid = culled;
     } else {
         h->inc_valid = false;
     }
     h->last_tiling = tiling;
     if (tiling == 3 && h->tile_bounds >= 2) {  // 2.5-opt, culled: box + cull (with gains) + list sweep
         CUDA_TRY(launch_box_cull(h->cgeo, h->d_P, h->d_E, h->d_G, h->n, h->d_ctiles, h->nctiles, h->d_rbox, h->d_cbox,
-                                 h->d_list, in, apply ? 1 : 0, h->stream));
+                                 h->d_list, in, apply ? 1 : 0, h->d_ctilebest, flags, h->stream));
         CUDA_TRY(launch_sweep25_list(h->cgeo, h->d_P, h->d_E, h->d_G, h->n, h->d_list, h->list25_grid, in,
-                                     apply ? 1 : 0, h->stream));
+                                     apply ? 1 : 0, h->d_ctilebest, flags, h->stream));
     } else if (tiling == 3) {  // 2.5-opt: dense tiling (R = 7), per-tile bound unless TILE_BOUNDS = 0
         CUDA_TRY(launch_sweep25(h->geo, h->d_P, h->d_E, h->d_G, h->n, h->d_tiles, h->ntiles, in, apply ? 1 : 0,
                                 h->tile_bounds != 0 ? kSweepTileBounds : 0, h->stream));

@@ -79,7 +79,8 @@ cudaError_t launch_sweep25(const Geometry& g, const float2* P, const int* E, con
 cudaError_t launch_gain(const float2* P, int* G, int n, int lo, int hi, cudaStream_t st);
 int sweep25_list_grid(const Geometry& g, int ntiles);
 cudaError_t launch_sweep25_list(const Geometry& g, const float2* P, const int* E, const int* G, int n,
-                                const int4* list, int grid, Slot* slot, int respect_done, cudaStream_t st);
+                                const int4* list, int grid, Slot* slot, int respect_done,
+                                unsigned long long* tilebest, int flags, cudaStream_t st);
 cudaError_t launch_decide25(const float2* P, const int* E, const int* G, Slot* slot, cudaStream_t st);
 cudaError_t launch_apply25(float2* P, int* E, int* G, int* tour, int n, const Slot* in, Slot* out,
                            long long max_moves, int explicit_move, int ei, int ej, int etype,
@@ -97,7 +98,8 @@ cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n
 int sweep_list_grid(const Geometry& g, int ntiles);
 // box + cull only (the 2.5-opt list sweep follows); G != NULL adds the gain term to the cull
 cudaError_t launch_box_cull(const Geometry& g, const float2* P, const int* E, const int* G, int n, const int2* tiles,
-                            int ntiles, Box* rbox, Box* cbox, int4* list, Slot* slot, int respect_done, cudaStream_t st);
+                            int ntiles, Box* rbox, Box* cbox, int4* list, Slot* slot, int respect_done,
+                            unsigned long long* tilebest, int flags, cudaStream_t st);
 cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles,
                               int ntiles, int grid, Box* rbox, Box* cbox, int4* list, Slot* slot, int respect_done,
                               unsigned long long* tilebest, int flags, cudaStream_t st);

@@ -138,7 +138,8 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* 
 __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, const int* __restrict__ E,
                                                   const int* __restrict__ G, int n, int TI, int nrb, int TJ, int ncc,
                                                   Box* __restrict__ rbox, Box* __restrict__ cbox,
-                                                  Slot* __restrict__ slot, int respect_done, int incremental)
+                                                  Slot* __restrict__ slot, int respect_done, int incremental,
+                                                  int halo)
 {
     pdl_trigger();
     pdl_wait();
@@ -147,8 +148,8 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
     int dlo = 0, dhi = n;
     if (incremental && *(volatile const int*)&slot->seed_ok) {
         const unsigned long long mv = *(volatile const unsigned long long*)&slot->last_key;
-        dlo = key_i(mv);
-        dhi = key_j(mv);
+        dlo = key_i(mv) - halo;  // halo 1 for 2.5-opt: the gains changed on [i, j+1]
+        dhi = key_j(mv) + halo;
     }
     // the cull and the list sweep that follow start from zeroed counters (a
     // best_move sweep leaves them set on the slot the next iteration reads)
@@ -217,7 +218,7 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
                                                    const Box* __restrict__ rbox, const Box* __restrict__ cbox,
                                                    Slot* __restrict__ slot, int4* __restrict__ list,
                                                    unsigned long long* __restrict__ tilebest, int flags,
-                                                   int respect_done, int n)
+                                                   int respect_done, int n, int halo)
 {
     pdl_trigger();
     pdl_wait();
@@ -233,8 +234,8 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
     int dlo = 0, dhi = n;
     if ((flags & kSweepIncremental) && !(flags & kSweepFull) && *(volatile int*)&slot->seed_ok) {
         const unsigned long long mv = *(volatile unsigned long long*)&slot->last_key;
-        dlo = key_i(mv);
-        dhi = key_j(mv);
+        dlo = key_i(mv) - halo;  // 2.5-opt (halo 1): a pair also reads g_{a+1}, g_b and D(a+1, b)
+        dhi = key_j(mv) + halo;
     }
     bool live = t < ntiles;
     unsigned long long clean_min = kKeyNone;
@@ -613,15 +614,17 @@ cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n
 }
 
 cudaError_t launch_box_cull(const Geometry& g, const float2* P, const int* E, const int* G, int n, const int2* tiles,
-                            int ntiles, Box* rbox, Box* cbox, int4* list, Slot* slot, int respect_done, cudaStream_t st)
+                            int ntiles, Box* rbox, Box* cbox, int4* list, Slot* slot, int respect_done,
+                            unsigned long long* tilebest, int flags, cudaStream_t st)
 {
     const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
     const int warps = nrb + ncc;
+    const bool inc = (flags & kSweepIncremental) != 0;
     cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, G, n, TI, nrb, g.tj, ncc,
-                               rbox, cbox, slot, respect_done, 0);
+                               rbox, cbox, slot, respect_done, inc && !(flags & kSweepFull) ? 1 : 0, 1);
     if (e != cudaSuccess) return e;
     e = launch_pdl(cull_kernel, dim3((ntiles + 255) / 256), dim3(256), 0, st, tiles, ntiles, TI, g.tj, rbox, cbox, slot,
-                   list, (unsigned long long*)nullptr, 0, respect_done, n);
+                   list, tilebest, flags, respect_done, n, 1);
     g_launches += 2;
     return e != cudaSuccess ? e : cudaGetLastError();
 }
@@ -650,10 +653,10 @@ cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, 
     const int warps = nrb + ncc;
     const bool inc = (flags & kSweepIncremental) != 0;
     cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, (const int*)nullptr, n, TI,
-                               nrb, g.tj, ncc, rbox, cbox, slot, respect_done, inc && !(flags & kSweepFull) ? 1 : 0);
+                               nrb, g.tj, ncc, rbox, cbox, slot, respect_done, inc && !(flags & kSweepFull) ? 1 : 0, 0);
     if (e != cudaSuccess) return e;
     e = launch_pdl(cull_kernel, dim3((ntiles + 255) / 256), dim3(256), 0, st, tiles, ntiles, TI, g.tj, rbox, cbox, slot,
-                   list, tilebest, flags, respect_done, n);
+                   list, tilebest, flags, respect_done, n, 0);
     if (e != cudaSuccess) return e;
     if (inc) flags = (flags | kSweepLocal) & ~kSweepSeed;  // tile-local minima, reusable while clean
     e = by_rows(g.rows, [&](auto r) {

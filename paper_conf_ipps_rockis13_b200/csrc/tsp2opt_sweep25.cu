@@ -284,7 +284,8 @@ __device__ __forceinline__ void reverse_range(float2* P, int* tour, int lo, int 
 // The caller synchronises the CTA before the shared chunk is reused.
 __device__ __forceinline__ void sweep25_tile(const float2* __restrict__ P, const int* __restrict__ E,
                                              const int* __restrict__ G, int n, int2 tile, int TJ,
-                                             Slot* __restrict__ slot, void* smem, int flags)
+                                             Slot* __restrict__ slot, void* smem, int flags,
+                                             unsigned long long* __restrict__ tilebest)
 {
     const int TI = 32 * R25 * (int)(blockDim.x >> 5);
     const Tile25Smem sm(smem, TJ, TI);
@@ -320,7 +321,8 @@ __device__ __forceinline__ void sweep25_tile(const float2* __restrict__ P, const
         sm.cole[c] = (float)__ldg(E + J0 + c);
         sm.colg[c] = (float)__ldg(G + J0 + c);
     }
-    const unsigned long long g = *(volatile unsigned long long*)&slot->key;
+    // kSweepLocal: the tile's own minimum (reused by the incremental sweep while clean)
+    const unsigned long long g = (flags & kSweepLocal) ? seed_key() : *(volatile unsigned long long*)&slot->key;
     const int dg = key_delta(g);
     if (active) {
 #pragma unroll
@@ -330,21 +332,32 @@ __device__ __forceinline__ void sweep25_tile(const float2* __restrict__ P, const
         }
     }
     __syncthreads();
-    if (!active) return;
     unsigned long long mykey = kKeyNone;
-    Bound25 b;
-    set_bound25(b, erow, grow, dg == 0 ? 0 : dg + 1);
-    const bool masked = (wrow0 + 32 * R25 - 1) >= jstart;
-    if (!(flags & kSweepTileBounds) || tile_may_pass25(rows, b, sm, jstart - J0, J1 - J0)) {
-        if (masked) walk25<true, false>(rows, b, row0, jstart, J0, J1, sm, my_rowe, my_rowg, P, mykey);
-        else walk25<false, false>(rows, b, row0, jstart, J0, J1, sm, my_rowe, my_rowg, P, mykey);
-    }
+    if (active) {
+        Bound25 b;
+        set_bound25(b, erow, grow, dg == 0 ? 0 : dg + 1);
+        const bool masked = (wrow0 + 32 * R25 - 1) >= jstart;
+        if (!(flags & kSweepTileBounds) || tile_may_pass25(rows, b, sm, jstart - J0, J1 - J0)) {
+            if (masked) walk25<true, false>(rows, b, row0, jstart, J0, J1, sm, my_rowe, my_rowg, P, mykey);
+            else walk25<false, false>(rows, b, row0, jstart, J0, J1, sm, my_rowe, my_rowg, P, mykey);
+        }
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        const unsigned long long other = __shfl_xor_sync(0xffffffffu, mykey, o);
-        mykey = other < mykey ? other : mykey;
+        for (int o = 16; o > 0; o >>= 1) {
+            const unsigned long long other = __shfl_xor_sync(0xffffffffu, mykey, o);
+            mykey = other < mykey ? other : mykey;
+        }
+        if (lane == 0 && mykey < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, mykey);
     }
-    if (lane == 0 && mykey < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, mykey);
+    if (tilebest) {  // the tile's minimum over its warps (incremental sweep)
+        __shared__ unsigned long long s_red25[kMaxWarps];
+        if (lane == 0) s_red25[warp] = mykey;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            unsigned long long m = s_red25[0];
+            for (int w = 1; w < (int)(blockDim.x >> 5); w++) m = s_red25[w] < m ? s_red25[w] : m;
+            *tilebest = m;
+        }
+    }
 }
 
 __global__ void __launch_bounds__(128, 4) sweep25_kernel(const float2* __restrict__ P, const int* __restrict__ E,
@@ -356,7 +369,7 @@ __global__ void __launch_bounds__(128, 4) sweep25_kernel(const float2* __restric
     pdl_trigger();
     pdl_wait();
     if (respect_done && *(volatile int*)&slot->done) return;  // converged: iteration is a no-op
-    sweep25_tile(P, E, G, n, tiles[blockIdx.x], TJ, slot, smem25, flags);
+    sweep25_tile(P, E, G, n, tiles[blockIdx.x], TJ, slot, smem25, flags, nullptr);
 }
 
 // The 2.5-opt sweep over the culled list (as sweep_list_kernel: first entry
@@ -364,7 +377,8 @@ __global__ void __launch_bounds__(128, 4) sweep25_kernel(const float2* __restric
 __global__ void __launch_bounds__(128, 4) sweep25_list_kernel(const float2* __restrict__ P,
                                                               const int* __restrict__ E, const int* __restrict__ G,
                                                               int n, const int4* __restrict__ list, int TJ,
-                                                              Slot* __restrict__ slot, int respect_done)
+                                                              Slot* __restrict__ slot, int respect_done,
+                                                              unsigned long long* __restrict__ tilebest, int flags)
 {
     extern __shared__ float4 smem25[];
     __shared__ int4 s_t;
@@ -378,7 +392,8 @@ __global__ void __launch_bounds__(128, 4) sweep25_list_kernel(const float2* __re
         __syncthreads();
         const int4 e = s_t;
         if (e.z < 0) break;
-        sweep25_tile(P, E, G, n, make_int2(e.x, e.y), TJ, slot, smem25, kSweepTileBounds);
+        sweep25_tile(P, E, G, n, make_int2(e.x, e.y), TJ, slot, smem25, flags | kSweepTileBounds,
+                     (flags & kSweepIncremental) ? tilebest + e.z : nullptr);
         if (threadIdx.x == 0) k = gridDim.x + atomicAdd(&slot->next_tile, 1u);
         __syncthreads();
     }
@@ -443,7 +458,7 @@ __global__ void __launch_bounds__(256) apply25_kernel(float2* __restrict__ P, in
             o.done = explicit_move ? (done & 4) : done;
             o.next_tile = 0;
             o.ncull = 0;
-            o.seed_ok = 0;
+            o.seed_ok = (apply && !explicit_move) ? 1 : 0;  // the incremental sweep may reuse clean tiles
             o.mtype = t;
             if (!explicit_move && !done) {
                 if (delta >= 0) o.done = 1;              // local minimum (reading R7)
@@ -510,12 +525,14 @@ int sweep25_list_grid(const Geometry& g, int ntiles)
 }
 
 cudaError_t launch_sweep25_list(const Geometry& g, const float2* P, const int* E, const int* G, int n,
-                                const int4* list, int grid, Slot* slot, int respect_done, cudaStream_t st)
+                                const int4* list, int grid, Slot* slot, int respect_done,
+                                unsigned long long* tilebest, int flags, cudaStream_t st)
 {
+    if (flags & kSweepIncremental) flags = (flags | kSweepLocal) & ~kSweepSeed;
     if (grid <= 0) return cudaSuccess;
     if (g.rows != R25) return cudaErrorInvalidValue;
     cudaError_t e = launch_kernel_pdl(sweep25_list_kernel, dim3(grid), dim3(32 * g.warps), sweep25_smem_bytes(g), st,
-                                      P, E, G, n, list, g.tj, slot, respect_done);
+                                      P, E, G, n, list, g.tj, slot, respect_done, tilebest, flags);
     if (e != cudaSuccess) return e;
     count_launch(1);
     return cudaGetLastError();

@@ -30,7 +30,7 @@ def test_best_move25_parity(gpu, n, kind):
             assert g.best_move(t) == (i, j, d)
 
 
-@pytest.mark.parametrize("bounds", ["0", "1", "2"])
+@pytest.mark.parametrize("bounds", ["0", "1", "2", "3"])
 @pytest.mark.parametrize("warps,tj", [(1, 2), (1, 3), (1, 32), (2, 64), (4, 128), (3, 7)])
 def test_best_move25_geometries(gpu, monkeypatch, warps, tj, bounds):
     monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", bounds)
@@ -64,12 +64,14 @@ def test_local_search25_trace(gpu, kind, n, seed):
     assert set(np.unique(want["trace"][:, 3]).tolist()) == {0, 1, 2}  # every move type occurs
 
 
+@pytest.mark.parametrize("bounds", ["2", "3"])
 @pytest.mark.parametrize("cull_tj", ["2", "3", "32", "64"])
 @pytest.mark.parametrize("kind,n,seed", [("uniform", 1002, 5), ("lattice", 2000, 6)])
-def test_local_search25_culled(gpu, monkeypatch, cull_tj, kind, n, seed):
+def test_local_search25_culled(gpu, monkeypatch, cull_tj, kind, n, seed, bounds):
     """The pre-sweep cull with the gain term (box + cull + list sweep), forced at
-    small n, with narrow and ragged column chunks."""
-    monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", "2")
+    small n, with narrow and ragged column chunks; bounds 3 keeps the tiles'
+    own minima and re-sweeps only the tiles the last move touched."""
+    monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", bounds)
     monkeypatch.setenv("TSP2OPT_CULL_TJ", cull_tj)
     c = inputs.make_coords(kind, n, seed)
     t = inputs.random_tour(n, seed)
@@ -112,10 +114,12 @@ def test_local_search25_max_iters(gpu):
             assert np.array_equal(res["tour"], want["tour"])
 
 
-def test_25opt_mixed_operations(gpu):
+@pytest.mark.parametrize("bounds", ["1", "3"])
+def test_25opt_mixed_operations(gpu, monkeypatch, bounds):
     """Explicit moves of every type (edges of the position range included),
     switching the mode off and on around device-side iterations, simulated
-    shards, and the error cases."""
+    shards, and the error cases; bounds 3: stored tile minima across all of it."""
+    monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", bounds)
     n = 1200
     c = inputs.make_coords("lattice", n, 5)
     t = inputs.random_tour(n, 5)
