@@ -231,18 +231,25 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
     // their cities and e_a, e_b their lengths, so every delta and the tile's
     // stored minimum stand.  Otherwise (or without a valid last move) it is
     // culled (minimum: none) or listed for the sweep.
+    // all independent loads first (the kernel is latency bound: one short chain per thread)
+    const bool inc = (flags & kSweepIncremental) && !(flags & kSweepFull);
+    const int seed_ok = inc ? *(volatile int*)&slot->seed_ok : 0;
+    const unsigned long long mv = inc ? *(volatile unsigned long long*)&slot->last_key : 0ull;
+    bool live = t < ntiles;
+    unsigned long long stored = kKeyNone;
+    if (live) {
+        tl = tiles[t];
+        if (inc) stored = tilebest[t];
+    }
     int dlo = 0, dhi = n;
-    if ((flags & kSweepIncremental) && !(flags & kSweepFull) && *(volatile int*)&slot->seed_ok) {
-        const unsigned long long mv = *(volatile unsigned long long*)&slot->last_key;
+    if (seed_ok) {
         dlo = key_i(mv) - halo;  // 2.5-opt (halo 1): a pair also reads g_{a+1}, g_b and D(a+1, b)
         dhi = key_j(mv) + halo;
     }
-    bool live = t < ntiles;
     unsigned long long clean_min = kKeyNone;
     if (live) {
-        tl = tiles[t];
         live = (tl.x <= dhi && tl.x + TI >= dlo) || (tl.y <= dhi && tl.y + TJ >= dlo);  // dirty
-        if (!live) clean_min = tilebest[t];  // a clean tile's stored minimum stands
+        if (!live) clean_min = stored;  // a clean tile's stored minimum stands
     }
     if (flags & kSweepIncremental) {
         // the clean tiles' share of the sweep's minimum (the re-swept tiles add
