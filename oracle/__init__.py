@@ -87,6 +87,10 @@ def _load():
             lib.oracle25_apply.restype = None
             lib.oracle25_local_search.argtypes = [p, i64, p, i64, p, p, p, i64]
             lib.oracle25_local_search.restype = ctypes.c_int
+            lib.oracle_first_move.argtypes = [p, i64, p, p, p, p]
+            lib.oracle_first_move.restype = None
+            lib.oracle_first_local_search.argtypes = [p, i64, p, i64, p, p, p, i64]
+            lib.oracle_first_local_search.restype = ctypes.c_int
             lib.oracle_num_threads.argtypes = []
             lib.oracle_num_threads.restype = ctypes.c_int
             _lib = lib
@@ -293,6 +297,27 @@ def local_search25(coords, tour, max_iters: int = -1, trace_cap: int = 0):
     tr = np.zeros((max(trace_cap, 1), 4), dtype=np.int64)
     st = _load().oracle25_local_search(_ptr(xy), xy.shape[0], _ptr(t), int(max_iters), _ptr(out[0:1]),
                                        _ptr(out[1:2]), _ptr(tr) if trace_cap > 0 else None, int(trace_cap))
+    it = int(out[1])
+    return dict(tour=t, length=int(out[0]), iterations=it, status=int(st), trace=tr[: min(it, trace_cap)].copy())
+
+
+def first_move(coords, tour):
+    """(i, j, delta): the improving pair with the lowest Fig. 3 cell, else (0, 1, 0) (reading R20)."""
+    xy = _xy(coords)
+    t = np.ascontiguousarray(tour, dtype=np.int32)
+    out = np.zeros(3, dtype=np.int64)
+    _load().oracle_first_move(_ptr(xy), xy.shape[0], _ptr(t), _ptr(out[0:1]), _ptr(out[1:2]), _ptr(out[2:3]))
+    return int(out[0]), int(out[1]), int(out[2])
+
+
+def first_local_search(coords, tour, max_iters: int = -1, trace_cap: int = 0):
+    """First-improvement 2-opt local search (reading R20); same return dict as local_search."""
+    xy = _xy(coords)
+    t = np.array(tour, dtype=np.int32, copy=True)
+    out = np.zeros(2, dtype=np.int64)
+    tr = np.zeros((max(trace_cap, 1), 3), dtype=np.int64)
+    st = _load().oracle_first_local_search(_ptr(xy), xy.shape[0], _ptr(t), int(max_iters), _ptr(out[0:1]),
+                                           _ptr(out[1:2]), _ptr(tr) if trace_cap > 0 else None, int(trace_cap))
     it = int(out[1])
     return dict(tour=t, length=int(out[0]), iterations=it, status=int(st), trace=tr[: min(it, trace_cap)].copy())
 

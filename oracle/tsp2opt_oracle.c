@@ -37,6 +37,9 @@
  *                        operations on city ids; the neighbourhood as a set of
  *                        cycles == 2-opt neighbours + node insertions; the
  *                        sweep == the per-move definition; global optima.
+ *   oracle_first_* (tests/test_oracle_first.py) -- first improvement: the
+ *                        first improving neighbour of an explicit scan in cell
+ *                        order; 2-opt local-minimum certificate.
  */
 #include <math.h>
 #include <stdint.h>
@@ -674,6 +677,54 @@ int oracle25_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64_t m
         L += d;
         if (trace && it < trace_cap) {
             trace[4 * it] = i; trace[4 * it + 1] = j; trace[4 * it + 2] = d; trace[4 * it + 3] = t;
+        }
+        it++;
+    }
+    *length = L;
+    *iterations = it;
+    return status;
+}
+
+/* ---------------------------------------------------------------------------
+ * First-improvement 2-opt.  Reading R20 (DESIGN.md
+ * §3): the paper's sequential loop visits the pairs in the Fig. 3 cell order
+ * (L14: "0,1 0  0,2 1  1,2 2 ..."); first improvement applies the first pair
+ * of that order with delta < 0 and restarts the scan, i.e. it takes the
+ * improving pair with the lowest cell number instead of the lowest delta.
+ * Same neighbourhood (reading R1), same apply, same termination (R7): at a
+ * local minimum it returns (0, 1, 0).
+ * ------------------------------------------------------------------------- */
+void oracle_first_move(const int32_t *xy, int64_t n, const int32_t *tour, int64_t *bi, int64_t *bj, int64_t *bdelta)
+{
+    for (int64_t j = 1; j < n; j++)
+        for (int64_t i = 0; i < j; i++) {
+            int64_t d = oracle_delta(xy, n, tour, i, j);
+            if (d < 0) {
+                *bi = i; *bj = j; *bdelta = d;
+                return;
+            }
+        }
+    *bi = 0; *bj = 1; *bdelta = 0;
+}
+
+int oracle_first_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64_t max_iters,
+                              int64_t *length, int64_t *iterations, int64_t *trace, int64_t trace_cap)
+{
+    int64_t L = oracle_tour_length(xy, n, tour);
+    int64_t it = 0;
+    int status = 0;
+    for (;;) {
+        int64_t i, j, d;
+        oracle_first_move(xy, n, tour, &i, &j, &d);
+        if (d >= 0) break;
+        if (max_iters >= 0 && it >= max_iters) { /* reading R8 */
+            status = 1;
+            break;
+        }
+        oracle_apply(tour, i, j);
+        L += d;
+        if (trace && it < trace_cap) {
+            trace[3 * it] = i; trace[3 * it + 1] = j; trace[3 * it + 2] = d;
         }
         it++;
     }
