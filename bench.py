@@ -215,11 +215,12 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms, sweep_avg_ms, e2e_total, tb_total_ms, tb_sweep_ms = t.tolist()
 
-    ls = ils = batch = batch_ils = pruned = or25 = None
+    ls = ils = batch = batch_ils = pruned = or25 = first = None
     if rank == 0 and world == 1 and not args.no_ls:
         ls = time_to_local_min(tsp2opt, args.ls_config)
         pruned = time_pruned(tsp2opt, args.pruned_config, not args.no_cpu) if args.pruned_config else None
         or25 = time_25opt(tsp2opt, args.or25_config, not args.no_cpu) if args.or25_config else None
+        first = time_first(tsp2opt, args.first_config) if args.first_config else None
         ils = time_ils(tsp2opt, args.ils_config) if args.ils_config else None
         batch = time_batch(tsp2opt, args.batch_config, not args.no_cpu) if args.batch_config else None
         batch_ils = time_batch_ils(tsp2opt, args.batch_ils_config, not args.no_cpu) if args.batch_ils_config else None
@@ -274,6 +275,8 @@ def run_ours(args):
             line["pruned_local_search"] = pruned
         if or25:
             line["local_search_25opt"] = or25
+        if first:
+            line["local_search_first_improvement"] = first
         if batch:
             line["batch_local_search"] = batch
         if batch_ils:
@@ -440,6 +443,30 @@ def time_25opt(tsp2opt, spec, with_oracle=True):
                                    "sample": f"{reps} oracle 2.5-opt sweeps of the MF tour; the local search "
                                              "estimate is per-sweep time x (moves + 1)"}
         out.append(entry)
+    return out
+
+
+def time_first(tsp2opt, spec):
+    """First-improvement 2-opt (TSP2OPT_OPT_FIRST_IMPROVEMENT; SURVEY §8(f) NEXT-4;
+    reading R20) to the local minimum, `cfg` (random start) or `cfg:mf` entries,
+    wall time of tsp2opt_local_search (as time_to_local_minimum)."""
+    out = []
+    for item in spec.split(","):
+        if not item:
+            continue
+        name, _, tk = item.partition(":")
+        coords, tour = inputs.config_instance(name, "random")
+        n = len(coords)
+        with tsp2opt.TSP2Opt(coords) as g:
+            if tk == "mf":
+                tour = g.mf_tour()["tour"]
+            g.set_option(tsp2opt.OPT_FIRST_IMPROVEMENT, 1)
+            g.local_search(tour, max_iters=2)  # warm-up
+            t0 = time.perf_counter()
+            r = g.local_search(tour)
+            dt = time.perf_counter() - t0
+        out.append({"config": name, "n": n, "start": tk or "random", "rule": "first improvement", "seconds": dt,
+                    "iterations": r["iterations"], "length": r["length"]})
     return out
 
 
@@ -638,6 +665,7 @@ def main():
     ap.add_argument("--ils-config", default="C1:200,C2:50", help="Iterated Local Search runs cfg:iterations")
     ap.add_argument("--pruned-config", default="C3:8,C4:8,C5:8,C5:16", help="pruned 2-opt from MF, cfg:K")
     ap.add_argument("--or25-config", default="C3,C4,C5", help="2.5-opt local search from MF, configs")
+    ap.add_argument("--first-config", default="C1,C2,C3:mf,C4:mf,C5:mf", help="first-improvement local search")
     ap.add_argument("--batch-config", default="100:4736,1002:592", help="batched local search n:instances")
     ap.add_argument("--batch-ils-config", default="C1:4736:100", help="batched ILS cfg:replicas:steps")
     ap.add_argument("--no-ls", action="store_true")

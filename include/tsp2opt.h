@@ -196,7 +196,8 @@ int tsp2opt_mf_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length, int32_t *ro
 /* Copy the current tour (host int32[n]) and its length out. */
 int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
 
-/* Execution options (none but TSP2OPT_OPT_NEIGHBOURS changes any result; all results stay bit-exact):
+/* Execution options (NEIGHBOURS, NODE_INSERTION and FIRST_IMPROVEMENT select the method; the others change
+ * no result; all results stay bit-exact with the corresponding oracle):
  *  TSP2OPT_OPT_TILE_BOUNDS (default 3 from 1e8 pairs per rank, else 1): 1 = skip a tile of the sweep when the
  *      bounding boxes of its row and column cities prove that no pair can pass
  *      the per-pair necessary condition; 2 = the same, plus a
@@ -239,6 +240,13 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
  *      moves.  Results equal oracle25_*.  Not with TSP2OPT_OPT_NEIGHBOURS > 0
  *      (EINVAL) or tsp2opt_ils; the sweep uses R = 7 rows per lane and the
  *      per-tile bound (no pre-sweep cull, no persistent loop).
+ *  TSP2OPT_OPT_FIRST_IMPROVEMENT (default 0): 1 = first improvement (SURVEY.md
+ *      §8(f) NEXT-4; reading R20): best_move returns the improving
+ *      pair with the lowest Fig. 3 cell (the first one the paper's sequential
+ *      pair order reaches) instead of the lowest delta, with its exact delta;
+ *      local_search applies it and restarts.  Not with TSP2OPT_OPT_NEIGHBOURS,
+ *      TSP2OPT_OPT_NODE_INSERTION or tsp2opt_ils (EINVAL).  Equals
+ *      oracle_first_*.
  * Returns TSP2OPT_EINVAL for an unknown option or value. */
 #define TSP2OPT_OPT_TILE_BOUNDS 1
 #define TSP2OPT_OPT_SEED 2
@@ -247,6 +255,7 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
 #define TSP2OPT_OPT_NEIGHBOURS 5
 #define TSP2OPT_MAX_NEIGHBOURS 16
 #define TSP2OPT_OPT_NODE_INSERTION 6
+#define TSP2OPT_OPT_FIRST_IMPROVEMENT 7
 int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value);
 
 /* Recorded move trace: writes min(count, cap) rows of int32 (i, j, delta) into

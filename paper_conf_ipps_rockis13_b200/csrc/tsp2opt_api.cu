@@ -94,6 +94,7 @@ struct tsp2opt_ctx {
     unsigned long long* d_knn = nullptr;  // [n * kMaxNeighbours] exact nearest-neighbour keys (d << 22 | c)
     int* d_pos = nullptr;       // [n] inverse permutation pos[tour[k]] = k (pruned sweep only)
     int or25 = 0;               // TSP2OPT_OPT_NODE_INSERTION: 1 = 2.5-opt (2-opt plus node insertion, reading R19)
+    int first = 0;              // TSP2OPT_OPT_FIRST_IMPROVEMENT: 1 = lowest improving cell (reading R20)
     int* d_G = nullptr;         // [n + 1 + pad] removal gains g_k (2.5-opt only)
     unsigned* d_bar25 = nullptr;  // [2] grid barrier of the 2.5-opt apply
     int* d_ttype = nullptr;     // [trace_cap] move types of the traced moves (2.5-opt)
@@ -314,8 +315,8 @@ int load_host_tour(tsp2opt_ctx* h, const int32_t* tour)
 
 int sweep_flags(const tsp2opt_ctx* h)
 {
-    return (h->seed_next ? kSweepSeed : 0) | (h->tile_bounds != 0 ? kSweepTileBounds : 0) |
-           (h->tile_bounds == 3 ? kSweepIncremental : 0);
+    return (h->seed_next && !h->first ? kSweepSeed : 0) | (h->tile_bounds != 0 ? kSweepTileBounds : 0) |
+           (h->tile_bounds == 3 ? kSweepIncremental : 0) | (h->first ? kSweepFirst : 0);
 }
 
 // One iteration: sweep (a4/a5) -> allreduce-min (a6) -> apply (a7/a8).
@@ -364,7 +365,7 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         const int p0 = (int)((long long)h->n * h->shard_rank / h->shard_world);
         const int p1 = (int)((long long)h->n * (h->shard_rank + 1) / h->shard_world);
         CUDA_TRY(launch_pruned_sweep(h->d_P, h->d_E, h->d_tour, h->d_pos, h->d_knn, h->nbr_k, h->n, p0, p1, in,
-                                     apply ? 1 : 0, h->stream));
+                                     apply ? 1 : 0, h->first, h->stream));
     } else if (tiling) {  // cull first, then sweep the kept tiles only
         CUDA_TRY(launch_cull_sweep(h->cgeo, h->d_P, h->d_E, h->n, h->d_ctiles, h->nctiles, h->list_grid, h->d_rbox,
                                    h->d_cbox, h->d_list, in, apply ? 1 : 0, h->d_ctilebest, flags, h->stream));
@@ -377,6 +378,8 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         ncclResult_t r = ncclAllReduce(&in->key, &in->key, 1, ncclUint64, ncclMin, h->comm, h->stream);
         if (r != ncclSuccess) return nccl_fail(r, "ncclAllReduce");
     }
+    // first improvement: the min carries the marker delta; the exact delta of the winner
+    if (h->first) CUDA_TRY(launch_first_fix(h->d_P, h->d_E, in, apply ? 1 : 0, h->stream));
     if (apply && h->or25) {
         Slot* out = h->d_slots + (h->parity ^ 1);
         CUDA_TRY(launch_apply25(h->d_P, h->d_E, h->d_G, h->d_tour, h->n, in, out, max_moves, 0, 0, 0, 0, h->d_trace,
@@ -402,7 +405,7 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
     // n ~ 7e3 where the per-sweep kernels pack tiles better); TSP2OPT_PERSISTENT
     // = 0 / 1 forces either loop, 2 (default) chooses by pair count.
     const bool use_persistent =
-        !h->comm && h->nbr_k == 0 && !h->or25 && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
+        !h->comm && h->nbr_k == 0 && !h->or25 && !h->first && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
     if (use_persistent) {
         h->inc_valid = false;
         // One persistent cooperative launch runs sweep -> apply to the local
@@ -795,8 +798,8 @@ int tsp2opt_batch_ils_async(const int32_t* d_coords_xy, int32_t n, int32_t batch
 int tsp2opt_ils(tsp2opt_t h, int32_t* tour, int64_t iterations, uint64_t seed, int64_t* length, int64_t* lengths)
 {
     if (!h || !tour || !length || iterations < 0) return TSP2OPT_EINVAL;
-    if (h->nbr_k > 0 || h->or25) {  // ILS is defined (and pinned) on the full 2-opt neighbourhood only
-        g_last_error = "tsp2opt_ils: set TSP2OPT_OPT_NEIGHBOURS and TSP2OPT_OPT_NODE_INSERTION to 0 first";
+    if (h->nbr_k > 0 || h->or25 || h->first) {  // ILS is defined (and pinned) for best-improvement 2-opt only
+        g_last_error = "tsp2opt_ils: set TSP2OPT_OPT_NEIGHBOURS, _NODE_INSERTION and _FIRST_IMPROVEMENT to 0 first";
         return TSP2OPT_EINVAL;
     }
     int rc = load_host_tour(h, tour);
@@ -899,8 +902,15 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
         if (value < 0 || value > 2) return TSP2OPT_EINVAL;
         h->persistent = (int)value;
         break;
+    case TSP2OPT_OPT_FIRST_IMPROVEMENT: {
+        if (value < 0 || value > 1 || (value && (h->or25 || h->nbr_k > 0))) return TSP2OPT_EINVAL;
+        h->first = (int)value;
+        if (h->has_tour) CUDA_TRY(launch_reset_key(h->d_slots + h->parity, h->stream));  // pending key: other rule
+        CUDA_TRY(cudaStreamSynchronize(h->stream));
+        break;
+    }
     case TSP2OPT_OPT_NODE_INSERTION: {
-        if (value < 0 || value > 1 || (value && h->nbr_k > 0)) return TSP2OPT_EINVAL;
+        if (value < 0 || value > 1 || (value && (h->nbr_k > 0 || h->first))) return TSP2OPT_EINVAL;
         CUDA_TRY(cudaStreamSynchronize(h->stream));
         if (value && !h->d_G) {
             const size_t np = (size_t)h->n + 1 + kPad;
@@ -929,7 +939,7 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
         break;
     }
     case TSP2OPT_OPT_NEIGHBOURS: {
-        if (value < 0 || value > kMaxNeighbours || (value && h->or25)) return TSP2OPT_EINVAL;
+        if (value < 0 || value > kMaxNeighbours || (value && (h->or25 || h->first))) return TSP2OPT_EINVAL;
         if (value > 0) {
             if (!h->d_knn) {  // exact candidate lists, once per handle (coordinates never change)
                 unsigned long long* knn = nullptr;

@@ -29,6 +29,10 @@ constexpr int kSweepLocal = 4;       // tile-local bound (start at delta < 0, ig
                                      // minimum is then exact on its own and can be reused while the tile is clean
 constexpr int kSweepIncremental = 8; // culled sweep: only tiles the last applied move touched are re-swept
 constexpr int kSweepFull = 16;       // incremental sweep whose stored minima are not valid yet: re-sweep all
+// First improvement (reading R20): improving pairs enter the min with this
+// delta, so the min is the lowest cell; first_fix_kernel writes the real delta.
+constexpr int kFirstDelta = -1;
+constexpr int kSweepFirst = 32;      // first improvement: the lowest improving cell instead of the lowest delta
 
 // Bounding box of a run of route positions (unbiased integer coordinates) and
 // the largest tour edge leaving it: the summaries the tile cull compares.

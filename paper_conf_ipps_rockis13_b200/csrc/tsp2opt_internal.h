@@ -68,7 +68,7 @@ cudaError_t launch_knn(const int* coords, int n, unsigned long long* knn, cudaSt
 constexpr int kMaxNeighbours = kMfK;
 cudaError_t launch_pruned_sweep(const float2* P, const int* E, const int* tour, const int* pos,
                                 const unsigned long long* knn, int K, int n, int p0, int p1, Slot* slot,
-                                int respect_done, cudaStream_t st);
+                                int respect_done, int first, cudaStream_t st);
 cudaError_t launch_pos(const int* tour, int* pos, int n, cudaStream_t st);
 // 2.5-opt (tsp2opt_sweep25.cu; reading R19): sweep over the dense tiling with R = kRowsSmall,
 // per-position removal gains G, cooperative apply resolving the move type.
@@ -90,6 +90,7 @@ cudaError_t sweep_prepare();
 cudaError_t launch_load_tour(const int* coords, const int* tour_src, int* tour_dst, float2* P, int* E, int n,
                              Slot* slot, unsigned* stamp, unsigned epoch, cudaStream_t st);
 cudaError_t launch_reset_key(Slot* slot, cudaStream_t st);
+cudaError_t launch_first_fix(const float2* P, const int* E, Slot* slot, int respect_done, cudaStream_t st);
 cudaError_t launch_double_bridge(const int* in, int* out, int n, int a, int b, int c, cudaStream_t st);
 cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
                          Slot* slot, int respect_done, unsigned long long* tilebest, int flags, cudaStream_t st);

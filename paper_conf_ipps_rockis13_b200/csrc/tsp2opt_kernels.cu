@@ -96,7 +96,7 @@ __global__ void reset_key_kernel(Slot* slot)
 #ifndef TSP2OPT_MINB
 #define TSP2OPT_MINB 4  // CTAs of 128 threads per SM the register allocation must allow
 #endif
-template <int R>
+template <int R, bool FIRST>
 __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* __restrict__ P, const int* __restrict__ E, int n,
                                                      const int2* __restrict__ tiles, int TJ, Slot* __restrict__ slot,
                                                      int respect_done, unsigned long long* __restrict__ tilebest,
@@ -107,7 +107,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* 
     pdl_trigger();
     pdl_wait();
     if (respect_done && *(volatile int*)&slot->done) return;  // converged: iteration is a no-op
-    sweep_tile<R, false>(P, E, n, tiles[blockIdx.x], TJ, slot, sm, tilebest + blockIdx.x, flags);
+    sweep_tile<R, false, FIRST>(P, E, n, tiles[blockIdx.x], TJ, slot, sm, tilebest + blockIdx.x, flags);
 }
 
 // ===========================================================================
@@ -287,7 +287,7 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
 // slot->next_tile (dynamic scheduling: the kept tiles of a coherent tour
 // cluster along the diagonal, per-tile claims keep the CTAs balanced) until
 // the list is done.
-template <int R>
+template <int R, bool FIRST>
 __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const float2* __restrict__ P,
                                                                       const int* __restrict__ E, int n,
                                                                       const int2* __restrict__ tiles,
@@ -311,7 +311,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const flo
         __syncthreads();
         const int4 e = s_t;
         if (e.z < 0) break;
-        sweep_tile<R, false>(P, E, n, make_int2(e.x, e.y), TJ, slot, sm, tilebest + e.z, flags);
+        sweep_tile<R, false, FIRST>(P, E, n, make_int2(e.x, e.y), TJ, slot, sm, tilebest + e.z, flags);
         if (threadIdx.x == 0) k = gridDim.x + atomicAdd(&slot->next_tile, 1u);
         __syncthreads();  // before the next tile overwrites the shared chunk (and s_t)
     }
@@ -565,6 +565,29 @@ cudaError_t launch_double_bridge(const int* in, int* out, int n, int a, int b, i
     return cudaGetLastError();
 }
 
+// First improvement (reading R20): the sweep's min carries the marker delta
+// kFirstDelta; replace it by the exact delta of the winning pair before the
+// apply (length bookkeeping, trace) and the host read it.
+__global__ void first_fix_kernel(const float2* __restrict__ P, const int* __restrict__ E, Slot* __restrict__ slot,
+                                 int respect_done)
+{
+    pdl_trigger();
+    pdl_wait();
+    if (respect_done && *(volatile int*)&slot->done) return;
+    const unsigned long long k = slot->key;
+    if (key_delta(k) >= 0) return;  // the seed: no improving pair
+    const int i = key_i(k), j = key_j(k);
+    const int d = exact_dist_biased(P[i], P[j]) + exact_dist_biased(P[i + 1], P[j + 1]) - E[i] - E[j];
+    slot->key = pack_key(d, i, j);
+}
+
+cudaError_t launch_first_fix(const float2* P, const int* E, Slot* slot, int respect_done, cudaStream_t st)
+{
+    cudaError_t e = launch_pdl(first_fix_kernel, dim3(1), dim3(32), 0, st, P, E, slot, respect_done);
+    g_launches += 1;
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
+
 cudaError_t launch_reset_key(Slot* slot, cudaStream_t st)
 {
     reset_key_kernel<<<1, 1, 0, st>>>(slot);
@@ -585,20 +608,32 @@ static auto by_rows(int rows, F&& f)
                               : f(std::integral_constant<int, kRowsLarge>{});
 }
 
+// (R, first improvement) instantiations of the sweep kernels
+template <typename F>
+static auto by_rows_first(int rows, bool first, F&& f)
+{
+    return by_rows(rows, [&](auto r) {
+        return first ? f(r, std::true_type{}) : f(r, std::false_type{});
+    });
+}
+
 cudaError_t sweep_prepare()
 {
     for (int R : {kRowsSmall, kRowsLarge}) {
         const Geometry gmax{R, kMaxWarps, kMaxTJ};
-        cudaError_t e = by_rows(R, [&](auto r) {
-            return cudaFuncSetAttribute(sweep_kernel<decltype(r)::value>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                        (int)sweep_smem_bytes(gmax));
-        });
-        if (e != cudaSuccess) return e;
-        e = by_rows(R, [&](auto r) {
-            return cudaFuncSetAttribute(sweep_list_kernel<decltype(r)::value>,
-                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sweep_smem_bytes(gmax));
-        });
-        if (e != cudaSuccess) return e;
+        for (bool first : {false, true}) {
+            cudaError_t e = by_rows_first(R, first, [&](auto r, auto f) {
+                return cudaFuncSetAttribute(sweep_kernel<decltype(r)::value, decltype(f)::value>,
+                                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sweep_smem_bytes(gmax));
+            });
+            if (e != cudaSuccess) return e;
+            e = by_rows_first(R, first, [&](auto r, auto f) {
+                return cudaFuncSetAttribute(sweep_list_kernel<decltype(r)::value, decltype(f)::value>,
+                                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sweep_smem_bytes(gmax));
+            });
+            if (e != cudaSuccess) return e;
+        }
+        cudaError_t e;
         e = by_rows(R, [&](auto r) {
             return cudaFuncSetAttribute(local_search_kernel<decltype(r)::value>,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sweep_smem_bytes(gmax));
@@ -612,9 +647,9 @@ cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n
                          Slot* slot, int respect_done, unsigned long long* tilebest, int flags, cudaStream_t st)
 {
     if (ntiles <= 0) return cudaSuccess;
-    by_rows(g.rows, [&](auto r) {
-        return launch_pdl(sweep_kernel<decltype(r)::value>, dim3(ntiles), dim3(32 * g.warps), sweep_smem_bytes(g),
-                          st, P, E, n, tiles, g.tj, slot, respect_done, tilebest, flags);
+    by_rows_first(g.rows, (flags & kSweepFirst) != 0, [&](auto r, auto f) {
+        return launch_pdl(sweep_kernel<decltype(r)::value, decltype(f)::value>, dim3(ntiles), dim3(32 * g.warps),
+                          sweep_smem_bytes(g), st, P, E, n, tiles, g.tj, slot, respect_done, tilebest, flags);
     });
     g_launches += 1;
     return cudaGetLastError();
@@ -640,7 +675,7 @@ int sweep_list_grid(const Geometry& g, int ntiles)
 {
     int per_sm = 0;
     cudaError_t e = by_rows(g.rows, [&](auto r) {
-        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sweep_list_kernel<decltype(r)::value>,
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sweep_list_kernel<decltype(r)::value, false>,
                                                              32 * g.warps, sweep_smem_bytes(g));
     });
     if (e != cudaSuccess) return 0;
@@ -666,9 +701,9 @@ cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, 
                    list, tilebest, flags, respect_done, n, 0);
     if (e != cudaSuccess) return e;
     if (inc) flags = (flags | kSweepLocal) & ~kSweepSeed;  // tile-local minima, reusable while clean
-    e = by_rows(g.rows, [&](auto r) {
-        return launch_pdl(sweep_list_kernel<decltype(r)::value>, dim3(grid), dim3(32 * g.warps), sweep_smem_bytes(g),
-                          st, P, E, n, tiles, list, g.tj, slot, respect_done, tilebest, flags);
+    e = by_rows_first(g.rows, (flags & kSweepFirst) != 0, [&](auto r, auto f) {
+        return launch_pdl(sweep_list_kernel<decltype(r)::value, decltype(f)::value>, dim3(grid), dim3(32 * g.warps),
+                          sweep_smem_bytes(g), st, P, E, n, tiles, list, g.tj, slot, respect_done, tilebest, flags);
     });
     g_launches += 3;
     if (e != cudaSuccess) return e;

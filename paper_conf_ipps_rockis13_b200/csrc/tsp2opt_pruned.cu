@@ -54,12 +54,15 @@ __device__ __forceinline__ unsigned long long umin64(unsigned long long a, unsig
 // Key of the move (i, j) = sorted(x, y) whose other new edge joins ax and ay;
 // dn is the exact length of the candidate edge, ex and ey the two removed edges.
 // delta >= dn - ex - ey (the other new edge is >= 0): no sqrt when that is >= 0.
-__device__ __forceinline__ unsigned long long move_key(int x, int y, float2 ax, float2 ay, int dn, int ex, int ey)
+// first != 0 (first improvement, reading R20): improving moves enter the min
+// with the marker delta kFirstDelta, so the min is the lowest cell.
+__device__ __forceinline__ unsigned long long move_key(int x, int y, float2 ax, float2 ay, int dn, int ex, int ey,
+                                                       int first)
 {
     const int lo = dn - ex - ey;
     if (lo >= 0) return kKeyNone;
     const int d = lo + exact_edge(ax, ay);
-    return d < 0 ? pack_key(d, min(x, y), max(x, y)) : kKeyNone;
+    return d < 0 ? pack_key(first ? kFirstDelta : d, min(x, y), max(x, y)) : kKeyNone;
 }
 
 }  // namespace
@@ -70,7 +73,7 @@ template <int TP>
 __global__ void __launch_bounds__(kPrunedThreads) pruned_sweep_kernel(
     const float2* __restrict__ P, const int* __restrict__ E, const int* __restrict__ tour, const int* __restrict__ pos,
     const unsigned long long* __restrict__ knn, int K, int n, int p0, int p1, Slot* __restrict__ slot,
-    int respect_done)
+    int respect_done, int first)
 {
     constexpr int kSlots = kMaxNeighbours / TP;
     pdl_trigger();
@@ -103,8 +106,8 @@ __global__ void __launch_bounds__(kPrunedThreads) pruned_sweep_kernel(
             const int qq = q[r], qp = qq == 0 ? n - 1 : qq - 1, dac = (int)(nk[r] >> 22);
             const float2 c1 = __ldg(P + qq + 1), c0 = __ldg(P + qp);
             const int ec1 = __ldg(E + qq), ec0 = __ldg(E + qp);
-            best = umin64(best, move_key(pa, qq, a1, c1, dac, ea1, ec1));  // {t[i], t[j]} = {a, c}
-            best = umin64(best, move_key(pp, qp, a0, c0, dac, ea0, ec0));  // {t[i+1], t[j+1]} = {a, c}
+            best = umin64(best, move_key(pa, qq, a1, c1, dac, ea1, ec1, first));  // {t[i], t[j]} = {a, c}
+            best = umin64(best, move_key(pp, qp, a0, c0, dac, ea0, ec0, first));  // {t[i+1], t[j+1]} = {a, c}
         }
     }
 #pragma unroll
@@ -138,14 +141,15 @@ static int pruned_tp(int n)
 
 cudaError_t launch_pruned_sweep(const float2* P, const int* E, const int* tour, const int* pos,
                                 const unsigned long long* knn, int K, int n, int p0, int p1, Slot* slot,
-                                int respect_done, cudaStream_t st)
+                                int respect_done, int first, cudaStream_t st)
 {
     const int tp = pruned_tp(n);
     const long long threads = (long long)std::max(0, p1 - p0) * tp;
     const dim3 grid((unsigned)std::max(1LL, (threads + kPrunedThreads - 1) / kPrunedThreads)), block(kPrunedThreads);
     cudaError_t e;
 #define TSP2OPT_PRUNED_LAUNCH(T) \
-    launch_kernel_pdl(pruned_sweep_kernel<T>, grid, block, 0, st, P, E, tour, pos, knn, K, n, p0, p1, slot, respect_done)
+    launch_kernel_pdl(pruned_sweep_kernel<T>, grid, block, 0, st, P, E, tour, pos, knn, K, n, p0, p1, slot, respect_done, \
+                      first)
     switch (tp) {
     case 1: e = TSP2OPT_PRUNED_LAUNCH(1); break;
     case 2: e = TSP2OPT_PRUNED_LAUNCH(2); break;

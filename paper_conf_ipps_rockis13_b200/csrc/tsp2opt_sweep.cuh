@@ -147,7 +147,7 @@ __device__ __forceinline__ bool step_any(const Bound<R>& b, const float (&cur)[R
 // exhaustively by tsp2opt_selftest) is covered by a 0.5 slack.  Survivors are
 // evaluated with integer nint distances -- the oracle's arithmetic -- and
 // accepted iff delta < B, in increasing cell order.
-template <int R, bool MASK, bool PS>
+template <int R, bool MASK, bool PS, bool FIRST>
 __device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1], const float (&nxt)[R + 1],
                                            float scol, int row0, int j, float4 c0, float4 c1, float ej,
                                            const float* my_rowe, const float2* P, unsigned long long& mykey)
@@ -182,19 +182,27 @@ __device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1
         if (!nint_from_float(fmaf(dx1, dx1, dy1 * dy1), d2))
             d2 = (float)exact_dist_xy(unbias(pi1.x), unbias(pi1.y), xj1, yj1);
         const float d = (d1 + d2) - (my_rowe[r] + ej);  // exact: integers < 2^24
+        if (FIRST) {
+            // first improvement (reading R20): the lane's first improving pair is its
+            // lowest cell; the key's delta is the marker kFirstDelta (resolved later)
+            if (d < 0.0f && mykey == kKeyNone) mykey = pack_key(kFirstDelta, row0 + r, j);
+            continue;
+        }
         if (d < Bf) {
             Bf = d;
             mykey = pack_key((int)d, row0 + r, j);
         }
     }
-    if (Bf < b.Bf) {
+    if (!FIRST && Bf < b.Bf) {
         b.B = (int)Bf;
         b.Bf = Bf;
     }
 }
 
-template <int R, bool MASK, bool PS>
-__device__ __forceinline__ void column_step(const Rows<R>& rows, Bound<R>& b, const float (&cur)[R + 1],
+// Returns true (FIRST only) once some lane of the warp holds an improving
+// pair: every later column has higher cell numbers, so the walk can stop.
+template <int R, bool MASK, bool PS, bool FIRST>
+__device__ __forceinline__ bool column_step(const Rows<R>& rows, Bound<R>& b, const float (&cur)[R + 1],
                                             float (&nxt)[R + 1], int row0, int j, int J0, const TileSmem& sm,
                                             const float* my_rowe, const float2* P, unsigned long long& mykey)
 {
@@ -211,15 +219,18 @@ __device__ __forceinline__ void column_step(const Rows<R>& rows, Bound<R>& b, co
         if ((threadIdx.x & 31) == 0) atomicAdd(&g_stats[1], 1ULL);
 #endif
         const int B0 = b.B;
-        if (any) exact_step<R, MASK, PS>(b, cur, nxt, scol, row0, j, sm.colxy[j - J0], c1, ej, my_rowe, P, mykey);
+        if (any)
+            exact_step<R, MASK, PS, FIRST>(b, cur, nxt, scol, row0, j, sm.colxy[j - J0], c1, ej, my_rowe, P, mykey);
+        if (FIRST) return __any_sync(0xffffffffu, mykey != kKeyNone);
         // share the warp's best: a lane may accept delta <= (best of another lane)
         const int wb = __reduce_min_sync(0xffffffffu, b.B);
         const int nb = min(b.B, wb + 1);
         if (nb < B0) reset_bound<R>(b, my_rowe, nb);
     }
+    return false;
 }
 
-template <int R, bool MASK, bool PS>
+template <int R, bool MASK, bool PS, bool FIRST>
 __device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0, int jstart, int J0, int J1,
                                      const TileSmem& sm, const float* my_rowe, const float2* P,
                                      unsigned long long& mykey)
@@ -228,10 +239,10 @@ __device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0,
     column_sq<R>(sa, rows, sm.colxy[jstart - J0]);
     int j = jstart;
     for (; j + 1 < J1; j += 2) {
-        column_step<R, MASK, PS>(rows, b, sa, sb, row0, j, J0, sm, my_rowe, P, mykey);
-        column_step<R, MASK, PS>(rows, b, sb, sa, row0, j + 1, J0, sm, my_rowe, P, mykey);
+        if (column_step<R, MASK, PS, FIRST>(rows, b, sa, sb, row0, j, J0, sm, my_rowe, P, mykey)) return;
+        if (column_step<R, MASK, PS, FIRST>(rows, b, sb, sa, row0, j + 1, J0, sm, my_rowe, P, mykey)) return;
     }
-    if (j < J1) column_step<R, MASK, PS>(rows, b, sa, sb, row0, j, J0, sm, my_rowe, P, mykey);
+    if (j < J1) column_step<R, MASK, PS, FIRST>(rows, b, sa, sb, row0, j, J0, sm, my_rowe, P, mykey);
 }
 
 // Tile-level form of the same exact necessary condition (a bound on all of the
@@ -305,7 +316,7 @@ __host__ __device__ inline size_t tile_smem_bytes(int TJ, int TI)
 // deterministic).  The caller synchronises the CTA before reusing `sm`.
 constexpr int kMaxWarpsPerTile = 4;
 
-template <int R, bool PS>
+template <int R, bool PS, bool FIRST = false>
 __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n, int2 tile, int TJ, Slot* slot,
                                            const TileSmem& sm, unsigned long long* tilebest, int flags)
 {
@@ -345,7 +356,7 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     // kSweepLocal: the tile's own minimum over its improving pairs, independent
     // of every other tile (reused by the incremental sweep while the tile is clean)
     unsigned long long g = (flags & kSweepLocal) ? seed_key() : *(volatile unsigned long long*)&slot->key;
-    if (!(flags & kSweepLocal) && (flags & kSweepSeed) && *(volatile int*)&slot->seed_ok) {
+    if (!FIRST && !(flags & kSweepLocal) && (flags & kSweepSeed) && *(volatile int*)&slot->seed_ok) {
         const unsigned long long mv = *(volatile unsigned long long*)&slot->last_key;
         const unsigned long long k = surviving_key(*(volatile unsigned long long*)tilebest, key_i(mv), key_j(mv));
         if (k < g) {
@@ -361,16 +372,19 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     __syncthreads();
 
     unsigned long long mykey = kKeyNone;
-    if (active) {
+    // FIRST: a tile whose lowest cell is above an improving pair already found
+    // (the global key) cannot hold the first improving pair
+    const bool skip = FIRST && g < pack_key(kFirstDelta, wrow0, jstart);
+    if (active && !skip) {
         Bound<R> b;
-        set_bound<R>(b, erow, dg == 0 ? 0 : dg + 1);
+        set_bound<R>(b, erow, FIRST ? 0 : (dg == 0 ? 0 : dg + 1));
         const bool masked = (wrow0 + 32 * R - 1) >= jstart;  // warp-uniform: some row >= some j
         if (!(flags & kSweepTileBounds) || tile_may_pass<R>(rows, b, sm, jstart - J0, J1 - J0)) {
 #ifdef TSP2OPT_STATS
             if (lane == 0) atomicAdd(&g_stats[3], 1ULL);
 #endif
-            if (masked) walk<R, true, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
-            else walk<R, false, PS>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
+            if (masked) walk<R, true, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
+            else walk<R, false, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
         }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {

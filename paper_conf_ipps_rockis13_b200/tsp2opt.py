@@ -286,6 +286,7 @@ def get_tour(h, n: int):
 
 
 OPT_TILE_BOUNDS, OPT_SEED, OPT_PERSISTENT, OPT_TRACE, OPT_NEIGHBOURS, OPT_NODE_INSERTION = 1, 2, 3, 4, 5, 6
+OPT_FIRST_IMPROVEMENT = 7
 MAX_NEIGHBOURS = 16  # TSP2OPT_MAX_NEIGHBOURS
 
 
