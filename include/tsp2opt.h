@@ -244,8 +244,9 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
  *      §8(f) NEXT-4; reading R20): best_move returns the improving
  *      pair with the lowest Fig. 3 cell (the first one the paper's sequential
  *      pair order reaches) instead of the lowest delta, with its exact delta;
- *      local_search applies it and restarts.  Not with TSP2OPT_OPT_NEIGHBOURS,
- *      TSP2OPT_OPT_NODE_INSERTION or tsp2opt_ils (EINVAL).  Equals
+ *      local_search applies it and restarts.  With TSP2OPT_OPT_NEIGHBOURS it
+ *      is the lowest improving cell of M_K (oracle_pruned_first_move).  Not
+ *      with TSP2OPT_OPT_NODE_INSERTION or tsp2opt_ils (EINVAL).  Equals
  *      oracle_first_*.
  * Returns TSP2OPT_EINVAL for an unknown option or value. */
 #define TSP2OPT_OPT_TILE_BOUNDS 1

@@ -77,6 +77,8 @@ def _load():
             lib.oracle_pruned_best_move_plain.restype = None
             lib.oracle_pruned_best_move.argtypes = [p, i64, p, p, i64, p, p, p]
             lib.oracle_pruned_best_move.restype = None
+            lib.oracle_pruned_first_move.argtypes = [p, i64, p, p, i64, p, p, p]
+            lib.oracle_pruned_first_move.restype = None
             lib.oracle_pruned_local_search.argtypes = [p, i64, p, i64, i64, ctypes.c_int, p, p, p, i64]
             lib.oracle_pruned_local_search.restype = ctypes.c_int
             lib.oracle25_delta.argtypes = [p, i64, p, i64, i64, ctypes.c_int]
@@ -250,15 +252,29 @@ def pruned_best_move(coords, tour, K: int, plain: bool = False, nbr=None):
     return int(out[0]), int(out[1]), int(out[2])
 
 
-def pruned_local_search(coords, tour, K: int, max_iters: int = -1, trace_cap: int = 0, plain: bool = False):
-    """Best-improvement local search over M_K; same return dict as local_search."""
+def pruned_first_move(coords, tour, K: int, nbr=None):
+    """(i, j, delta): the improving pair of M_K with the lowest Fig. 3 cell (readings R18 + R20)."""
+    xy = _xy(coords)
+    K = _check_k(K)
+    t = np.ascontiguousarray(tour, dtype=np.int32)
+    nb = knn(xy, K) if nbr is None else np.ascontiguousarray(nbr, dtype=np.int32)
+    out = np.zeros(3, dtype=np.int64)
+    _load().oracle_pruned_first_move(_ptr(xy), xy.shape[0], _ptr(t), _ptr(nb), K, _ptr(out[0:1]), _ptr(out[1:2]),
+                                     _ptr(out[2:3]))
+    return int(out[0]), int(out[1]), int(out[2])
+
+
+def pruned_local_search(coords, tour, K: int, max_iters: int = -1, trace_cap: int = 0, plain: bool = False,
+                        first: bool = False):
+    """Local search over M_K (best improvement, or first improvement with first=True);
+    same return dict as local_search."""
     xy = _xy(coords)
     K = _check_k(K)
     t = np.array(tour, dtype=np.int32, copy=True)
     out = np.zeros(2, dtype=np.int64)
     tr = np.zeros((max(trace_cap, 1), 3), dtype=np.int64)
     st = _load().oracle_pruned_local_search(
-        _ptr(xy), xy.shape[0], _ptr(t), K, int(max_iters), 1 if plain else 0,
+        _ptr(xy), xy.shape[0], _ptr(t), K, int(max_iters), (1 if plain else 0) | (2 if first else 0),
         _ptr(out[0:1]), _ptr(out[1:2]), _ptr(tr) if trace_cap > 0 else None, int(trace_cap),
     )
     it = int(out[1])

@@ -521,9 +521,29 @@ void oracle_pruned_best_move(const int32_t *xy, int64_t n, const int32_t *tour, 
     *bi = best_i; *bj = best_j; *bdelta = best_d;
 }
 
-/* Best-improvement local search over M_K (same loop, status and trace
- * conventions as oracle_local_search).  plain != 0 uses the plain sweep. */
-int oracle_pruned_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64_t K, int64_t max_iters, int plain,
+/* First improvement over M_K (readings R18 + R20): the pair of M_K with
+ * delta < 0 and the lowest Fig. 3 cell, scanning the pairs in cell order. */
+void oracle_pruned_first_move(const int32_t *xy, int64_t n, const int32_t *tour, const int32_t *nbr, int64_t K,
+                              int64_t *bi, int64_t *bj, int64_t *bdelta)
+{
+    for (int64_t j = 1; j < n; j++)
+        for (int64_t i = 0; i < j; i++) {
+            if (!in_candidate_edges(nbr, K, tour[i], tour[j]) &&
+                !in_candidate_edges(nbr, K, tour[i + 1], tour[(j + 1) % n]))
+                continue;
+            int64_t d = oracle_delta(xy, n, tour, i, j);
+            if (d < 0) {
+                *bi = i; *bj = j; *bdelta = d;
+                return;
+            }
+        }
+    *bi = 0; *bj = 1; *bdelta = 0;
+}
+
+/* Local search over M_K (same loop, status and trace conventions as
+ * oracle_local_search).  mode bit 0: the plain all-pairs scan instead of the
+ * list enumeration (best improvement); bit 1: first improvement (R20). */
+int oracle_pruned_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64_t K, int64_t max_iters, int mode,
                                int64_t *length, int64_t *iterations, int64_t *trace, int64_t trace_cap)
 {
     int32_t *nbr = (int32_t *)malloc(sizeof(int32_t) * n * K);
@@ -533,7 +553,8 @@ int oracle_pruned_local_search(const int32_t *xy, int64_t n, int32_t *tour, int6
     int status = 0;
     for (;;) {
         int64_t i, j, d;
-        if (plain) oracle_pruned_best_move_plain(xy, n, tour, nbr, K, &i, &j, &d);
+        if (mode & 2) oracle_pruned_first_move(xy, n, tour, nbr, K, &i, &j, &d);
+        else if (mode & 1) oracle_pruned_best_move_plain(xy, n, tour, nbr, K, &i, &j, &d);
         else oracle_pruned_best_move(xy, n, tour, nbr, K, &i, &j, &d);
         if (d >= 0) break;
         if (max_iters >= 0 && it >= max_iters) { /* reading R8 */

@@ -903,7 +903,7 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
         h->persistent = (int)value;
         break;
     case TSP2OPT_OPT_FIRST_IMPROVEMENT: {
-        if (value < 0 || value > 1 || (value && (h->or25 || h->nbr_k > 0))) return TSP2OPT_EINVAL;
+        if (value < 0 || value > 1 || (value && h->or25)) return TSP2OPT_EINVAL;
         h->first = (int)value;
         if (h->has_tour) CUDA_TRY(launch_reset_key(h->d_slots + h->parity, h->stream));  // pending key: other rule
         CUDA_TRY(cudaStreamSynchronize(h->stream));
@@ -939,7 +939,7 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
         break;
     }
     case TSP2OPT_OPT_NEIGHBOURS: {
-        if (value < 0 || value > kMaxNeighbours || (value && (h->or25 || h->first))) return TSP2OPT_EINVAL;
+        if (value < 0 || value > kMaxNeighbours || (value && h->or25)) return TSP2OPT_EINVAL;
         if (value > 0) {
             if (!h->d_knn) {  // exact candidate lists, once per handle (coordinates never change)
                 unsigned long long* knn = nullptr;

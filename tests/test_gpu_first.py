@@ -112,9 +112,8 @@ def test_first_mixed_operations(gpu, monkeypatch, bounds):
             g.debug_set_shard(0, 1)
             _, i, j, d = min(keys)
             assert (i, j, d) == want, world
-        for opt in (tsp2opt.OPT_NEIGHBOURS, tsp2opt.OPT_NODE_INSERTION):
-            with pytest.raises(tsp2opt.TSP2OptError):
-                g.set_option(opt, 1 if opt == tsp2opt.OPT_NODE_INSERTION else 8)
+        with pytest.raises(tsp2opt.TSP2OptError):
+            g.set_option(tsp2opt.OPT_NODE_INSERTION, 1)
         with pytest.raises(tsp2opt.TSP2OptError):
             g.ils(t, 2, 1)
 
@@ -145,3 +144,33 @@ def test_first_full_size_from_mf(gpu, cfg, nsamples):
         L += d
     assert np.array_equal(tour, res["tour"]) and L == res["length"] == oracle.tour_length(c, tour)
     assert oracle.best_move(c, res["tour"]) == (0, 1, 0)
+
+
+@pytest.mark.parametrize("n", [5, 33, 481, 2500])
+@pytest.mark.parametrize("K", [1, 4, 8, 16])
+def test_pruned_first_move_parity(gpu, n, K):
+    """First improvement over the pruned neighbourhood M_K (readings R18 + R20)."""
+    c = inputs.make_coords("lattice" if n % 2 else "uniform", n, 3)
+    nb = oracle.knn(c, K)
+    mid = oracle.local_search(c, inputs.random_tour(n, 4), max_iters=n)["tour"]
+    with _handle(c) as g:
+        g.set_option(tsp2opt.OPT_NEIGHBOURS, K)
+        for t in (inputs.random_tour(n, 3), inputs.hilbert_tour(c), mid):
+            assert g.best_move(t) == oracle.pruned_first_move(c, t, K, nbr=nb)
+
+
+@pytest.mark.parametrize("kind,n,seed,K,cap", [("uniform", 200, 1, 4, -1), ("lattice", 500, 2, 8, -1),
+                                               ("uniform", 1002, 3, 16, 2000)])
+def test_pruned_first_local_search(gpu, kind, n, seed, K, cap):
+    c = inputs.make_coords(kind, n, seed)
+    t = inputs.random_tour(n, seed)
+    want = oracle.pruned_local_search(c, t, K, first=True, max_iters=cap, trace_cap=40 * n)
+    with _handle(c) as g:
+        g.set_option(tsp2opt.OPT_NEIGHBOURS, K)
+        g.set_option(tsp2opt.OPT_TRACE, 40 * n)
+        res = g.local_search(t, max_iters=None if cap < 0 else cap)
+        trace = g.get_trace(40 * n)
+    assert res["status"] == want["status"]
+    assert (res["iterations"], res["length"]) == (want["iterations"], want["length"])
+    assert np.array_equal(res["tour"], want["tour"])
+    assert np.array_equal(np.asarray(trace, dtype=np.int64), want["trace"])

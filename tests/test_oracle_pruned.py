@@ -174,3 +174,43 @@ def test_pruned_max_iters_status():
         assert r["iterations"] == cap and r["status"] == 1
     r = oracle.pruned_local_search(c, t, 5, max_iters=full["iterations"])
     assert r["status"] == 0 and r["length"] == full["length"]
+
+
+def brute_pruned_first(coords, tour, K):
+    """First 2-opt neighbour in cell order that creates an edge of E_K and shortens the tour."""
+    coords = [tuple(map(int, c)) for c in coords]
+    tour = [int(c) for c in tour]
+    n = len(tour)
+    E = candidate_edges(py_knn(coords, K))
+    L0 = py_length(coords, tour)
+    old = edge_set(tour)
+    for j in range(1, n):
+        for i in range(j):
+            t2 = tour[: i + 1] + tour[i + 1 : j + 1][::-1] + tour[j + 1 :]
+            if (edge_set(t2) - old) & E and py_length(coords, t2) - L0 < 0:
+                return i, j, py_length(coords, t2) - L0
+    return 0, 1, 0
+
+
+@pytest.mark.parametrize("name,coords,tour", _instances(), ids=lambda v: v if isinstance(v, str) else "")
+def test_pruned_first_move_brute_force(name, coords, tour):
+    n = len(coords)
+    for K in (1, 2, 3, 5, n - 1):
+        assert oracle.pruned_first_move(coords, tour, K) == brute_pruned_first(coords, tour, K), K
+    assert oracle.pruned_first_move(coords, tour, max(1, n - 1)) == oracle.first_move(coords, tour)
+
+
+@pytest.mark.parametrize("kind,n,seed,K", [("uniform", 80, 1, 4), ("lattice", 120, 2, 8)])
+def test_pruned_first_local_search(kind, n, seed, K):
+    c = inputs.make_coords(kind, n, seed)
+    t0 = inputs.random_tour(n, seed)
+    res = oracle.pruned_local_search(c, t0, K, trace_cap=100_000, first=True)
+    t = [int(x) for x in t0]
+    for step, (i, j, d) in enumerate(res["trace"].tolist()):
+        if step % 10 == 0:
+            assert brute_pruned_first(c, t, K) == (i, j, d)
+        t = t[: i + 1] + t[i + 1 : j + 1][::-1] + t[j + 1 :]
+    assert t == res["tour"].tolist()
+    assert oracle.pruned_best_move(c, res["tour"], K) == (0, 1, 0)  # the same M_K local minimum certificate
+    full = oracle.pruned_local_search(c, t0, n - 1, first=True)
+    assert full["length"] == oracle.first_local_search(c, t0)["length"]
