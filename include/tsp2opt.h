@@ -65,7 +65,9 @@ int tsp2opt_create(const int32_t *coords_xy, int32_t n, tsp2opt_t *out);
  * §8(e); L18 §VI "dividing the 2-opt task between multiple devices").
  * nccl_id: TSP2OPT_NCCL_ID_BYTES bytes from tsp2opt_nccl_unique_id() on rank 0,
  * broadcast by the caller.  Every rank must make the same sequence of calls;
- * outputs are identical on all ranks.  world == 1 is allowed (no NCCL). */
+ * outputs are identical on all ranks.  world == 1 is allowed: with
+ * nccl_id == NULL there is no NCCL; with an id, a one-rank communicator runs
+ * the same allreduce path (the sharded code path on a single GPU). */
 int tsp2opt_create_sharded(const int32_t *coords_xy, int32_t n, int32_t rank, int32_t world,
                            const void *nccl_id, tsp2opt_t *out);
 

@@ -520,7 +520,7 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     }
     rc = upload_shard(h, rank, world);
     if (rc) return fail(rc);
-    if (world > 1) {
+    if (world > 1 || nccl_id) {  // world 1 with an id: a one-rank communicator (the sharded path on one GPU)
         ncclUniqueId id;
         memcpy(&id, nccl_id, sizeof(id));
         ncclResult_t r = ncclCommInitRank(&h->comm, world, id, rank);

@@ -372,7 +372,8 @@ class TSP2Opt:
     def __init__(self, coords, rank: int = 0, world: int = 1, nccl_id: bytes | None = None):
         xy = _i32(coords).reshape(-1, 2)
         self.n = xy.shape[0]
-        self.h = create(xy) if world == 1 else create_sharded(xy, rank, world, nccl_id)
+        # world 1 with an NCCL id: a one-rank communicator (the sharded path on one GPU)
+        self.h = create(xy) if (world == 1 and nccl_id is None) else create_sharded(xy, rank, world, nccl_id)
 
     def close(self):
         if self.h:
