@@ -353,7 +353,7 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         h->inc_valid = false;
     }
     h->last_tiling = tiling;
-    if (tiling == 3 && h->tile_bounds >= 2) {  // 2.5-opt, culled: box + cull (with gains) + list sweep
+    if (tiling == 3 && h->tile_bounds >= 2 && h->cgeo.rows == kRowsSmall) {  // 2.5-opt, culled (R = 7 tiling only)
         CUDA_TRY(launch_box_cull(h->cgeo, h->d_P, h->d_E, h->d_G, h->n, h->d_ctiles, h->nctiles, h->d_rbox, h->d_cbox,
                                  h->d_list, in, apply ? 1 : 0, h->d_ctilebest, flags, h->stream));
         CUDA_TRY(launch_sweep25_list(h->cgeo, h->d_P, h->d_E, h->d_G, h->n, h->d_list, h->list25_grid, in,
@@ -969,7 +969,7 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
             CUDA_TRY(cudaMalloc(&h->d_bar25, sizeof(unsigned) * 2));
             CUDA_TRY(cudaMemset(h->d_bar25, 0, sizeof(unsigned) * 2));
         }
-            // the 2.5-opt sweep is instantiated for R = 7 only; the 2-opt geometry comes back with value 0
+        // the 2.5-opt sweep is instantiated for R = 7 only; the 2-opt geometry comes back with value 0
         const long long total_pairs = (long long)h->n * (h->n - 1) / 2;
         Geometry g = choose_geometry(total_pairs / h->world);
         if (value) g.rows = kRowsSmall;
