@@ -137,7 +137,9 @@ int tsp2opt_local_search(tsp2opt_t h, int32_t *tour, int64_t max_iters, int64_t 
  * l_k = 1 + out % max(1, (n-1)/3); a = l0, b = a + l1, c = b + l2; s' = A C B D
  * for s* = A B C D cut at a < b < c (no perturbation when n < 8).
  * tour: host int32[n], in = start tour, out = best tour; *length its length;
- * lengths (NULL or int64[iterations+1]) = best length after each step. */
+ * lengths (NULL or int64[iterations+1]) = best length after each step.
+ * local_search is the handle's variant (set_option: pruned, first improvement,
+ * 2.5-opt; oracle_ils_mode), best-improvement 2-opt by default. */
 int tsp2opt_ils(tsp2opt_t h, int32_t *tour, int64_t iterations, uint64_t seed, int64_t *length,
                 int64_t *lengths);
 
@@ -228,7 +230,7 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
  *      else (0, 1, 0).  O(nK) per sweep instead of C(n,2); the result equals
  *      oracle_pruned_best_move, not the full sweep's.  The exact candidate
  *      lists are built on the device on first use (8 * 16 * n bytes).
- *      0 restores the full neighbourhood.  tsp2opt_ils needs K = 0 (EINVAL).
+ *      0 restores the full neighbourhood.
  *  TSP2OPT_OPT_NODE_INSERTION (default 0): 1 switches best_move / apply /
  *      iterate_async / local_search to best-improvement 2.5-opt (SURVEY.md
  *      §8(f) NEXT-4; L26 §VII "more complex local search algorithms such as
@@ -240,16 +242,17 @@ int tsp2opt_get_tour(tsp2opt_t h, int32_t *tour_out, int64_t *length);
  *      reaching delta at (i, j) (tsp2opt_best_move_typed reports it).  Type 1
  *      rotates positions i+1..j left by one, type 2 right by one; t[0] never
  *      moves.  Results equal oracle25_*.  Not with TSP2OPT_OPT_NEIGHBOURS > 0
- *      (EINVAL) or tsp2opt_ils; the sweep uses R = 7 rows per lane and the
- *      per-tile bound (no pre-sweep cull, no persistent loop).
+ *      or first improvement (EINVAL); the sweep uses R = 7 rows per lane (no
+ *      persistent loop).
  *  TSP2OPT_OPT_FIRST_IMPROVEMENT (default 0): 1 = first improvement (SURVEY.md
  *      §8(f) NEXT-4; reading R20): best_move returns the improving
  *      pair with the lowest Fig. 3 cell (the first one the paper's sequential
  *      pair order reaches) instead of the lowest delta, with its exact delta;
  *      local_search applies it and restarts.  With TSP2OPT_OPT_NEIGHBOURS it
  *      is the lowest improving cell of M_K (oracle_pruned_first_move).  Not
- *      with TSP2OPT_OPT_NODE_INSERTION or tsp2opt_ils (EINVAL).  Equals
- *      oracle_first_*.
+ *      with TSP2OPT_OPT_NODE_INSERTION (EINVAL).  Equals oracle_first_*.
+ *  tsp2opt_ils runs its local searches with the handle's variant
+ *      (oracle_ils_mode).
  * Returns TSP2OPT_EINVAL for an unknown option or value. */
 #define TSP2OPT_OPT_TILE_BOUNDS 1
 #define TSP2OPT_OPT_SEED 2

@@ -93,6 +93,8 @@ def _load():
             lib.oracle_first_move.restype = None
             lib.oracle_first_local_search.argtypes = [p, i64, p, i64, p, p, p, i64]
             lib.oracle_first_local_search.restype = ctypes.c_int
+            lib.oracle_ils_mode.argtypes = [p, i64, p, i64, ctypes.c_uint64, ctypes.c_int, i64, p, p]
+            lib.oracle_ils_mode.restype = None
             lib.oracle_num_threads.argtypes = []
             lib.oracle_num_threads.restype = ctypes.c_int
             _lib = lib
@@ -201,13 +203,23 @@ def double_bridge(tour, a: int, b: int, c: int) -> np.ndarray:
     return out
 
 
-def ils(coords, tour, iterations: int, seed: int):
+def ils(coords, tour, iterations: int, seed: int, neighbours: int = 0, first: bool = False,
+        node_insertion: bool = False):
     """Iterated Local Search (L10 Algorithm 1; readings R14-R16).
-    Returns dict(tour, length, lengths) -- lengths[t] = best length after t steps."""
+    Returns dict(tour, length, lengths) -- lengths[t] = best length after t steps.
+    neighbours / first / node_insertion select the local search (R18 / R20 / R19)."""
     xy = _xy(coords)
     t = np.array(tour, dtype=np.int32, copy=True)
     out = np.zeros(1, dtype=np.int64)
     lengths = np.zeros(iterations + 1, dtype=np.int64)
+    if neighbours or first or node_insertion:
+        if node_insertion and (neighbours or first):
+            raise ValueError("2.5-opt combines with neither pruning nor first improvement")
+        mode = 4 if node_insertion else (3 if neighbours and first else 1 if neighbours else 2)
+        _load().oracle_ils_mode(_ptr(xy), xy.shape[0], _ptr(t), int(iterations),
+                                ctypes.c_uint64(seed & 0xFFFFFFFFFFFFFFFF), mode, int(neighbours), _ptr(out),
+                                _ptr(lengths))
+        return dict(tour=t, length=int(out[0]), lengths=lengths)
     _load().oracle_ils(_ptr(xy), xy.shape[0], _ptr(t), int(iterations), ctypes.c_uint64(seed & 0xFFFFFFFFFFFFFFFF),
                        _ptr(out), _ptr(lengths))
     return dict(tour=t, length=int(out[0]), lengths=lengths)

@@ -753,3 +753,46 @@ int oracle_first_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64
     *iterations = it;
     return status;
 }
+
+
+/* ---------------------------------------------------------------------------
+ * Iterated Local Search over any of the local searches above (L10 Algorithm 1
+ * with "2optLocalSearch" replaced by the variant; L26 §VII names 2.5-opt as
+ * the next local search).  Same perturbation, acceptance and termination as
+ * oracle_ils (readings R14-R16).  mode: 0 best-improvement 2-opt (== oracle_ils),
+ * 1 pruned to K neighbours (R18), 2 first improvement (R20), 3 pruned + first,
+ * 4 2.5-opt (R19).
+ * ------------------------------------------------------------------------- */
+static void ls_mode(const int32_t *xy, int64_t n, int32_t *tour, int mode, int64_t K, int64_t *L)
+{
+    int64_t it;
+    if (mode == 0) oracle_local_search(xy, n, tour, -1, L, &it, NULL, 0);
+    else if (mode == 1) oracle_pruned_local_search(xy, n, tour, K, -1, 0, L, &it, NULL, 0);
+    else if (mode == 2) oracle_first_local_search(xy, n, tour, -1, L, &it, NULL, 0);
+    else if (mode == 3) oracle_pruned_local_search(xy, n, tour, K, -1, 2, L, &it, NULL, 0);
+    else oracle25_local_search(xy, n, tour, -1, L, &it, NULL, 0);
+}
+
+void oracle_ils_mode(const int32_t *xy, int64_t n, int32_t *tour, int64_t iterations, uint64_t seed, int mode,
+                     int64_t K, int64_t *length, int64_t *lengths)
+{
+    int64_t L;
+    ls_mode(xy, n, tour, mode, K, &L);
+    if (lengths) lengths[0] = L;
+    int32_t *cand = (int32_t *)malloc(sizeof(int32_t) * n);
+    for (int64_t t = 0; t < iterations; t++) {
+        if (n >= 8) {
+            int64_t a, b, c, L2;
+            oracle_double_bridge_cuts(n, seed, t, &a, &b, &c);
+            oracle_double_bridge(tour, n, a, b, c, cand);
+            ls_mode(xy, n, cand, mode, K, &L2);
+            if (L2 < L) {
+                memcpy(tour, cand, sizeof(int32_t) * n);
+                L = L2;
+            }
+        }
+        if (lengths) lengths[t + 1] = L;
+    }
+    free(cand);
+    *length = L;
+}

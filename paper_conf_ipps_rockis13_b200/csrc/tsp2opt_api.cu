@@ -848,10 +848,8 @@ int tsp2opt_batch_ils_async(const int32_t* d_coords_xy, int32_t n, int32_t batch
 int tsp2opt_ils(tsp2opt_t h, int32_t* tour, int64_t iterations, uint64_t seed, int64_t* length, int64_t* lengths)
 {
     if (!h || !tour || !length || iterations < 0) return TSP2OPT_EINVAL;
-    if (h->nbr_k > 0 || h->or25 || h->first) {  // ILS is defined (and pinned) for best-improvement 2-opt only
-        g_last_error = "tsp2opt_ils: set TSP2OPT_OPT_NEIGHBOURS, _NODE_INSERTION and _FIRST_IMPROVEMENT to 0 first";
-        return TSP2OPT_EINVAL;
-    }
+    // The local search of each step is the handle's: 2-opt, pruned (R18), first
+    // improvement (R20) or 2.5-opt (R19) -- oracle_ils_mode
     int rc = load_host_tour(h, tour);
     if (rc) return rc;
     if (!h->d_best) CUDA_TRY(cudaMalloc(&h->d_best, sizeof(int) * (size_t)h->n));

@@ -167,8 +167,6 @@ def test_25opt_mixed_operations(gpu, monkeypatch, bounds):
         g.debug_set_shard(0, 1)
         with pytest.raises(tsp2opt.TSP2OptError):
             g.set_option(tsp2opt.OPT_NEIGHBOURS, 8)  # exclusive modes
-        with pytest.raises(tsp2opt.TSP2OptError):
-            g.ils(t, 2, 1)
 
 
 @pytest.mark.parametrize("cfg,nsamples", [("C3", 4), ("C4", 3), ("C5", 2)])

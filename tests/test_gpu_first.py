@@ -114,8 +114,6 @@ def test_first_mixed_operations(gpu, monkeypatch, bounds):
             assert (i, j, d) == want, world
         with pytest.raises(tsp2opt.TSP2OptError):
             g.set_option(tsp2opt.OPT_NODE_INSERTION, 1)
-        with pytest.raises(tsp2opt.TSP2OptError):
-            g.ils(t, 2, 1)
 
 
 @pytest.mark.parametrize("cfg,nsamples", [("C3", 6), ("C4", 4), ("C5", 2)])

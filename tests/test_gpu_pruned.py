@@ -130,8 +130,9 @@ def test_pruned_option_errors(gpu):
             with pytest.raises(tsp2opt.TSP2OptError):
                 g.set_option(tsp2opt.OPT_NEIGHBOURS, bad)
         g.set_option(tsp2opt.OPT_NEIGHBOURS, 4)
+        g.set_option(tsp2opt.OPT_NODE_INSERTION, 0)  # switching a mode off is always valid
         with pytest.raises(tsp2opt.TSP2OptError):
-            g.ils(inputs.random_tour(50, 1), 3, 7)
+            g.set_option(tsp2opt.OPT_NODE_INSERTION, 1)  # exclusive with pruning
 
 
 @pytest.mark.parametrize("cfg", ["C4", "C5"])

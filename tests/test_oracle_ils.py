@@ -74,3 +74,32 @@ def test_ils_invariants_medium():
     assert oracle.best_move(coords, res["tour"])[2] == 0  # a 2-opt local minimum
     assert sorted(res["tour"].tolist()) == list(range(200)) and res["tour"][0] == t0[0]
     assert Ls[-1] <= oracle.local_search(coords, t0)["length"]
+
+
+@pytest.mark.parametrize("kw", [dict(neighbours=6), dict(first=True), dict(neighbours=6, first=True),
+                                dict(node_insertion=True)])
+def test_ils_over_variants(kw):
+    """ILS with another local search: the same perturbation / acceptance as a
+    Python restatement of Algorithm 1 around the variant's oracle local search."""
+    c = inputs.make_coords("uniform", 60, 5)
+    t0 = inputs.random_tour(60, 5)
+
+    def ls(t):
+        if kw.get("node_insertion"):
+            return oracle.local_search25(c, t)
+        if kw.get("neighbours"):
+            return oracle.pruned_local_search(c, t, kw["neighbours"], first=kw.get("first", False))
+        return oracle.first_local_search(c, t)
+
+    r = ls(t0)
+    best, L = r["tour"], r["length"]
+    lengths = [L]
+    for it in range(6):
+        a, b, cc = oracle.double_bridge_cuts(60, 99, it)
+        r = ls(oracle.double_bridge(best, a, b, cc))
+        if r["length"] < L:
+            best, L = r["tour"], r["length"]
+        lengths.append(L)
+    got = oracle.ils(c, t0, 6, 99, **kw)
+    assert got["length"] == L and np.array_equal(got["tour"], best)
+    assert got["lengths"].tolist() == lengths
