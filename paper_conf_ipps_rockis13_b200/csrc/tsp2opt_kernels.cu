@@ -143,21 +143,24 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
 {
     pdl_trigger();
     pdl_wait();
-    // incremental: only the summaries of blocks the last applied move touched
-    // (P changed on [i+1, j], E on [i, j]) are recomputed; the others stand
-    int dlo = 0, dhi = n;
-    if (incremental && *(volatile const int*)&slot->seed_ok) {
-        const unsigned long long mv = *(volatile const unsigned long long*)&slot->last_key;
-        dlo = key_i(mv) - halo;  // halo 1 for 2.5-opt: the gains changed on [i, j+1]
-        dhi = key_j(mv) + halo;
-    }
+    // the slot's fields are read together (one L2 round trip; the kernel is latency bound)
+    const int done = respect_done ? *(volatile const int*)&slot->done : 0;
+    const int seed_ok = incremental ? *(volatile const int*)&slot->seed_ok : 0;
+    const unsigned long long mv = incremental ? *(volatile const unsigned long long*)&slot->last_key : 0ull;
     // the cull and the list sweep that follow start from zeroed counters (a
     // best_move sweep leaves them set on the slot the next iteration reads)
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         slot->ncull = 0;
         slot->next_tile = 0;
     }
-    if (respect_done && *(volatile const int*)&slot->done) return;
+    if (done) return;
+    // incremental: only the summaries of blocks the last applied move touched
+    // (P changed on [i+1, j], E on [i, j]) are recomputed; the others stand
+    int dlo = 0, dhi = n;
+    if (seed_ok) {
+        dlo = key_i(mv) - halo;  // halo 1 for 2.5-opt: the gains changed on [i, j+1]
+        dhi = key_j(mv) + halo;
+    }
     const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
     int k0, ke;
     Box* out;
@@ -222,7 +225,7 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
 {
     pdl_trigger();
     pdl_wait();
-    if (respect_done && *(volatile int*)&slot->done) return;  // grid-uniform
+    const int done = respect_done ? *(volatile int*)&slot->done : 0;  // read with the other fields below
     const int t = blockIdx.x * blockDim.x + threadIdx.x;
     bool keep = false;
     int2 tl = make_int2(0, 0);
@@ -241,6 +244,7 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
         tl = tiles[t];
         if (inc) stored = tilebest[t];
     }
+    if (done) return;  // grid-uniform
     int dlo = 0, dhi = n;
     if (seed_ok) {
         dlo = key_i(mv) - halo;  // 2.5-opt (halo 1): a pair also reads g_{a+1}, g_b and D(a+1, b)
@@ -261,7 +265,7 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
         __syncthreads();
         if (threadIdx.x == 0) {
             for (int w = 1; w < (int)(blockDim.x >> 5); w++) clean_min = min(clean_min, s_min[w]);
-            if (clean_min < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, clean_min);
+            if (clean_min != kKeyNone) atomicMin(&slot->key, clean_min);  // no read-back: a RED, no round trip
         }
     }
     if (live) {
@@ -301,8 +305,9 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const flo
     __shared__ int4 s_t;
     pdl_trigger();
     pdl_wait();
-    if (respect_done && *(volatile int*)&slot->done) return;
+    const int done = respect_done ? *(volatile int*)&slot->done : 0;  // both fields in one round trip
     const unsigned count = *(volatile unsigned*)&slot->ncull;
+    if (done) return;
     // first entry static (entry blockIdx.x: no burst of 3k atomics on one
     // address at kernel start), then dynamic claims past the first wave
     unsigned k = blockIdx.x;

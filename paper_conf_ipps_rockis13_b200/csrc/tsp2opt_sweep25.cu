@@ -384,8 +384,9 @@ __global__ void __launch_bounds__(128, 4) sweep25_list_kernel(const float2* __re
     __shared__ int4 s_t;
     pdl_trigger();
     pdl_wait();
-    if (respect_done && *(volatile int*)&slot->done) return;
+    const int done = respect_done ? *(volatile int*)&slot->done : 0;  // both fields in one round trip
     const unsigned count = *(volatile unsigned*)&slot->ncull;
+    if (done) return;
     unsigned k = blockIdx.x;
     for (;;) {
         if (threadIdx.x == 0) s_t = k < count ? list[k] : make_int4(0, 0, -1, 0);
