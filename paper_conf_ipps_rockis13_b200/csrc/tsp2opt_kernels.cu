@@ -217,32 +217,41 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
 // with delta < 0; kept tiles (I0, J0, index) are appended to list[] (warp-aggregated
 // atomic on slot->ncull).  With seeding or the incremental sweep, a culled
 // tile's minimum is "none".
+constexpr int kCullPerThread = 4;  // tiles per thread, their loads batched (the kernel is latency bound)
+
 __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tiles, int ntiles, int TI, int TJ,
                                                    const Box* __restrict__ rbox, const Box* __restrict__ cbox,
                                                    Slot* __restrict__ slot, int4* __restrict__ list,
                                                    unsigned long long* __restrict__ tilebest, int flags,
                                                    int respect_done, int n, int halo)
 {
+    constexpr int V = kCullPerThread;
     pdl_trigger();
     pdl_wait();
-    const int done = respect_done ? *(volatile int*)&slot->done : 0;  // read with the other fields below
-    const int t = blockIdx.x * blockDim.x + threadIdx.x;
-    bool keep = false;
-    int2 tl = make_int2(0, 0);
     // kSweepIncremental: a tile whose pairs (a, b) all have a, b outside the
     // last applied move's [i, j] is clean -- positions a, a+1, b, b+1 kept
     // their cities and e_a, e_b their lengths, so every delta and the tile's
     // stored minimum stand.  Otherwise (or without a valid last move) it is
     // culled (minimum: none) or listed for the sweep.
-    // all independent loads first (the kernel is latency bound: one short chain per thread)
+    // All independent loads first (the slot's fields, then V tiles per thread).
     const bool inc = (flags & kSweepIncremental) && !(flags & kSweepFull);
+    const int done = respect_done ? *(volatile int*)&slot->done : 0;
     const int seed_ok = inc ? *(volatile int*)&slot->seed_ok : 0;
     const unsigned long long mv = inc ? *(volatile unsigned long long*)&slot->last_key : 0ull;
-    bool live = t < ntiles;
-    unsigned long long stored = kKeyNone;
-    if (live) {
-        tl = tiles[t];
-        if (inc) stored = tilebest[t];
+    const int gid = blockIdx.x * blockDim.x + threadIdx.x, stride = gridDim.x * blockDim.x;
+    int2 tl[V];
+    unsigned long long stored[V];
+    bool live[V];
+#pragma unroll
+    for (int k = 0; k < V; k++) {
+        const int t = gid + k * stride;
+        live[k] = t < ntiles;
+        tl[k] = make_int2(0, 0);
+        stored[k] = kKeyNone;
+        if (live[k]) {
+            tl[k] = tiles[t];
+            if (inc) stored[k] = tilebest[t];
+        }
     }
     if (done) return;  // grid-uniform
     int dlo = 0, dhi = n;
@@ -251,10 +260,12 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
         dhi = key_j(mv) + halo;
     }
     unsigned long long clean_min = kKeyNone;
-    if (live) {
-        live = (tl.x <= dhi && tl.x + TI >= dlo) || (tl.y <= dhi && tl.y + TJ >= dlo);  // dirty
-        if (!live) clean_min = stored;  // a clean tile's stored minimum stands
-    }
+#pragma unroll
+    for (int k = 0; k < V; k++)
+        if (live[k]) {
+            live[k] = (tl[k].x <= dhi && tl[k].x + TI >= dlo) || (tl[k].y <= dhi && tl[k].y + TJ >= dlo);  // dirty
+            if (!live[k]) clean_min = min(clean_min, stored[k]);  // a clean tile's stored minimum stands
+        }
     if (flags & kSweepIncremental) {
         // the clean tiles' share of the sweep's minimum (the re-swept tiles add
         // theirs from the list sweep); one atomic per block at most
@@ -268,21 +279,33 @@ __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tile
             if (clean_min != kKeyNone) atomicMin(&slot->key, clean_min);  // no read-back: a RED, no round trip
         }
     }
-    if (live) {
-        const Box r = rbox[tl.x / TI], c = cbox[tl.y / TJ];
-        const long long gx = max(0, max(c.xlo - r.xhi, r.xlo - c.xhi));
-        const long long gy = max(0, max(c.ylo - r.yhi, r.ylo - c.yhi));
-        const long long T = (long long)max(max(r.emax, c.emax), max(r.pad[0], c.pad[0])) - 1;  // pad[0]: gneg
-        keep = T >= 0 && gx * gx + gy * gy <= T * T + T;
-        if (!keep && (flags & (kSweepSeed | kSweepIncremental))) tilebest[t] = kKeyNone;
-    }
-    const unsigned m = __ballot_sync(0xffffffffu, keep);
-    if (m) {
-        const int lane = threadIdx.x & 31, leader = __ffs(m) - 1;
-        unsigned base = 0;
-        if (lane == leader) base = atomicAdd(&slot->ncull, (unsigned)__popc(m));
-        base = __shfl_sync(0xffffffffu, base, leader);
-        if (keep) list[base + __popc(m & ((1u << lane) - 1u))] = make_int4(tl.x, tl.y, t, 0);
+    Box r[V], c[V];
+#pragma unroll
+    for (int k = 0; k < V; k++)
+        if (live[k]) {
+            r[k] = rbox[tl[k].x / TI];
+            c[k] = cbox[tl[k].y / TJ];
+        }
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int k = 0; k < V; k++) {
+        bool keep = false;
+        if (live[k]) {
+            const long long gx = max(0, max(c[k].xlo - r[k].xhi, r[k].xlo - c[k].xhi));
+            const long long gy = max(0, max(c[k].ylo - r[k].yhi, r[k].ylo - c[k].yhi));
+            const long long T =
+                (long long)max(max(r[k].emax, c[k].emax), max(r[k].pad[0], c[k].pad[0])) - 1;  // pad[0]: gneg
+            keep = T >= 0 && gx * gx + gy * gy <= T * T + T;
+            if (!keep && (flags & (kSweepSeed | kSweepIncremental))) tilebest[gid + k * stride] = kKeyNone;
+        }
+        const unsigned m = __ballot_sync(0xffffffffu, keep);
+        if (m) {
+            const int leader = __ffs(m) - 1;
+            unsigned base = 0;
+            if (lane == leader) base = atomicAdd(&slot->ncull, (unsigned)__popc(m));
+            base = __shfl_sync(0xffffffffu, base, leader);
+            if (keep) list[base + __popc(m & ((1u << lane) - 1u))] = make_int4(tl[k].x, tl[k].y, gid + k * stride, 0);
+        }
     }
 }
 
@@ -670,8 +693,8 @@ cudaError_t launch_box_cull(const Geometry& g, const float2* P, const int* E, co
     cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, G, n, TI, nrb, g.tj, ncc,
                                rbox, cbox, slot, respect_done, inc && !(flags & kSweepFull) ? 1 : 0, 1);
     if (e != cudaSuccess) return e;
-    e = launch_pdl(cull_kernel, dim3((ntiles + 255) / 256), dim3(256), 0, st, tiles, ntiles, TI, g.tj, rbox, cbox, slot,
-                   list, tilebest, flags, respect_done, n, 1);
+    e = launch_pdl(cull_kernel, dim3((ntiles + 256 * kCullPerThread - 1) / (256 * kCullPerThread)), dim3(256), 0, st,
+                   tiles, ntiles, TI, g.tj, rbox, cbox, slot, list, tilebest, flags, respect_done, n, 1);
     g_launches += 2;
     return e != cudaSuccess ? e : cudaGetLastError();
 }
@@ -702,8 +725,8 @@ cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, 
     cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, (const int*)nullptr, n, TI,
                                nrb, g.tj, ncc, rbox, cbox, slot, respect_done, inc && !(flags & kSweepFull) ? 1 : 0, 0);
     if (e != cudaSuccess) return e;
-    e = launch_pdl(cull_kernel, dim3((ntiles + 255) / 256), dim3(256), 0, st, tiles, ntiles, TI, g.tj, rbox, cbox, slot,
-                   list, tilebest, flags, respect_done, n, 0);
+    e = launch_pdl(cull_kernel, dim3((ntiles + 256 * kCullPerThread - 1) / (256 * kCullPerThread)), dim3(256), 0, st,
+                   tiles, ntiles, TI, g.tj, rbox, cbox, slot, list, tilebest, flags, respect_done, n, 0);
     if (e != cudaSuccess) return e;
     if (inc) flags = (flags | kSweepLocal) & ~kSweepSeed;  // tile-local minima, reusable while clean
     e = by_rows_first(g.rows, (flags & kSweepFirst) != 0, [&](auto r, auto f) {
