@@ -161,63 +161,71 @@ __global__ void __launch_bounds__(256) box_kernel(const float2* __restrict__ P, 
         dlo = key_i(mv) - halo;  // halo 1 for 2.5-opt: the gains changed on [i, j+1]
         dhi = key_j(mv) + halo;
     }
-    const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
-    int k0, ke;
-    Box* out;
-    if (w < nrb) {
-        k0 = w * TI;
-        ke = min(k0 + TI, n - 1);
-        out = rbox + w;
-    } else if (w < nrb + ncc) {
-        k0 = (w - nrb) * TJ;
-        ke = min(k0 + TJ, n);
-        out = cbox + (w - nrb);
-    } else {
-        return;  // whole warps only
-    }
-    if (ke < dlo || k0 > dhi) return;  // clean: its summary stands (whole warp)
-    int xlo = 1 << 30, xhi = -1, ylo = 1 << 30, yhi = -1, emax = 0, gneg = 0;
-    // up to kBoxIters positions per lane, all loads issued before the first use
-    constexpr int kBoxIters = (32 * kRowsLarge * kMaxWarps + 1 + 31) / 32;
-#pragma unroll
-    for (int it = 0; it < kBoxIters; it++) {
-        const int k = k0 + lane + 32 * it;
-        if (k <= ke) {
-            const float2 p = P[k];
-            const int x = unbias(p.x), y = unbias(p.y);
-            xlo = min(xlo, x);
-            xhi = max(xhi, x);
-            ylo = min(ylo, y);
-            yhi = max(yhi, y);
-            if (k < ke) emax = max(emax, E[k]);
-            if (G) gneg = max(gneg, -G[k == n ? 0 : k]);
+    const int lane = threadIdx.x & 31;
+    const int nwarps = (int)(gridDim.x * blockDim.x) >> 5;
+    // grid-stride over the summaries: a small grid, most summaries are clean and skipped
+    for (int w = (int)(blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nrb + ncc; w += nwarps) {
+        int k0, ke;
+        Box* out;
+        if (w < nrb) {
+            k0 = w * TI;
+            ke = min(k0 + TI, n - 1);
+            out = rbox + w;
+        } else {
+            k0 = (w - nrb) * TJ;
+            ke = min(k0 + TJ, n);
+            out = cbox + (w - nrb);
         }
-    }
-    const unsigned full = 0xffffffffu;
-    xlo = __reduce_min_sync(full, xlo);
-    xhi = __reduce_max_sync(full, xhi);
-    ylo = __reduce_min_sync(full, ylo);
-    yhi = __reduce_max_sync(full, yhi);
-    emax = __reduce_max_sync(full, emax);
-    gneg = __reduce_max_sync(full, gneg);
-    if (lane == 0) {
-        Box b;
-        b.xlo = xlo;
-        b.xhi = xhi;
-        b.ylo = ylo;
-        b.yhi = yhi;
-        b.emax = emax;
-        b.pad[0] = gneg;  // 0 without G
-        b.pad[1] = b.pad[2] = 0;
-        *out = b;
+        if (ke < dlo || k0 > dhi) continue;  // clean: its summary stands (whole warp)
+        int xlo = 1 << 30, xhi = -1, ylo = 1 << 30, yhi = -1, emax = 0, gneg = 0;
+        // up to kBoxIters positions per lane, all loads issued before the first use
+        constexpr int kBoxIters = (32 * kRowsLarge * kMaxWarps + 1 + 31) / 32;
+#pragma unroll
+        for (int it = 0; it < kBoxIters; it++) {
+            const int k = k0 + lane + 32 * it;
+            if (k <= ke) {
+                const float2 p = P[k];
+                const int x = unbias(p.x), y = unbias(p.y);
+                xlo = min(xlo, x);
+                xhi = max(xhi, x);
+                ylo = min(ylo, y);
+                yhi = max(yhi, y);
+                if (k < ke) emax = max(emax, E[k]);
+                if (G) gneg = max(gneg, -G[k == n ? 0 : k]);
+            }
+        }
+        const unsigned full = 0xffffffffu;
+        xlo = __reduce_min_sync(full, xlo);
+        xhi = __reduce_max_sync(full, xhi);
+        ylo = __reduce_min_sync(full, ylo);
+        yhi = __reduce_max_sync(full, yhi);
+        emax = __reduce_max_sync(full, emax);
+        gneg = __reduce_max_sync(full, gneg);
+        if (lane == 0) {
+            Box b;
+            b.xlo = xlo;
+            b.xhi = xhi;
+            b.ylo = ylo;
+            b.yhi = yhi;
+            b.emax = emax;
+            b.pad[0] = gneg;  // 0 without G
+            b.pad[1] = b.pad[2] = 0;
+            *out = b;
+        }
     }
 }
 
+#ifndef TSP2OPT_CULL_V
+#define TSP2OPT_CULL_V 4
+#endif
+#ifndef TSP2OPT_BOX_BLOCKS
+#define TSP2OPT_BOX_BLOCKS 64  // box kernel grid cap (grid-stride over the summaries)
+#endif
 // One thread per tile of the shard: keep the tile iff its boxes allow a pair
 // with delta < 0; kept tiles (I0, J0, index) are appended to list[] (warp-aggregated
 // atomic on slot->ncull).  With seeding or the incremental sweep, a culled
 // tile's minimum is "none".
-constexpr int kCullPerThread = 4;  // tiles per thread, their loads batched (the kernel is latency bound)
+constexpr int kCullPerThread = TSP2OPT_CULL_V;  // tiles per thread, their loads batched (the kernel is latency bound)
 
 __global__ void __launch_bounds__(256) cull_kernel(const int2* __restrict__ tiles, int ntiles, int TI, int TJ,
                                                    const Box* __restrict__ rbox, const Box* __restrict__ cbox,
@@ -690,7 +698,7 @@ cudaError_t launch_box_cull(const Geometry& g, const float2* P, const int* E, co
     const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
     const int warps = nrb + ncc;
     const bool inc = (flags & kSweepIncremental) != 0;
-    cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, G, n, TI, nrb, g.tj, ncc,
+    cudaError_t e = launch_pdl(box_kernel, dim3(std::min((warps + 7) / 8, TSP2OPT_BOX_BLOCKS)), dim3(256), 0, st, P, E, G, n, TI, nrb, g.tj, ncc,
                                rbox, cbox, slot, respect_done, inc && !(flags & kSweepFull) ? 1 : 0, 1);
     if (e != cudaSuccess) return e;
     e = launch_pdl(cull_kernel, dim3((ntiles + 256 * kCullPerThread - 1) / (256 * kCullPerThread)), dim3(256), 0, st,
@@ -722,7 +730,7 @@ cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, 
     const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
     const int warps = nrb + ncc;
     const bool inc = (flags & kSweepIncremental) != 0;
-    cudaError_t e = launch_pdl(box_kernel, dim3((warps + 7) / 8), dim3(256), 0, st, P, E, (const int*)nullptr, n, TI,
+    cudaError_t e = launch_pdl(box_kernel, dim3(std::min((warps + 7) / 8, TSP2OPT_BOX_BLOCKS)), dim3(256), 0, st, P, E, (const int*)nullptr, n, TI,
                                nrb, g.tj, ncc, rbox, cbox, slot, respect_done, inc && !(flags & kSweepFull) ? 1 : 0, 0);
     if (e != cudaSuccess) return e;
     e = launch_pdl(cull_kernel, dim3((ntiles + 256 * kCullPerThread - 1) / (256 * kCullPerThread)), dim3(256), 0, st,
