@@ -214,6 +214,8 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
     h->d_list = nullptr;
     if (h->nctiles > 0) CUDA_TRY(cudaMalloc(&h->d_list, sizeof(int4) * (size_t)h->nctiles));
     h->list_grid = sweep_list_grid(h->cgeo, h->nctiles);
+    if (const char* el = getenv("TSP2OPT_LIST_GRID"))  // experiment: cap the list sweep's co-resident grid
+        if (atoi(el) > 0) h->list_grid = std::min(h->list_grid, atoi(el));
     h->list25_grid = sweep25_list_grid(h->cgeo, h->nctiles);
     h->last_tiling = -1;
     h->inc_valid = false;
