@@ -568,7 +568,9 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     h->all_tiles = build_tiles(n, h->geo);
     // Culled-sweep tiling: R = 7 rows per lane and narrow column chunks (measured,
     // local search from MF).
-    h->cgeo = Geometry{kRowsSmall, 1, total_pairs / world >= 1000000000LL ? 64 : 32};
+    // (incremental culled sweep, measured without per-sweep events: n = 85900 TJ 32 28.6 vs 64 30.6 us
+    // per iteration, n = 33810 TJ 16 20.6 vs 32 22.7 us; profiles/r01_inc_tiling.jsonl)
+    h->cgeo = Geometry{kRowsSmall, 1, total_pairs / world >= 1000000000LL ? 32 : 16};
     if (const char* er = getenv("TSP2OPT_CULL_ROWS")) h->cgeo.rows = atoi(er) == kRowsSmall ? kRowsSmall : kRowsLarge;
     if (const char* ec = getenv("TSP2OPT_CULL_TJ"))
         if (atoi(ec) >= 2 && atoi(ec) <= kMaxTJ) h->cgeo.tj = atoi(ec);

@@ -20,12 +20,15 @@ for cfg in cfgs:
         with tsp2opt.TSP2Opt(c) as g:
             g.set_option(tsp2opt.OPT_TILE_BOUNDS, 3)
             g.local_search(t, max_iters=3)
-            g.profile(True)
             t0 = time.perf_counter()
             r = g.local_search(t)
             dt = time.perf_counter() - t0
-            ms, launches = g.profile_read()
-            g.profile(False)
+            ms, launches = 0.0, 1
+            if os.environ.get("EXP_PROFILE"):
+                g.profile(True)
+                g.local_search(t)
+                ms, launches = g.profile_read()
+                g.profile(False)
         print(json.dumps({"cfg": cfg, "rows": int(rows), "tj": int(tj), "iters": r["iterations"], "length": r["length"],
                           "s": dt, "us_per_iter": 1e6 * dt / max(1, r["iterations"]),
                           "sweep_us": 1e3 * ms / max(1, launches)}), flush=True)
