@@ -269,21 +269,13 @@ int validate_coords(const int32_t* xy, int32_t n)
     return TSP2OPT_OK;
 }
 
-// Permutation check with per-thread epoch stamps (no allocation or clearing per call).
 int validate_tour(const int32_t* t, int n)
 {
     if (!t) return TSP2OPT_EINVAL;
-    thread_local std::vector<uint32_t> stamp;
-    thread_local uint32_t epoch = 0;
-    if (stamp.size() < (size_t)n) stamp.assign((size_t)n, 0u);
-    if (++epoch == 0) {  // wrap-around: clear and restart
-        std::fill(stamp.begin(), stamp.end(), 0u);
-        epoch = 1;
-    }
+    std::vector<unsigned char> seen(n, 0);  // bytes: the check stays in the host's L2
     for (int k = 0; k < n; k++) {
-        const int32_t c = t[k];
-        if (c < 0 || c >= n || stamp[c] == epoch) return TSP2OPT_ENOTPERM;
-        stamp[c] = epoch;
+        if (t[k] < 0 || t[k] >= n || seen[t[k]]) return TSP2OPT_ENOTPERM;
+        seen[t[k]] = 1;
     }
     return TSP2OPT_OK;
 }
