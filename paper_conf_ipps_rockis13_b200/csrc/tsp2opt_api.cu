@@ -86,6 +86,8 @@ struct tsp2opt_ctx {
     int list25_grid = 0;        // CTAs of the 2.5-opt culled sweep
     int last_tiling = -1;       // tiling of the previous sweep (0 dense, 1 cull): seeds are per tiling
     bool inc_valid = false;     // the stored per-tile minima are those of an incremental sweep of the current tiling
+    bool global_seed = false;   // TSP2OPT_GLOBAL_SEED=1: dense sweeps start from the best surviving tile minimum
+                                // (measured: C4 random 8 % faster, C2 / C3 2-10 % slower; profiles/r01_global_seed.jsonl)
     unsigned long long* d_trace = nullptr;  // [trace_cap] keys of the applied moves (TSP2OPT_OPT_TRACE)
     int* d_best = nullptr;      // [n] best tour of an ILS run
     void* d_mf_ws = nullptr;    // Multiple Fragment workspace (mf_workspace_bytes), allocated on first use
@@ -391,6 +393,9 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         Slot* out = h->d_slots + (h->parity ^ 1);
         CUDA_TRY(launch_apply(h->d_P, h->d_E, h->d_tour, h->n, in, out, max_moves, 0, 0, 0, h->d_trace,
                               h->trace_cap, h->nbr_k > 0 ? h->d_pos : nullptr, h->stream));
+        // dense best-improvement sweep: start the next one from the best surviving tile minimum
+        if (tiling == 0 && !h->first && h->global_seed)
+            CUDA_TRY(launch_global_seed(h->d_tilebest, h->ntiles, out, h->stream));
         h->parity ^= 1;
     }
     return TSP2OPT_OK;
@@ -540,6 +545,7 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     CTRY(cudaHostAlloc(&h->h_ctl, sizeof(int), cudaHostAllocDefault));
     if (const char* ep = getenv("TSP2OPT_PERSISTENT")) h->persistent = atoi(ep);
     if (const char* es = getenv("TSP2OPT_SEED")) h->seed_next = atoi(es) != 0;
+    if (const char* eg = getenv("TSP2OPT_GLOBAL_SEED")) h->global_seed = atoi(eg) != 0;
 
     CTRY(cudaMemset(h->d_slots, 0, sizeof(Slot) * 2));
     {

@@ -624,6 +624,45 @@ cudaError_t launch_first_fix(const float2* P, const int* E, Slot* slot, int resp
     return e != cudaSuccess ? e : cudaGetLastError();
 }
 
+// Global seed of the dense sweep (tiling 0): after a move (i, j) is applied,
+// every tile minimum of the sweep that found it whose pair the reversal leaves
+// intact (surviving_key) is a real pair of the new tour with its exact delta.
+// Their min starts the next sweep's bound for every tile at once, instead of
+// the seed (0, 1, 0) that only tightens as tiles finish.  The sweep still
+// examines every pair: any pair with a lower (delta, cell) replaces it.
+__global__ void __launch_bounds__(256) global_seed_kernel(const unsigned long long* __restrict__ tilebest, int ntiles,
+                                                          Slot* __restrict__ slot)
+{
+    pdl_trigger();
+    pdl_wait();
+    const int ok = *(volatile int*)&slot->seed_ok;
+    const int done = *(volatile int*)&slot->done;
+    const unsigned long long mv = *(volatile unsigned long long*)&slot->last_key;
+    if (!ok || done) return;
+    const int i = key_i(mv), j = key_j(mv);
+    unsigned long long m = kKeyNone;
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < ntiles; t += gridDim.x * blockDim.x)
+        m = min(m, surviving_key(tilebest[t], i, j));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
+    __shared__ unsigned long long s_m[8];
+    if ((threadIdx.x & 31) == 0) s_m[threadIdx.x >> 5] = m;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int w = 1; w < (int)(blockDim.x >> 5); w++) m = min(m, s_m[w]);
+        if (m != kKeyNone) atomicMin(&slot->key, m);
+    }
+}
+
+cudaError_t launch_global_seed(const unsigned long long* tilebest, int ntiles, Slot* slot, cudaStream_t st)
+{
+    if (ntiles <= 0) return cudaSuccess;
+    const int grid = std::max(1, std::min(148, (ntiles + 255) / 256));
+    cudaError_t e = launch_pdl(global_seed_kernel, dim3(grid), dim3(256), 0, st, tilebest, ntiles, slot);
+    g_launches += 1;
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
+
 cudaError_t launch_reset_key(Slot* slot, cudaStream_t st)
 {
     reset_key_kernel<<<1, 1, 0, st>>>(slot);

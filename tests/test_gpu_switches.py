@@ -48,3 +48,20 @@ def test_pruned_threads_per_position(gpu, monkeypatch, tp):
         res = g.local_search(t)
     want = oracle.pruned_local_search(c, t, 16)
     assert (res["iterations"], res["length"]) == (want["iterations"], want["length"])
+
+
+@pytest.mark.parametrize("kind,n,seed", [("uniform", 1002, 31), ("lattice", 3001, 32)])
+def test_global_seed_switch(gpu, monkeypatch, kind, n, seed):
+    """TSP2OPT_GLOBAL_SEED=1: each dense sweep starts from the best tile minimum
+    of the previous sweep that the applied reversal leaves intact."""
+    monkeypatch.setenv("TSP2OPT_GLOBAL_SEED", "1")
+    monkeypatch.setenv("TSP2OPT_PERSISTENT", "0")
+    c = inputs.make_coords(kind, n, seed)
+    t = inputs.random_tour(n, seed)
+    want = oracle.local_search(c, t, trace_cap=10 * n)
+    with tsp2opt.TSP2Opt(c) as g:
+        g.set_option(tsp2opt.OPT_TRACE, 10 * n)
+        res = g.local_search(t)
+        trace = g.get_trace(10 * n)
+    assert (res["iterations"], res["length"]) == (want["iterations"], want["length"])
+    assert np.array_equal(np.asarray(trace, dtype=np.int64), want["trace"])
