@@ -89,6 +89,14 @@ def _load():
             lib.oracle25_apply.restype = None
             lib.oracle25_local_search.argtypes = [p, i64, p, i64, p, p, p, i64]
             lib.oracle25_local_search.restype = ctypes.c_int
+            lib.oracleor_delta.argtypes = [p, i64, p, i64, i64, ctypes.c_int]
+            lib.oracleor_delta.restype = i64
+            lib.oracleor_best_move.argtypes = [p, i64, p, p, p, p, p]
+            lib.oracleor_best_move.restype = None
+            lib.oracleor_apply.argtypes = [p, i64, i64, ctypes.c_int]
+            lib.oracleor_apply.restype = None
+            lib.oracleor_local_search.argtypes = [p, i64, p, i64, p, p, p, i64]
+            lib.oracleor_local_search.restype = ctypes.c_int
             lib.oracle_first_move.argtypes = [p, i64, p, p, p, p]
             lib.oracle_first_move.restype = None
             lib.oracle_first_local_search.argtypes = [p, i64, p, i64, p, p, p, i64]
@@ -324,6 +332,41 @@ def local_search25(coords, tour, max_iters: int = -1, trace_cap: int = 0):
     out = np.zeros(2, dtype=np.int64)
     tr = np.zeros((max(trace_cap, 1), 4), dtype=np.int64)
     st = _load().oracle25_local_search(_ptr(xy), xy.shape[0], _ptr(t), int(max_iters), _ptr(out[0:1]),
+                                       _ptr(out[1:2]), _ptr(tr) if trace_cap > 0 else None, int(trace_cap))
+    it = int(out[1])
+    return dict(tour=t, length=int(out[0]), iterations=it, status=int(st), trace=tr[: min(it, trace_cap)].copy())
+
+
+def delta_or(coords, tour, i: int, j: int, typ: int) -> int:
+    """delta of Or-opt move (i, j, type) (reading R21); a huge value if not a move."""
+    xy = _xy(coords)
+    t = np.ascontiguousarray(tour, dtype=np.int32)
+    return int(_load().oracleor_delta(_ptr(xy), xy.shape[0], _ptr(t), i, j, typ))
+
+
+def best_move_or(coords, tour):
+    """(i, j, type, delta) of the best Or-opt move (reading R21: 2-opt plus segment moves, L <= 3)."""
+    xy = _xy(coords)
+    t = np.ascontiguousarray(tour, dtype=np.int32)
+    out = np.zeros(4, dtype=np.int64)
+    _load().oracleor_best_move(_ptr(xy), xy.shape[0], _ptr(t), _ptr(out[0:1]), _ptr(out[1:2]), _ptr(out[2:3]),
+                               _ptr(out[3:4]))
+    return int(out[0]), int(out[1]), int(out[2]), int(out[3])
+
+
+def apply_or(tour, i: int, j: int, typ: int) -> np.ndarray:
+    t = np.array(tour, dtype=np.int32, copy=True)
+    _load().oracleor_apply(_ptr(t), i, j, typ)
+    return t
+
+
+def local_search_or(coords, tour, max_iters: int = -1, trace_cap: int = 0):
+    """Best-improvement Or-opt local search; trace int64[k, 4] rows (i, j, delta, type)."""
+    xy = _xy(coords)
+    t = np.array(tour, dtype=np.int32, copy=True)
+    out = np.zeros(2, dtype=np.int64)
+    tr = np.zeros((max(trace_cap, 1), 4), dtype=np.int64)
+    st = _load().oracleor_local_search(_ptr(xy), xy.shape[0], _ptr(t), int(max_iters), _ptr(out[0:1]),
                                        _ptr(out[1:2]), _ptr(tr) if trace_cap > 0 else None, int(trace_cap))
     it = int(out[1])
     return dict(tour=t, length=int(out[0]), iterations=it, status=int(st), trace=tr[: min(it, trace_cap)].copy())

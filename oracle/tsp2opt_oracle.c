@@ -796,3 +796,124 @@ void oracle_ils_mode(const int32_t *xy, int64_t n, int32_t *tour, int64_t iterat
     free(cand);
     *length = L;
 }
+
+/* ---------------------------------------------------------------------------
+ * Or-opt ("2.5-opt/Or-opt variants"; L18 §V "more
+ * sophisticated algorithms such as 3-opt, k-opt or LK"; L26 §VII "2.5-opt,
+ * 3-opt and Lin-Kernighan").  The paper gives no definition; reading R21
+ * takes Or's textbook neighbourhood -- 2-opt plus moving a
+ * segment of L = 1, 2 or 3 consecutive cities, in either orientation, into
+ * another edge -- over the same pairs 0 <= i < j <= n-1 as the 2-opt sweep
+ * (reading R1).  Types (13 per pair):
+ *   type 0                     the 2-opt move (reverse positions i+1..j);
+ *   type 1 + 4(L-1) + 2 dir + rev, for j >= i+L+1:
+ *     dir 0 (forward):  segment t[i+1..i+L] moves between t[j] and t[j+1];
+ *     dir 1 (backward): segment t[j-L+1..j] moves between t[i] and t[i+1];
+ *     rev 1: the segment is inserted reversed.
+ * With a = the segment's first city and b its last (rev swaps them):
+ *   forward:  delta = d(t_i, t_{i+L+1}) - d(t_i, t_{i+1}) - d(t_{i+L}, t_{i+L+1})
+ *                   + d(t_j, a) + d(b, t_{j+1}) - d(t_j, t_{j+1});
+ *   backward: delta = d(t_{j-L}, t_{j+1}) - d(t_{j-L}, t_{j-L+1}) - d(t_j, t_{j+1})
+ *                   + d(t_i, a) + d(b, t_{i+1}) - d(t_i, t_{i+1}).
+ * L = 1 forward / backward are 2.5-opt's types 1 / 2 (reading R19); for
+ * L = 1 the reversed types equal the plain ones and lose the type tie-break.
+ * Best = the lowest (delta, Fig. 3 cell, type) with delta < 0, else
+ * (0, 1, type 0, delta 0).  Only positions i+1..j move, so t[0] never moves
+ * (reading R6): segments containing t[0] are not moved.
+ * ------------------------------------------------------------------------- */
+int64_t oracleor_delta(const int32_t *xy, int64_t n, const int32_t *tour, int64_t i, int64_t j, int type)
+{
+    if (type == 0) return oracle_delta(xy, n, tour, i, j);
+    if (type < 0 || type > 12) return INT64_MAX;
+    const int64_t L = 1 + (type - 1) / 4, dir = ((type - 1) / 2) & 1, rev = (type - 1) & 1;
+    if (j < i + L + 1) return INT64_MAX; /* not a move */
+    if (dir == 0) {
+        const int64_t a = rev ? i + L : i + 1, b = rev ? i + 1 : i + L;
+        return dpos(xy, tour, n, i, i + L + 1) - dpos(xy, tour, n, i, i + 1) - dpos(xy, tour, n, i + L, i + L + 1)
+             + dpos(xy, tour, n, j, a) + dpos(xy, tour, n, b, j + 1) - dpos(xy, tour, n, j, j + 1);
+    }
+    const int64_t a = rev ? j : j - L + 1, b = rev ? j - L + 1 : j;
+    return dpos(xy, tour, n, j - L, j + 1) - dpos(xy, tour, n, j - L, j - L + 1) - dpos(xy, tour, n, j, j + 1)
+         + dpos(xy, tour, n, i, a) + dpos(xy, tour, n, b, i + 1) - dpos(xy, tour, n, i, i + 1);
+}
+
+/* One exhaustive Or-opt sweep: every (j, i, type) in increasing (cell, type)
+ * order, oracleor_delta per move, strict '<' keeps the lowest. */
+void oracleor_best_move(const int32_t *xy, int64_t n, const int32_t *tour,
+                        int64_t *bi, int64_t *bj, int64_t *btype, int64_t *bdelta)
+{
+    int64_t best_d = 0, best_i = 0, best_j = 1, best_t = 0;
+#pragma omp parallel
+    {
+        int64_t td = 0, ti = 0, tj = 1, tt = 0;
+#pragma omp for schedule(dynamic, 16) nowait
+        for (int64_t j = 1; j < n; j++)
+            for (int64_t i = 0; i < j; i++)
+                for (int t = 0; t <= 12; t++) {
+                    const int64_t d = oracleor_delta(xy, n, tour, i, j, t);
+                    if (d < td || (d == td && (oracle_cell(i, j) < oracle_cell(ti, tj) ||
+                                               (oracle_cell(i, j) == oracle_cell(ti, tj) && t < tt)))) {
+                        td = d; ti = i; tj = j; tt = t;
+                    }
+                }
+#pragma omp critical
+        {
+            if (td < best_d || (td == best_d && (oracle_cell(ti, tj) < oracle_cell(best_i, best_j) ||
+                                                 (oracle_cell(ti, tj) == oracle_cell(best_i, best_j) && tt < best_t)))) {
+                best_d = td; best_i = ti; best_j = tj; best_t = tt;
+            }
+        }
+    }
+    *bi = best_i; *bj = best_j; *btype = best_t; *bdelta = best_d;
+}
+
+/* Apply move (i, j, type) by writing positions i+1..j in their new order:
+ * the rest of the span first (forward) or last (backward), the segment in
+ * its (possibly reversed) order in the edge it moves into. */
+void oracleor_apply(int32_t *tour, int64_t i, int64_t j, int type)
+{
+    if (type == 0) {
+        oracle_apply(tour, i, j);
+        return;
+    }
+    const int64_t L = 1 + (type - 1) / 4, dir = ((type - 1) / 2) & 1, rev = (type - 1) & 1;
+    const int64_t m = j - i;
+    int32_t *span = (int32_t *)malloc(sizeof(int32_t) * m);
+    int64_t w = 0;
+    if (dir == 0) {
+        for (int64_t k = i + L + 1; k <= j; k++) span[w++] = tour[k];
+        for (int64_t q = 0; q < L; q++) span[w++] = tour[rev ? i + L - q : i + 1 + q];
+    } else {
+        for (int64_t q = 0; q < L; q++) span[w++] = tour[rev ? j - q : j - L + 1 + q];
+        for (int64_t k = i + 1; k <= j - L; k++) span[w++] = tour[k];
+    }
+    memcpy(tour + i + 1, span, sizeof(int32_t) * m);
+    free(span);
+}
+
+/* Best-improvement Or-opt local search; trace rows (i, j, delta, type). */
+int oracleor_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64_t max_iters,
+                          int64_t *length, int64_t *iterations, int64_t *trace, int64_t trace_cap)
+{
+    int64_t L = oracle_tour_length(xy, n, tour);
+    int64_t it = 0;
+    int status = 0;
+    for (;;) {
+        int64_t i, j, t, d;
+        oracleor_best_move(xy, n, tour, &i, &j, &t, &d);
+        if (d >= 0) break;
+        if (max_iters >= 0 && it >= max_iters) { /* reading R8 */
+            status = 1;
+            break;
+        }
+        oracleor_apply(tour, i, j, (int)t);
+        L += d;
+        if (trace && it < trace_cap) {
+            trace[4 * it] = i; trace[4 * it + 1] = j; trace[4 * it + 2] = d; trace[4 * it + 3] = t;
+        }
+        it++;
+    }
+    *length = L;
+    *iterations = it;
+    return status;
+}
