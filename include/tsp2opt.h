@@ -186,6 +186,37 @@ int tsp2opt_batch_ils_async(const int32_t *d_coords_xy, int32_t n, int32_t batch
                             int64_t iterations, const uint64_t *d_seeds, int64_t *d_lengths, int64_t *d_history,
                             void *stream);
 
+/* Or-opt local search (SURVEY §8(f) NEXT-4 "2.5-opt/Or-opt variants"; L18 §V
+ * "more sophisticated algorithms such as 3-opt, k-opt or LK"; L26 §VII; the
+ * paper gives no definition: reading R21).  The
+ * neighbourhood is 2-opt plus moving a segment of L = 1, 2 or 3 cities, in
+ * either orientation, into another edge, over the pairs 0 <= i < j <= n-1 of
+ * reading R1, 13 moves per pair:
+ *   type 0: the 2-opt move (reverse positions i+1..j);
+ *   type 1 + 4(L-1) + 2*dir + rev (needs j >= i+L+1): dir 0 moves
+ *   t[i+1..i+L] between t[j] and t[j+1], dir 1 moves t[j-L+1..j] between
+ *   t[i] and t[i+1]; rev = 1 inserts the segment reversed.
+ * Best improvement: each step applies the lowest (delta, Fig. 3 cell
+ * j(j-1)/2+i, type) with delta < 0; t[0] never moves.  Stateless (no handle;
+ * current CUDA device, legacy default stream).  coords_xy: host int32[2n] in
+ * [0, 2^15); tour: host int32[n], in = start tour, out = the Or-opt local
+ * minimum (or the tour after max_iters moves); *length / *iterations (or NULL)
+ * = final length and moves applied; trace_ijdt (NULL iff trace_cap == 0):
+ * int32[4*trace_cap] rows (i, j, delta, type) of the first trace_cap moves.
+ * 3 <= n <= TSP2OPT_OROPT_MAX_N (the key packs i and j in 20 bits).  Returns
+ * TSP2OPT_OK at a local minimum, TSP2OPT_MAXITER when capped with an
+ * improving move left; errors as tsp2opt_create / set_tour, or EINVAL
+ * (max_iters < 0, trace_cap < 0); nothing is written on error. */
+#define TSP2OPT_OROPT_MAX_N (1 << 20)
+int tsp2opt_oropt_local_search(const int32_t *coords_xy, int32_t n, int32_t *tour, int64_t max_iters,
+                               int64_t *length, int64_t *iterations, int32_t *trace_ijdt, int64_t trace_cap);
+
+/* One Or-opt sweep: the best move (i, j, type, delta) of `tour` (host
+ * int32[n], not modified), (0, 1, 0, 0) at a local minimum.  Arguments and
+ * errors as tsp2opt_oropt_local_search. */
+int tsp2opt_oropt_best_move(const int32_t *coords_xy, int32_t n, const int32_t *tour, int32_t *i, int32_t *j,
+                            int32_t *type, int32_t *delta);
+
 /* Multiple Fragment (greedy) start tour, computed on the device (SURVEY §8(f)
  * NEXT-1; L22 §V "an initial solution based on the Multiple Fragment(Greedy)
  * heuristic[18]"; definition, tie-break and orientation: DESIGN.md R17 --

@@ -1217,3 +1217,103 @@ const char* tsp2opt_strerror(int code)
 const char* tsp2opt_last_error(void) { return g_last_error.c_str(); }
 
 }  // extern "C"
+
+// ---------------------------------------------------------------------------
+// Or-opt (reading R21; tsp2opt_oropt.cu).  Stateless:
+// upload, then per move one dense sweep, an 8-byte key read and the apply.
+namespace {
+
+int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters, int64_t* length,
+           int64_t* iterations, int32_t* trace, int64_t trace_cap, unsigned long long* first_key)
+{
+    int rc = validate_coords(coords_xy, n);
+    if (rc) return rc;
+    rc = validate_tour(tour, n);
+    if (rc) return rc;
+    int* d_xy = nullptr;
+    int* d_t = nullptr;
+    int* d_span = nullptr;
+    int2* d_q = nullptr;
+    unsigned long long* d_slot = nullptr;  // [0] key, [1] length
+    auto cleanup = [&]() {
+        cudaFree(d_xy);
+        cudaFree(d_t);
+        cudaFree(d_span);
+        cudaFree(d_q);
+        cudaFree(d_slot);
+    };
+    auto fail = [&](cudaError_t e, const char* what) {
+        cleanup();
+        return cuda_fail(e, what);
+    };
+    cudaError_t e;
+    const size_t nb = sizeof(int) * (size_t)n;
+    if ((e = cudaMalloc(&d_xy, 2 * nb)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMalloc(&d_t, nb)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMalloc(&d_span, nb)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMalloc(&d_q, sizeof(int2) * oropt_q_entries(n))) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMalloc(&d_slot, 2 * sizeof(unsigned long long))) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMemcpy(d_xy, coords_xy, 2 * nb, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "H2D");
+    if ((e = cudaMemcpy(d_t, tour, nb, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "H2D");
+    if ((e = launch_or_load(d_xy, d_t, d_q, n, d_slot + 1, nullptr)) != cudaSuccess) return fail(e, "or_load");
+    unsigned long long len = 0;
+    if ((e = cudaMemcpy(&len, d_slot + 1, sizeof(len), cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
+    long long L = (long long)len, it = 0;
+    int status = TSP2OPT_OK;
+    for (;;) {
+        if ((e = launch_or_sweep(d_q, n, d_slot, nullptr)) != cudaSuccess) return fail(e, "or_sweep_kernel");
+        unsigned long long key = 0;
+        if ((e = cudaMemcpy(&key, d_slot, sizeof(key), cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
+        if (first_key && it == 0) *first_key = key;
+        int i, j, type, d;
+        or_unpack(key, &i, &j, &type, &d);
+        if (d >= 0) break;
+        if (it >= max_iters) {  // reading R8
+            status = TSP2OPT_MAXITER;
+            break;
+        }
+        if ((e = launch_or_apply(d_xy, d_t, d_q, d_span, n, i, j, type, nullptr)) != cudaSuccess)
+            return fail(e, "or_apply");
+        if (trace && it < trace_cap) {
+            trace[4 * it] = i;
+            trace[4 * it + 1] = j;
+            trace[4 * it + 2] = d;
+            trace[4 * it + 3] = type;
+        }
+        L += d;
+        it++;
+    }
+    if ((e = cudaMemcpy(tour, d_t, nb, cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
+    cleanup();
+    if (length) *length = L;
+    if (iterations) *iterations = it;
+    return status;
+}
+
+}  // namespace
+
+int tsp2opt_oropt_local_search(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters,
+                               int64_t* length, int64_t* iterations, int32_t* trace_ijdt, int64_t trace_cap)
+{
+    if (!coords_xy || !tour || max_iters < 0 || trace_cap < 0 || (trace_cap > 0 && !trace_ijdt)) return TSP2OPT_EINVAL;
+    if (n < 3 || n > TSP2OPT_OROPT_MAX_N) return TSP2OPT_EINVAL;
+    return or_run(coords_xy, n, tour, max_iters, length, iterations, trace_ijdt, trace_cap, nullptr);
+}
+
+int tsp2opt_oropt_best_move(const int32_t* coords_xy, int32_t n, const int32_t* tour, int32_t* i, int32_t* j,
+                            int32_t* type, int32_t* delta)
+{
+    if (!coords_xy || !tour || !i || !j || !type || !delta) return TSP2OPT_EINVAL;
+    if (n < 3 || n > TSP2OPT_OROPT_MAX_N) return TSP2OPT_EINVAL;
+    std::vector<int32_t> t(tour, tour + n);
+    unsigned long long key = 0;
+    int rc = or_run(coords_xy, n, t.data(), 0, nullptr, nullptr, nullptr, 0, &key);
+    if (rc < 0) return rc;
+    int ii, jj, tt, dd;
+    or_unpack(key, &ii, &jj, &tt, &dd);
+    *i = ii;
+    *j = jj;
+    *type = tt;
+    *delta = dd;
+    return TSP2OPT_OK;
+}

@@ -85,6 +85,13 @@ cudaError_t launch_decide25(const float2* P, const int* E, const int* G, Slot* s
 cudaError_t launch_apply25(float2* P, int* E, int* G, int* tour, int n, const Slot* in, Slot* out,
                            long long max_moves, int explicit_move, int ei, int ej, int etype,
                            unsigned long long* trace, int* ttype, long long trace_cap, unsigned* bar, cudaStream_t st);
+// Or-opt (tsp2opt_oropt.cu; reading R21): route-ordered int2 Q[n + 5], dense sweep, span apply.
+size_t oropt_q_entries(int n);
+cudaError_t launch_or_load(const int* coords, const int* tour, int2* Q, int n, unsigned long long* len, cudaStream_t st);
+cudaError_t launch_or_sweep(const int2* Q, int n, unsigned long long* slot, cudaStream_t st);
+cudaError_t launch_or_apply(const int* coords, int* tour, int2* Q, int* span, int n, int i, int j, int type,
+                            cudaStream_t st);
+void or_unpack(unsigned long long key, int* i, int* j, int* type, int* delta);
 size_t sweep_smem_bytes(const Geometry& g);
 cudaError_t sweep_prepare();
 cudaError_t launch_load_tour(const int* coords, const int* tour_src, int* tour_dst, float2* P, int* E, int n,

@@ -1,0 +1,184 @@
+// tsp2opt_oropt.cu -- Or-opt sweep and apply (SURVEY.md §8(f) NEXT-4,
+// "2.5-opt/Or-opt variants"; L26 §VII; reading R21 and §5.15).
+//
+// Neighbourhood (reading R21): the pairs 0 <= i < j <= n-1 of the closed tour
+// (reading R1), 13 moves per pair: type 0 the 2-opt move, and for
+// type = 1 + 4(L-1) + 2 dir + rev with j >= i+L+1 the move of a segment of
+// L = 1..3 cities (dir 0: t[i+1..i+L] into the edge (t_j, t_{j+1}); dir 1:
+// t[j-L+1..j] into the edge (t_i, t_{i+1})), reversed iff rev.  Best = the
+// lowest (delta, Fig. 3 cell, type) with delta < 0, else (0, 1, type 0).
+//
+// Layout: Q[p] = coords[tour[p]] for p < n + 5 (positions mod n: the closed
+// array of reading R10 plus the halo a segment of three past position n-1
+// can reach), int2.  One thread per cell, grid-stride over the cells of a
+// 148-multiple grid; the packed key (delta + 2^18) << 44 | j << 24 | i << 4 |
+// type (n <= 2^20) reduces per warp by shuffles, per CTA in shared memory and
+// per GPU with one 64-bit atomicMin.  Distances are the exact EUC_2D nint of
+// tsp2opt_device.cuh.  The apply writes positions i+1..j in their new order
+// into a scratch span, then copies it back (two launches, no grid barrier).
+#include "tsp2opt_internal.h"
+
+namespace tsp2opt {
+
+constexpr int kOrHalo = 5;
+constexpr int kOrThreads = 256;
+
+__host__ __device__ __forceinline__ unsigned long long or_pack(int delta, int i, int j, int type)
+{
+    return ((unsigned long long)(delta + kDeltaBias) << 44) | ((unsigned long long)j << 24) |
+           ((unsigned long long)i << 4) | (unsigned long long)type;
+}
+
+__device__ __forceinline__ int or_d(int2 a, int2 b) { return exact_dist_xy(a.x, a.y, b.x, b.y); }
+
+// Q[p] = coords[tour[p mod n]] for p < n + kOrHalo
+__global__ void or_gather_kernel(const int* __restrict__ coords, const int* __restrict__ tour, int2* __restrict__ Q,
+                                 int n)
+{
+    for (int p = blockIdx.x * blockDim.x + threadIdx.x; p < n + kOrHalo; p += gridDim.x * blockDim.x) {
+        const int c = tour[p % n];
+        Q[p] = make_int2(coords[2 * c], coords[2 * c + 1]);
+    }
+}
+
+// Tour length: sum of d(Q[p], Q[p+1]), p < n, into *len (zeroed by the caller)
+__global__ void or_length_kernel(const int2* __restrict__ Q, int n, unsigned long long* len)
+{
+    unsigned long long s = 0;
+    for (int p = blockIdx.x * blockDim.x + threadIdx.x; p < n; p += gridDim.x * blockDim.x) s += or_d(Q[p], Q[p + 1]);
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if ((threadIdx.x & 31) == 0 && s) atomicAdd(len, s);
+}
+
+__global__ void __launch_bounds__(kOrThreads) or_sweep_kernel(const int2* __restrict__ Q, int n, long long cells,
+                                                              unsigned long long* slot)
+{
+    unsigned long long best = or_pack(0, 0, 1, 0);
+    for (long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x; k < cells;
+         k += (long long)gridDim.x * blockDim.x) {
+        // cell k = j(j-1)/2 + i (Fig. 3): j = floor((1 + sqrt(1 + 8k)) / 2), fixed up exactly
+        int j = (int)((1.0 + sqrt(1.0 + 8.0 * (double)k)) * 0.5);
+        while ((long long)j * (j - 1) / 2 > k) j--;
+        while ((long long)(j + 1) * j / 2 <= k) j++;
+        const int i = (int)(k - (long long)j * (j - 1) / 2);
+        const int2 a0 = Q[i], a1 = Q[i + 1], bj = Q[j], bj1 = Q[j + 1];
+        const int ei = or_d(a0, a1), ej = or_d(bj, bj1);
+        int d = or_d(a0, bj) + or_d(a1, bj1) - ei - ej;  // type 0
+        unsigned long long key = or_pack(d, i, j, 0);
+        if (key < best) best = key;
+#pragma unroll
+        for (int L = 1; L <= 3; L++) {
+            if (j < i + L + 1) break;
+            // forward: t[i+1..i+L] into (t_j, t_{j+1})
+            const int2 s0 = Q[i + 1], sL = Q[i + L], nx = Q[i + L + 1];
+            const int rem_f = or_d(a0, nx) - ei - or_d(sL, nx) - ej;
+            // backward: t[j-L+1..j] into (t_i, t_{i+1})
+            const int2 pv = Q[j - L], u0 = Q[j - L + 1];
+            const int rem_b = or_d(pv, bj1) - or_d(pv, u0) - ej - ei;
+            const int df0 = rem_f + or_d(bj, s0) + or_d(sL, bj1);
+            const int df1 = rem_f + or_d(bj, sL) + or_d(s0, bj1);
+            const int db0 = rem_b + or_d(a0, u0) + or_d(bj, a1);
+            const int db1 = rem_b + or_d(a0, bj) + or_d(u0, a1);
+            const int t0 = 1 + 4 * (L - 1);
+            key = or_pack(df0, i, j, t0);
+            if (key < best) best = key;
+            key = or_pack(df1, i, j, t0 + 1);
+            if (key < best) best = key;
+            key = or_pack(db0, i, j, t0 + 2);
+            if (key < best) best = key;
+            key = or_pack(db1, i, j, t0 + 3);
+            if (key < best) best = key;
+        }
+    }
+    for (int o = 16; o; o >>= 1) {
+        const unsigned long long other = __shfl_xor_sync(0xffffffffu, best, o);
+        best = other < best ? other : best;
+    }
+    __shared__ unsigned long long red[kOrThreads / 32];
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = best;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int w = 1; w < kOrThreads / 32; w++) best = red[w] < best ? red[w] : best;
+        atomicMin(slot, best);
+    }
+}
+
+// span[p - i - 1] = the tour city that lands on position p in [i+1, j] (oracleor_apply's order)
+__global__ void or_span_kernel(const int* __restrict__ tour, int* __restrict__ span, int i, int j, int type)
+{
+    const int m = j - i;
+    const int L = 1 + (type - 1) / 4, dir = ((type - 1) / 2) & 1, rev = (type - 1) & 1;
+    for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < m; q += gridDim.x * blockDim.x) {
+        const int p = i + 1 + q;
+        int src;
+        if (type == 0) src = i + 1 + j - p;
+        else if (dir == 0) src = p <= j - L ? p + L : (rev ? i + L - (p - (j - L + 1)) : i + 1 + (p - (j - L + 1)));
+        else src = p <= i + L ? (rev ? j - (p - i - 1) : j - L + 1 + (p - i - 1)) : p - L;
+        span[q] = tour[src];
+    }
+}
+
+__global__ void or_commit_kernel(const int* __restrict__ coords, const int* __restrict__ span, int* __restrict__ tour,
+                                 int2* __restrict__ Q, int n, int i, int j)
+{
+    for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < j - i; q += gridDim.x * blockDim.x) {
+        const int p = i + 1 + q, c = span[q];
+        tour[p] = c;
+        const int2 v = make_int2(coords[2 * c], coords[2 * c + 1]);
+        Q[p] = v;
+        if (p < kOrHalo) Q[n + p] = v;  // the halo copies of positions 1..4
+    }
+}
+
+static int or_grid(long long work, int per_cta, int cap)
+{
+    int sms = 148;
+    int dev = 0;
+    if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const long long need = (work + per_cta - 1) / per_cta;
+    const long long g = std::min<long long>(need, (long long)sms * cap);
+    return (int)std::max<long long>(1, g);
+}
+
+size_t oropt_q_entries(int n) { return (size_t)n + kOrHalo; }
+
+cudaError_t launch_or_load(const int* coords, const int* tour, int2* Q, int n, unsigned long long* len, cudaStream_t st)
+{
+    cudaError_t e = cudaMemsetAsync(len, 0, sizeof(unsigned long long), st);
+    if (e != cudaSuccess) return e;
+    or_gather_kernel<<<or_grid(n + kOrHalo, 256, 4), 256, 0, st>>>(coords, tour, Q, n);
+    or_length_kernel<<<or_grid(n, 256, 4), 256, 0, st>>>(Q, n, len);
+    count_launch(2);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_or_sweep(const int2* Q, int n, unsigned long long* slot, cudaStream_t st)
+{
+    const unsigned long long seed = or_pack(0, 0, 1, 0);
+    cudaError_t e = cudaMemcpyAsync(slot, &seed, sizeof(seed), cudaMemcpyHostToDevice, st);
+    if (e != cudaSuccess) return e;
+    const long long cells = (long long)n * (n - 1) / 2;
+    or_sweep_kernel<<<or_grid(cells, kOrThreads, 8), kOrThreads, 0, st>>>(Q, n, cells, slot);
+    count_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_or_apply(const int* coords, int* tour, int2* Q, int* span, int n, int i, int j, int type,
+                            cudaStream_t st)
+{
+    const int g = or_grid(j - i, 256, 4);
+    or_span_kernel<<<g, 256, 0, st>>>(tour, span, i, j, type);
+    or_commit_kernel<<<g, 256, 0, st>>>(coords, span, tour, Q, n, i, j);
+    count_launch(2);
+    return cudaGetLastError();
+}
+
+void or_unpack(unsigned long long key, int* i, int* j, int* type, int* delta)
+{
+    *delta = (int)(key >> 44) - kDeltaBias;
+    *j = (int)((key >> 24) & 0xFFFFF);
+    *i = (int)((key >> 4) & 0xFFFFF);
+    *type = (int)(key & 0xF);
+}
+
+}  // namespace tsp2opt

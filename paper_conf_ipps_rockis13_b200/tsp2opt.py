@@ -69,6 +69,8 @@ def _L():
             "tsp2opt_batch_local_search_async": ([P, I32, I32, P, I64, P, P, P], I32),
             "tsp2opt_batch_ils": ([P, I32, I32, P, I64, P, P, P], I32),
             "tsp2opt_batch_ils_async": ([P, I32, I32, P, I64, P, P, P, P], I32),
+            "tsp2opt_oropt_local_search": ([P, I32, P, I64, pI64, pI64, P, I64], I32),
+            "tsp2opt_oropt_best_move": ([P, I32, P, pI32, pI32, pI32, pI32], I32),
             "tsp2opt_plan_shard": ([I32, I32, I32, pI32, pI32, pI32, P, I64, pI64, pI64], I32),
             "tsp2opt_get_geometry": ([P, pI32, pI32, pI32, pI64, pI64], I32),
             "tsp2opt_selftest": ([pI64, pI64, pI64, pI64], I32),
@@ -217,6 +219,32 @@ def local_search_current(h, max_iters: int | None = None):
     mi = MAX_ITERS_UNBOUNDED if max_iters is None else int(max_iters)
     st = _check(_L().tsp2opt_local_search(h, None, mi, ctypes.byref(L), ctypes.byref(it)), "tsp2opt_local_search")
     return dict(length=L.value, iterations=it.value, status=st)
+
+
+def oropt_local_search(coords, tour, max_iters: int | None = None, trace_cap: int = 0):
+    """Or-opt local search (reading R21), stateless: coords int32[n, 2], tour int32[n] ->
+    dict(tour, length, iterations, status, trace int32[k, 4] rows (i, j, delta, type))."""
+    xy = _i32(coords)
+    n = xy.shape[0]
+    t = np.array(tour, dtype=np.int32, copy=True).reshape(n)
+    tr = np.zeros((max(trace_cap, 1), 4), dtype=np.int32)
+    L, it = ctypes.c_int64(), ctypes.c_int64()
+    mi = MAX_ITERS_UNBOUNDED if max_iters is None else int(max_iters)
+    st = _check(_L().tsp2opt_oropt_local_search(_ptr(xy), n, _ptr(t), mi, ctypes.byref(L), ctypes.byref(it),
+                                                _ptr(tr) if trace_cap > 0 else None, int(trace_cap)),
+                "tsp2opt_oropt_local_search")
+    return dict(tour=t, length=L.value, iterations=it.value, status=st, trace=tr[: min(it.value, trace_cap)].copy())
+
+
+def oropt_best_move(coords, tour):
+    """(i, j, type, delta) of the best Or-opt move of `tour` (one device sweep)."""
+    xy = _i32(coords)
+    n = xy.shape[0]
+    t = np.ascontiguousarray(tour, dtype=np.int32).reshape(n)
+    i, j, ty, d = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+    _check(_L().tsp2opt_oropt_best_move(_ptr(xy), n, _ptr(t), ctypes.byref(i), ctypes.byref(j), ctypes.byref(ty),
+                                        ctypes.byref(d)), "tsp2opt_oropt_best_move")
+    return i.value, j.value, ty.value, d.value
 
 
 def batch_local_search(coords, tours, max_iters: int | None = None):

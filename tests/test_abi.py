@@ -73,6 +73,23 @@ def test_argument_validation_without_gpu():
     badt[1, 4] = 5
     assert bls(xy2.ctypes.data, 10, 2, badt.ctypes.data, 5, L.ctypes.data, L.ctypes.data) == tsp2opt.ENOTPERM
     assert lib.tsp2opt_strerror(tsp2opt.ENOTPERM) == b"tour is not a permutation of 0..n-1"
+    # Or-opt entries (reading R21): validated on the host before any device work
+    orl, orb = lib.tsp2opt_oropt_local_search, lib.tsp2opt_oropt_best_move
+    t1 = np.arange(10, dtype=np.int32)
+    i32 = ctypes.c_int32()
+    assert orl(None, 10, t1.ctypes.data, 5, None, None, None, 0) == tsp2opt.EINVAL
+    for n in (2, (1 << 20) + 1):
+        assert orl(xy.ctypes.data, n, t1.ctypes.data, 5, None, None, None, 0) == tsp2opt.EINVAL
+    assert orl(xy.ctypes.data, 10, t1.ctypes.data, -1, None, None, None, 0) == tsp2opt.EINVAL
+    assert orl(xy.ctypes.data, 10, t1.ctypes.data, 5, None, None, None, 3) == tsp2opt.EINVAL
+    bad = np.zeros(20, np.int32)
+    bad[3] = 1 << 15
+    assert orl(bad.ctypes.data, 10, t1.ctypes.data, 5, None, None, None, 0) == tsp2opt.ERANGE
+    bt = t1.copy()
+    bt[2] = 3
+    assert orl(xy.ctypes.data, 10, bt.ctypes.data, 5, None, None, None, 0) == tsp2opt.ENOTPERM
+    assert orb(xy.ctypes.data, 10, bt.ctypes.data, *([ctypes.byref(i32)] * 4)) == tsp2opt.ENOTPERM
+    assert orb(xy.ctypes.data, 10, t1.ctypes.data, None, None, None, None) == tsp2opt.EINVAL
 
 
 def test_key_layout_constants_match_header():

@@ -1,0 +1,76 @@
+"""GPU parity of best-improvement Or-opt (tsp2opt_oropt_*; SURVEY.md §8(f)
+NEXT-4 "2.5-opt/Or-opt variants"; L26 §VII; reading R21) against
+oracle.*_or -- bit-exact: (i, j, type, delta) per sweep, the traced moves,
+final tour, length and move count, through the C ABI."""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_ipps_rockis13_b200 import inputs, tsp2opt
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("n", [3, 4, 5, 6, 7, 16, 33, 100, 481, 1002, 2500])
+@pytest.mark.parametrize("kind", ["uniform", "lattice"])
+def test_oropt_best_move_parity(gpu, n, kind):
+    c = inputs.make_coords(kind, n, 7)
+    for t in (inputs.random_tour(n, 7), inputs.random_tour(n, 8), inputs.hilbert_tour(c)):
+        assert tsp2opt.oropt_best_move(c, t) == oracle.best_move_or(c, t)
+
+
+def test_oropt_best_move_c3_sized(gpu):
+    n = 7397  # pla7397-shaped: several thousand CTAs of cells and the 2^20-bit key fields
+    c = inputs.make_coords("lattice", n, 1)
+    for t in (inputs.random_tour(n, 1), inputs.hilbert_tour(c)):
+        assert tsp2opt.oropt_best_move(c, t) == oracle.best_move_or(c, t)
+
+
+@pytest.mark.parametrize("kind,n,seed", [("uniform", 8, 1), ("uniform", 50, 2), ("lattice", 100, 1),
+                                         ("uniform", 100, 3), ("lattice", 257, 2), ("uniform", 300, 4)])
+def test_oropt_local_search_parity(gpu, kind, n, seed):
+    c = inputs.make_coords(kind, n, seed)
+    t0 = inputs.random_tour(n, seed)
+    ref = oracle.local_search_or(c, t0, trace_cap=100_000)
+    got = tsp2opt.oropt_local_search(c, t0, trace_cap=100_000)
+    assert got["status"] == ref["status"] == 0
+    assert got["iterations"] == ref["iterations"]
+    assert got["length"] == ref["length"]
+    assert np.array_equal(got["tour"], ref["tour"])
+    assert np.array_equal(got["trace"].astype(np.int64), ref["trace"])
+
+
+def test_oropt_duplicates_and_collinear(gpu):
+    dup = inputs.make_coords("uniform", 40, 4)
+    dup[5] = dup[2]
+    dup[17] = dup[2]
+    line = np.array([[53 * k % 900, 7] for k in range(41)], dtype=np.int32)
+    for c in (dup, line):
+        t0 = inputs.random_tour(len(c), 6)
+        ref = oracle.local_search_or(c, t0)
+        got = tsp2opt.oropt_local_search(c, t0)
+        assert (got["length"], got["iterations"]) == (ref["length"], ref["iterations"])
+        assert np.array_equal(got["tour"], ref["tour"])
+
+
+def test_oropt_max_iters(gpu):
+    c = inputs.make_coords("uniform", 120, 5)
+    t0 = inputs.random_tour(120, 5)
+    for cap in (0, 1, 9):
+        ref = oracle.local_search_or(c, t0, max_iters=cap)
+        got = tsp2opt.oropt_local_search(c, t0, max_iters=cap)
+        assert got["status"] == ref["status"] == 1
+        assert got["iterations"] == cap and got["length"] == ref["length"]
+        assert np.array_equal(got["tour"], ref["tour"])
+
+
+def test_oropt_local_search_c2_hilbert(gpu):
+    # pr1002-shaped from the Hilbert start: full trace parity at a size spanning many CTAs
+    n = 1002
+    c = inputs.make_coords("uniform", n, 1)
+    t0 = inputs.hilbert_tour(c)
+    ref = oracle.local_search_or(c, t0, trace_cap=100_000)
+    got = tsp2opt.oropt_local_search(c, t0, trace_cap=100_000)
+    assert (got["status"], got["iterations"], got["length"]) == (ref["status"], ref["iterations"], ref["length"])
+    assert np.array_equal(got["tour"], ref["tour"])
+    assert np.array_equal(got["trace"].astype(np.int64), ref["trace"])
