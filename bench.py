@@ -215,12 +215,13 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms, sweep_avg_ms, e2e_total, tb_total_ms, tb_sweep_ms = t.tolist()
 
-    ls = ils = batch = batch_ils = pruned = or25 = first = None
+    ls = ils = batch = batch_ils = pruned = or25 = first = oropt = None
     if rank == 0 and world == 1 and not args.no_ls:
         ls = time_to_local_min(tsp2opt, args.ls_config)
         pruned = time_pruned(tsp2opt, args.pruned_config, not args.no_cpu) if args.pruned_config else None
         or25 = time_25opt(tsp2opt, args.or25_config, not args.no_cpu) if args.or25_config else None
         first = time_first(tsp2opt, args.first_config) if args.first_config else None
+        oropt = time_oropt(tsp2opt, args.oropt_config, not args.no_cpu) if args.oropt_config else None
         ils = time_ils(tsp2opt, args.ils_config) if args.ils_config else None
         batch = time_batch(tsp2opt, args.batch_config, not args.no_cpu) if args.batch_config else None
         batch_ils = time_batch_ils(tsp2opt, args.batch_ils_config, not args.no_cpu) if args.batch_ils_config else None
@@ -277,6 +278,8 @@ def run_ours(args):
             line["local_search_25opt"] = or25
         if first:
             line["local_search_first_improvement"] = first
+        if oropt:
+            line["local_search_oropt"] = oropt
         if batch:
             line["batch_local_search"] = batch
         if batch_ils:
@@ -448,6 +451,42 @@ def time_25opt(tsp2opt, spec, with_oracle=True):
             entry["cpu_oracle"] = {"sweep_seconds": per, "est_ls_seconds": per * (r["iterations"] + 1),
                                    "cores": oracle.num_threads(), "kind": "oracle",
                                    "sample": f"{reps} oracle 2.5-opt sweeps of the MF tour; the local search "
+                                             "estimate is per-sweep time x (moves + 1)"}
+        out.append(entry)
+    return out
+
+
+def time_oropt(tsp2opt, spec, with_oracle=True):
+    """Best-improvement Or-opt (tsp2opt_oropt_local_search; SURVEY §8(f) NEXT-4
+    "2.5-opt/Or-opt variants"; reading R21), `cfg` (random start) or
+    `cfg:hilbert` entries: wall time of the stateless C-ABI call, host tour in
+    and out, with the oracle's per-sweep time on the start tour beside it."""
+    out = []
+    for item in spec.split(","):
+        if not item:
+            continue
+        name, _, tk = item.partition(":")
+        coords, tour = inputs.config_instance(name, tk or "random")
+        n = len(coords)
+        tsp2opt.oropt_local_search(coords, tour, max_iters=2)  # warm-up
+        t0 = time.perf_counter()
+        r = tsp2opt.oropt_local_search(coords, tour)
+        sec = time.perf_counter() - t0
+        cells = n * (n - 1) // 2
+        entry = {"config": name, "n": n, "start": tk or "random", "moves": "2-opt + Or-opt segments of 1..3 cities",
+                 "seconds": sec, "iterations": r["iterations"], "length": r["length"],
+                 "s_per_iteration": sec / (r["iterations"] + 1),
+                 "pair_checks_per_s": cells * (r["iterations"] + 1) / sec, "moves_per_pair": 13}
+        if with_oracle and n <= 20000:
+            import oracle
+            reps = 3 if n > 5000 else 10
+            o0 = time.perf_counter()
+            for _ in range(reps):
+                oracle.best_move_or(coords, tour)
+            per = (time.perf_counter() - o0) / reps
+            entry["cpu_oracle"] = {"sweep_seconds": per, "est_ls_seconds": per * (r["iterations"] + 1),
+                                   "cores": oracle.num_threads(), "kind": "oracle",
+                                   "sample": f"{reps} oracle Or-opt sweeps of the start tour; the local search "
                                              "estimate is per-sweep time x (moves + 1)"}
         out.append(entry)
     return out
@@ -672,6 +711,7 @@ def main():
     ap.add_argument("--ils-config", default="C1:200,C2:50", help="Iterated Local Search runs cfg:iterations")
     ap.add_argument("--pruned-config", default="C3:8,C4:8,C5:8,C5:16", help="pruned 2-opt from MF, cfg:K")
     ap.add_argument("--or25-config", default="C3,C4,C5", help="2.5-opt local search from MF, configs")
+    ap.add_argument("--oropt-config", default="C1,C2,C3:hilbert", help="Or-opt local search, cfg[:hilbert]")
     ap.add_argument("--first-config", default="C1,C2,C3:mf,C4:mf,C5:mf", help="first-improvement local search")
     ap.add_argument("--batch-config", default="100:4736,1002:592", help="batched local search n:instances")
     ap.add_argument("--batch-ils-config", default="C1:4736:100", help="batched ILS cfg:replicas:steps")

@@ -37,6 +37,12 @@
  *                        operations on city ids; the neighbourhood as a set of
  *                        cycles == 2-opt neighbours + node insertions; the
  *                        sweep == the per-move definition; global optima.
+ *   oracleor_* (tests/test_oracle_oropt.py) -- Or-opt (reading R21): brute
+ *                        force over neighbours built from the move's wording
+ *                        (cut a segment of L cities, insert it after a city);
+ *                        the neighbourhood as a set of cycles == 2-opt
+ *                        neighbours + all segment moves; L = 1 == 2.5-opt's
+ *                        insertions; the optimum admits no improving move.
  *   oracle_first_* (tests/test_oracle_first.py) -- first improvement: the
  *                        first improving neighbour of an explicit scan in cell
  *                        order; 2-opt local-minimum certificate.
