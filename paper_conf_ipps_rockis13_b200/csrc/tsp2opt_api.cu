@@ -1234,8 +1234,10 @@ int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters
     int* d_t = nullptr;
     int* d_span = nullptr;
     int2* d_q = nullptr;
+    int4* d_c = nullptr;  // per-position sweep constants CR | CC
     unsigned long long* d_slot = nullptr;  // [0] key, [1] length
     auto cleanup = [&]() {
+        cudaFree(d_c);
         cudaFree(d_xy);
         cudaFree(d_t);
         cudaFree(d_span);
@@ -1253,6 +1255,7 @@ int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters
     if ((e = cudaMalloc(&d_span, nb)) != cudaSuccess) return fail(e, "cudaMalloc");
     if ((e = cudaMalloc(&d_q, sizeof(int2) * oropt_q_entries(n))) != cudaSuccess) return fail(e, "cudaMalloc");
     if ((e = cudaMalloc(&d_slot, 2 * sizeof(unsigned long long))) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMalloc(&d_c, 2 * sizeof(int4) * oropt_const_entries(n))) != cudaSuccess) return fail(e, "cudaMalloc");
     if ((e = cudaMemcpy(d_xy, coords_xy, 2 * nb, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "H2D");
     if ((e = cudaMemcpy(d_t, tour, nb, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "H2D");
     if ((e = launch_or_load(d_xy, d_t, d_q, n, d_slot + 1, nullptr)) != cudaSuccess) return fail(e, "or_load");
@@ -1261,7 +1264,7 @@ int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters
     long long L = (long long)len, it = 0;
     int status = TSP2OPT_OK;
     for (;;) {
-        if ((e = launch_or_sweep(d_q, n, d_slot, nullptr)) != cudaSuccess) return fail(e, "or_sweep_kernel");
+        if ((e = launch_or_sweep(d_q, d_c, d_c + oropt_const_entries(n), n, d_slot, nullptr)) != cudaSuccess) return fail(e, "or_sweep_kernel");
         unsigned long long key = 0;
         if ((e = cudaMemcpy(&key, d_slot, sizeof(key), cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
         if (first_key && it == 0) *first_key = key;

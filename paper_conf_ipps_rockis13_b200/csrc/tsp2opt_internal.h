@@ -88,7 +88,8 @@ cudaError_t launch_apply25(float2* P, int* E, int* G, int* tour, int n, const Sl
 // Or-opt (tsp2opt_oropt.cu; reading R21): route-ordered int2 Q[n + 5], dense sweep, span apply.
 size_t oropt_q_entries(int n);
 cudaError_t launch_or_load(const int* coords, const int* tour, int2* Q, int n, unsigned long long* len, cudaStream_t st);
-cudaError_t launch_or_sweep(const int2* Q, int n, unsigned long long* slot, cudaStream_t st);
+size_t oropt_const_entries(int n);
+cudaError_t launch_or_sweep(const int2* Q, int4* CR, int4* CC, int n, unsigned long long* slot, cudaStream_t st);
 cudaError_t launch_or_apply(const int* coords, int* tour, int2* Q, int* span, int n, int i, int j, int type,
                             cudaStream_t st);
 void or_unpack(unsigned long long key, int* i, int* j, int* type, int* delta);

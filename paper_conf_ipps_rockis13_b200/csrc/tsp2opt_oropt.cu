@@ -16,6 +16,9 @@
 // per GPU with one 64-bit atomicMin.  Distances are the exact EUC_2D nint of
 // tsp2opt_device.cuh.  The apply writes positions i+1..j in their new order
 // into a scratch span, then copies it back (two launches, no grid barrier).
+#include <climits>
+#include <cstdlib>
+
 #include "tsp2opt_internal.h"
 
 namespace tsp2opt {
@@ -103,6 +106,122 @@ __global__ void __launch_bounds__(kOrThreads) or_sweep_kernel(const int2* __rest
     }
 }
 
+// Per-position constants of the tiled sweep, rebuilt before every sweep (O(n)):
+//   CR[p] = (e_p, rf_1, rf_2, rf_3) with rf_L = d(t_p, t_{p+L+1}) - e_p - d(t_{p+L}, t_{p+L+1})
+//           (the row part of a forward move's removal gain);
+//   CC[p] = (e_p, rb_1, rb_2, rb_3) with rb_L = d(t_{p-L}, t_{p+1}) - d(t_{p-L}, t_{p-L+1}) - e_p
+//           (the column part of a backward move's removal gain; p - L >= 0 only is ever read).
+__global__ void or_consts_kernel(const int2* __restrict__ Q, int n, int4* __restrict__ CR, int4* __restrict__ CC)
+{
+    for (int p = blockIdx.x * blockDim.x + threadIdx.x; p < n; p += gridDim.x * blockDim.x) {
+        const int e = or_d(Q[p], Q[p + 1]);
+        int rf[3], rb[3];
+#pragma unroll
+        for (int L = 1; L <= 3; L++) {
+            rf[L - 1] = or_d(Q[p], Q[p + L + 1]) - e - or_d(Q[p + L], Q[p + L + 1]);
+            rb[L - 1] = p - L >= 0 ? or_d(Q[p - L], Q[p + 1]) - or_d(Q[p - L], Q[p - L + 1]) - e : 0;
+        }
+        CR[p] = make_int4(e, rf[0], rf[1], rf[2]);
+        CC[p] = make_int4(e, rb[0], rb[1], rb[2]);
+    }
+}
+
+constexpr int kOrTileI = 256;  // rows per tile = threads per CTA (one row city per thread)
+constexpr int kOrTileJ = 256;  // columns per tile
+
+// Tiled sweep: CTA = one (row block, column block) tile of the upper triangle,
+// thread = row i, walking the tile's columns j in increasing order.  Every
+// distance of a pair's 13 moves is d(t_{i+r}, t_c) for r in 0..3 and c in
+// j-2..j+1 (or a per-position constant), so a 4 x 4 register window slides
+// along j and each column step computes only the 4 distances to t_{j+1}.
+// The thread keeps its lowest (delta, cell, type): per pair the min of
+// delta << 4 | type (lowest type among equal deltas), replacing the thread's
+// best only on a strictly lower delta (cells increase along the walk).
+__global__ void __launch_bounds__(kOrTileI) or_tile_kernel(const int2* __restrict__ Q, const int4* __restrict__ CR,
+                                                           const int4* __restrict__ CC, int n, int nbj,
+                                                           unsigned long long* slot)
+{
+    // tile t -> (ib <= jb) over the upper triangle of blocks, t = jb(jb+1)/2 + ib
+    const int t = blockIdx.x;
+    int jb = (int)((sqrtf(8.0f * (float)t + 1.0f) - 1.0f) * 0.5f);
+    while (jb * (jb + 1) / 2 > t) jb--;
+    while ((jb + 1) * (jb + 2) / 2 <= t) jb++;
+    const int ib = t - jb * (jb + 1) / 2;
+    const int i = ib * kOrTileI + threadIdx.x;
+    const int j0 = max(jb * kOrTileJ, i + 1), j1 = min(n, (jb + 1) * kOrTileJ);
+    int best = INT_MAX, bj = 0, bt = 0;  // best delta, its column and type
+    if (i < n - 1 && j0 < j1) {
+        const int2 r0 = Q[i], r1 = Q[i + 1], r2 = Q[i + 2], r3 = Q[i + 3];
+        const int4 cr = CR[i];
+        // window D[r][k]: d(t_{i+r}, t_{j-2+k}), k = 0..3 (columns j-2, j-1, j, j+1); columns < 0 are never read
+        int D0[4], D1[4], D2[4], D3[4];
+#pragma unroll
+        for (int k = 0; k < 3; k++) {
+            const int2 c = Q[max(0, j0 - 2 + k)];
+            D0[k + 1] = or_d(r0, c);
+            D1[k + 1] = or_d(r1, c);
+            D2[k + 1] = or_d(r2, c);
+            D3[k + 1] = or_d(r3, c);
+        }
+        for (int j = j0; j < j1; j++) {
+#pragma unroll
+            for (int k = 0; k < 3; k++) {
+                D0[k] = D0[k + 1];
+                D1[k] = D1[k + 1];
+                D2[k] = D2[k + 1];
+                D3[k] = D3[k + 1];
+            }
+            const int2 c = Q[j + 1];
+            D0[3] = or_d(r0, c);
+            D1[3] = or_d(r1, c);
+            D2[3] = or_d(r2, c);
+            D3[3] = or_d(r3, c);
+            const int4 cc = CC[j];
+            const int base = -cr.x - cc.x;
+            int v = (D0[2] + D1[3] + base) * 16;  // type 0
+            const int gap = j - i;                // moves of length L need gap >= L + 1
+            // forward L: rf_L - e_j + d(t_j, a) + d(b, t_{j+1}); a, b = t_{i+1}, t_{i+L} (rev: swapped)
+            // backward L: rb_L - e_i + d(t_i, a) + d(b, t_{i+1}); a, b = t_{j-L+1}, t_j (rev: swapped)
+            if (gap >= 2) {
+                const int f = cr.y - cc.x, b = cc.y - cr.x;
+                v = min(v, (f + D1[2] + D1[3]) * 16 + 1);
+                v = min(v, (b + D0[2] + D1[2]) * 16 + 3);
+            }
+            if (gap >= 3) {
+                const int f = cr.z - cc.x, b = cc.z - cr.x;
+                v = min(v, (f + D1[2] + D2[3]) * 16 + 5);
+                v = min(v, (f + D2[2] + D1[3]) * 16 + 6);
+                v = min(v, (b + D0[1] + D1[2]) * 16 + 7);
+                v = min(v, (b + D0[2] + D1[1]) * 16 + 8);
+            }
+            if (gap >= 4) {
+                const int f = cr.w - cc.x, b = cc.w - cr.x;
+                v = min(v, (f + D1[2] + D3[3]) * 16 + 9);
+                v = min(v, (f + D3[2] + D1[3]) * 16 + 10);
+                v = min(v, (b + D0[0] + D1[2]) * 16 + 11);
+                v = min(v, (b + D0[2] + D1[0]) * 16 + 12);
+            }
+            if ((v >> 4) < best) {
+                best = v >> 4;
+                bt = v & 15;
+                bj = j;
+            }
+        }
+    }
+    unsigned long long key = best < 0 ? or_pack(best, i, bj, bt) : or_pack(0, 0, 1, 0);
+    for (int o = 16; o; o >>= 1) {
+        const unsigned long long other = __shfl_xor_sync(0xffffffffu, key, o);
+        key = other < key ? other : key;
+    }
+    __shared__ unsigned long long red[kOrTileI / 32];
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = key;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int w = 1; w < kOrTileI / 32; w++) key = red[w] < key ? red[w] : key;
+        if (key < or_pack(0, 0, 1, 0)) atomicMin(slot, key);
+    }
+}
+
 // span[p - i - 1] = the tour city that lands on position p in [i+1, j] (oracleor_apply's order)
 __global__ void or_span_kernel(const int* __restrict__ tour, int* __restrict__ span, int i, int j, int type)
 {
@@ -152,14 +271,33 @@ cudaError_t launch_or_load(const int* coords, const int* tour, int2* Q, int n, u
     return cudaGetLastError();
 }
 
-cudaError_t launch_or_sweep(const int2* Q, int n, unsigned long long* slot, cudaStream_t st)
+static bool or_naive()
+{
+    static const bool v = [] {
+        const char* s = getenv("TSP2OPT_OROPT_NAIVE");
+        return s && s[0] == '1';
+    }();
+    return v;
+}
+
+size_t oropt_const_entries(int n) { return (size_t)n; }
+
+cudaError_t launch_or_sweep(const int2* Q, int4* CR, int4* CC, int n, unsigned long long* slot, cudaStream_t st)
 {
     const unsigned long long seed = or_pack(0, 0, 1, 0);
     cudaError_t e = cudaMemcpyAsync(slot, &seed, sizeof(seed), cudaMemcpyHostToDevice, st);
     if (e != cudaSuccess) return e;
-    const long long cells = (long long)n * (n - 1) / 2;
-    or_sweep_kernel<<<or_grid(cells, kOrThreads, 8), kOrThreads, 0, st>>>(Q, n, cells, slot);
-    count_launch();
+    if (or_naive()) {  // TSP2OPT_OROPT_NAIVE=1: the one-thread-per-cell kernel (experiment switch, same result)
+        const long long cells = (long long)n * (n - 1) / 2;
+        or_sweep_kernel<<<or_grid(cells, kOrThreads, 8), kOrThreads, 0, st>>>(Q, n, cells, slot);
+        count_launch();
+        return cudaGetLastError();
+    }
+    or_consts_kernel<<<or_grid(n, 256, 4), 256, 0, st>>>(Q, n, CR, CC);
+    const int nbj = (n + kOrTileJ - 1) / kOrTileJ;  // kOrTileI == kOrTileJ: row block b covers column block b
+    const long long tiles = (long long)nbj * (nbj + 1) / 2;
+    or_tile_kernel<<<(unsigned)tiles, kOrTileI, 0, st>>>(Q, CR, CC, n, nbj, slot);
+    count_launch(2);
     return cudaGetLastError();
 }
 
