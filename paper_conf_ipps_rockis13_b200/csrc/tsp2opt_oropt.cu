@@ -126,10 +126,18 @@ __global__ void or_consts_kernel(const int2* __restrict__ Q, int n, int4* __rest
     }
 }
 
-constexpr int kOrTileI = 256;  // rows per tile = threads per CTA (one row city per thread)
-constexpr int kOrTileJ = 256;  // columns per tile
+constexpr int kOrMaxTI = 256;  // rows per tile = threads per CTA (one row city per thread), upper bound
 
-// Tiled sweep: CTA = one (row block, column block) tile of the upper triangle,
+// Tile geometry by size: enough CTAs to fill 148 SMs at small n, long column
+// walks (few window warm-ups) at large n.
+static void or_tiles(int n, int* ti, int* tj)
+{
+    if (n <= 2048) { *ti = 64; *tj = 16; }
+    else if (n <= 16384) { *ti = 128; *tj = 32; }
+    else { *ti = 256; *tj = 128; }
+}
+
+// Tiled sweep: CTA = one (row block blockIdx.y, column chunk blockIdx.x) tile,
 // thread = row i, walking the tile's columns j in increasing order.  Every
 // distance of a pair's 13 moves is d(t_{i+r}, t_c) for r in 0..3 and c in
 // j-2..j+1 (or a per-position constant), so a 4 x 4 register window slides
@@ -137,18 +145,15 @@ constexpr int kOrTileJ = 256;  // columns per tile
 // The thread keeps its lowest (delta, cell, type): per pair the min of
 // delta << 4 | type (lowest type among equal deltas), replacing the thread's
 // best only on a strictly lower delta (cells increase along the walk).
-__global__ void __launch_bounds__(kOrTileI) or_tile_kernel(const int2* __restrict__ Q, const int4* __restrict__ CR,
-                                                           const int4* __restrict__ CC, int n, int nbj,
+__global__ void __launch_bounds__(kOrMaxTI) or_tile_kernel(const int2* __restrict__ Q, const int4* __restrict__ CR,
+                                                           const int4* __restrict__ CC, int n, int tj,
                                                            unsigned long long* slot)
 {
-    // tile t -> (ib <= jb) over the upper triangle of blocks, t = jb(jb+1)/2 + ib
-    const int t = blockIdx.x;
-    int jb = (int)((sqrtf(8.0f * (float)t + 1.0f) - 1.0f) * 0.5f);
-    while (jb * (jb + 1) / 2 > t) jb--;
-    while ((jb + 1) * (jb + 2) / 2 <= t) jb++;
-    const int ib = t - jb * (jb + 1) / 2;
-    const int i = ib * kOrTileI + threadIdx.x;
-    const int j0 = max(jb * kOrTileJ, i + 1), j1 = min(n, (jb + 1) * kOrTileJ);
+    const int ti = blockDim.x;
+    const int row0 = blockIdx.y * ti, col1 = (blockIdx.x + 1) * tj;
+    if (col1 - 1 <= row0) return;  // below the diagonal: no pair i < j (uniform over the CTA)
+    const int i = row0 + threadIdx.x;
+    const int j0 = max(blockIdx.x * tj, i + 1), j1 = min(n, col1);
     int best = INT_MAX, bj = 0, bt = 0;  // best delta, its column and type
     if (i < n - 1 && j0 < j1) {
         const int2 r0 = Q[i], r1 = Q[i + 1], r2 = Q[i + 2], r3 = Q[i + 3];
@@ -213,11 +218,11 @@ __global__ void __launch_bounds__(kOrTileI) or_tile_kernel(const int2* __restric
         const unsigned long long other = __shfl_xor_sync(0xffffffffu, key, o);
         key = other < key ? other : key;
     }
-    __shared__ unsigned long long red[kOrTileI / 32];
+    __shared__ unsigned long long red[kOrMaxTI / 32];
     if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = key;
     __syncthreads();
     if (threadIdx.x == 0) {
-        for (int w = 1; w < kOrTileI / 32; w++) key = red[w] < key ? red[w] : key;
+        for (int w = 1; w < (int)(blockDim.x >> 5); w++) key = red[w] < key ? red[w] : key;
         if (key < or_pack(0, 0, 1, 0)) atomicMin(slot, key);
     }
 }
@@ -294,9 +299,10 @@ cudaError_t launch_or_sweep(const int2* Q, int4* CR, int4* CC, int n, unsigned l
         return cudaGetLastError();
     }
     or_consts_kernel<<<or_grid(n, 256, 4), 256, 0, st>>>(Q, n, CR, CC);
-    const int nbj = (n + kOrTileJ - 1) / kOrTileJ;  // kOrTileI == kOrTileJ: row block b covers column block b
-    const long long tiles = (long long)nbj * (nbj + 1) / 2;
-    or_tile_kernel<<<(unsigned)tiles, kOrTileI, 0, st>>>(Q, CR, CC, n, nbj, slot);
+    int ti, tj;
+    or_tiles(n, &ti, &tj);
+    const dim3 grid((n + tj - 1) / tj, (n + ti - 1) / ti);
+    or_tile_kernel<<<grid, ti, 0, st>>>(Q, CR, CC, n, tj, slot);
     count_launch(2);
     return cudaGetLastError();
 }
