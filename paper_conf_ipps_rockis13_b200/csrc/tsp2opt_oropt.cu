@@ -137,6 +137,71 @@ static void or_tiles(int n, int* ti, int* tj)
     else { *ti = 256; *tj = 128; }
 }
 
+// The 13 moves of pair (i, j) from the window D_r[k] = d(t_{i+r}, t_{j-2+k})
+// (columns j-2, j-1, j, j+1) and the per-position constants: min over the
+// valid types of delta * 16 + type.
+//   forward L:  rf_L - e_j + d(t_j, a) + d(b, t_{j+1}); a, b = t_{i+1}, t_{i+L} (rev: swapped)
+//   backward L: rb_L - e_i + d(t_i, a) + d(b, t_{i+1}); a, b = t_{j-L+1}, t_j (rev: swapped)
+// (moves of length L need gap = j - i >= L + 1; the L = 1 reversed types
+// duplicate types 1 and 3 and never win the type tie-break.)
+__device__ __forceinline__ int or_eval_exact(const int* D0, const int* D1, const int* D2, const int* D3, int4 cr,
+                                             int4 cc, int gap)
+{
+    int v = (D0[2] + D1[3] - cr.x - cc.x) * 16;  // type 0
+    if (gap >= 2) {
+        const int f = cr.y - cc.x, b = cc.y - cr.x;
+        v = min(v, (f + D1[2] + D1[3]) * 16 + 1);
+        v = min(v, (b + D0[2] + D1[2]) * 16 + 3);
+    }
+    if (gap >= 3) {
+        const int f = cr.z - cc.x, b = cc.z - cr.x;
+        v = min(v, (f + D1[2] + D2[3]) * 16 + 5);
+        v = min(v, (f + D2[2] + D1[3]) * 16 + 6);
+        v = min(v, (b + D0[1] + D1[2]) * 16 + 7);
+        v = min(v, (b + D0[2] + D1[1]) * 16 + 8);
+    }
+    if (gap >= 4) {
+        const int f = cr.w - cc.x, b = cc.w - cr.x;
+        v = min(v, (f + D1[2] + D3[3]) * 16 + 9);
+        v = min(v, (f + D3[2] + D1[3]) * 16 + 10);
+        v = min(v, (b + D0[0] + D1[2]) * 16 + 11);
+        v = min(v, (b + D0[2] + D1[0]) * 16 + 12);
+    }
+    return v;
+}
+
+// The same minimum over the types in FP32 from approximate distances
+// sqrt_approx(s_f), without the type.  Each distance is within 0.53 of its
+// nint (0.5 rounding + 0.03 MUFU / s_f error, tsp2opt_selftest_sqrt), a move
+// has two varying distances, and the three FP32 additions of values below
+// 2^18 round by at most 0.05, so every exact delta is >= this value - 1.11.
+__device__ __forceinline__ float or_eval_float(const float* F0, const float* F1, const float* F2, const float* F3,
+                                               int4 cr, int4 cc, int gap)
+{
+    float m = F0[2] + F1[3] + (float)(-cr.x - cc.x);
+    if (gap >= 2) {
+        const float f = (float)(cr.y - cc.x), b = (float)(cc.y - cr.x);
+        m = fminf(m, fminf(f + (F1[2] + F1[3]), b + (F0[2] + F1[2])));
+    }
+    if (gap >= 3) {
+        const float f = (float)(cr.z - cc.x), b = (float)(cc.z - cr.x);
+        m = fminf(m, fminf(f + fminf(F1[2] + F2[3], F2[2] + F1[3]), b + fminf(F0[1] + F1[2], F0[2] + F1[1])));
+    }
+    if (gap >= 4) {
+        const float f = (float)(cr.w - cc.x), b = (float)(cc.w - cr.x);
+        m = fminf(m, fminf(f + fminf(F1[2] + F3[3], F3[2] + F1[3]), b + fminf(F0[0] + F1[2], F0[2] + F1[0])));
+    }
+    return m;
+}
+
+constexpr float kOrSlack = 1.25f;  // > 1.11: a pair can beat `best` only if its float minimum <= best - 1 + kOrSlack
+
+__device__ __forceinline__ float or_df(float2 a, float2 b)
+{
+    const float dx = a.x - b.x, dy = a.y - b.y;
+    return sqrt_approx(fmaf(dx, dx, dy * dy));
+}
+
 // Tiled sweep: CTA = one (row block blockIdx.y, column chunk blockIdx.x) tile,
 // thread = row i, walking the tile's columns j in increasing order.  Every
 // distance of a pair's 13 moves is d(t_{i+r}, t_c) for r in 0..3 and c in
@@ -145,6 +210,10 @@ static void or_tiles(int n, int* ti, int* tj)
 // The thread keeps its lowest (delta, cell, type): per pair the min of
 // delta << 4 | type (lowest type among equal deltas), replacing the thread's
 // best only on a strictly lower delta (cells increase along the walk).
+// FILTER: the window holds FP32 approximate distances; a pair is evaluated
+// exactly (12 exact distances from the coordinates) only when its FP32
+// minimum can beat the thread's best (or_eval_float's bound).
+template <bool FILTER>
 __global__ void __launch_bounds__(kOrMaxTI) or_tile_kernel(const int2* __restrict__ Q, const int4* __restrict__ CR,
                                                            const int4* __restrict__ CC, int n, int tj,
                                                            unsigned long long* slot)
@@ -154,8 +223,62 @@ __global__ void __launch_bounds__(kOrMaxTI) or_tile_kernel(const int2* __restric
     if (col1 - 1 <= row0) return;  // below the diagonal: no pair i < j (uniform over the CTA)
     const int i = row0 + threadIdx.x;
     const int j0 = max(blockIdx.x * tj, i + 1), j1 = min(n, col1);
-    int best = INT_MAX, bj = 0, bt = 0;  // best delta, its column and type
-    if (i < n - 1 && j0 < j1) {
+    // Seed the thread's bound with the sweep's best so far (other CTAs'
+    // atomicMin): only pairs with delta <= that delta can still win, and an
+    // equal delta may win on a lower cell, so the bound is one above it.
+    const int gd = (int)(*(volatile const unsigned long long*)slot >> 44) - kDeltaBias;
+    int best = gd < 0 ? gd + 1 : 0, bj = 0, bt = 0;  // record a pair iff its delta < best; its column and type
+    if (FILTER && i < n - 1 && j0 < j1) {
+        const int2 r0 = Q[i], r1 = Q[i + 1], r2 = Q[i + 2], r3 = Q[i + 3];
+        const float2 g0 = make_float2(r0.x, r0.y), g1 = make_float2(r1.x, r1.y), g2 = make_float2(r2.x, r2.y),
+                     g3 = make_float2(r3.x, r3.y);
+        const int4 cr = CR[i];
+        float F0[4], F1[4], F2[4], F3[4];
+#pragma unroll
+        for (int k = 0; k < 3; k++) {
+            const int2 q = Q[max(0, j0 - 2 + k)];
+            const float2 c = make_float2(q.x, q.y);
+            F0[k + 1] = or_df(g0, c);
+            F1[k + 1] = or_df(g1, c);
+            F2[k + 1] = or_df(g2, c);
+            F3[k + 1] = or_df(g3, c);
+        }
+        for (int j = j0; j < j1; j++) {
+#pragma unroll
+            for (int k = 0; k < 3; k++) {
+                F0[k] = F0[k + 1];
+                F1[k] = F1[k + 1];
+                F2[k] = F2[k + 1];
+                F3[k] = F3[k + 1];
+            }
+            const int2 q = Q[j + 1];
+            const float2 c = make_float2(q.x, q.y);
+            F0[3] = or_df(g0, c);
+            F1[3] = or_df(g1, c);
+            F2[3] = or_df(g2, c);
+            F3[3] = or_df(g3, c);
+            const int4 cc = CC[j];
+            const int gap = j - i;
+            if (or_eval_float(F0, F1, F2, F3, cr, cc, gap) <= (float)(best - 1) + kOrSlack) {
+                int D0[4], D1[4], D2[4], D3[4];
+#pragma unroll
+                for (int k = 0; k < 4; k++) {
+                    const int2 w = Q[max(0, j - 2 + k)];
+                    D0[k] = or_d(r0, w);
+                    D1[k] = or_d(r1, w);
+                    D2[k] = or_d(r2, w);
+                    D3[k] = or_d(r3, w);
+                }
+                const int v = or_eval_exact(D0, D1, D2, D3, cr, cc, gap);
+                if ((v >> 4) < best) {
+                    best = v >> 4;
+                    bt = v & 15;
+                    bj = j;
+                }
+            }
+        }
+    }
+    if (!FILTER && i < n - 1 && j0 < j1) {
         const int2 r0 = Q[i], r1 = Q[i + 1], r2 = Q[i + 2], r3 = Q[i + 3];
         const int4 cr = CR[i];
         // window D[r][k]: d(t_{i+r}, t_{j-2+k}), k = 0..3 (columns j-2, j-1, j, j+1); columns < 0 are never read
@@ -181,31 +304,7 @@ __global__ void __launch_bounds__(kOrMaxTI) or_tile_kernel(const int2* __restric
             D1[3] = or_d(r1, c);
             D2[3] = or_d(r2, c);
             D3[3] = or_d(r3, c);
-            const int4 cc = CC[j];
-            const int base = -cr.x - cc.x;
-            int v = (D0[2] + D1[3] + base) * 16;  // type 0
-            const int gap = j - i;                // moves of length L need gap >= L + 1
-            // forward L: rf_L - e_j + d(t_j, a) + d(b, t_{j+1}); a, b = t_{i+1}, t_{i+L} (rev: swapped)
-            // backward L: rb_L - e_i + d(t_i, a) + d(b, t_{i+1}); a, b = t_{j-L+1}, t_j (rev: swapped)
-            if (gap >= 2) {
-                const int f = cr.y - cc.x, b = cc.y - cr.x;
-                v = min(v, (f + D1[2] + D1[3]) * 16 + 1);
-                v = min(v, (b + D0[2] + D1[2]) * 16 + 3);
-            }
-            if (gap >= 3) {
-                const int f = cr.z - cc.x, b = cc.z - cr.x;
-                v = min(v, (f + D1[2] + D2[3]) * 16 + 5);
-                v = min(v, (f + D2[2] + D1[3]) * 16 + 6);
-                v = min(v, (b + D0[1] + D1[2]) * 16 + 7);
-                v = min(v, (b + D0[2] + D1[1]) * 16 + 8);
-            }
-            if (gap >= 4) {
-                const int f = cr.w - cc.x, b = cc.w - cr.x;
-                v = min(v, (f + D1[2] + D3[3]) * 16 + 9);
-                v = min(v, (f + D3[2] + D1[3]) * 16 + 10);
-                v = min(v, (b + D0[0] + D1[2]) * 16 + 11);
-                v = min(v, (b + D0[2] + D1[0]) * 16 + 12);
-            }
+            const int v = or_eval_exact(D0, D1, D2, D3, CR[i], CC[j], j - i);
             if ((v >> 4) < best) {
                 best = v >> 4;
                 bt = v & 15;
@@ -213,7 +312,7 @@ __global__ void __launch_bounds__(kOrMaxTI) or_tile_kernel(const int2* __restric
             }
         }
     }
-    unsigned long long key = best < 0 ? or_pack(best, i, bj, bt) : or_pack(0, 0, 1, 0);
+    unsigned long long key = bj > 0 ? or_pack(best, i, bj, bt) : or_pack(0, 0, 1, 0);
     for (int o = 16; o; o >>= 1) {
         const unsigned long long other = __shfl_xor_sync(0xffffffffu, key, o);
         key = other < key ? other : key;
@@ -285,6 +384,18 @@ static bool or_naive()
     return v;
 }
 
+// The FP32 filter pays from the 128 x 32 tiles up (measured: C3 / C4 sweeps
+// 1.3x / 1.6x faster); the 16-column walks of n <= 2048 re-seed too often.
+// TSP2OPT_OROPT_FILTER=0 / 1 forces it off / on (experiment switch, same result).
+static bool or_filter(int n)
+{
+    static const int mode = [] {
+        const char* s = getenv("TSP2OPT_OROPT_FILTER");
+        return s && (s[0] == '0' || s[0] == '1') ? s[0] - '0' : -1;
+    }();
+    return mode < 0 ? n > 2048 : mode == 1;
+}
+
 size_t oropt_const_entries(int n) { return (size_t)n; }
 
 cudaError_t launch_or_sweep(const int2* Q, int4* CR, int4* CC, int n, unsigned long long* slot, cudaStream_t st)
@@ -302,7 +413,10 @@ cudaError_t launch_or_sweep(const int2* Q, int4* CR, int4* CC, int n, unsigned l
     int ti, tj;
     or_tiles(n, &ti, &tj);
     const dim3 grid((n + tj - 1) / tj, (n + ti - 1) / ti);
-    or_tile_kernel<<<grid, ti, 0, st>>>(Q, CR, CC, n, tj, slot);
+    if (or_filter(n))
+        or_tile_kernel<true><<<grid, ti, 0, st>>>(Q, CR, CC, n, tj, slot);
+    else
+        or_tile_kernel<false><<<grid, ti, 0, st>>>(Q, CR, CC, n, tj, slot);
     count_launch(2);
     return cudaGetLastError();
 }
