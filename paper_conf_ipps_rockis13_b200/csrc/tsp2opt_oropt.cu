@@ -10,12 +10,17 @@
 //
 // Layout: Q[p] = coords[tour[p]] for p < n + 5 (positions mod n: the closed
 // array of reading R10 plus the halo a segment of three past position n-1
-// can reach), int2.  One thread per cell, grid-stride over the cells of a
-// 148-multiple grid; the packed key (delta + 2^18) << 44 | j << 24 | i << 4 |
-// type (n <= 2^20) reduces per warp by shuffles, per CTA in shared memory and
-// per GPU with one 64-bit atomicMin.  Distances are the exact EUC_2D nint of
+// can reach), int2, and per-position removal-gain constants CR / CC.  The
+// sweep (or_tile_kernel) walks (row block x column chunk)
+// tiles, one row city per thread, with a 4 x 4 register window of distances
+// sliding along the columns; from n > 2048 the window is FP32 with an exact
+// fallback.  The packed key (delta + 2^18) << 44 | j << 24 | i << 4 | type
+// (n <= 2^20) reduces per warp by shuffles, per CTA in shared memory and per
+// GPU with one 64-bit atomicMin.  Exact distances are the EUC_2D nint of
 // tsp2opt_device.cuh.  The apply writes positions i+1..j in their new order
 // into a scratch span, then copies it back (two launches, no grid barrier).
+// or_sweep_kernel (one thread per cell) is the first version, kept behind
+// TSP2OPT_OROPT_NAIVE=1.
 #include <climits>
 #include <cstdlib>
 
