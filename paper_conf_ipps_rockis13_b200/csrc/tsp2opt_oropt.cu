@@ -116,8 +116,10 @@ __global__ void __launch_bounds__(kOrThreads) or_sweep_kernel(const int2* __rest
 //           (the row part of a forward move's removal gain);
 //   CC[p] = (e_p, rb_1, rb_2, rb_3) with rb_L = d(t_{p-L}, t_{p+1}) - d(t_{p-L}, t_{p-L+1}) - e_p
 //           (the column part of a backward move's removal gain; p - L >= 0 only is ever read).
-__global__ void or_consts_kernel(const int2* __restrict__ Q, int n, int4* __restrict__ CR, int4* __restrict__ CC)
+__global__ void or_consts_kernel(const int2* __restrict__ Q, int n, int4* __restrict__ CR, int4* __restrict__ CC,
+                                 unsigned long long* slot)
 {
+    if (blockIdx.x == 0 && threadIdx.x == 0) *slot = or_pack(0, 0, 1, 0);  // the sweep's seed key (reading R7)
     for (int p = blockIdx.x * blockDim.x + threadIdx.x; p < n; p += gridDim.x * blockDim.x) {
         const int e = or_d(Q[p], Q[p + 1]);
         int rf[3], rb[3];
@@ -405,16 +407,16 @@ size_t oropt_const_entries(int n) { return (size_t)n; }
 
 cudaError_t launch_or_sweep(const int2* Q, int4* CR, int4* CC, int n, unsigned long long* slot, cudaStream_t st)
 {
-    const unsigned long long seed = or_pack(0, 0, 1, 0);
-    cudaError_t e = cudaMemcpyAsync(slot, &seed, sizeof(seed), cudaMemcpyHostToDevice, st);
-    if (e != cudaSuccess) return e;
     if (or_naive()) {  // TSP2OPT_OROPT_NAIVE=1: the one-thread-per-cell kernel (experiment switch, same result)
+        const unsigned long long seed = or_pack(0, 0, 1, 0);
+        cudaError_t e = cudaMemcpyAsync(slot, &seed, sizeof(seed), cudaMemcpyHostToDevice, st);
+        if (e != cudaSuccess) return e;
         const long long cells = (long long)n * (n - 1) / 2;
         or_sweep_kernel<<<or_grid(cells, kOrThreads, 8), kOrThreads, 0, st>>>(Q, n, cells, slot);
         count_launch();
         return cudaGetLastError();
     }
-    or_consts_kernel<<<or_grid(n, 256, 4), 256, 0, st>>>(Q, n, CR, CC);
+    or_consts_kernel<<<or_grid(n, 256, 4), 256, 0, st>>>(Q, n, CR, CC, slot);  // also writes the seed key
     int ti, tj;
     or_tiles(n, &ti, &tj);
     const dim3 grid((n + tj - 1) / tj, (n + ti - 1) / ti);
