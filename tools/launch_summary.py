@@ -14,7 +14,7 @@ def main(path):
             k = d["Kernel Name"].split("(")[0]
             agg[k][0] += 1
             agg[k][1] += float(d["Metric Value"]) * (1e-3 if d["Metric Unit"] == "ns" else 1.0)
-    ours = {k: v for k, v in agg.items() if "tsp2opt" in k}
+    ours = {k: v for k, v in agg.items() if "tsp2opt" in k or k.split("<")[0].split()[-1].startswith("or_")}
     tot_ours = sum(v[1] for v in ours.values())
     print(f"# {path}: per-kernel device time (cold-cache, serialised; compare shares)")
     print(f"{'launches':>8} {'total_us':>12} {'avg_us':>10} {'share_of_ours':>13}  kernel")
