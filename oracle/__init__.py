@@ -103,6 +103,10 @@ def _load():
             lib.oracle_first_local_search.restype = ctypes.c_int
             lib.oracle_ils_mode.argtypes = [p, i64, p, i64, ctypes.c_uint64, ctypes.c_int, i64, p, p]
             lib.oracle_ils_mode.restype = None
+            lib.oracle_radius_best_move.argtypes = [p, i64, p, ctypes.c_int, p, p, p, p]
+            lib.oracle_radius_best_move.restype = None
+            lib.oracle_radius_local_search.argtypes = [p, i64, p, i64, ctypes.c_int, p, p, p, i64]
+            lib.oracle_radius_local_search.restype = ctypes.c_int
             lib.oracle_num_threads.argtypes = []
             lib.oracle_num_threads.restype = ctypes.c_int
             _lib = lib
@@ -234,11 +238,12 @@ def ils(coords, tour, iterations: int, seed: int, neighbours: int = 0, first: bo
 
 
 def mf_tour(coords) -> np.ndarray:
-    """Multiple Fragment (greedy) start tour (L22 §V; reading R17), n <= 20000."""
+    """Multiple Fragment (greedy) start tour (L22 §V; reading R17).  Plain: all
+    C(n,2) edges sorted, 8 C(n,2) bytes of host memory (4.6 GB at C4, 29.5 GB at C5)."""
     xy = _xy(coords)
     t = np.zeros(xy.shape[0], dtype=np.int32)
     if _load().oracle_mf_tour(_ptr(xy), xy.shape[0], _ptr(t)) != 0:
-        raise ValueError("oracle_mf_tour: n out of range [3, 20000] or out of memory")
+        raise ValueError("oracle_mf_tour: n out of range [3, 2^22] or out of memory")
     return t
 
 
@@ -389,6 +394,43 @@ def first_local_search(coords, tour, max_iters: int = -1, trace_cap: int = 0):
     tr = np.zeros((max(trace_cap, 1), 3), dtype=np.int64)
     st = _load().oracle_first_local_search(_ptr(xy), xy.shape[0], _ptr(t), int(max_iters), _ptr(out[0:1]),
                                            _ptr(out[1:2]), _ptr(tr) if trace_cap > 0 else None, int(trace_cap))
+    it = int(out[1])
+    return dict(tour=t, length=int(out[0]), iterations=it, status=int(st), trace=tr[: min(it, trace_cap)].copy())
+
+
+def _radius_mode(first: bool, node_insertion: bool) -> int:
+    if first and node_insertion:
+        raise ValueError("the radius oracle has no first-improvement 2.5-opt")
+    return 2 if node_insertion else (1 if first else 0)
+
+
+def radius_best_move(coords, tour, first: bool = False, node_insertion: bool = False):
+    """The exact radius-pruned sweep (SURVEY.md §8(c) lemma): equal to best_move (default),
+    first_move (first=True) -> (i, j, delta), or best_move25 (node_insertion=True) ->
+    (i, j, type, delta)."""
+    xy = _xy(coords)
+    t = np.ascontiguousarray(tour, dtype=np.int32)
+    out = np.zeros(4, dtype=np.int64)
+    mode = _radius_mode(first, node_insertion)
+    _load().oracle_radius_best_move(_ptr(xy), xy.shape[0], _ptr(t), mode, _ptr(out[0:1]), _ptr(out[1:2]),
+                                    _ptr(out[2:3]), _ptr(out[3:4]))
+    if node_insertion:
+        return int(out[0]), int(out[1]), int(out[2]), int(out[3])
+    return int(out[0]), int(out[1]), int(out[3])
+
+
+def radius_local_search(coords, tour, max_iters: int = -1, trace_cap: int = 0, first: bool = False,
+                        node_insertion: bool = False):
+    """Local search with the exact radius-pruned sweep; the same return dict (and trace
+    rows) as local_search / first_local_search / local_search25."""
+    xy = _xy(coords)
+    t = np.array(tour, dtype=np.int32, copy=True)
+    out = np.zeros(2, dtype=np.int64)
+    w = 4 if node_insertion else 3
+    tr = np.zeros((max(trace_cap, 1), w), dtype=np.int64)
+    st = _load().oracle_radius_local_search(_ptr(xy), xy.shape[0], _ptr(t), int(max_iters),
+                                            _radius_mode(first, node_insertion), _ptr(out[0:1]), _ptr(out[1:2]),
+                                            _ptr(tr) if trace_cap > 0 else None, int(trace_cap))
     it = int(out[1])
     return dict(tour=t, length=int(out[0]), iterations=it, status=int(st), trace=tr[: min(it, trace_cap)].copy())
 

@@ -317,8 +317,9 @@ void oracle_ils(const int32_t *xy, int64_t n, int32_t *tour, int64_t iterations,
  * cycle; the n-1 kept edges form a Hamiltonian path, closed by the edge
  * between its two ends.  Tour: start at city 0, step to its lower-id
  * neighbour, then follow the cycle.  Plain version: all C(n,2) edges, one
- * sort, union-find -- O(n^2 log n) time and 8 C(n,2) bytes, for n <= 20000.
- * Returns 0, or -1 if n is out of range or memory runs out.
+ * sort, union-find -- O(n^2 log n) time and 8 C(n,2) bytes (4.6 GB at n = 33810,
+ * 29.5 GB at n = 85900; golden files only).  Returns 0, or -1 if n is out of
+ * range [3, 2^22] or memory runs out.
  * ------------------------------------------------------------------------- */
 static int cmp_u64(const void *a, const void *b)
 {
@@ -337,7 +338,7 @@ static int64_t uf_find(int64_t *parent, int64_t x)
 
 int oracle_mf_tour(const int32_t *xy, int64_t n, int32_t *tour)
 {
-    if (n < 3 || n > 20000) return -1;
+    if (n < 3 || n > (1 << 22)) return -1; /* key packing below; memory: 4 n(n-1) bytes */
     const int64_t m = n * (n - 1) / 2;
     uint64_t *key = (uint64_t *)malloc(sizeof(uint64_t) * m);
     int64_t *parent = (int64_t *)malloc(sizeof(int64_t) * n);
@@ -919,6 +920,226 @@ int oracleor_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64_t m
         }
         it++;
     }
+    *length = L;
+    *iterations = it;
+    return status;
+}
+
+/* ---------------------------------------------------------------------------
+ * Exact radius-pruned sweeps (SURVEY.md §8(c) "Exact pruned oracle for large
+ * n").  These return EXACTLY what the plain all-pairs sweeps above return --
+ * they are not a different neighbourhood -- but visit only the pairs that can
+ * improve, so whole C4/C5 local searches from a constructive start finish in
+ * minutes instead of hours.  They exist to write golden traces at those sizes
+ * (tests/golden/make_golden.py) and are pinned move by move against the plain
+ * sweeps (tests/test_oracle_radius.py).
+ *
+ * Lemma (2-opt, L12 Fig. 2 delta, reading R2):
+ *   delta(i,j) = [D(t_i,t_j) - e_i] + [D(t_{i+1},t_{j+1}) - e_j] < 0
+ *   implies D(t_i,t_j) < e_i  or  D(t_{i+1},t_{j+1}) < e_j
+ * (if both brackets are >= 0 the sum is >= 0).  So the improving pairs are
+ * among
+ *   (A) i = p, j = q > p       with D(t_p, t_q) < e_p, and
+ *   (B) i = a-1, j = b-1, a < b with D(t_a, t_b) < e_{b-1}   (b = n is t_0).
+ * 2.5-opt (reading R19): delta_1 = [g_{i+1} + D(t_{i+1},t_j)] + [D(t_{i+1},t_{j+1}) - e_j]
+ * and delta_2 = [g_j + D(t_j,t_{i+1})] + [D(t_i,t_j) - e_i], so add
+ *   (C) i = p-1, j = q >= p+1  with D(t_p, t_q) < -g_p, and
+ *   (D) i = p-1, j = q, 1 <= p <= q-1 with D(t_q, t_p) < -g_q.
+ * Every candidate gets its exact delta(s); the result is the minimum over the
+ * candidates with delta < 0 of the same key as the plain sweep -- (delta, Fig. 3
+ * cell) for best improvement (reading R5), the cell alone for first improvement
+ * (reading R20), (delta, cell, type) for 2.5-opt (R19) -- else (0, 1, 0): the
+ * plain sweep's answer when no pair improves (reading R7).  A pair found twice
+ * is harmless (the minimum is idempotent).
+ *
+ * "All cities within distance < r of a point" is a plain scan of the cells of
+ * a uniform grid that intersect the square [x-r, x+r] x [y-r, y+r]
+ * (D < r implies |dx|, |dy| <= sqrt(s) < r + 1/2), testing the exact
+ * oracle_dist of every city found there.
+ * ------------------------------------------------------------------------- */
+typedef struct {
+    int64_t G, w;          /* G x G cells of width w */
+    int64_t *start;        /* cell c holds city[start[c] .. start[c+1]) */
+    int32_t *city;
+} oracle_grid;
+
+static void grid_build(oracle_grid *g, const int32_t *xy, int64_t n)
+{
+    int64_t G = (int64_t)sqrt((double)n / 2.0);
+    if (G < 1) G = 1;
+    g->G = G;
+    g->w = (32768 + G - 1) / G;
+    g->start = (int64_t *)calloc(G * G + 1, sizeof(int64_t));
+    g->city = (int32_t *)malloc(sizeof(int32_t) * (n > 0 ? n : 1));
+    for (int64_t c = 0; c < n; c++) g->start[(xy[2 * c + 1] / g->w) * G + xy[2 * c] / g->w + 1]++;
+    for (int64_t k = 0; k < G * G; k++) g->start[k + 1] += g->start[k];
+    int64_t *fill = (int64_t *)malloc(sizeof(int64_t) * (G * G + 1));
+    memcpy(fill, g->start, sizeof(int64_t) * (G * G + 1));
+    for (int64_t c = 0; c < n; c++) g->city[fill[(xy[2 * c + 1] / g->w) * G + xy[2 * c] / g->w]++] = (int32_t)c;
+    free(fill);
+}
+
+static void grid_free(oracle_grid *g)
+{
+    free(g->start);
+    free(g->city);
+}
+
+/* Appends to out[] every city c with oracle_dist((x, y), c) < r; returns the count.
+ * out must hold n entries. */
+static int64_t grid_within(const oracle_grid *g, const int32_t *xy, int64_t x, int64_t y, int64_t r, int32_t *out)
+{
+    int64_t m = 0;
+    if (r <= 0) return 0;
+    int64_t cx0 = x - r < 0 ? 0 : (x - r) / g->w, cx1 = (x + r) / g->w;
+    int64_t cy0 = y - r < 0 ? 0 : (y - r) / g->w, cy1 = (y + r) / g->w;
+    if (cx1 > g->G - 1) cx1 = g->G - 1;
+    if (cy1 > g->G - 1) cy1 = g->G - 1;
+    for (int64_t cy = cy0; cy <= cy1; cy++)
+        for (int64_t cx = cx0; cx <= cx1; cx++)
+            for (int64_t k = g->start[cy * g->G + cx]; k < g->start[cy * g->G + cx + 1]; k++) {
+                const int32_t c = g->city[k];
+                if (oracle_dist(x, y, xy[2 * c], xy[2 * c + 1]) < r) out[m++] = c;
+            }
+    return m;
+}
+
+/* the running minimum of one thread: (delta, cell, type), or the cell alone (first improvement) */
+typedef struct {
+    int64_t d, i, j, t;
+} radius_best;
+
+static void radius_offer(radius_best *b, int first, int64_t d, int64_t i, int64_t j, int64_t t)
+{
+    if (d >= 0) return; /* only improving moves compete; none -> (0, 1, 0) */
+    const int64_t k = oracle_cell(i, j), kb = oracle_cell(b->i, b->j);
+    int better;
+    if (b->d >= 0) better = 1;
+    else if (first) better = k < kb;
+    else better = d < b->d || (d == b->d && (k < kb || (k == kb && t < b->t)));
+    if (better) {
+        b->d = d; b->i = i; b->j = j; b->t = t;
+    }
+}
+
+/* One radius-pruned sweep over the route arrays px/py (n+1 entries, closed),
+ * e (edges), g (2.5-opt gains, mode 2 only) and pos (city -> position).
+ * mode 0: best-improvement 2-opt; 1: first-improvement 2-opt; 2: 2.5-opt. */
+static void radius_sweep(const int32_t *xy, int64_t n, const oracle_grid *grid, const int64_t *px, const int64_t *py,
+                         const int64_t *e, const int64_t *g, const int64_t *pos, int mode,
+                         int64_t *bi, int64_t *bj, int64_t *btype, int64_t *bdelta)
+{
+    radius_best best = {0, 0, 1, 0};
+#pragma omp parallel
+    {
+        radius_best tb = {0, 0, 1, 0};
+        int32_t *near = (int32_t *)malloc(sizeof(int32_t) * n);
+#pragma omp for schedule(dynamic, 64) nowait
+        for (int64_t p = 0; p <= n; p++) {
+            /* the candidate pairs (i, j) of rules A-D anchored at position p */
+            for (int rule = 0; rule < 4; rule++) {
+                int64_t r;
+                if (rule == 0) r = p <= n - 2 ? e[p] : 0;                  /* A: i = p */
+                else if (rule == 1) r = p >= 2 ? e[p - 1] : 0;              /* B: j + 1 = p */
+                else if (mode != 2) r = 0;
+                else if (rule == 2) r = (p >= 1 && p <= n - 2) ? -g[p] : 0; /* C: i + 1 = p */
+                else r = (p >= 2 && p <= n - 1) ? -g[p] : 0;                 /* D: j = p */
+                const int64_t m = grid_within(grid, xy, px[p], py[p], r, near);
+                for (int64_t k = 0; k < m; k++) {
+                    const int64_t q = pos[near[k]];
+                    int64_t i, j;
+                    if (rule == 0) { if (q <= p) continue; i = p; j = q; }
+                    else if (rule == 1) { if (q < 1 || q >= p) continue; i = q - 1; j = p - 1; }
+                    else if (rule == 2) { if (q < p + 1) continue; i = p - 1; j = q; }
+                    else { if (q < 1 || q > p - 1) continue; i = q - 1; j = p; }
+                    const int64_t dij = oracle_dist(px[i], py[i], px[j], py[j]);
+                    const int64_t di1j1 = oracle_dist(px[i + 1], py[i + 1], px[j + 1], py[j + 1]);
+                    radius_offer(&tb, mode == 1, dij + di1j1 - e[i] - e[j], i, j, 0);
+                    if (mode == 2 && j >= i + 2) {
+                        const int64_t di1j = oracle_dist(px[i + 1], py[i + 1], px[j], py[j]);
+                        radius_offer(&tb, 0, g[i + 1] + di1j + di1j1 - e[j], i, j, 1);
+                        radius_offer(&tb, 0, g[j] + dij + di1j - e[i], i, j, 2);
+                    }
+                }
+            }
+        }
+        free(near);
+#pragma omp critical
+        {
+            if (tb.d < 0) radius_offer(&best, mode == 1, tb.d, tb.i, tb.j, tb.t);
+        }
+    }
+    *bi = best.i; *bj = best.j; *btype = best.t; *bdelta = best.d;
+}
+
+/* route arrays of `tour`: P[k] = coords[t[k mod n]] for k <= n, e_k, g_k (R19), pos */
+static void radius_route(const int32_t *xy, int64_t n, const int32_t *tour, int64_t *px, int64_t *py, int64_t *e,
+                         int64_t *g, int64_t *pos)
+{
+    for (int64_t k = 0; k <= n; k++) {
+        const int64_t c = tour[k % n];
+        px[k] = xy[2 * c];
+        py[k] = xy[2 * c + 1];
+    }
+    for (int64_t k = 0; k < n; k++) e[k] = oracle_dist(px[k], py[k], px[k + 1], py[k + 1]);
+    for (int64_t k = 0; k < n; k++) {
+        const int64_t km = (k + n - 1) % n;
+        g[k] = oracle_dist(px[km], py[km], px[k + 1], py[k + 1]) - e[km] - e[k];
+    }
+    for (int64_t k = 0; k < n; k++) pos[tour[k]] = k;
+}
+
+/* One sweep from scratch: (i, j, type, delta), equal to oracle_best_move (mode 0),
+ * oracle_first_move (mode 1) or oracle25_best_move (mode 2). */
+void oracle_radius_best_move(const int32_t *xy, int64_t n, const int32_t *tour, int mode,
+                             int64_t *bi, int64_t *bj, int64_t *btype, int64_t *bdelta)
+{
+    oracle_grid grid;
+    grid_build(&grid, xy, n);
+    int64_t *buf = (int64_t *)malloc(sizeof(int64_t) * (5 * n + 2));
+    int64_t *px = buf, *py = buf + n + 1, *e = buf + 2 * n + 2, *g = buf + 3 * n + 2, *pos = buf + 4 * n + 2;
+    radius_route(xy, n, tour, px, py, e, g, pos);
+    radius_sweep(xy, n, &grid, px, py, e, g, pos, mode, bi, bj, btype, bdelta);
+    free(buf);
+    grid_free(&grid);
+}
+
+/* Local search with the radius-pruned sweep: the same loop, status and trace
+ * conventions as oracle_local_search / oracle_first_local_search (mode 0 / 1;
+ * trace rows (i, j, delta)) and oracle25_local_search (mode 2; rows (i, j,
+ * delta, type)).  The grid indexes cities, which never move, so it is built
+ * once; the route arrays are rebuilt from the tour before every sweep. */
+int oracle_radius_local_search(const int32_t *xy, int64_t n, int32_t *tour, int64_t max_iters, int mode,
+                               int64_t *length, int64_t *iterations, int64_t *trace, int64_t trace_cap)
+{
+    oracle_grid grid;
+    grid_build(&grid, xy, n);
+    int64_t *buf = (int64_t *)malloc(sizeof(int64_t) * (5 * n + 2));
+    int64_t *px = buf, *py = buf + n + 1, *e = buf + 2 * n + 2, *g = buf + 3 * n + 2, *pos = buf + 4 * n + 2;
+    const int w = mode == 2 ? 4 : 3;
+    int64_t L = oracle_tour_length(xy, n, tour);
+    int64_t it = 0;
+    int status = 0;
+    for (;;) {
+        int64_t i, j, t, d;
+        radius_route(xy, n, tour, px, py, e, g, pos);
+        radius_sweep(xy, n, &grid, px, py, e, g, pos, mode, &i, &j, &t, &d);
+        if (d >= 0) break;
+        if (max_iters >= 0 && it >= max_iters) { /* reading R8 */
+            status = 1;
+            break;
+        }
+        if (mode == 2) oracle25_apply(tour, i, j, (int)t);
+        else oracle_apply(tour, i, j);
+        L += d;
+        if (trace && it < trace_cap) {
+            trace[w * it] = i; trace[w * it + 1] = j; trace[w * it + 2] = d;
+            if (w == 4) trace[w * it + 3] = t;
+        }
+        it++;
+    }
+    free(buf);
+    grid_free(&grid);
     *length = L;
     *iterations = it;
     return status;
