@@ -51,6 +51,21 @@ __global__ void k(float* out, float seed, long long* cyc)
                 int q = __float_as_int(v[2 * c]);
                 asm volatile("add.s32 %0, %0, %1;" : "+r"(q) : "r"(__float_as_int(a)));
                 v[2 * c] = __int_as_float(q);
+            } else if (OP == 8) {  // MUFU.SQRT (sqrt.approx.ftz.f32): the XU pipe
+                asm volatile("sqrt.approx.ftz.f32 %0, %0;" : "+f"(v[2 * c]));
+            } else if (OP == 9) {  // MUFU.RSQ
+                asm volatile("rsqrt.approx.ftz.f32 %0, %0;" : "+f"(v[2 * c]));
+            } else if (OP == 10) {  // ISETP (OR-accumulate, signed compare of float bits)
+                int q = p[c];
+                asm volatile("{.reg .pred t, u; setp.ne.u32 u, %0, 0; setp.le.or.s32 t, %1, %2, u; selp.u32 %0, 1, 0, t;}"
+                             : "+r"(q) : "r"(__float_as_int(v[2 * c])), "r"(__float_as_int(a)));
+                p[c] = q;
+            } else if (OP == 11) {  // FMNMX3 (3-input min)
+                asm volatile("min.f32 %0, %0, %1, %2;" : "+f"(v[2 * c]) : "f"(v[2 * c + 1]), "f"(a));
+            } else if (OP == 12) {  // F2I (cvt.rni.s32.f32), the conversion pipe
+                int q;
+                asm volatile("cvt.rni.s32.f32 %0, %1;" : "=r"(q) : "f"(v[2 * c]));
+                v[2 * c] = __int_as_float(q) ;
             }
         }
     }
@@ -86,6 +101,7 @@ int main()
     for (int w : {8, 16, 32}) {
         run<0>("FFMA", w); run<6>("FMUL", w); run<1>("FFMA2", w); run<2>("FADD2", w);
         run<3>("FSETP", w); run<4>("FMNMX", w); run<5>("FFMA2+SETP", w); run<7>("IADD", w);
+        run<8>("MUFU.SQRT", w); run<9>("MUFU.RSQ", w); run<10>("ISETP", w); run<11>("FMNMX3", w); run<12>("F2I", w);
     }
     return 0;
 }
