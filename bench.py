@@ -36,7 +36,8 @@ from paper_conf_ipps_rockis13_b200 import inputs  # noqa: E402
 
 METRIC = "2-opt pair checks/sec and time-to-local-minimum at 1/2/4/8 B200 vs roofline"
 UNIT = "pair checks/s"
-PAIRS_PER_CLK_SM = 8  # north_star roofline: ~2 distance evaluations (16 issue slots, 2 XU ops) per pair
+PAIRS_PER_CLK_SM = 8  # north_star's per-pair model: ~2 distance evaluations (16 issue slots, 2 XU ops) per pair
+ISSUE_PER_CLK_SM = 4  # warp-instruction issue slots per clock per SM (4 SMSPs) -- the sweep's real ceiling
 N_SM = 148
 
 
@@ -215,9 +216,13 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms, sweep_avg_ms, e2e_total, tb_total_ms, tb_sweep_ms = t.tolist()
 
-    ls = ils = batch = batch_ils = pruned = or25 = first = oropt = None
+    ls = ils = batch = batch_ils = pruned = or25 = first = oropt = sharded = balance = None
+    if world > 1 and not args.no_ls:  # collective: every rank runs it
+        sharded = time_sharded_ls(tsp2opt, rank, world, args.sharded_config)
+    if rank == 0 and world == 1 and not args.no_ls and args.balance_config:
+        balance = shard_balance(tsp2opt, args.balance_config)
     if rank == 0 and world == 1 and not args.no_ls:
-        ls = time_to_local_min(tsp2opt, args.ls_config)
+        ls = time_to_local_min(tsp2opt, args.ls_config, not args.no_cpu)
         pruned = time_pruned(tsp2opt, args.pruned_config, not args.no_cpu) if args.pruned_config else None
         or25 = time_25opt(tsp2opt, args.or25_config, not args.no_cpu) if args.or25_config else None
         first = time_first(tsp2opt, args.first_config) if args.first_config else None
@@ -230,9 +235,15 @@ def run_ours(args):
         prof = ncu_profile_summary(args.config, args.tour)
         pk = peaks()
         sm_max = clocks.get("sm_max_mhz") or pk.get("sm_max_mhz") or 1965.0
-        peak = PAIRS_PER_CLK_SM * N_SM * sm_max * 1e6 * world  # aggregate over ranks
-        achieved = geo["pairs"] * world / (sweep_avg_ms * 1e-3)  # per launch, all ranks
+        pair_peak = PAIRS_PER_CLK_SM * N_SM * sm_max * 1e6 * world  # north_star's per-pair model, all ranks
+        pair_rate = geo["pairs"] * world / (sweep_avg_ms * 1e-3)  # pairs per second of sweep launch, all ranks
         value = total_pairs * args.steps / (total_ms * 1e-3)
+        # Roofline: the sweep is issue-bound, so `frac` is the issue-slot
+        # fraction -- the warp instructions ONE sweep launch executes (ncu, committed
+        # profile of this workload) over the live launch time, against 4 warp-inst/clk/SM.
+        issue_peak = ISSUE_PER_CLK_SM * N_SM * sm_max * 1e6  # warp-instructions/s per GPU
+        winst = prof.get("warp_inst")
+        issue_rate = winst / (sweep_avg_ms * 1e-3) if winst else None
         line = {
             "metric": METRIC,
             "value": value,
@@ -251,12 +262,22 @@ def run_ours(args):
                                    f"{'allreduce-min + ' if world > 1 else ''}apply",
                        "n": n, "pairs_per_step": total_pairs, "l2": "flushed (256 MiB write) between timed steps",
                        "geometry": geo, "parallelism": f"tile-shard x{world}"},
-            "roofline": {"bound": "alu", "achieved": achieved / 1e9, "peak": peak / 1e9, "unit": "Gpair/s",
-                         "frac": achieved / peak, "traffic": prof.get("traffic"),
-                         "kernel": "sweep_kernel", "peak_def": f"{PAIRS_PER_CLK_SM} pairs/clk/SM x {N_SM} SMs x "
-                         f"{sm_max:.0f} MHz (north_star: ~2 distance evaluations per pair; DESIGN.md §7)",
-                         "issue_util_ncu": prof.get("issue_util"), "ncu_profile": prof.get("path"),
-                         "sweep_ms_avg": sweep_avg_ms, "sweep_share_of_step": sweep_avg_ms / (total_ms / args.steps)},
+            "roofline": {"bound": "alu", "achieved": issue_rate / 1e12 if issue_rate else None,
+                         "peak": issue_peak / 1e12, "unit": "Twarp-inst/s",
+                         "frac": issue_rate / issue_peak if issue_rate else None, "traffic": prof.get("traffic"),
+                         "kernel": "sweep_kernel",
+                         "peak_def": f"{ISSUE_PER_CLK_SM} warp-instructions/clk/SM (4 SMSPs x 1 issue) x {N_SM} SMs x "
+                                     f"{sm_max:.0f} MHz: the sweep is issue-bound (DESIGN.md §5.4, §7)",
+                         "achieved_def": "warp instructions per C5 sweep launch (ncu smsp__inst_executed.sum of the "
+                                         "committed profile) / live sweep-launch time (CUDA events, this run)",
+                         "warp_inst_per_launch": winst, "inst_per_pair": (32 * winst / geo["pairs"]) if winst else None,
+                         "ncu_profile": prof.get("path"), "ncu_issue_active": prof.get("issue_util"),
+                         "sweep_ms_avg": sweep_avg_ms, "sweep_share_of_step": sweep_avg_ms / (total_ms / args.steps),
+                         "pair_rate": pair_rate / 1e9, "pair_rate_unit": "Gpair/s (all ranks)",
+                         "model_ratio": pair_rate / pair_peak,
+                         "model_def": f"pair rate / ({PAIRS_PER_CLK_SM} pairs/clk/SM x {N_SM} x {sm_max:.0f} MHz x "
+                                      f"{world}), north_star's ~2 distance evaluations per pair; > 1 means fewer "
+                                      "instructions per pair than that model, not above the hardware limit"},
             "e2e": {"value": total_pairs * len(e2e_ms) / (e2e_total * 1e-3), "unit": UNIT,
                     "h2d_bytes_per_step": 4 * n, "d2h_bytes_per_step": 2 * 64,
                     "api": "tsp2opt_best_move(host tour) + tsp2opt_apply"},
@@ -270,6 +291,10 @@ def run_ours(args):
         }
         if ls:
             line["time_to_local_minimum"] = ls
+        if sharded:
+            line["time_to_local_minimum_sharded"] = sharded
+        if balance:
+            line["shard_load_balance"] = balance
         if ils:
             line["ils"] = ils
         if pruned:
@@ -303,6 +328,8 @@ def ncu_profile_summary(cfg, tour):
     for line in open(paths[-1]):
         if line.startswith("ipc_per_sm"):
             vals["ipc_per_sm"] = float(line.split()[3])
+        elif line.startswith("warp_inst_total"):
+            vals["warp_inst"] = float(line.split()[1])
         elif line.startswith(("dram_read", "dram_write")):
             name, num, unit = (line.split() + ["byte"])[:3]
             vals[name] = float(num) * {"Mbyte": 1e6, "Kbyte": 1e3, "byte": 1.0, "Gbyte": 1e9}.get(unit, 1.0)
@@ -311,15 +338,49 @@ def ncu_profile_summary(cfg, tour):
         out["traffic"] = vals["dram_read"] + vals.get("dram_write", 0.0)
     if "ipc_per_sm" in vals:
         out["issue_util"] = vals["ipc_per_sm"] / 4.0
+    if "warp_inst" in vals:
+        out["warp_inst"] = vals["warp_inst"]
     return out
 
 
-def time_to_local_min(tsp2opt, cfg_name):
+def oracle_ttlm(name, tk, coords, tour):
+    """The oracle's time to the same local minimum (Table II "Time to first
+    minimum"; SURVEY §8(d) "full local search for C1-C3"): C1 and C2 run live on this
+    box's host cores; C3-C5 are too slow for a bench run, so their figure is the
+    oracle_seconds recorded by tests/golden/make_golden.py (labelled with its
+    threads and, for C4 / C5, the exact radius-pruned oracle it used)."""
+    import oracle
+
+    n = len(coords)
+    if n <= 2000:
+        if tour is None:  # the Multiple Fragment start: the oracle's own (never the device's)
+            tour = oracle.mf_tour(coords)
+        t0 = time.perf_counter()
+        r = oracle.local_search(coords, tour)
+        return {"seconds": time.perf_counter() - t0, "iterations": r["iterations"], "length": r["length"],
+                "cores": oracle.num_threads(), "kind": "oracle", "sample": "the whole local search, live"}
+    gdir = os.path.join(ROOT, "tests", "golden")
+    cands = [(f"ls_{name}_lattice_{tk}_s1.npz", "plain all-pairs oracle"),
+             (f"ls_radius_{name}_lattice_{tk}_s1.npz", "exact radius-pruned oracle (SURVEY §8(c) lemma; same moves)")]
+    for fname, what in cands:
+        path = os.path.join(gdir, fname)
+        if os.path.exists(path):
+            g = np.load(path)
+            return {"seconds": float(g["oracle_seconds"]), "iterations": int(g["iterations"]),
+                    "length": int(g["length"]), "cores": int(g["oracle_threads"]), "kind": "oracle",
+                    "sample": f"recorded by tests/golden/make_golden.py on the 8-core dev host, {what}"}
+    return None
+
+
+def time_to_local_min(tsp2opt, cfg_name, with_oracle=True):
     """Wall time of tsp2opt_local_search (host tour in, host tour out) per config.
     Start `mf`: the paper's Table II protocol (L22 "time needed from an initial
     solution based on the Multiple Fragment(Greedy) heuristic ... to the local
     minimum"): tsp2opt_mf_tour on the device, then the local search from it;
-    both inside the timed region (coordinates already on the device)."""
+    both inside the timed region (coordinates already on the device).
+    `pairs_covered_per_s` = C(n,2) x sweeps / time: with the tile bounds and the
+    culled / incremental sweeps most pairs are covered by a tile-level proof, not
+    tested one by one, so it is NOT a pair-check rate (that is the dense `value`)."""
     out = []
     for name in cfg_name.split(","):
         name, _, tk = name.partition(":")
@@ -334,10 +395,16 @@ def time_to_local_min(tsp2opt, cfg_name):
                 r = g.local_search_current()
                 t2 = time.perf_counter()
             n = len(coords)
-            out.append({"config": name, "n": n, "start": "mf", "seconds": t2 - t0, "mf_seconds": t1 - t0,
-                        "ls_seconds": t2 - t1, "mf_length": m["length"], "mf_rounds": m["rounds"],
-                        "iterations": r["iterations"], "length": r["length"],
-                        "pair_checks_per_s": (r["iterations"] + 1) * n * (n - 1) / 2 / (t2 - t1)})
+            entry = {"config": name, "n": n, "start": "mf", "seconds": t2 - t0, "mf_seconds": t1 - t0,
+                     "ls_seconds": t2 - t1, "mf_length": m["length"], "mf_rounds": m["rounds"],
+                     "iterations": r["iterations"], "length": r["length"],
+                     "us_per_move": 1e6 * (t2 - t1) / max(1, r["iterations"]),
+                     "pairs_covered_per_s": (r["iterations"] + 1) * n * (n - 1) / 2 / (t2 - t1)}
+            if with_oracle:
+                o = oracle_ttlm(name, "mf", coords, None)
+                if o:
+                    entry["cpu_oracle"] = o
+            out.append(entry)
             continue
         coords, tour = inputs.config_instance(name, tk or None)
         with tsp2opt.TSP2Opt(coords) as g:
@@ -346,9 +413,93 @@ def time_to_local_min(tsp2opt, cfg_name):
             r = g.local_search(tour)
             dt = time.perf_counter() - t0
         n = len(tour)
-        out.append({"config": name, "n": n, "start": tk or inputs.CONFIGS[name]["tour"], "seconds": dt,
+        tk = tk or inputs.CONFIGS[name]["tour"]
+        entry = {"config": name, "n": n, "start": tk, "seconds": dt,
+                 "iterations": r["iterations"], "length": r["length"],
+                 "us_per_move": 1e6 * dt / max(1, r["iterations"]),
+                 "pairs_covered_per_s": (r["iterations"] + 1) * n * (n - 1) / 2 / dt}
+        if with_oracle:
+            o = oracle_ttlm(name, tk, coords, tour)
+            if o:
+                entry["cpu_oracle"] = o
+        out.append(entry)
+    return out
+
+
+def time_sharded_ls(tsp2opt, rank, world, spec):
+    """Time to local minimum on sharded handles (§VI "dividing the 2-opt task
+    between multiple devices"): every rank runs tsp2opt_local_search on its
+    tile shard with one allreduce-min per sweep.  seconds = max over ranks of each rank's
+    wall time of the call, the ranks started together by a barrier.  Every rank's final
+    tour must be identical (tour hash all-gathered) and equal to the length / move count
+    a world-1 run reports (checked by tests/test_gpu_multirank.py)."""
+    import hashlib
+
+    import torch
+    import torch.distributed as dist
+
+    out = []
+    for item in spec.split(","):
+        if not item:
+            continue
+        name, _, tk = item.partition(":")
+        coords, tour = inputs.config_instance(name, "random" if tk == "mf" else (tk or None))
+        obj = [tsp2opt.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        with tsp2opt.TSP2Opt(coords, rank, world, obj[0]) as g:
+            if tk == "mf":
+                tour = g.mf_tour()["tour"]
+            g.local_search(tour, max_iters=2)  # warm-up (graphs, NCCL channels)
+            dist.barrier()
+            t0 = time.perf_counter()
+            r = g.local_search(tour)
+            dt = time.perf_counter() - t0
+        t = torch.tensor([dt], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        h = hashlib.sha1(r["tour"].tobytes()).hexdigest()[:16]
+        hs = [None] * world
+        dist.all_gather_object(hs, (h, r["iterations"], r["length"]))
+        n = len(coords)
+        out.append({"config": name, "n": n, "start": tk or "random", "ranks": world, "seconds": t.item(),
                     "iterations": r["iterations"], "length": r["length"],
-                    "pair_checks_per_s": (r["iterations"] + 1) * n * (n - 1) / 2 / dt})
+                    "us_per_move": 1e6 * t.item() / max(1, r["iterations"]),
+                    "tours_agree": all(x == hs[0] for x in hs), "tour_sha1_16": h,
+                    "timing": "max over ranks of the per-rank wall time of tsp2opt_local_search"})
+    return out
+
+
+def shard_balance(tsp2opt, spec):
+    """Load balance of the equal-pair LPT tile split, measured on ONE GPU:
+    for world = 2, 4, 8 every shard r of the dense C4 / C5 sweep (random tour, tile bounds
+    off, the bench's `value` workload) is timed alone with tsp2opt_debug_set_shard(r, world)
+    and the library's CUDA events; reported as max / mean shard time.  The min over the
+    shards' moves must equal the full sweep's move.  A load-balance check of the split,
+    not a multi-GPU measurement."""
+    out = []
+    for name in spec.split(","):
+        if not name:
+            continue
+        coords, tour = inputs.config_instance(name, "random")
+        with tsp2opt.TSP2Opt(coords) as g:
+            g.set_option(tsp2opt.OPT_TILE_BOUNDS, 0)
+            full = g.best_move(tour)
+            for world in (2, 4, 8):
+                times, moves = [], []
+                for r in range(world):
+                    g.debug_set_shard(r, world)
+                    g.best_move(tour)
+                    g.profile(True)
+                    for _ in range(3):
+                        mv = g.best_move()
+                    ms, k = g.profile_read()
+                    g.profile(False)
+                    times.append(ms / k)
+                    moves.append(mv)
+                g.debug_set_shard(0, 1)
+                best = min(moves, key=lambda m: (m[2], m[1] * (m[1] - 1) // 2 + m[0]))
+                out.append({"config": name, "world": world, "shard_ms": times,
+                            "max_over_mean": max(times) / (sum(times) / world),
+                            "min_of_shards_equals_full": best == full})
     return out
 
 
@@ -476,7 +627,7 @@ def time_oropt(tsp2opt, spec, with_oracle=True):
         entry = {"config": name, "n": n, "start": tk or "random", "moves": "2-opt + Or-opt segments of 1..3 cities",
                  "seconds": sec, "iterations": r["iterations"], "length": r["length"],
                  "s_per_iteration": sec / (r["iterations"] + 1),
-                 "pair_checks_per_s": cells * (r["iterations"] + 1) / sec, "moves_per_pair": 13}
+                 "pairs_covered_per_s": cells * (r["iterations"] + 1) / sec, "moves_per_pair": 13}
         if with_oracle and n <= 20000:
             import oracle
             reps = 3 if n > 5000 else 10
@@ -565,9 +716,13 @@ def time_batch(tsp2opt, spec, with_oracle=True):
                 dev.append(e0.elapsed_time(e1) * 1e-3)
         dev_s = float(np.median(dev))
         moves = int(di.sum())
-        t0 = time.perf_counter()
-        r = tsp2opt.batch_local_search(cs, ts)
-        host_s = time.perf_counter() - t0
+        tsp2opt.batch_local_search(cs[:2], ts[:2])  # warm-up of the host entry
+        host = []
+        for _ in range(3):  # median of 3 host-API runs
+            t0 = time.perf_counter()
+            r = tsp2opt.batch_local_search(cs, ts)
+            host.append(time.perf_counter() - t0)
+        host_s = float(np.median(host))
         ok = bool((r["lengths"] == dl.cpu().numpy()).all())
         item_out = {"n": n, "instances": B, "coords": "uniform seeds 1..B", "start": "random",
                     "device_s": dev_s, "instances_per_s": B / dev_s,
@@ -622,9 +777,13 @@ def time_batch_ils(tsp2opt, spec, with_oracle=True):
             if rep:
                 dev.append(e0.elapsed_time(e1) * 1e-3)
         dev_s = float(np.median(dev))
-        t0 = time.perf_counter()
-        r = tsp2opt.batch_ils(cs, ts, T, seeds, history=False)
-        host_s = time.perf_counter() - t0
+        tsp2opt.batch_ils(cs[:2], ts[:2], 1, seeds[:2], history=False)  # warm-up of the host entry
+        host = []
+        for _ in range(3):  # median of 3 host-API runs
+            t0 = time.perf_counter()
+            r = tsp2opt.batch_ils(cs, ts, T, seeds, history=False)
+            host.append(time.perf_counter() - t0)
+        host_s = float(np.median(host))
         L = dl.cpu().numpy()
         item_out = {"config": name, "n": n, "replicas": R, "ils_steps": T, "device_s": dev_s,
                     "ils_steps_per_s": R * T / dev_s, "best_length": int(L.min()), "mean_length": float(L.mean()),
@@ -688,7 +847,8 @@ def run_reference(args):
             break
     k = len(times)
     value = total_pairs * k / sum(times)
-    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": k, "warmup": args.warmup,
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": max(world, args.gpus), "steps": k,
+            "warmup": args.warmup,
             "ms_per_step": 1e3 * sum(times) / k, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "int64", "data": "synthetic", "impl": "reference",
             "config": {"workload": f"{args.config} n={n} {cfg['coords']} coords, {args.tour} tour; one step = "
@@ -697,6 +857,26 @@ def run_reference(args):
                              "sample": f"{k} step(s) of the workload (capped at {args.ref_seconds:.0f} s)"},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def launch_ranks(n: int) -> int:
+    import socket
+
+    try:
+        import torch
+
+        have = torch.cuda.device_count()
+    except Exception:  # pragma: no cover
+        have = 0
+    if have < n:
+        print(json.dumps({"metric": METRIC, "error": f"--gpus {n} but {have} CUDA device(s) visible"}), flush=True)
+        return 2
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 def main():
@@ -708,6 +888,9 @@ def main():
     ap.add_argument("--config", default="C5")
     ap.add_argument("--tour", default="random", choices=["random", "hilbert"])
     ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert,C5:hilbert,C2:mf,C3:mf,C4:mf,C5:mf", help="configs timed to a local minimum (rank 0, N=1)")
+    ap.add_argument("--sharded-config", default="C4:hilbert,C5:hilbert,C4:mf,C5:mf",
+                    help="time to local minimum on the sharded handle, N > 1 (every rank)")
+    ap.add_argument("--balance-config", default="C4,C5", help="per-shard sweep times of the LPT split, N = 1")
     ap.add_argument("--ils-config", default="C1:200,C2:50", help="Iterated Local Search runs cfg:iterations")
     ap.add_argument("--pruned-config", default="C3:8,C4:8,C5:8,C5:16", help="pruned 2-opt from MF, cfg:K")
     ap.add_argument("--or25-config", default="C3,C4,C5", help="2.5-opt local search from MF, configs")
@@ -722,6 +905,10 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         args.warmup = 3
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl == "ours":
+        # `bench.py --gpus N` without an external launcher: start the N ranks here
+        # (one process per GPU, rendezvous on 127.0.0.1), exactly as torchrun would.
+        raise SystemExit(launch_ranks(args.gpus))
     if args.impl == "reference":
         run_reference(args)
     else:

@@ -217,6 +217,15 @@ int tsp2opt_oropt_local_search(const int32_t *coords_xy, int32_t n, int32_t *tou
 int tsp2opt_oropt_best_move(const int32_t *coords_xy, int32_t n, const int32_t *tour, int32_t *i, int32_t *j,
                             int32_t *type, int32_t *delta);
 
+/* Or-opt sweep kernel selection for this process (no result depends on it;
+ * DESIGN.md §5.15): filter -1 = by size (the FP32 filter from n > 2048), 0 =
+ * exact walk only, 1 = FP32 filter + seeded bound; naive 1 = the one-thread-
+ * per-cell kernel (filter ignored), 0 = the tiled kernel.  Overrides the
+ * TSP2OPT_OROPT_FILTER / TSP2OPT_OROPT_NAIVE environment defaults.  Not
+ * thread-safe against a concurrent Or-opt call.  Returns EINVAL for other
+ * values. */
+int tsp2opt_oropt_config(int32_t filter, int32_t naive);
+
 /* Multiple Fragment (greedy) start tour, computed on the device (SURVEY §8(f)
  * NEXT-1; L22 §V "an initial solution based on the Multiple Fragment(Greedy)
  * heuristic[18]"; definition, tie-break and orientation: DESIGN.md R17 --

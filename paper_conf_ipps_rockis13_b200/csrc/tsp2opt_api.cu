@@ -81,6 +81,9 @@ struct tsp2opt_ctx {
     int2* d_ctiles = nullptr;   // this shard's cull tiles
     unsigned long long* d_ctilebest = nullptr;  // their per-tile minima (seeds)
     int4* d_list = nullptr;     // kept cull tiles (I0, J0, index) [nctiles]
+    int* d_tmap = nullptr;      // [nrb * ncc] (row block, column chunk) -> this shard's cull-tile index, -1 if none
+    int inc_grid = 0;           // one-warp CTAs of the fused incremental sweep (co-resident)
+    bool inc_fused = true;      // TSP2OPT_INC_FUSED=0: the box + cull + list kernels on every iteration
     int nctiles = 0;
     int list_grid = 0;          // CTAs of the culled sweep (co-resident)
     int list25_grid = 0;        // CTAs of the 2.5-opt culled sweep
@@ -215,6 +218,19 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
     cudaFree(h->d_list);
     h->d_list = nullptr;
     if (h->nctiles > 0) CUDA_TRY(cudaMalloc(&h->d_list, sizeof(int4) * (size_t)h->nctiles));
+    {  // (row block, column chunk) -> index in this shard's cull-tile array (the fused incremental sweep)
+        const int TI = h->cgeo.ti(), TJ = h->cgeo.tj;
+        const int nrb = (h->n - 1 + TI - 1) / TI, ncc = (h->n + TJ - 1) / TJ;
+        std::vector<int> map((size_t)nrb * ncc, -1);
+        long long unused = 0;
+        std::vector<Tile> mine = shard_tiles(h->all_ctiles, rank, world, &unused);
+        for (size_t k = 0; k < mine.size(); k++) map[(size_t)(mine[k].i0 / TI) * ncc + mine[k].j0 / TJ] = (int)k;
+        cudaFree(h->d_tmap);
+        h->d_tmap = nullptr;
+        CUDA_TRY(cudaMalloc(&h->d_tmap, sizeof(int) * map.size()));
+        CUDA_TRY(cudaMemcpy(h->d_tmap, map.data(), sizeof(int) * map.size(), cudaMemcpyHostToDevice));
+        h->inc_grid = inc_sweep_grid(h->cgeo);
+    }
     h->list_grid = sweep_list_grid(h->cgeo, h->nctiles);
     if (const char* el = getenv("TSP2OPT_LIST_GRID"))  // experiment: cap the list sweep's co-resident grid
         if (atoi(el) > 0) h->list_grid = std::min(h->list_grid, atoi(el));
@@ -246,6 +262,7 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_ctiles);
     cudaFree(h->d_ctilebest);
     cudaFree(h->d_list);
+    cudaFree(h->d_tmap);
     cudaFree(h->d_rbox);
     cudaFree(h->d_cbox);
     cudaFree(h->d_trace);
@@ -370,6 +387,11 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
         const int p1 = (int)((long long)h->n * (h->shard_rank + 1) / h->shard_world);
         CUDA_TRY(launch_pruned_sweep(h->d_P, h->d_E, h->d_tour, h->d_pos, h->d_knn, h->nbr_k, h->n, p0, p1, in,
                                      apply ? 1 : 0, h->first, h->stream));
+    } else if (tiling && (flags & kSweepIncremental) && !(flags & kSweepFull) && h->inc_fused &&
+               h->cgeo.rows == kRowsSmall && h->cgeo.warps == 1 && h->inc_grid > 0) {
+        // incremental: dirty tiles only, enumerated from the last move; box, cull and sweep in one launch
+        CUDA_TRY(launch_inc_sweep(h->cgeo, h->d_P, h->d_E, h->n, h->d_ctiles, h->nctiles, h->d_tmap, h->inc_grid,
+                                  h->d_rbox, h->d_cbox, in, apply ? 1 : 0, h->d_ctilebest, flags, h->stream));
     } else if (tiling) {  // cull first, then sweep the kept tiles only
         CUDA_TRY(launch_cull_sweep(h->cgeo, h->d_P, h->d_E, h->n, h->d_ctiles, h->nctiles, h->list_grid, h->d_rbox,
                                    h->d_cbox, h->d_list, in, apply ? 1 : 0, h->d_ctilebest, flags, h->stream));
@@ -457,7 +479,9 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
         // first-improvement and 2.5-opt loops; 20 % slower for the dense best-improvement
         // sweep (C3 from random), which keeps plain stream launches.
         const bool dense_best = !h->or25 && h->nbr_k == 0 && !h->first && h->tile_bounds < 2;
-        const bool use_graph = graphs_enabled() && !h->comm && !h->profiling && !dense_best;
+        // Sharded handles capture the ncclAllReduce into the same graph (NCCL supports
+        // stream capture of collectives): one graph launch per 64 iterations on every rank.
+        const bool use_graph = graphs_enabled() && !h->profiling && !dense_best;
         auto drop_graph = [&]() {
             if (gexec) cudaGraphExecDestroy(gexec);
             gexec = nullptr;
@@ -546,6 +570,7 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     if (const char* ep = getenv("TSP2OPT_PERSISTENT")) h->persistent = atoi(ep);
     if (const char* es = getenv("TSP2OPT_SEED")) h->seed_next = atoi(es) != 0;
     if (const char* eg = getenv("TSP2OPT_GLOBAL_SEED")) h->global_seed = atoi(eg) != 0;
+    if (const char* ef = getenv("TSP2OPT_INC_FUSED")) h->inc_fused = atoi(ef) != 0;
 
     CTRY(cudaMemset(h->d_slots, 0, sizeof(Slot) * 2));
     {
@@ -561,14 +586,17 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     // n = 85900 39 vs 65 (cull) vs 212 (in-sweep bound) us per iteration, n = 33810 26 vs 36 vs
     // 79 us; n = 7397 23 vs 25 vs 18 us, where the extra launches cost more than the skipped
     // tiles; profiles/r01_ls_incremental.jsonl).
-    h->tile_bounds = total_pairs / world >= 100000000LL ? 3 : 1;
+    // The level follows the instance, not the shard: a coherent tour keeps a few percent of
+    // the tiles on EVERY rank, and a rank's shard of a large instance is still a spread-out
+    // subset of its tiles, so C4 at 8 ranks keeps the incremental culled sweep.
+    h->tile_bounds = total_pairs >= 100000000LL ? 3 : 1;
     if (const char* eb = getenv("TSP2OPT_TILE_BOUNDS")) h->tile_bounds = std::min(3, std::max(0, atoi(eb)));
     h->all_tiles = build_tiles(n, h->geo);
     // Culled-sweep tiling: R = 7 rows per lane and narrow column chunks (measured,
     // local search from MF).
     // (incremental culled sweep, measured without per-sweep events: n = 85900 TJ 32 28.6 vs 64 30.6 us
     // per iteration, n = 33810 TJ 16 20.6 vs 32 22.7 us; profiles/r01_inc_tiling.jsonl)
-    h->cgeo = Geometry{kRowsSmall, 1, total_pairs / world >= 1000000000LL ? 32 : 16};
+    h->cgeo = Geometry{kRowsSmall, 1, total_pairs >= 1000000000LL ? 32 : 16};
     if (const char* er = getenv("TSP2OPT_CULL_ROWS")) h->cgeo.rows = atoi(er) == kRowsSmall ? kRowsSmall : kRowsLarge;
     if (const char* ec = getenv("TSP2OPT_CULL_TJ"))
         if (atoi(ec) >= 2 && atoi(ec) <= kMaxTJ) h->cgeo.tj = atoi(ec);
@@ -1263,6 +1291,7 @@ int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters
     if ((e = cudaMemcpy(&len, d_slot + 1, sizeof(len), cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
     long long L = (long long)len, it = 0;
     int status = TSP2OPT_OK;
+    std::vector<int32_t> tr;  // copied to the caller only on success (nothing is written on error)
     for (;;) {
         if ((e = launch_or_sweep(d_q, d_c, d_c + oropt_const_entries(n), n, d_slot, nullptr)) != cudaSuccess) return fail(e, "or_sweep_kernel");
         unsigned long long key = 0;
@@ -1277,17 +1306,13 @@ int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters
         }
         if ((e = launch_or_apply(d_xy, d_t, d_q, d_span, n, i, j, type, nullptr)) != cudaSuccess)
             return fail(e, "or_apply");
-        if (trace && it < trace_cap) {
-            trace[4 * it] = i;
-            trace[4 * it + 1] = j;
-            trace[4 * it + 2] = d;
-            trace[4 * it + 3] = type;
-        }
+        if (trace && it < trace_cap) tr.insert(tr.end(), {i, j, d, type});
         L += d;
         it++;
     }
     if ((e = cudaMemcpy(tour, d_t, nb, cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
     cleanup();
+    if (trace && !tr.empty()) memcpy(trace, tr.data(), sizeof(int32_t) * tr.size());
     if (length) *length = L;
     if (iterations) *iterations = it;
     return status;
@@ -1301,6 +1326,13 @@ int tsp2opt_oropt_local_search(const int32_t* coords_xy, int32_t n, int32_t* tou
     if (!coords_xy || !tour || max_iters < 0 || trace_cap < 0 || (trace_cap > 0 && !trace_ijdt)) return TSP2OPT_EINVAL;
     if (n < 3 || n > TSP2OPT_OROPT_MAX_N) return TSP2OPT_EINVAL;
     return or_run(coords_xy, n, tour, max_iters, length, iterations, trace_ijdt, trace_cap, nullptr);
+}
+
+int tsp2opt_oropt_config(int32_t filter, int32_t naive)
+{
+    if (filter < -1 || filter > 1 || naive < 0 || naive > 1) return TSP2OPT_EINVAL;
+    or_config(filter, naive);
+    return TSP2OPT_OK;
 }
 
 int tsp2opt_oropt_best_move(const int32_t* coords_xy, int32_t n, const int32_t* tour, int32_t* i, int32_t* j,

@@ -89,6 +89,7 @@ cudaError_t launch_apply25(float2* P, int* E, int* G, int* tour, int n, const Sl
 size_t oropt_q_entries(int n);
 cudaError_t launch_or_load(const int* coords, const int* tour, int2* Q, int n, unsigned long long* len, cudaStream_t st);
 size_t oropt_const_entries(int n);
+void or_config(int filter, int naive);
 cudaError_t launch_or_sweep(const int2* Q, int4* CR, int4* CC, int n, unsigned long long* slot, cudaStream_t st);
 cudaError_t launch_or_apply(const int* coords, int* tour, int2* Q, int* span, int n, int i, int j, int type,
                             cudaStream_t st);
@@ -113,6 +114,13 @@ cudaError_t launch_box_cull(const Geometry& g, const float2* P, const int* E, co
 cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles,
                               int ntiles, int grid, Box* rbox, Box* cbox, int4* list, Slot* slot, int respect_done,
                               unsigned long long* tilebest, int flags, cudaStream_t st);
+// Fused incremental culled sweep (after the first iteration of a TILE_BOUNDS = 3 search):
+// dirty tiles enumerated from the last move via tmap, boxes recomputed in place, cull and sweep
+// in one launch of `grid` one-warp CTAs (inc_sweep_grid), clean minima folded into the key.
+int inc_sweep_grid(const Geometry& g);
+cudaError_t launch_inc_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
+                             const int* tmap, int grid, Box* rbox, Box* cbox, Slot* slot, int respect_done,
+                             unsigned long long* tilebest, int flags, cudaStream_t st);
 cudaError_t launch_apply(float2* P, int* E, int* tour, int n, const Slot* in, Slot* out, long long max_moves,
                          int explicit_move, int ei, int ej, unsigned long long* trace, long long trace_cap,
                          int* pos, cudaStream_t st);

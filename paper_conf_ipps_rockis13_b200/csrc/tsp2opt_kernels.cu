@@ -354,6 +354,149 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const flo
 }
 
 // ===========================================================================
+// Fused incremental culled sweep (TSP2OPT_OPT_TILE_BOUNDS = 3, every iteration
+// after the first of a local search).  One launch replaces box + cull + list
+// sweep: the dirty tiles -- those whose row block or column chunk meets the
+// last applied move's [i, j] -- are ENUMERATED from (i, j) by index arithmetic
+// (tmap: (row block, column chunk) -> this shard's tile index, -1 if none), not
+// found by scanning all tiles; the warp that owns a dirty tile recomputes the
+// boxes of its dirty blocks from P / E on the spot (no box kernel, no list),
+// applies the cull test of cull_kernel and, if the tile is kept, sweeps it with
+// its tile-local bound right away (kSweepLocal: the stored minimum stays exact
+// while the tile is clean).  Every CTA also folds a share of the clean tiles'
+// stored minima into the slot key.  Exactness: the same cull condition, the
+// same tile sweep and the same clean / dirty rule as box_kernel + cull_kernel
+// + sweep_list_kernel.
+// ===========================================================================
+__device__ __forceinline__ Box warp_box(const float2* __restrict__ P, const int* __restrict__ E, int k0, int ke)
+{
+    // positions k0..ke (cities), edges k0..ke-1; every lane returns the box
+    int xlo = 1 << 30, xhi = -1, ylo = 1 << 30, yhi = -1, emax = 0;
+    const int lane = threadIdx.x & 31;
+    for (int k = k0 + lane; k <= ke; k += 32) {
+        const float2 p = P[k];
+        const int x = unbias(p.x), y = unbias(p.y);
+        xlo = min(xlo, x);
+        xhi = max(xhi, x);
+        ylo = min(ylo, y);
+        yhi = max(yhi, y);
+        if (k < ke) emax = max(emax, E[k]);
+    }
+    const unsigned full = 0xffffffffu;
+    Box b;
+    b.xlo = __reduce_min_sync(full, xlo);
+    b.xhi = __reduce_max_sync(full, xhi);
+    b.ylo = __reduce_min_sync(full, ylo);
+    b.yhi = __reduce_max_sync(full, yhi);
+    b.emax = __reduce_max_sync(full, emax);
+    b.pad[0] = b.pad[1] = b.pad[2] = 0;
+    return b;
+}
+
+template <int R, bool FIRST>
+__global__ void __launch_bounds__(32, 16) inc_sweep_kernel(const float2* __restrict__ P, const int* __restrict__ E,
+                                                           int n, const int2* __restrict__ tiles, int ntiles,
+                                                           const int* __restrict__ tmap, int TI, int TJ, int nrb,
+                                                           int ncc, Box* __restrict__ rbox, Box* __restrict__ cbox,
+                                                           Slot* __restrict__ slot, int respect_done,
+                                                           unsigned long long* __restrict__ tilebest, int flags)
+{
+    extern __shared__ float4 smem[];
+    const TileSmem sm(smem, TJ);
+    pdl_trigger();
+    pdl_wait();
+    const int done = respect_done ? *(volatile const int*)&slot->done : 0;
+    const int seed_ok = *(volatile const int*)&slot->seed_ok;
+    const unsigned long long mv = *(volatile const unsigned long long*)&slot->last_key;
+    if (done) return;
+    int dlo = 0, dhi = n;  // no valid last move: every tile is dirty
+    if (seed_ok) {
+        dlo = key_i(mv);
+        dhi = key_j(mv);
+    }
+    const int lane = threadIdx.x & 31;
+    // (1) the clean tiles' stored minima (a tile is clean iff neither its row
+    //     range nor its column range meets [dlo, dhi]), one grid-stride pass
+    {
+        unsigned long long m = kKeyNone;
+        constexpr int V = 4;  // loads in flight per lane
+        for (int t0 = blockIdx.x * 32 * V; t0 < ntiles; t0 += gridDim.x * 32 * V) {
+            int2 tl[V];
+            unsigned long long kb[V];
+#pragma unroll
+            for (int v = 0; v < V; v++) {
+                const int t = t0 + v * 32 + lane;
+                tl[v] = t < ntiles ? tiles[t] : make_int2(0, 0);
+                kb[v] = t < ntiles ? tilebest[t] : kKeyNone;
+            }
+#pragma unroll
+            for (int v = 0; v < V; v++) {
+                const bool dirty = (tl[v].x <= dhi && tl[v].x + TI >= dlo) || (tl[v].y <= dhi && tl[v].y + TJ >= dlo);
+                if (!dirty) m = min(m, kb[v]);
+            }
+        }
+        for (int o = 16; o > 0; o >>= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
+        if (lane == 0 && m != kKeyNone && m < *(volatile unsigned long long*)&slot->key) atomicMin(&slot->key, m);
+    }
+    // (2) the dirty tiles: rows [rlo, rhi] x every chunk, then every row block x
+    //     chunks [clo, chi] without the rows already covered
+    const int rlo = max(0, (dlo - TI + TI - 1) >= 0 ? (dlo - TI + TI - 1) / TI : 0), rhi = min(nrb - 1, dhi / TI);
+    const int clo = max(0, (dlo - TJ + TJ - 1) >= 0 ? (dlo - TJ + TJ - 1) / TJ : 0), chi = min(ncc - 1, dhi / TJ);
+    const long long nA = rlo <= rhi ? (long long)(rhi - rlo + 1) * ncc : 0;
+    const long long nB = clo <= chi ? (long long)nrb * (chi - clo + 1) : 0;
+    for (long long u = blockIdx.x; u < nA + nB; u += gridDim.x) {
+        int rb, cc;
+        if (u < nA) {
+            rb = rlo + (int)(u / ncc);
+            cc = (int)(u % ncc);
+        } else {
+            const long long v = u - nA;
+            rb = (int)(v / (chi - clo + 1));
+            cc = clo + (int)(v % (chi - clo + 1));
+            if (rb >= rlo && rb <= rhi) continue;  // already in part A
+        }
+        const int t = tmap[(long long)rb * ncc + cc];
+        if (t < 0) continue;  // below the diagonal, or another rank's tile
+        const bool rdirty = rb >= rlo && rb <= rhi, cdirty = cc >= clo && cc <= chi;
+        Box r, c;
+        if (rdirty) {
+            r = warp_box(P, E, rb * TI, min(rb * TI + TI, n - 1));
+            if (lane == 0) rbox[rb] = r;  // every warp of this row writes the same box
+        } else {
+            r = rbox[rb];
+        }
+        if (cdirty) {
+            c = warp_box(P, E, cc * TJ, min(cc * TJ + TJ, n));
+            if (lane == 0) cbox[cc] = c;
+        } else {
+            c = cbox[cc];
+        }
+        const long long gx = max(0, max(c.xlo - r.xhi, r.xlo - c.xhi));
+        const long long gy = max(0, max(c.ylo - r.yhi, r.ylo - c.yhi));
+        const long long T = (long long)max(r.emax, c.emax) - 1;
+        const bool keep = T >= 0 && gx * gx + gy * gy <= T * T + T;
+        if (keep) {
+            sweep_tile<R, false, FIRST>(P, E, n, make_int2(rb * TI, cc * TJ), TJ, slot, sm, tilebest + t,
+                                        flags | kSweepLocal);
+            __syncthreads();  // before the next tile overwrites the shared chunk
+        } else if (lane == 0) {
+            tilebest[t] = kKeyNone;
+        }
+    }
+}
+
+template <int R, bool FIRST>
+static cudaError_t launch_inc_sweep_t(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles,
+                                      int ntiles, const int* tmap, int grid, Box* rbox, Box* cbox, Slot* slot,
+                                      int respect_done, unsigned long long* tilebest, int flags, cudaStream_t st)
+{
+    const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
+    return launch_kernel_pdl(inc_sweep_kernel<R, FIRST>, dim3(grid), dim3(32), sweep_smem_bytes(g), st, P, E, n,
+                             tiles, ntiles, tmap, TI, g.tj, nrb, ncc, rbox, cbox, slot, respect_done, tilebest,
+                             flags & ~kSweepSeed);
+}
+
+// ===========================================================================
 // a7 + a8: apply the best move of slot_in (or an explicit (i, j)) and write
 // the next iteration's state into slot_out.  Reverses P and tour on [i+1, j]
 // and e on [i+1, j-1]; the two new edges are exact distances of the
@@ -709,6 +852,14 @@ cudaError_t sweep_prepare()
             if (e != cudaSuccess) return e;
         }
         cudaError_t e;
+        if (R == kRowsSmall) {
+            e = cudaFuncSetAttribute(inc_sweep_kernel<kRowsSmall, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)sweep_smem_bytes(gmax));
+            if (e == cudaSuccess)
+                e = cudaFuncSetAttribute(inc_sweep_kernel<kRowsSmall, true>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sweep_smem_bytes(gmax));
+            if (e != cudaSuccess) return e;
+        }
         e = by_rows(R, [&](auto r) {
             return cudaFuncSetAttribute(local_search_kernel<decltype(r)::value>,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sweep_smem_bytes(gmax));
@@ -744,6 +895,33 @@ cudaError_t launch_box_cull(const Geometry& g, const float2* P, const int* E, co
                    tiles, ntiles, TI, g.tj, rbox, cbox, slot, list, tilebest, flags, respect_done, n, 1);
     g_launches += 2;
     return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+cudaError_t launch_inc_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
+                             const int* tmap, int grid, Box* rbox, Box* cbox, Slot* slot, int respect_done,
+                             unsigned long long* tilebest, int flags, cudaStream_t st)
+{
+    if (ntiles <= 0 || grid <= 0) return cudaSuccess;
+    if (g.rows != kRowsSmall || g.warps != 1) return cudaErrorInvalidValue;  // instantiated for R = 7, one warp
+    cudaError_t e = (flags & kSweepFirst)
+                        ? launch_inc_sweep_t<kRowsSmall, true>(g, P, E, n, tiles, ntiles, tmap, grid, rbox, cbox, slot,
+                                                               respect_done, tilebest, flags, st)
+                        : launch_inc_sweep_t<kRowsSmall, false>(g, P, E, n, tiles, ntiles, tmap, grid, rbox, cbox,
+                                                                slot, respect_done, tilebest, flags, st);
+    g_launches += 1;
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+int inc_sweep_grid(const Geometry& g)
+{
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, inc_sweep_kernel<kRowsSmall, false>, 32,
+                                                      sweep_smem_bytes(g)) != cudaSuccess)
+        return 0;
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    return per_sm * sms;
 }
 
 int sweep_list_grid(const Geometry& g, int ntiles)

@@ -21,6 +21,7 @@
 // into a scratch span, then copies it back (two launches, no grid barrier).
 // or_sweep_kernel (one thread per cell) is the first version, kept behind
 // TSP2OPT_OROPT_NAIVE=1.
+#include <atomic>
 #include <climits>
 #include <cstdlib>
 
@@ -382,25 +383,40 @@ cudaError_t launch_or_load(const int* coords, const int* tour, int2* Q, int n, u
     return cudaGetLastError();
 }
 
-static bool or_naive()
-{
-    static const bool v = [] {
-        const char* s = getenv("TSP2OPT_OROPT_NAIVE");
-        return s && s[0] == '1';
-    }();
-    return v;
-}
-
+// Kernel and filter selection of the Or-opt sweep (none changes a result).
+// Defaults come from TSP2OPT_OROPT_NAIVE / TSP2OPT_OROPT_FILTER, read once;
+// tsp2opt_oropt_config overrides them (tests run every mode in one process).
 // The FP32 filter pays from the 128 x 32 tiles up (measured: C3 / C4 sweeps
 // 1.3x / 1.6x faster); the 16-column walks of n <= 2048 re-seed too often.
-// TSP2OPT_OROPT_FILTER=0 / 1 forces it off / on (experiment switch, same result).
+static std::atomic<int> g_or_filter{-2};  // -2 unset, -1 auto (n > 2048), 0 off, 1 on
+static std::atomic<int> g_or_naive{-1};   // -1 unset, 0 tiled kernel, 1 one thread per cell
+
+static bool or_naive()
+{
+    int v = g_or_naive.load();
+    if (v < 0) {
+        const char* s = getenv("TSP2OPT_OROPT_NAIVE");
+        v = (s && s[0] == '1') ? 1 : 0;
+        g_or_naive.store(v);
+    }
+    return v == 1;
+}
+
 static bool or_filter(int n)
 {
-    static const int mode = [] {
+    int m = g_or_filter.load();
+    if (m == -2) {
         const char* s = getenv("TSP2OPT_OROPT_FILTER");
-        return s && (s[0] == '0' || s[0] == '1') ? s[0] - '0' : -1;
-    }();
-    return mode < 0 ? n > 2048 : mode == 1;
+        m = s && (s[0] == '0' || s[0] == '1') ? s[0] - '0' : -1;
+        g_or_filter.store(m);
+    }
+    return m < 0 ? n > 2048 : m == 1;
+}
+
+void or_config(int filter, int naive)
+{
+    g_or_filter.store(filter);
+    g_or_naive.store(naive);
 }
 
 size_t oropt_const_entries(int n) { return (size_t)n; }

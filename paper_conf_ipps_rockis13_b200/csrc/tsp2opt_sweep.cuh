@@ -65,6 +65,7 @@ struct Bound {
     int B;          // accept delta < B (lane-local running bound)
     float Bf;       // B as float (exact)
     float a2f;      // column offset a2 = (B - 2) - a1
+    int a2;
     float srow[R];  // row thresholds: D(i_r, j) <= e_{i_r} + a1  <=>  s <= srow[r]
 };
 
@@ -82,6 +83,7 @@ __device__ __forceinline__ void set_bound(Bound<R>& b, const float* erowf, int B
     const int a1 = (c - 1) >> 1;
     const int a2 = c - 1 - a1;
     b.a2f = (float)a2;
+    b.a2 = a2;
     const float a1f = (float)a1;
 #pragma unroll
     for (int r = 0; r < R; r++) b.srow[r] = sq_threshold(erowf[r] + a1f);
@@ -89,17 +91,35 @@ __device__ __forceinline__ void set_bound(Bound<R>& b, const float* erowf, int B
 
 // Shared memory of one tile: the column chunk (the paper's coordinate range
 // "B", L20 Listing 2) and the edges of the CTA's rows (range "A").
+constexpr int kMaxWarpsPerTile = 4;
+
+// One staged column c = j - J0 is a record of kColRec float4 (48 bytes):
+//   [0] (-x, -x, -y, -y)  biased floats, negated
+//   [1] (e_j, thr_0, thr_1, thr_2), [2] (thr_3, -, -, -)
+// thr_w = sq_threshold(e_j + a2w) is warp w's column threshold (fill_colthr).
+// Interleaving them lets the walk step ONE shared-memory pointer per column
+// (immediate offsets for xy, the next column and the threshold).
+constexpr int kColRec = 3;
+
 struct TileSmem {
-    float4* colxy;  // [TJ + 2]: (-x, -x, -y, -y) of columns J0..J1 and one spare (biased floats)
-    float* cole;    // [TJ + 2]: e_j as float
-    float* rowe;    // [32 * R * warps]: e_i of the CTA's rows, as float
+    float4* col;  // [TJ + 2] column records: columns J0..J1 and one spare
+    float* rowe;  // [32 * R * warps]: e_i of the CTA's rows, as float
     __device__ TileSmem(void* base, int TJ)
-        : colxy(reinterpret_cast<float4*>(base)),
-          cole(reinterpret_cast<float*>(colxy + TJ + 2)),
-          rowe(cole + TJ + 2)
+        : col(reinterpret_cast<float4*>(base)), rowe(reinterpret_cast<float*>(col + kColRec * (TJ + 2)))
     {
     }
+    __device__ float4 xy(int c) const { return col[kColRec * c]; }
+    __device__ float e(int c) const { return reinterpret_cast<const float*>(col + kColRec * c + 1)[0]; }
+    __device__ void put(int c, float2 p, float e) const
+    {
+        col[kColRec * c] = make_float4(-p.x, -p.x, -p.y, -p.y);
+        reinterpret_cast<float*>(col + kColRec * c + 1)[0] = e;
+    }
 };
+
+// Column record accessors for a walk's running pointer (rec = &col[kColRec * c]).
+__device__ __forceinline__ float rec_e(const float4* rec) { return reinterpret_cast<const float*>(rec + 1)[0]; }
+__device__ __forceinline__ float rec_thr(const float4* rec, int w) { return reinterpret_cast<const float*>(rec + 1)[1 + w]; }
 
 // Same as set_bound, from the lane's row edges in shared memory (rare: the
 // bound dropped mid-tile).
@@ -123,7 +143,14 @@ __device__ __forceinline__ bool step_any(const Bound<R>& b, const float (&cur)[R
         bool a0 = m <= scol, a1 = false, a2 = false, a3 = false;
 #pragma unroll
         for (int r = 0; r < R; r++) {
+#ifndef TSP2OPT_ROWTEST_FLOAT
+            // cur >= +0 and srow is either >= +0 or negative (t < 0, sq_threshold), so the
+            // signed integer order of the IEEE bits equals the float order here (ISETP runs
+            // at full rate on the ALU pipe, FSETP at half)
+            const bool t = __float_as_int(cur[r]) <= __float_as_int(b.srow[r]);
+#else
             const bool t = cur[r] <= b.srow[r];
+#endif
             if ((r & 3) == 0) a0 |= t;
             else if ((r & 3) == 1) a1 |= t;
             else if ((r & 3) == 2) a2 |= t;
@@ -199,17 +226,38 @@ __device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1
     }
 }
 
-// Returns true (FIRST only) once some lane of the warp holds an improving
-// pair: every later column has higher cell numbers, so the walk can stop.
+// The column thresholds of this warp's walk, thr_w of columns rec[0 .. count)
+// = sq_threshold(e_j + a2w) with a2w the largest column offset a2 of the
+// warp's lanes: a larger a2 only weakens each lane's necessary condition (its
+// own a1 + a2 >= c - 1 still holds), so one threshold per column serves the
+// whole warp.  Written when the walk starts and again after a lane's bound
+// dropped (rare); it saves the walk four FP32 instructions per column step.
+// Returns a2w.
+__device__ __forceinline__ int fill_colthr(int a2, float4* rec, int w, int count)
+{
+    const int a2w = __reduce_max_sync(0xffffffffu, a2);
+    const float a2wf = (float)a2w;
+    for (int k = (int)(threadIdx.x & 31); k < count; k += 32) {
+        float* r = reinterpret_cast<float*>(rec + kColRec * k + 1);
+        r[1 + w] = sq_threshold(r[0] + a2wf);
+    }
+    __syncwarp();
+    return a2w;
+}
+
+// One column step of the walk at column j, rec = its record.  Returns true
+// (FIRST only) once some lane of the warp holds an improving pair: every later
+// column has higher cell numbers, so the walk can stop.  left = columns from j
+// to the end of the chunk.
 template <int R, bool MASK, bool PS, bool FIRST>
 __device__ __forceinline__ bool column_step(const Rows<R>& rows, Bound<R>& b, const float (&cur)[R + 1],
-                                            float (&nxt)[R + 1], int row0, int j, int J0, const TileSmem& sm,
-                                            const float* my_rowe, const float2* P, unsigned long long& mykey)
+                                            float (&nxt)[R + 1], int row0, int j, float4* rec, int w, int left,
+                                            int& a2w, const float* my_rowe, const float2* P,
+                                            unsigned long long& mykey)
 {
-    const float4 c1 = sm.colxy[j + 1 - J0];
+    const float4 c1 = rec[kColRec];
     column_sq<R>(nxt, rows, c1);
-    const float ej = sm.cole[j - J0];
-    const float scol = sq_threshold(ej + b.a2f);
+    const float scol = rec_thr(rec, w);
     const bool any = step_any<R, MASK>(b, cur, nxt, scol, row0, j);
 #ifdef TSP2OPT_STATS
     if ((threadIdx.x & 31) == 0) atomicAdd(&g_stats[0], 1ULL);
@@ -219,13 +267,13 @@ __device__ __forceinline__ bool column_step(const Rows<R>& rows, Bound<R>& b, co
         if ((threadIdx.x & 31) == 0) atomicAdd(&g_stats[1], 1ULL);
 #endif
         const int B0 = b.B;
-        if (any)
-            exact_step<R, MASK, PS, FIRST>(b, cur, nxt, scol, row0, j, sm.colxy[j - J0], c1, ej, my_rowe, P, mykey);
+        if (any) exact_step<R, MASK, PS, FIRST>(b, cur, nxt, scol, row0, j, rec[0], c1, rec_e(rec), my_rowe, P, mykey);
         if (FIRST) return __any_sync(0xffffffffu, mykey != kKeyNone);
         // share the warp's best: a lane may accept delta <= (best of another lane)
         const int wb = __reduce_min_sync(0xffffffffu, b.B);
         const int nb = min(b.B, wb + 1);
         if (nb < B0) reset_bound<R>(b, my_rowe, nb);
+        if (__reduce_max_sync(0xffffffffu, b.a2) != a2w) a2w = fill_colthr(b.a2, rec + kColRec, w, left - 1);
     }
     return false;
 }
@@ -235,14 +283,19 @@ __device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0,
                                      const TileSmem& sm, const float* my_rowe, const float2* P,
                                      unsigned long long& mykey)
 {
+    const int w = threadIdx.x >> 5;
+    float4* rec = sm.col + kColRec * (jstart - J0);
+    int a2w = fill_colthr(b.a2, rec, w, J1 - jstart);
     float sa[R + 1], sb[R + 1];
-    column_sq<R>(sa, rows, sm.colxy[jstart - J0]);
+    column_sq<R>(sa, rows, rec[0]);
     int j = jstart;
-    for (; j + 1 < J1; j += 2) {
-        if (column_step<R, MASK, PS, FIRST>(rows, b, sa, sb, row0, j, J0, sm, my_rowe, P, mykey)) return;
-        if (column_step<R, MASK, PS, FIRST>(rows, b, sb, sa, row0, j + 1, J0, sm, my_rowe, P, mykey)) return;
+    for (; j + 1 < J1; j += 2, rec += 2 * kColRec) {
+        if (column_step<R, MASK, PS, FIRST>(rows, b, sa, sb, row0, j, rec, w, J1 - j, a2w, my_rowe, P, mykey)) return;
+        if (column_step<R, MASK, PS, FIRST>(rows, b, sb, sa, row0, j + 1, rec + kColRec, w, J1 - j - 1, a2w, my_rowe,
+                                            P, mykey))
+            return;
     }
-    if (j < J1) column_step<R, MASK, PS, FIRST>(rows, b, sa, sb, row0, j, J0, sm, my_rowe, P, mykey);
+    if (j < J1) column_step<R, MASK, PS, FIRST>(rows, b, sa, sb, row0, j, rec, w, J1 - j, a2w, my_rowe, P, mykey);
 }
 
 // Tile-level form of the same exact necessary condition (a bound on all of the
@@ -273,12 +326,12 @@ __device__ __forceinline__ bool tile_may_pass(const Rows<R>& rows, const Bound<R
     // column cities are staged negated: colxy = (-x, -x, -y, -y)
     float cxlo = 3.0e38f, cxhi = -3.0e38f, cylo = 3.0e38f, cyhi = -3.0e38f, emax = -1.0f;
     for (int c = cbeg + (int)(threadIdx.x & 31); c <= cend; c += 32) {
-        const float4 v = sm.colxy[c];
+        const float4 v = sm.xy(c);
         cxlo = fminf(cxlo, -v.x);
         cxhi = fmaxf(cxhi, -v.x);
         cylo = fminf(cylo, -v.z);
         cyhi = fmaxf(cyhi, -v.z);
-        if (c < cend) emax = fmaxf(emax, sm.cole[c]);  // e_j of the step's own column j < J1
+        if (c < cend) emax = fmaxf(emax, sm.e(c));  // e_j of the step's own column j < J1
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
@@ -304,7 +357,7 @@ __device__ __forceinline__ bool tile_may_pass(const Rows<R>& rows, const Bound<R
 // Shared memory bytes of a tile with TJ columns and TI rows.
 __host__ __device__ inline size_t tile_smem_bytes(int TJ, int TI)
 {
-    return (size_t)(TJ + 2) * (sizeof(float4) + sizeof(float)) + (size_t)TI * sizeof(float);
+    return (size_t)(TJ + 2) * kColRec * sizeof(float4) + (size_t)TI * sizeof(float);
 }
 
 // One tile.  All global loads of the tile (the lane's rows and row edges, the
@@ -314,7 +367,6 @@ __host__ __device__ inline size_t tile_smem_bytes(int TJ, int TI)
 // minima are published with one atomicMin each (L16 Fig. 4 "Get best local
 // pair ... Get best global pair"; min is order-independent, so the result is
 // deterministic).  The caller synchronises the CTA before reusing `sm`.
-constexpr int kMaxWarpsPerTile = 4;
 
 template <int R, bool PS, bool FIRST = false>
 __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n, int2 tile, int TJ, Slot* slot,
@@ -345,8 +397,7 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     for (int c = threadIdx.x; c <= ncol + 1; c += blockDim.x) {  // J1 <= n: P[n] = P[0]; + 1 spare column
         const float2 p = gld<PS>(P + J0 + c);
         const int e = gld<PS>(E + J0 + c);
-        sm.colxy[c] = make_float4(-p.x, -p.x, -p.y, -p.y);
-        sm.cole[c] = (float)e;
+        sm.put(c, p, (float)e);
     }
     // The slot key is the seed (0, cell 0) or a real pair of this sweep, so a
     // pair of ours can only win with delta < 0 (key delta 0) or delta <= key delta.

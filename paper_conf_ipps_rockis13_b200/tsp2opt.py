@@ -71,6 +71,7 @@ def _L():
             "tsp2opt_batch_ils_async": ([P, I32, I32, P, I64, P, P, P, P], I32),
             "tsp2opt_oropt_local_search": ([P, I32, P, I64, pI64, pI64, P, I64], I32),
             "tsp2opt_oropt_best_move": ([P, I32, P, pI32, pI32, pI32, pI32], I32),
+            "tsp2opt_oropt_config": ([I32, I32], I32),
             "tsp2opt_plan_shard": ([I32, I32, I32, pI32, pI32, pI32, P, I64, pI64, pI64], I32),
             "tsp2opt_get_geometry": ([P, pI32, pI32, pI32, pI64, pI64], I32),
             "tsp2opt_selftest": ([pI64, pI64, pI64, pI64], I32),
@@ -234,6 +235,12 @@ def oropt_local_search(coords, tour, max_iters: int | None = None, trace_cap: in
                                                 _ptr(tr) if trace_cap > 0 else None, int(trace_cap)),
                 "tsp2opt_oropt_local_search")
     return dict(tour=t, length=L.value, iterations=it.value, status=st, trace=tr[: min(it.value, trace_cap)].copy())
+
+
+def oropt_config(filter: int = -1, naive: int = 0) -> None:
+    """Or-opt kernel selection (no result depends on it): filter -1 by size, 0 off, 1 on;
+    naive 1 selects the one-thread-per-cell kernel."""
+    _check(_L().tsp2opt_oropt_config(int(filter), int(naive)), "tsp2opt_oropt_config")
 
 
 def oropt_best_move(coords, tour):

@@ -71,7 +71,7 @@ def main():
     ap.add_argument("--coords", default=None)
     ap.add_argument("--tour", default=None)
     ap.add_argument("--seed", type=int, default=None)
-    ap.add_argument("--variant", default="2opt")
+    ap.add_argument("--variant", default="2opt", help="comma-separated list")
     a = ap.parse_args()
     c = dict(inputs.CONFIGS[a.config])
     kind = a.coords or c["coords"]
@@ -81,17 +81,17 @@ def main():
     t0 = time.time()
     tour = start_tour(tk, coords, seed)
     t_start = time.time() - t0
-    t0 = time.time()
-    res = run(a.variant, coords, tour)
-    dt = time.time() - t0
-    out = golden_path(a.config, kind, tk, seed, a.variant)
-    np.savez_compressed(out, start=tour, tour=res["tour"], length=res["length"], iterations=res["iterations"],
-                        status=res["status"], trace=res["trace"].astype(np.int64),
-                        oracle_seconds=dt, start_seconds=t_start, oracle_threads=oracle.num_threads(),
-                        variant=a.variant)
-    print(out, res["length"], res["iterations"], f"{dt:.1f}s (start {t_start:.1f}s)", oracle.num_threads(),
-          "threads", flush=True)
-
+    print(f"{a.config} {tk} start: {t_start:.1f}s", flush=True)
+    for variant in a.variant.split(","):
+        t0 = time.time()
+        res = run(variant, coords, tour)
+        dt = time.time() - t0
+        out = golden_path(a.config, kind, tk, seed, variant)
+        np.savez_compressed(out, start=tour, tour=res["tour"], length=res["length"], iterations=res["iterations"],
+                            status=res["status"], trace=res["trace"].astype(np.int64),
+                            oracle_seconds=dt, start_seconds=t_start, oracle_threads=oracle.num_threads(),
+                            variant=variant)
+        print(out, res["length"], res["iterations"], f"{dt:.1f}s", oracle.num_threads(), "threads", flush=True)
 
 if __name__ == "__main__":
     main()

@@ -74,3 +74,62 @@ def test_oropt_local_search_c2_hilbert(gpu):
     assert (got["status"], got["iterations"], got["length"]) == (ref["status"], ref["iterations"], ref["length"])
     assert np.array_equal(got["tour"], ref["tour"])
     assert np.array_equal(got["trace"].astype(np.int64), ref["trace"])
+
+
+@pytest.fixture
+def or_mode():
+    """Select the Or-opt kernel for one test (tsp2opt_oropt_config), then restore the default."""
+    yield tsp2opt.oropt_config
+    tsp2opt.oropt_config(-1, 0)
+
+
+@pytest.mark.parametrize("filt", [0, 1])
+@pytest.mark.parametrize("kind,n,seed,start", [("uniform", 300, 1, "random"), ("lattice", 700, 2, "random"),
+                                               ("uniform", 1002, 3, "hilbert"), ("lattice", 2500, 4, "hilbert"),
+                                               ("uniform", 2049, 5, "hilbert")])
+def test_oropt_local_search_filter_modes(gpu, or_mode, filt, kind, n, seed, start):
+    """The whole local search -- every move down to the local minimum, where the deltas
+    approach 0 and the FP32 filter's margin matters most -- with the filter forced off
+    and on, on both sides of the n > 2048 default switch."""
+    or_mode(filt, 0)
+    c = inputs.make_coords(kind, n, seed)
+    t0 = inputs.make_tour(start, c, seed)
+    ref = oracle.local_search_or(c, t0, trace_cap=100_000)
+    got = tsp2opt.oropt_local_search(c, t0, trace_cap=100_000)
+    assert (got["status"], got["iterations"], got["length"]) == (ref["status"], ref["iterations"], ref["length"])
+    assert np.array_equal(got["trace"].astype(np.int64), ref["trace"])
+    assert np.array_equal(got["tour"], ref["tour"])
+
+
+def test_oropt_naive_kernel_mode(gpu, or_mode):
+    or_mode(-1, 1)
+    c = inputs.make_coords("lattice", 400, 9)
+    t0 = inputs.random_tour(400, 9)
+    ref = oracle.local_search_or(c, t0, trace_cap=100_000)
+    got = tsp2opt.oropt_local_search(c, t0, trace_cap=100_000)
+    assert np.array_equal(got["trace"].astype(np.int64), ref["trace"]) and np.array_equal(got["tour"], ref["tour"])
+
+
+def test_oropt_config_errors(gpu):
+    for bad in ((-2, 0), (2, 0), (0, 2), (0, -1)):
+        with pytest.raises(tsp2opt.TSP2OptError):
+            tsp2opt.oropt_config(*bad)
+
+
+@pytest.mark.parametrize("filt", [-1, 0])
+def test_oropt_c3_hilbert_golden(gpu, or_mode, filt):
+    """pla7397-shaped C3 from the Hilbert start -- the bench's Or-opt workload -- in the
+    default mode (FP32 filter, n > 2048) and the exact walk: every move, the final tour,
+    length and move count equal the committed golden (plain oracle, make_golden.py)."""
+    import os
+    path = os.path.join(os.path.dirname(__file__), "golden", "ls_oropt_C3_lattice_hilbert_s1.npz")
+    gold = np.load(path)
+    or_mode(filt, 0)
+    c, _ = inputs.config_instance("C3")
+    t0 = inputs.hilbert_tour(c)
+    assert np.array_equal(gold["start"], t0)
+    k = int(gold["iterations"])
+    got = tsp2opt.oropt_local_search(c, t0, trace_cap=k + 10)
+    assert (got["status"], got["iterations"], got["length"]) == (0, k, int(gold["length"]))
+    assert np.array_equal(got["trace"].astype(np.int64), gold["trace"][:k])
+    assert np.array_equal(got["tour"], gold["tour"])

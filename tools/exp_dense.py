@@ -13,7 +13,8 @@ import time
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ipps_rockis13_b200 import inputs, tsp2opt  # noqa: E402
 
-out = {"label": sys.argv[1] if len(sys.argv) > 1 else "default", "lib": os.path.basename(tsp2opt.LIB)}
+out = {"label": sys.argv[1] if len(sys.argv) > 1 else "default", "lib": os.path.basename(tsp2opt.LIB),
+       "env": {k: v for k, v in os.environ.items() if k.startswith("TSP2OPT_") and k != "TSP2OPT_LIB"}}
 for cfg in ("C5", "C4"):
     c, t = inputs.config_instance(cfg, "random")
     n = len(t)

@@ -11,6 +11,7 @@
 #   launches:NAME:CMD     ncu launch list (gpu__time_duration) of CMD (commas for spaces) -> NAME.csv/.txt
 #   ncu:NAME:REGEX:CMD    ncu --set full of the first REGEX launch after one skip -> NAME.ncu-rep + .txt
 #   py:CMD                any python command (commas for spaces)
+#   env:K=V               export K=V for the tasks that follow
 cd "$(dirname "$0")/.."
 mkdir -p gpurun_out
 for task in "$@"; do
@@ -36,6 +37,7 @@ for task in "$@"; do
     ncu) name="${arg%%:*}"; rest="${arg#*:}"; rx="${rest%%:*}"; cmd="${rest#*:}"
            timeout 1800 ncu --set full --clock-control none --import-source on -k regex:$rx -s 1 -c 1 -o gpurun_out/$name -f ${cmd//,/ } > gpurun_out/$name.log 2>&1
            echo "ncu $name rc=$?"; python tools/ncu_summary.py gpurun_out/$name.ncu-rep > gpurun_out/$name.txt 2>&1;;
+    env) export "$arg"; echo "env $arg";;
     py) timeout 2400 python ${arg//,/ } 2>&1 | tail -40; echo "py rc=${PIPESTATUS[0]}";;
     *) echo "unknown task $task";;
   esac
