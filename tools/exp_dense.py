@@ -28,14 +28,23 @@ for cfg in ("C5", "C4"):
         out[f"{cfg}_dense_ms"] = round(ms / k, 4)
         out[f"{cfg}_Tpairs"] = round(n * (n - 1) / 2 / (ms / k) / 1e9, 4)
         out[f"{cfg}_move"] = mv
-for cfg, tk in (("C3", "random"), ("C5", "hilbert")):
+for cfg, tk in (("C3", "random"), ("C4", "hilbert"), ("C5", "hilbert"), ("C5", "mf")):
     if os.environ.get("EXP_NO_LS"):
         break
-    c, t = inputs.config_instance(cfg, tk)
+    c, t = inputs.config_instance(cfg, "random" if tk == "mf" else tk)
     with tsp2opt.TSP2Opt(c) as g:
-        g.local_search(t, max_iters=3)
-        t0 = time.perf_counter()
-        r = g.local_search(t)
-        out[f"LS_{cfg}_{tk}_s"] = round(time.perf_counter() - t0, 4)
+        if tk == "mf":
+            g.mf_tour()
+            g.local_search_current(max_iters=3)
+            g.mf_tour()
+            t0 = time.perf_counter()
+            r = g.local_search_current()
+        else:
+            g.local_search(t, max_iters=3)
+            t0 = time.perf_counter()
+            r = g.local_search(t)
+        dt = time.perf_counter() - t0
+        out[f"LS_{cfg}_{tk}_s"] = round(dt, 4)
+        out[f"LS_{cfg}_{tk}_us_per_move"] = round(1e6 * dt / max(1, r["iterations"]), 2)
         out[f"LS_{cfg}_{tk}"] = [r["iterations"], r["length"]]
 print(json.dumps(out), flush=True)
