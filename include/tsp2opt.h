@@ -74,6 +74,31 @@ int tsp2opt_create_sharded(const int32_t *coords_xy, int32_t n, int32_t rank, in
 /* Write an NCCL unique id (TSP2OPT_NCCL_ID_BYTES bytes) into out. */
 int tsp2opt_nccl_unique_id(void *out);
 
+/* Sharded handle whose per-sweep allreduce-min (L18
+ * §VI "dividing the 2-opt task between multiple devices") runs over PEER
+ * MEMORY instead of NCCL: each rank's key is stored into every other rank's
+ * mailbox (CUDA IPC mapping: NVLink / NVSwitch peer memory across GPUs, the
+ * same HBM for ranks sharing a GPU) and each rank takes the minimum of what
+ * arrived -- one 32-thread kernel per sweep, no NCCL.  Same tiling, results
+ * and call discipline as tsp2opt_create_sharded.  1 <= world <=
+ * TSP2OPT_P2P_MAX_WORLD.  The handle is unusable (ESTATE) until every rank
+ * has called tsp2opt_p2p_connect with all ranks' exported mailboxes.
+ * A rank that stops issuing sweeps makes its peers' exchange time out after
+ * about 30 s: the call returns ECUDA and the handle must be destroyed. */
+#define TSP2OPT_P2P_MAX_WORLD 8
+#define TSP2OPT_P2P_HANDLE_BYTES 64
+int tsp2opt_create_sharded_p2p(const int32_t *coords_xy, int32_t n, int32_t rank, int32_t world, tsp2opt_t *out);
+
+/* Export this rank's mailbox (a cudaIpcMemHandle_t, TSP2OPT_P2P_HANDLE_BYTES
+ * bytes) into out; the caller all-gathers the world exports in rank order. */
+int tsp2opt_p2p_export(tsp2opt_t h, void *out);
+
+/* Map the other ranks' mailboxes: handles = world * TSP2OPT_P2P_HANDLE_BYTES
+ * bytes in rank order (this rank's own entry is ignored).  EINVAL for a
+ * handle not created by tsp2opt_create_sharded_p2p, ESTATE if already
+ * connected, ECUDA if a mailbox cannot be mapped (nothing stays mapped). */
+int tsp2opt_p2p_connect(tsp2opt_t h, const void *handles);
+
 /* Release all device memory, streams, graphs and the NCCL communicator. */
 void tsp2opt_destroy(tsp2opt_t h);
 

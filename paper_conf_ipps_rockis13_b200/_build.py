@@ -14,7 +14,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libtsp2opt.so")
-SOURCES = [os.path.join(CSRC, f) for f in ("tsp2opt_kernels.cu", "tsp2opt_batch.cu", "tsp2opt_mf.cu", "tsp2opt_pruned.cu", "tsp2opt_sweep25.cu", "tsp2opt_oropt.cu",
+SOURCES = [os.path.join(CSRC, f) for f in ("tsp2opt_kernels.cu", "tsp2opt_batch.cu", "tsp2opt_mf.cu", "tsp2opt_pruned.cu", "tsp2opt_sweep25.cu", "tsp2opt_oropt.cu", "tsp2opt_p2p.cu",
                                                     "tsp2opt_api.cu")]
 HEADERS = [os.path.join(CSRC, f) for f in ("tsp2opt_device.cuh", "tsp2opt_internal.h", "tsp2opt_sweep.cuh")] + [
     os.path.join(ROOT, "include", "tsp2opt.h")

@@ -113,6 +113,12 @@ struct tsp2opt_ctx {
     int ntiles = 0;               // tiles of this shard
     long long shard_pairs = 0;
     ncclComm_t comm = nullptr;
+    // peer-memory exchange (tsp2opt_create_sharded_p2p): own mailbox, the peers' mapped ones
+    bool p2p = false;
+    bool p2p_ready = false;
+    Mailbox* d_mbox = nullptr;
+    Mailbox** d_peers = nullptr;           // [world] device array of mailbox pointers (own at [rank])
+    std::vector<void*> p2p_opened;         // peers' mailboxes opened with cudaIpcOpenMemHandle
     bool profiling = false;
     std::vector<cudaEvent_t> ev_pool;  // pairs (start, stop) of recorded sweep launches
     size_t ev_used = 0;
@@ -226,6 +232,10 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
         std::vector<Tile> mine = shard_tiles(h->all_ctiles, rank, world, &unused);
         for (size_t k = 0; k < mine.size(); k++) map[(size_t)(mine[k].i0 / TI) * ncc + mine[k].j0 / TJ] = (int)k;
         cudaFree(h->d_tmap);
+    for (void* p : h->p2p_opened)
+        if (p) cudaIpcCloseMemHandle(p);
+    cudaFree(h->d_peers);
+    cudaFree(h->d_mbox);
         h->d_tmap = nullptr;
         CUDA_TRY(cudaMalloc(&h->d_tmap, sizeof(int) * map.size()));
         CUDA_TRY(cudaMemcpy(h->d_tmap, map.data(), sizeof(int) * map.size(), cudaMemcpyHostToDevice));
@@ -263,6 +273,10 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_ctilebest);
     cudaFree(h->d_list);
     cudaFree(h->d_tmap);
+    for (void* p : h->p2p_opened)
+        if (p) cudaIpcCloseMemHandle(p);
+    cudaFree(h->d_peers);
+    cudaFree(h->d_mbox);
     cudaFree(h->d_rbox);
     cudaFree(h->d_cbox);
     cudaFree(h->d_trace);
@@ -303,6 +317,10 @@ int read_slot(tsp2opt_ctx* h)
 {
     CUDA_TRY(cudaMemcpyAsync(h->h_slot, h->d_slots + h->parity, sizeof(Slot), cudaMemcpyDeviceToHost, h->stream));
     CUDA_TRY(cudaStreamSynchronize(h->stream));
+    if (h->h_slot->done & kDoneExchangeTimeout) {
+        g_last_error = "peer-memory exchange timed out (a rank stopped issuing sweeps)";
+        return TSP2OPT_ECUDA;
+    }
     if (h->h_slot->done & 4) {
         h->has_tour = false;
         g_last_error = "device tour is not a permutation";
@@ -343,6 +361,10 @@ int sweep_flags(const tsp2opt_ctx* h)
 // One iteration: sweep (a4/a5) -> allreduce-min (a6) -> apply (a7/a8).
 int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
 {
+    if (h->p2p && !h->p2p_ready) {
+        g_last_error = "peer-memory handle used before tsp2opt_p2p_connect";
+        return TSP2OPT_ESTATE;
+    }
     Slot* in = h->d_slots + h->parity;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     if (h->profiling) {
@@ -403,6 +425,8 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
     if (h->comm) {
         ncclResult_t r = ncclAllReduce(&in->key, &in->key, 1, ncclUint64, ncclMin, h->comm, h->stream);
         if (r != ncclSuccess) return nccl_fail(r, "ncclAllReduce");
+    } else if (h->p2p) {
+        CUDA_TRY(launch_p2p_min(in, h->d_peers, h->rank, h->world, apply ? 1 : 0, h->stream));
     }
     // first improvement: the min carries the marker delta; the exact delta of the winner
     if (h->first) CUDA_TRY(launch_first_fix(h->d_P, h->d_E, in, apply ? 1 : 0, h->stream));
@@ -442,7 +466,7 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
     // n ~ 7e3 where the per-sweep kernels pack tiles better); TSP2OPT_PERSISTENT
     // = 0 / 1 forces either loop, 2 (default) chooses by pair count.
     const bool use_persistent =
-        !h->comm && h->nbr_k == 0 && !h->or25 && !h->first && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
+        !h->comm && !h->p2p && h->nbr_k == 0 && !h->or25 && !h->first && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
     if (use_persistent) {
         h->inc_valid = false;
         // One persistent cooperative launch runs sweep -> apply to the local
@@ -528,13 +552,14 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
     return (h->h_slot->done & 3) == 2 ? TSP2OPT_MAXITER : TSP2OPT_OK;
 }
 
-int create_common(const int32_t* xy, int32_t n, int rank, int world, const void* nccl_id, tsp2opt_t* out)
+int create_common(const int32_t* xy, int32_t n, int rank, int world, const void* nccl_id, bool p2p, tsp2opt_t* out)
 {
     if (!out) return TSP2OPT_EINVAL;
     *out = nullptr;
     int rc = validate_coords(xy, n);
     if (rc) return rc;
-    if (world < 1 || rank < 0 || rank >= world || (world > 1 && !nccl_id)) return TSP2OPT_EINVAL;
+    if (world < 1 || rank < 0 || rank >= world || (world > 1 && !nccl_id && !p2p)) return TSP2OPT_EINVAL;
+    if (p2p && (nccl_id || world > kP2PMaxWorld)) return TSP2OPT_EINVAL;
     tsp2opt_ctx* h = new tsp2opt_ctx();
     h->n = n;
     h->rank = rank;
@@ -608,7 +633,13 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     }
     rc = upload_shard(h, rank, world);
     if (rc) return fail(rc);
-    if (world > 1 || nccl_id) {  // world 1 with an id: a one-rank communicator (the sharded path on one GPU)
+    if (p2p) {  // peer-memory exchange: the mailbox now, the peers at tsp2opt_p2p_connect
+        h->p2p = true;
+        CTRY(cudaMalloc(&h->d_mbox, sizeof(Mailbox)));
+        CTRY(cudaMemset(h->d_mbox, 0, sizeof(Mailbox)));
+        CTRY(cudaMalloc(&h->d_peers, sizeof(Mailbox*) * kP2PMaxWorld));
+        CTRY(cudaDeviceSynchronize());
+    } else if (world > 1 || nccl_id) {  // world 1 with an id: a one-rank communicator (the sharded path on one GPU)
         ncclUniqueId id;
         memcpy(&id, nccl_id, sizeof(id));
         ncclResult_t r = ncclCommInitRank(&h->comm, world, id, rank);
@@ -628,13 +659,13 @@ extern "C" {
 
 int tsp2opt_create(const int32_t* coords_xy, int32_t n, tsp2opt_t* out)
 {
-    return create_common(coords_xy, n, 0, 1, nullptr, out);
+    return create_common(coords_xy, n, 0, 1, nullptr, false, out);
 }
 
 int tsp2opt_create_sharded(const int32_t* coords_xy, int32_t n, int32_t rank, int32_t world, const void* nccl_id,
                            tsp2opt_t* out)
 {
-    return create_common(coords_xy, n, rank, world, nccl_id, out);
+    return create_common(coords_xy, n, rank, world, nccl_id, false, out);
 }
 
 int tsp2opt_nccl_unique_id(void* out)
@@ -645,6 +676,47 @@ int tsp2opt_nccl_unique_id(void* out)
     ncclResult_t r = ncclGetUniqueId(&id);
     if (r != ncclSuccess) return nccl_fail(r, "ncclGetUniqueId");
     memcpy(out, &id, sizeof(id));
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_create_sharded_p2p(const int32_t* coords_xy, int32_t n, int32_t rank, int32_t world, tsp2opt_t* out)
+{
+    return create_common(coords_xy, n, rank, world, nullptr, true, out);
+}
+
+int tsp2opt_p2p_export(tsp2opt_t h, void* out)
+{
+    if (!h || !out || !h->p2p) return TSP2OPT_EINVAL;
+    cudaIpcMemHandle_t m;
+    CUDA_TRY(cudaIpcGetMemHandle(&m, h->d_mbox));
+    memcpy(out, &m, sizeof(m));
+    return TSP2OPT_OK;
+}
+
+int tsp2opt_p2p_connect(tsp2opt_t h, const void* handles)
+{
+    if (!h || !handles || !h->p2p) return TSP2OPT_EINVAL;
+    if (h->p2p_ready) return TSP2OPT_ESTATE;
+    std::vector<Mailbox*> peers(kP2PMaxWorld, nullptr);
+    for (int r = 0; r < h->world; r++) {
+        if (r == h->rank) {
+            peers[r] = h->d_mbox;
+            continue;
+        }
+        cudaIpcMemHandle_t m;
+        memcpy(&m, (const char*)handles + (size_t)r * sizeof(cudaIpcMemHandle_t), sizeof(m));
+        void* p = nullptr;
+        const cudaError_t e = cudaIpcOpenMemHandle(&p, m, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) {
+            for (void* q : h->p2p_opened) cudaIpcCloseMemHandle(q);
+            h->p2p_opened.clear();
+            return cuda_fail(e, "cudaIpcOpenMemHandle");
+        }
+        h->p2p_opened.push_back(p);
+        peers[r] = (Mailbox*)p;
+    }
+    CUDA_TRY(cudaMemcpy(h->d_peers, peers.data(), sizeof(Mailbox*) * kP2PMaxWorld, cudaMemcpyHostToDevice));
+    h->p2p_ready = true;
     return TSP2OPT_OK;
 }
 

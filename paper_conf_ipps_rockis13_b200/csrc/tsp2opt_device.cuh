@@ -273,13 +273,26 @@ struct __align__(64) Slot {
     unsigned long long last_key;  // key of the most recent finished sweep
     long long moves;              // moves applied since the tour was loaded
     long long length;             // current tour length (int64: n * 46340 > 2^31)
-    int done;                     // 0 running, 1 local minimum, 2 capped, bit 2 (4): invalid tour
+    int done;                     // 0 running, 1 local minimum, 2 capped, bit 2 (4): invalid tour,
+                                  // bit 3 (8): peer exchange timed out
     unsigned next_tile;           // culled sweep: next entry of the kept-tile list to claim
     int seed_ok;                  // 1: last_key is the move just applied to the tour the tile minima of the
                                   //    previous sweep were measured on (they may seed this sweep)
     unsigned ncull;               // culled sweep: number of kept tiles in the list
     int mtype;                    // 2.5-opt: type of the move last applied / decided (reading R19)
     int pad[3];
+};
+
+// Slot::done bit set when a peer-memory exchange timed out (tsp2opt_p2p.cu).
+constexpr int kDoneExchangeTimeout = 8;
+
+// Peer-memory exchange of the per-sweep key (tsp2opt_p2p.cu): written by the
+// peers, polled by the owner; [parity][source rank].
+constexpr int kP2PMaxWorld = 8;
+struct __align__(64) Mailbox {
+    unsigned long long key[2][kP2PMaxWorld];
+    unsigned long long seq[2][kP2PMaxWorld];
+    unsigned long long counter;  // exchanges completed by the owner
 };
 
 // Software grid barrier for co-resident grids (cooperative launches): arrive

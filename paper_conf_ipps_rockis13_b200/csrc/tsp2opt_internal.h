@@ -128,6 +128,10 @@ cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour,
                                 Slot* slots, int parity, long long max_moves, long long budget, unsigned* bar,
                                 int* ctl, unsigned long long* tilebest, int flags, unsigned long long* trace,
                                 long long trace_cap, cudaStream_t st);
+// Allreduce-min of the slot key over peer-memory mailboxes (tsp2opt_p2p.cu): peers[r] = rank r's
+// mailbox mapped into this process (peers[rank] = the own one).
+cudaError_t launch_p2p_min(Slot* slot, Mailbox* const* peers, int rank, int world, int respect_done,
+                           cudaStream_t st);
 cudaError_t read_stats(long long* out4, int reset);
 cudaError_t run_selftest_sqrt(double* max_rel, int* zero_ok);
 cudaError_t run_selftest(long long* out4);  // dist_bad, filter_bad, first bad s, first bad dx<<15|dy

@@ -278,6 +278,38 @@ __device__ __forceinline__ bool column_step(const Rows<R>& rows, Bound<R>& b, co
     return false;
 }
 
+// The rare path of column step j for the grouped walk below: the step's
+// squared distances are recomputed from the lane's rows and the column records
+// (the walk's arrays have moved on), then exactly as column_step's rare branch.
+template <int R, bool MASK, bool PS, bool FIRST>
+__device__ __forceinline__ bool rare_step(const Rows<R>& rows, Bound<R>& b, int row0, int j, float4* rec, int w,
+                                          int left, int& a2w, const float* my_rowe, const float2* P,
+                                          unsigned long long& mykey)
+{
+    float cur[R + 1], nxt[R + 1];
+    column_sq<R>(cur, rows, rec[0]);
+    const float4 c1 = rec[kColRec];
+    column_sq<R>(nxt, rows, c1);
+    const float scol = rec_thr(rec, w);
+    const bool any = step_any<R, MASK>(b, cur, nxt, scol, row0, j);
+    if (!__any_sync(0xffffffffu, any)) return false;
+#ifdef TSP2OPT_STATS
+    if ((threadIdx.x & 31) == 0) atomicAdd(&g_stats[1], 1ULL);
+#endif
+    const int B0 = b.B;
+    if (any) exact_step<R, MASK, PS, FIRST>(b, cur, nxt, scol, row0, j, rec[0], c1, rec_e(rec), my_rowe, P, mykey);
+    if (FIRST) return __any_sync(0xffffffffu, mykey != kKeyNone);
+    const int wb = __reduce_min_sync(0xffffffffu, b.B);
+    const int nb = min(b.B, wb + 1);
+    if (nb < B0) reset_bound<R>(b, my_rowe, nb);
+    if (__reduce_max_sync(0xffffffffu, b.a2) != a2w) a2w = fill_colthr(b.a2, rec + kColRec, w, left - 1);
+    return false;
+}
+
+#ifndef TSP2OPT_VOTE_STEPS
+#define TSP2OPT_VOTE_STEPS 2  // column steps per warp vote (even; 1 = a vote every step)
+#endif
+
 template <int R, bool MASK, bool PS, bool FIRST>
 __device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0, int jstart, int J0, int J1,
                                      const TileSmem& sm, const float* my_rowe, const float2* P,
@@ -289,6 +321,34 @@ __device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0,
     float sa[R + 1], sb[R + 1];
     column_sq<R>(sa, rows, rec[0]);
     int j = jstart;
+    constexpr int V = TSP2OPT_VOTE_STEPS;
+    static_assert(V == 1 || V % 2 == 0, "grouped steps keep sa as the next group's current column");
+    if constexpr (V > 1) {
+        // V column steps per warp vote: one straight-line region of V steps for the
+        // scheduler and one VOTE + branch per group; a group with a candidate re-runs
+        // its steps one by one on the rare path (rare_step), in increasing cell order.
+        for (; j + V <= J1; j += V, rec += V * kColRec) {
+            bool any = false;
+#pragma unroll
+            for (int v = 0; v < V; v++) {
+                float(&cur)[R + 1] = (v & 1) ? sb : sa;
+                float(&nxt)[R + 1] = (v & 1) ? sa : sb;
+                column_sq<R>(nxt, rows, rec[(v + 1) * kColRec]);
+                any |= step_any<R, MASK>(b, cur, nxt, rec_thr(rec + v * kColRec, w), row0, j + v);
+            }
+#ifdef TSP2OPT_STATS
+            if ((threadIdx.x & 31) == 0) atomicAdd(&g_stats[0], (unsigned long long)V);
+#endif
+            if (__builtin_expect(__any_sync(0xffffffffu, any), 0)) {
+#pragma unroll 1
+                for (int v = 0; v < V; v++)
+                    if (rare_step<R, MASK, PS, FIRST>(rows, b, row0, j + v, rec + v * kColRec, w, J1 - j - v, a2w,
+                                                      my_rowe, P, mykey))
+                        return;
+                column_sq<R>(sa, rows, rec[V * kColRec]);  // the next group's current column
+            }
+        }
+    }
     for (; j + 1 < J1; j += 2, rec += 2 * kColRec) {
         if (column_step<R, MASK, PS, FIRST>(rows, b, sa, sb, row0, j, rec, w, J1 - j, a2w, my_rowe, P, mykey)) return;
         if (column_step<R, MASK, PS, FIRST>(rows, b, sb, sa, row0, j + 1, rec + kColRec, w, J1 - j - 1, a2w, my_rowe,

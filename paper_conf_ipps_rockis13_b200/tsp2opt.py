@@ -47,6 +47,9 @@ def _L():
             "tsp2opt_create": ([P, I32, ctypes.POINTER(P)], I32),
             "tsp2opt_create_sharded": ([P, I32, I32, I32, P, ctypes.POINTER(P)], I32),
             "tsp2opt_nccl_unique_id": ([P], I32),
+            "tsp2opt_create_sharded_p2p": ([P, I32, I32, I32, ctypes.POINTER(P)], I32),
+            "tsp2opt_p2p_export": ([P, P], I32),
+            "tsp2opt_p2p_connect": ([P, P], I32),
             "tsp2opt_destroy": ([P], None),
             "tsp2opt_set_stream": ([P, P], I32),
             "tsp2opt_set_tour": ([P, P], I32),
@@ -127,6 +130,30 @@ def create_sharded(coords, rank: int, world: int, nccl_id: bytes | None) -> ctyp
     _check(_L().tsp2opt_create_sharded(_ptr(xy), xy.size // 2, rank, world, idbuf, ctypes.byref(h)),
            "tsp2opt_create_sharded")
     return h
+
+
+P2P_HANDLE_BYTES = 64
+
+
+def create_sharded_p2p(coords, rank: int, world: int) -> ctypes.c_void_p:
+    """Sharded handle with the peer-memory exchange (tsp2opt_create_sharded_p2p)."""
+    xy = _i32(coords).reshape(-1)
+    h = ctypes.c_void_p()
+    _check(_L().tsp2opt_create_sharded_p2p(_ptr(xy), xy.size // 2, rank, world, ctypes.byref(h)),
+           "tsp2opt_create_sharded_p2p")
+    return h
+
+
+def p2p_export(h) -> bytes:
+    buf = ctypes.create_string_buffer(P2P_HANDLE_BYTES)
+    _check(_L().tsp2opt_p2p_export(h, buf), "tsp2opt_p2p_export")
+    return buf.raw
+
+
+def p2p_connect(h, handles) -> None:
+    blob = b"".join(handles)
+    buf = ctypes.create_string_buffer(blob, len(blob))
+    _check(_L().tsp2opt_p2p_connect(h, buf), "tsp2opt_p2p_connect")
 
 
 def nccl_unique_id() -> bytes:
@@ -404,11 +431,22 @@ def launch_count() -> int:
 class TSP2Opt:
     """One library handle (one GPU / one rank)."""
 
-    def __init__(self, coords, rank: int = 0, world: int = 1, nccl_id: bytes | None = None):
+    def __init__(self, coords, rank: int = 0, world: int = 1, nccl_id: bytes | None = None, p2p_allgather=None):
+        """p2p_allgather: a callable bytes -> list of every rank's bytes (rank order), e.g. over
+        torch.distributed; selects the peer-memory exchange instead of NCCL."""
         xy = _i32(coords).reshape(-1, 2)
         self.n = xy.shape[0]
-        # world 1 with an NCCL id: a one-rank communicator (the sharded path on one GPU)
-        self.h = create(xy) if (world == 1 and nccl_id is None) else create_sharded(xy, rank, world, nccl_id)
+        if p2p_allgather is not None:
+            self.h = create_sharded_p2p(xy, rank, world)
+            try:
+                p2p_connect(self.h, p2p_allgather(p2p_export(self.h)))
+            except Exception:
+                destroy(self.h)
+                self.h = None
+                raise
+        else:
+            # world 1 with an NCCL id: a one-rank communicator (the sharded path on one GPU)
+            self.h = create(xy) if (world == 1 and nccl_id is None) else create_sharded(xy, rank, world, nccl_id)
 
     def close(self):
         if self.h:
