@@ -84,6 +84,7 @@ struct tsp2opt_ctx {
     int* d_tmap = nullptr;      // [nrb * ncc] (row block, column chunk) -> this shard's cull-tile index, -1 if none
     int inc_grid = 0;           // one-warp CTAs of the fused incremental sweep (co-resident)
     bool inc_fused = true;      // TSP2OPT_INC_FUSED=0: the box + cull + list kernels on every iteration
+    bool inc_persistent = true; // TSP2OPT_INC_PERSISTENT=0: per-iteration launches instead of one cooperative launch
     int nctiles = 0;
     int list_grid = 0;          // CTAs of the culled sweep (co-resident)
     int list25_grid = 0;        // CTAs of the 2.5-opt culled sweep
@@ -467,7 +468,35 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
     // = 0 / 1 forces either loop, 2 (default) chooses by pair count.
     const bool use_persistent =
         !h->comm && !h->p2p && h->nbr_k == 0 && !h->or25 && !h->first && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
-    if (use_persistent) {
+    // The incremental culled search of a single GPU in one cooperative launch per
+    // ~1M iterations (launch_inc_ls): no per-iteration launches, three grid barriers
+    // per move.  Sharded handles keep the per-iteration kernels (the exchange sits
+    // between sweep and apply).
+    const bool use_inc_ls = h->inc_persistent && !h->comm && !h->p2p && h->nbr_k == 0 && !h->or25 &&
+                            h->tile_bounds == 3 && h->cgeo.rows == kRowsSmall && h->cgeo.warps == 1 && !h->profiling &&
+                            h->shard_world == 1;
+    if (use_inc_ls) {
+        const int flags = sweep_flags(h);
+        int full = (h->inc_valid && h->last_tiling == 1) ? 0 : 1;
+        for (long long launches = 0;; launches++) {
+            if (launches > 1000000) {
+                g_last_error = "local search did not converge";
+                return TSP2OPT_ECUDA;
+            }
+            CUDA_TRY(launch_inc_ls(h->cgeo, h->d_P, h->d_E, h->d_tour, h->n, h->d_ctiles, h->nctiles, h->d_tmap,
+                                   h->d_rbox, h->d_cbox, h->d_slots, h->parity, max_iters, 1LL << 20, full, h->d_bar,
+                                   h->d_ctl, h->d_ctilebest, flags, h->d_trace, h->trace_cap, h->stream));
+            full = 0;
+            CUDA_TRY(cudaMemcpyAsync(h->h_ctl, h->d_ctl, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+            CUDA_TRY(cudaStreamSynchronize(h->stream));
+            h->parity = *h->h_ctl;
+            h->inc_valid = true;  // the stored tile minima are tile-local and exact for the current tour
+            h->last_tiling = 1;
+            rc = read_slot(h);
+            if (rc) return rc;
+            if (h->h_slot->done & 3) break;
+        }
+    } else if (use_persistent) {
         h->inc_valid = false;
         // One persistent cooperative launch runs sweep -> apply to the local
         // minimum; the per-launch iteration budget bounds a launch to roughly
@@ -596,6 +625,7 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     if (const char* es = getenv("TSP2OPT_SEED")) h->seed_next = atoi(es) != 0;
     if (const char* eg = getenv("TSP2OPT_GLOBAL_SEED")) h->global_seed = atoi(eg) != 0;
     if (const char* ef = getenv("TSP2OPT_INC_FUSED")) h->inc_fused = atoi(ef) != 0;
+    if (const char* ei = getenv("TSP2OPT_INC_PERSISTENT")) h->inc_persistent = atoi(ei) != 0;
 
     CTRY(cudaMemset(h->d_slots, 0, sizeof(Slot) * 2));
     {

@@ -118,6 +118,13 @@ cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, 
 // dirty tiles enumerated from the last move via tmap, boxes recomputed in place, cull and sweep
 // in one launch of `grid` one-warp CTAs (inc_sweep_grid), clean minima folded into the key.
 int inc_sweep_grid(const Geometry& g);
+// Persistent incremental local search (one cooperative launch, one CTA of 16 warps per SM):
+// up to `budget` iterations of {dirty boxes; clean minima + cull + kept-tile sweeps; apply};
+// full = 1 makes the first iteration the full culled sweep.  ctl[0] = the final slot parity.
+cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
+                          const int* tmap, Box* rbox, Box* cbox, Slot* slots, int parity, long long max_moves,
+                          long long budget, int full, unsigned* bar, int* ctl, unsigned long long* tilebest, int flags,
+                          unsigned long long* trace, long long trace_cap, cudaStream_t st);
 cudaError_t launch_inc_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
                              const int* tmap, int grid, Box* rbox, Box* cbox, Slot* slot, int respect_done,
                              unsigned long long* tilebest, int flags, cudaStream_t st);

@@ -368,7 +368,8 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const flo
 // same tile sweep and the same clean / dirty rule as box_kernel + cull_kernel
 // + sweep_list_kernel.
 // ===========================================================================
-__device__ __forceinline__ Box warp_box(const float2* __restrict__ P, const int* __restrict__ E, int k0, int ke)
+__device__ __forceinline__ Box warp_box(const float2* P, const int* E, int k0, int ke)  // coherent loads: P, E may
+                                                                                       // change within a launch
 {
     // positions k0..ke (cities), edges k0..ke-1; every lane returns the box
     int xlo = 1 << 30, xhi = -1, ylo = 1 << 30, yhi = -1, emax = 0;
@@ -634,6 +635,155 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
             s_in.length = *(volatile long long*)&in->length;
             s_in.done = *(volatile int*)&in->done;
             s_in.seed_ok = *(volatile int*)&in->seed_ok;
+        }
+        __syncthreads();
+        apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride, trace, trace_cap, nullptr);
+        p ^= 1;
+        grid_sync(bar, gridDim.x);
+    }
+    if (gtid == 0) ctl[0] = p;
+}
+
+// ===========================================================================
+// Persistent incremental local search (TSP2OPT_OPT_TILE_BOUNDS = 3, one GPU):
+// ONE cooperative launch runs the whole culled, incremental search of §5.6 --
+// per iteration
+//   (B) the boxes of the row blocks / column chunks the last move touched
+//       (one warp each),                                          grid barrier,
+//   (C) the clean tiles' stored minima folded into the key (every thread),
+//       the dirty tiles culled (one THREAD each, enumerated from the last move
+//       through tmap) and every kept tile swept by one WARP with its private
+//       shared memory and the tile-local bound (kSweepLocal),    grid barrier,
+//   (A) the apply of the winning move (apply_phase, every thread), grid barrier
+// -- instead of four launches per move.  Same boxes, cull test, tile sweep,
+// clean / dirty rule and apply as box_kernel + cull_kernel + sweep_list_kernel
+// + apply_kernel, so the result is the same move sequence.  A dirty tile's
+// lane index is warp-major (u = lane * warps + warp), so the kept tiles of
+// one move -- neighbours in u -- land on different warps.  The first iteration
+// of a launch with `full` set (or any without a valid last move) treats every
+// block and tile as dirty: the full culled sweep.
+// ===========================================================================
+template <int R, bool FIRST>
+__global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, int* __restrict__ E,
+                                                        int* __restrict__ tour, int n,
+                                                        const int2* __restrict__ tiles, int ntiles,
+                                                        const int* __restrict__ tmap, int TI, int TJ, int nrb,
+                                                        int ncc, Box* __restrict__ rbox, Box* __restrict__ cbox,
+                                                        Slot* __restrict__ slots, int parity, long long max_moves,
+                                                        long long budget, int full, unsigned* __restrict__ bar,
+                                                        int* __restrict__ ctl,
+                                                        unsigned long long* __restrict__ tilebest, int flags,
+                                                        unsigned long long* __restrict__ trace, long long trace_cap,
+                                                        int tile_bytes)
+{
+    extern __shared__ float4 smem[];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const TileSmem sm(reinterpret_cast<char*>(smem) + (size_t)wib * tile_bytes, TJ);  // this warp's tile memory
+    const int nwb = blockDim.x >> 5;
+    const int gw = blockIdx.x * nwb + wib, nw = gridDim.x * nwb;
+    const int gtid = blockIdx.x * blockDim.x + threadIdx.x, stride = gridDim.x * blockDim.x;
+    const int tflags = (flags | kSweepLocal) & ~kSweepSeed;
+    __shared__ Slot s_in;
+    __shared__ unsigned long long s_min[16];
+    int p = parity;
+    for (long long it = 0; it < budget; it++) {
+        Slot* in = slots + p;
+        if (threadIdx.x == 0) {
+            s_in.done = *(volatile int*)&in->done;
+            s_in.seed_ok = (full && it == 0) ? 0 : *(volatile int*)&in->seed_ok;
+            s_in.last_key = *(volatile unsigned long long*)&in->last_key;
+        }
+        __syncthreads();
+        if (s_in.done) break;  // uniform across the grid
+        int dlo = 0, dhi = n;
+        if (s_in.seed_ok) {
+            dlo = key_i(s_in.last_key);
+            dhi = key_j(s_in.last_key);
+        }
+        const int rlo = dlo >= 1 ? (dlo - 1) / TI : 0, rhi = min(nrb - 1, dhi / TI);
+        const int clo = dlo >= 1 ? (dlo - 1) / TJ : 0, chi = min(ncc - 1, dhi / TJ);
+        // (B) boxes of the dirty blocks
+        {
+            const int nR = rhi - rlo + 1, nC = chi - clo + 1;
+            for (int task = gw; task < nR + nC; task += nw) {
+                if (task < nR) {
+                    const int rb = rlo + task;
+                    const Box b = warp_box(P, E, rb * TI, min(rb * TI + TI, n - 1));
+                    if (lane == 0) rbox[rb] = b;
+                } else {
+                    const int cc = clo + task - nR;
+                    const Box b = warp_box(P, E, cc * TJ, min(cc * TJ + TJ, n));
+                    if (lane == 0) cbox[cc] = b;
+                }
+            }
+        }
+        grid_sync(bar, gridDim.x);
+        // (C1) the clean tiles' stored minima
+        unsigned long long m = kKeyNone;
+        if (s_in.seed_ok) {
+            for (int t = gtid; t < ntiles; t += stride) {
+                const int2 tl = tiles[t];
+                const bool dirty = (tl.x <= dhi && tl.x + TI >= dlo) || (tl.y <= dhi && tl.y + TJ >= dlo);
+                if (!dirty) m = min(m, tilebest[t]);
+            }
+        }
+        for (int o = 16; o > 0; o >>= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
+        if (lane == 0) s_min[wib] = m;
+        // (C2) the dirty tiles: cull per thread, sweep the kept ones per warp
+        const long long nA = (long long)(rhi - rlo + 1) * ncc;
+        const long long nB = (long long)nrb * (chi - clo + 1);
+        for (long long base = 0; base < nA + nB; base += (long long)nw * 32) {
+            const long long u = base + (long long)lane * nw + gw;
+            int t = -1, rb = 0, cc = 0;
+            if (u < nA + nB) {
+                if (u < nA) {
+                    rb = rlo + (int)(u / ncc);
+                    cc = (int)(u % ncc);
+                } else {
+                    const long long v = u - nA;
+                    rb = (int)(v / (chi - clo + 1));
+                    cc = clo + (int)(v % (chi - clo + 1));
+                }
+                if (u < nA || rb < rlo || rb > rhi) t = tmap[(long long)rb * ncc + cc];
+            }
+            bool keep = false;
+            if (t >= 0) {
+                const Box r = rbox[rb], c = cbox[cc];
+                const long long gx = max(0, max(c.xlo - r.xhi, r.xlo - c.xhi));
+                const long long gy = max(0, max(c.ylo - r.yhi, r.ylo - c.yhi));
+                const long long T = (long long)max(r.emax, c.emax) - 1;
+                keep = T >= 0 && gx * gx + gy * gy <= T * T + T;
+                if (!keep) tilebest[t] = kKeyNone;
+            }
+            unsigned kept = __ballot_sync(0xffffffffu, keep);
+            while (kept) {
+                const int src = __ffs(kept) - 1;
+                kept &= kept - 1;
+                const int kt = __shfl_sync(0xffffffffu, t, src);
+                const int krb = __shfl_sync(0xffffffffu, rb, src), kcc = __shfl_sync(0xffffffffu, cc, src);
+                sweep_tile<R, true, FIRST, true>(P, E, n, make_int2(krb * TI, kcc * TJ), TJ, in, sm, tilebest + kt,
+                                                 tflags);
+            }
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            unsigned long long bm = s_min[0];
+            for (int w = 1; w < nwb; w++) bm = min(bm, s_min[w]);
+            if (bm != kKeyNone) atomicMin(&in->key, bm);
+        }
+        grid_sync(bar, gridDim.x);
+        // (A) apply the winning move
+        if (threadIdx.x == 0) {
+            unsigned long long key = *(volatile unsigned long long*)&in->key;
+            if (FIRST && key_delta(key) == kFirstDelta) {  // the marker delta: the winner's exact delta (R20)
+                const int i = key_i(key), j = key_j(key);
+                const int d = exact_dist_biased(__ldcg(P + i), __ldcg(P + j)) +
+                              exact_dist_biased(__ldcg(P + i + 1), __ldcg(P + j + 1)) - __ldcg(E + i) - __ldcg(E + j);
+                key = pack_key(d, i, j);
+            }
+            s_in.key = key;
+            s_in.moves = *(volatile long long*)&in->moves;
+            s_in.length = *(volatile long long*)&in->length;
         }
         __syncthreads();
         apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride, trace, trace_cap, nullptr);
@@ -910,6 +1060,34 @@ cudaError_t launch_inc_sweep(const Geometry& g, const float2* P, const int* E, i
                                                                 slot, respect_done, tilebest, flags, st);
     g_launches += 1;
     return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+constexpr int kIncLsThreads = 512;  // 16 warps, one CTA per SM
+
+cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
+                          const int* tmap, Box* rbox, Box* cbox, Slot* slots, int parity, long long max_moves,
+                          long long budget, int full, unsigned* bar, int* ctl, unsigned long long* tilebest, int flags,
+                          unsigned long long* trace, long long trace_cap, cudaStream_t st)
+{
+    if (g.rows != kRowsSmall || g.warps != 1) return cudaErrorInvalidValue;
+    int TI = g.ti(), TJ = g.tj, nrb = (n - 1 + TI - 1) / TI, ncc = (n + TJ - 1) / TJ;
+    int tile_bytes = (int)((sweep_smem_bytes(g) + 15) / 16 * 16);
+    const size_t smem = (size_t)tile_bytes * (kIncLsThreads / 32);
+    auto kern = (flags & kSweepFirst) ? inc_ls_kernel<kRowsSmall, true> : inc_ls_kernel<kRowsSmall, false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kIncLsThreads, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) return cudaErrorInvalidConfiguration;
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int grid = sms;  // one CTA per SM (co-resident: cooperative launch)
+    void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &tmap, &TI, &TJ, &nrb, &ncc, &rbox, &cbox, &slots, &parity,
+                    &max_moves, &budget, &full, &bar, &ctl, &tilebest, &flags, &trace, &trace_cap, &tile_bytes};
+    g_launches += 1;
+    return cudaLaunchCooperativeKernel((const void*)kern, dim3(grid), dim3(kIncLsThreads), args, smem, st);
 }
 
 int inc_sweep_grid(const Geometry& g)

@@ -307,15 +307,15 @@ __device__ __forceinline__ bool rare_step(const Rows<R>& rows, Bound<R>& b, int 
 }
 
 #ifndef TSP2OPT_VOTE_STEPS
-#define TSP2OPT_VOTE_STEPS 2  // column steps per warp vote (even; 1 = a vote every step)
+#define TSP2OPT_VOTE_STEPS 1  // column steps per warp vote (even, or 1 = a vote every step; measured: 2 and 4
+                              // are 6 % and 8 % slower at C5, profiles/r02_exp_sweep.jsonl)
 #endif
 
 template <int R, bool MASK, bool PS, bool FIRST>
 __device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0, int jstart, int J0, int J1,
                                      const TileSmem& sm, const float* my_rowe, const float2* P,
-                                     unsigned long long& mykey)
+                                     unsigned long long& mykey, int w)
 {
-    const int w = threadIdx.x >> 5;
     float4* rec = sm.col + kColRec * (jstart - J0);
     int a2w = fill_colthr(b.a2, rec, w, J1 - jstart);
     float sa[R + 1], sb[R + 1];
@@ -428,19 +428,24 @@ __host__ __device__ inline size_t tile_smem_bytes(int TJ, int TI)
 // pair ... Get best global pair"; min is order-independent, so the result is
 // deterministic).  The caller synchronises the CTA before reusing `sm`.
 
-template <int R, bool PS, bool FIRST = false>
+//
+// WT (warp tile): the tile belongs to ONE warp with its own TileSmem (the
+// persistent incremental local search, where each warp of a large CTA sweeps
+// its own tiles); warp synchronisation instead of block barriers.
+template <int R, bool PS, bool FIRST = false, bool WT = false>
 __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n, int2 tile, int TJ, Slot* slot,
                                            const TileSmem& sm, unsigned long long* tilebest, int flags)
 {
     const int I0 = tile.x, J0 = tile.y;
     const int J1 = min(J0 + TJ, n);  // columns j in [J0, J1), j <= n-1
     const int ncol = J1 - J0;
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int warp = WT ? 0 : threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int tid = WT ? lane : threadIdx.x, nthr = WT ? 32 : blockDim.x;
     const int wrow0 = I0 + warp * 32 * R;
     const int row0 = wrow0 + lane * R;
     const int jstart = max(J0, wrow0 + 1);  // no pair of this warp has j <= wrow0
     const bool active = jstart < J1;        // warp-uniform
-    float* my_rowe = sm.rowe + threadIdx.x * R;  // stride R (odd): conflict-free
+    float* my_rowe = sm.rowe + tid * R;  // stride R (odd): conflict-free
 
     Rows<R> rows;
     float erow[R];
@@ -454,7 +459,7 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
 #pragma unroll
         for (int r = 0; r < R; r++) erow[r] = (float)gld<PS>(E + row0 + r);
     }
-    for (int c = threadIdx.x; c <= ncol + 1; c += blockDim.x) {  // J1 <= n: P[n] = P[0]; + 1 spare column
+    for (int c = tid; c <= ncol + 1; c += nthr) {  // J1 <= n: P[n] = P[0]; + 1 spare column
         const float2 p = gld<PS>(P + J0 + c);
         const int e = gld<PS>(E + J0 + c);
         sm.put(c, p, (float)e);
@@ -472,7 +477,7 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
         const unsigned long long k = surviving_key(*(volatile unsigned long long*)tilebest, key_i(mv), key_j(mv));
         if (k < g) {
             g = k;
-            if (threadIdx.x == 0) atomicMin(&slot->key, k);
+            if (tid == 0) atomicMin(&slot->key, k);
         }
     }
     const int dg = key_delta(g);
@@ -480,7 +485,8 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
 #pragma unroll
         for (int r = 0; r < R; r++) my_rowe[r] = erow[r];
     }
-    __syncthreads();
+    if (WT) __syncwarp();
+    else __syncthreads();
 
     unsigned long long mykey = kKeyNone;
     // FIRST: a tile whose lowest cell is above an improving pair already found
@@ -494,8 +500,8 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
 #ifdef TSP2OPT_STATS
             if (lane == 0) atomicAdd(&g_stats[3], 1ULL);
 #endif
-            if (masked) walk<R, true, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
-            else walk<R, false, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey);
+            if (masked) walk<R, true, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey, warp);
+            else walk<R, false, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey, warp);
         }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
@@ -506,6 +512,11 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     }
     // The tile's best (a real pair of this sweep, or none) is kept for the next
     // iteration's seed (apply_phase: moves the applied reversal leaves intact).
+    if (WT) {
+        if (lane == 0) *tilebest = active ? mykey : kKeyNone;  // mykey is the warp minimum here
+        __syncwarp();
+        return;
+    }
     __shared__ unsigned long long s_red[kMaxWarpsPerTile];
     if (lane == 0) s_red[warp] = mykey;
     __syncthreads();
