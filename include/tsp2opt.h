@@ -392,6 +392,13 @@ int tsp2opt_selftest_sqrt(double *max_rel_err, int32_t *zero_ok);
  * product builds.  reset != 0 zeroes them afterwards. */
 int tsp2opt_debug_stats(int64_t *out4, int32_t reset);
 
+/* Phase clocks of the persistent incremental local search in an instrumented
+ * build (-DTSP2OPT_PHASE_TIMING): out8[k] = SM clock cycles CTA 0 spent in
+ * [0] dirty boxes, [1] barrier, [6] clean-minimum scan, [2] cull + kept-tile
+ * sweeps, [3] barrier, [4] apply, [5] barrier, summed over iterations; -1 in
+ * product builds.  reset != 0 zeroes them afterwards. */
+int tsp2opt_debug_phases(int64_t *out8, int32_t reset);
+
 /* Number of this library's kernel launches since load (for gpu_launches). */
 int64_t tsp2opt_launch_count(void);
 

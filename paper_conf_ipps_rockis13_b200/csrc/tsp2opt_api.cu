@@ -1318,6 +1318,15 @@ int tsp2opt_selftest_sqrt(double* max_rel_err, int32_t* zero_ok)
     return TSP2OPT_OK;
 }
 
+int tsp2opt_debug_phases(int64_t* out8, int32_t reset)
+{
+    if (!out8) return TSP2OPT_EINVAL;
+    long long v[8];
+    CUDA_TRY(read_phases(v, reset));
+    for (int k = 0; k < 8; k++) out8[k] = v[k];
+    return TSP2OPT_OK;
+}
+
 int tsp2opt_debug_stats(int64_t* out4, int32_t reset)
 {
     if (!out4) return TSP2OPT_EINVAL;

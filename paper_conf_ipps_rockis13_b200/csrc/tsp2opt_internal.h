@@ -140,6 +140,7 @@ cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour,
 cudaError_t launch_p2p_min(Slot* slot, Mailbox* const* peers, int rank, int world, int respect_done,
                            cudaStream_t st);
 cudaError_t read_stats(long long* out4, int reset);
+cudaError_t read_phases(long long* out8, int reset);
 cudaError_t run_selftest_sqrt(double* max_rel, int* zero_ok);
 cudaError_t run_selftest(long long* out4);  // dist_bad, filter_bad, first bad s, first bad dx<<15|dy
 

@@ -15,6 +15,13 @@
 
 namespace tsp2opt {
 
+#ifdef TSP2OPT_PHASE_TIMING
+// Instrumented builds only: clock cycles CTA 0 spends in each phase of the
+// persistent incremental local search (boxes, barrier, sweep, barrier, apply,
+// barrier), summed over the iterations; read by tsp2opt_debug_stats.
+__device__ unsigned long long g_phase[8];
+#endif
+
 // ===========================================================================
 // a2 + a3: route-order gather and edge pass (L18 Fig. 6 "An array containing
 // coordinates in the route's order"; done on the device instead of the host).
@@ -103,7 +110,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* 
                                                      int flags)
 {
     extern __shared__ float4 smem[];
-    const TileSmem sm(smem, TJ);
+    const TileSmem sm(smem, TJ, R * (int)blockDim.x);
     pdl_trigger();
     pdl_wait();
     if (respect_done && *(volatile int*)&slot->done) return;  // converged: iteration is a no-op
@@ -332,7 +339,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const flo
                                                                       int flags)
 {
     extern __shared__ float4 smem[];
-    const TileSmem sm(smem, TJ);
+    const TileSmem sm(smem, TJ, R * (int)blockDim.x);
     __shared__ int4 s_t;
     pdl_trigger();
     pdl_wait();
@@ -371,17 +378,33 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const flo
 __device__ __forceinline__ Box warp_box(const float2* P, const int* E, int k0, int ke)  // coherent loads: P, E may
                                                                                        // change within a launch
 {
-    // positions k0..ke (cities), edges k0..ke-1; every lane returns the box
+    // positions k0..ke (cities), edges k0..ke-1; every lane returns the box.  Up to
+    // kWarpBoxBatch positions per lane have their loads issued before the first use
+    // (one L2 round trip for a 225-position row block, instead of one per position).
+    constexpr int kWarpBoxBatch = 8;
     int xlo = 1 << 30, xhi = -1, ylo = 1 << 30, yhi = -1, emax = 0;
     const int lane = threadIdx.x & 31;
-    for (int k = k0 + lane; k <= ke; k += 32) {
-        const float2 p = P[k];
-        const int x = unbias(p.x), y = unbias(p.y);
-        xlo = min(xlo, x);
-        xhi = max(xhi, x);
-        ylo = min(ylo, y);
-        yhi = max(yhi, y);
-        if (k < ke) emax = max(emax, E[k]);
+    for (int k1 = k0; k1 <= ke; k1 += 32 * kWarpBoxBatch) {
+        float2 p[kWarpBoxBatch];
+        int e[kWarpBoxBatch];
+#pragma unroll
+        for (int b = 0; b < kWarpBoxBatch; b++) {
+            const int k = k1 + lane + 32 * b;
+            p[b] = k <= ke ? P[k] : make_float2(0.f, 0.f);
+            e[b] = k < ke ? E[k] : 0;
+        }
+#pragma unroll
+        for (int b = 0; b < kWarpBoxBatch; b++) {
+            const int k = k1 + lane + 32 * b;
+            if (k <= ke) {
+                const int x = unbias(p[b].x), y = unbias(p[b].y);
+                xlo = min(xlo, x);
+                xhi = max(xhi, x);
+                ylo = min(ylo, y);
+                yhi = max(yhi, y);
+                emax = max(emax, e[b]);
+            }
+        }
     }
     const unsigned full = 0xffffffffu;
     Box b;
@@ -403,7 +426,7 @@ __global__ void __launch_bounds__(32, 16) inc_sweep_kernel(const float2* __restr
                                                            unsigned long long* __restrict__ tilebest, int flags)
 {
     extern __shared__ float4 smem[];
-    const TileSmem sm(smem, TJ);
+    const TileSmem sm(smem, TJ, R * (int)blockDim.x);
     pdl_trigger();
     pdl_wait();
     const int done = respect_done ? *(volatile const int*)&slot->done : 0;
@@ -611,7 +634,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
                                                            unsigned long long* __restrict__ trace, long long trace_cap)
 {
     extern __shared__ float4 smem[];
-    const TileSmem sm(smem, TJ);
+    const TileSmem sm(smem, TJ, R * (int)blockDim.x);
     __shared__ Slot s_in;
     const int gtid = blockIdx.x * blockDim.x + threadIdx.x;
     const int stride = gridDim.x * blockDim.x;
@@ -678,7 +701,7 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
 {
     extern __shared__ float4 smem[];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    const TileSmem sm(reinterpret_cast<char*>(smem) + (size_t)wib * tile_bytes, TJ);  // this warp's tile memory
+    const TileSmem sm(reinterpret_cast<char*>(smem) + (size_t)wib * tile_bytes, TJ, 32 * R);  // this warp's tile memory
     const int nwb = blockDim.x >> 5;
     const int gw = blockIdx.x * nwb + wib, nw = gridDim.x * nwb;
     const int gtid = blockIdx.x * blockDim.x + threadIdx.x, stride = gridDim.x * blockDim.x;
@@ -686,6 +709,21 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
     __shared__ Slot s_in;
     __shared__ unsigned long long s_min[16];
     int p = parity;
+#ifdef TSP2OPT_PHASE_TIMING
+    long long tp0 = clock64();
+#define PHASE_MARK(k)                                                                         \
+    do {                                                                                      \
+        if (blockIdx.x == 0 && threadIdx.x == 0) {                                            \
+            const long long tp1 = clock64();                                                  \
+            atomicAdd(&g_phase[k], (unsigned long long)(tp1 - tp0));                          \
+            tp0 = tp1;                                                                        \
+        }                                                                                     \
+    } while (0)
+#else
+#define PHASE_MARK(k) \
+    do {              \
+    } while (0)
+#endif
     for (long long it = 0; it < budget; it++) {
         Slot* in = slots + p;
         if (threadIdx.x == 0) {
@@ -717,18 +755,9 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
                 }
             }
         }
+        PHASE_MARK(0);
         grid_sync(bar, gridDim.x);
-        // (C1) the clean tiles' stored minima
-        unsigned long long m = kKeyNone;
-        if (s_in.seed_ok) {
-            for (int t = gtid; t < ntiles; t += stride) {
-                const int2 tl = tiles[t];
-                const bool dirty = (tl.x <= dhi && tl.x + TI >= dlo) || (tl.y <= dhi && tl.y + TJ >= dlo);
-                if (!dirty) m = min(m, tilebest[t]);
-            }
-        }
-        for (int o = 16; o > 0; o >>= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
-        if (lane == 0) s_min[wib] = m;
+        PHASE_MARK(1);
         // (C2) the dirty tiles: cull per thread, sweep the kept ones per warp
         const long long nA = (long long)(rhi - rlo + 1) * ncc;
         const long long nB = (long long)nrb * (chi - clo + 1);
@@ -765,6 +794,32 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
                                                  tflags);
             }
         }
+        PHASE_MARK(2);
+        // (C1) the clean tiles' stored minima -- after the sweeps, so that warps
+        // without kept tiles do it while the others still sweep; loads batched
+        unsigned long long m = kKeyNone;
+        if (s_in.seed_ok) {
+            constexpr int V = 4;
+            for (int t0 = gtid; t0 < ntiles; t0 += V * stride) {
+                int2 tl[V];
+                unsigned long long kb[V];
+#pragma unroll
+                for (int v = 0; v < V; v++) {
+                    const int t = t0 + v * stride;
+                    tl[v] = t < ntiles ? tiles[t] : make_int2(-(1 << 30), -(1 << 30));
+                    kb[v] = t < ntiles ? tilebest[t] : kKeyNone;
+                }
+#pragma unroll
+                for (int v = 0; v < V; v++) {
+                    const bool dirty =
+                        (tl[v].x <= dhi && tl[v].x + TI >= dlo) || (tl[v].y <= dhi && tl[v].y + TJ >= dlo);
+                    if (!dirty) m = min(m, kb[v]);
+                }
+            }
+        }
+        for (int o = 16; o > 0; o >>= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
+        if (lane == 0) s_min[wib] = m;
+        PHASE_MARK(6);
         __syncthreads();
         if (threadIdx.x == 0) {
             unsigned long long bm = s_min[0];
@@ -772,6 +827,7 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
             if (bm != kKeyNone) atomicMin(&in->key, bm);
         }
         grid_sync(bar, gridDim.x);
+        PHASE_MARK(3);
         // (A) apply the winning move
         if (threadIdx.x == 0) {
             unsigned long long key = *(volatile unsigned long long*)&in->key;
@@ -788,9 +844,12 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
         __syncthreads();
         apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride, trace, trace_cap, nullptr);
         p ^= 1;
+        PHASE_MARK(4);
         grid_sync(bar, gridDim.x);
+        PHASE_MARK(5);
     }
     if (gtid == 0) ctl[0] = p;
+#undef PHASE_MARK
 }
 
 // ===========================================================================
@@ -1205,9 +1264,28 @@ cudaError_t run_selftest_sqrt(double* max_rel, int* zero_ok)
     return err;
 }
 
+cudaError_t read_phases(long long* out8, int reset)
+{
+#ifdef TSP2OPT_PHASE_TIMING
+    unsigned long long ph[8];
+    cudaError_t ep = cudaMemcpyFromSymbol(ph, g_phase, sizeof(ph));
+    if (ep != cudaSuccess) return ep;
+    for (int k = 0; k < 8; k++) out8[k] = (long long)ph[k];
+    if (reset) {
+        const unsigned long long z[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        ep = cudaMemcpyToSymbol(g_phase, z, sizeof(z));
+    }
+    return ep;
+#else
+    (void)reset;
+    for (int k = 0; k < 8; k++) out8[k] = -1;
+    return cudaSuccess;
+#endif
+}
+
 cudaError_t read_stats(long long* out4, int reset)
 {
-#ifdef TSP2OPT_STATS
+#if defined(TSP2OPT_STATS)
     unsigned long long h[4];
     cudaError_t e = cudaMemcpyFromSymbol(h, g_stats, sizeof(h));
     if (e != cudaSuccess) return e;

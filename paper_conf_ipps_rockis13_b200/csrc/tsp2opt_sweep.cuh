@@ -102,10 +102,14 @@ constexpr int kMaxWarpsPerTile = 4;
 constexpr int kColRec = 3;
 
 struct TileSmem {
-    float4* col;  // [TJ + 2] column records: columns J0..J1 and one spare
-    float* rowe;  // [32 * R * warps]: e_i of the CTA's rows, as float
-    __device__ TileSmem(void* base, int TJ)
-        : col(reinterpret_cast<float4*>(base)), rowe(reinterpret_cast<float*>(col + kColRec * (TJ + 2)))
+    float4* col;   // [TJ + 2] column records: columns J0..J1 and one spare
+    float* rowe;   // [TI = 32 * R * warps]: e_i of the CTA's rows, as float
+    float2* rowp;  // [32 * warps * (R + 1)]: each lane's R + 1 row cities (biased), for the rare path --
+                   // shared memory, not a reload of P that may miss L1 (persistent kernels invalidate it)
+    __device__ TileSmem(void* base, int TJ, int TI)
+        : col(reinterpret_cast<float4*>(base)),
+          rowe(reinterpret_cast<float*>(col + kColRec * (TJ + 2))),
+          rowp(reinterpret_cast<float2*>(rowe + TI))
     {
     }
     __device__ float4 xy(int c) const { return col[kColRec * c]; }
@@ -145,8 +149,8 @@ __device__ __forceinline__ bool step_any(const Bound<R>& b, const float (&cur)[R
         for (int r = 0; r < R; r++) {
 #ifndef TSP2OPT_ROWTEST_FLOAT
             // cur >= +0 and srow is either >= +0 or negative (t < 0, sq_threshold), so the
-            // signed integer order of the IEEE bits equals the float order here (ISETP runs
-            // at full rate on the ALU pipe, FSETP at half)
+            // signed integer order of the IEEE bits equals the float order here (ISETP and
+            // FSETP share the ALU pipe's half rate; measured 1 % faster, r02_exp_sweep.jsonl)
             const bool t = __float_as_int(cur[r]) <= __float_as_int(b.srow[r]);
 #else
             const bool t = cur[r] <= b.srow[r];
@@ -177,7 +181,7 @@ __device__ __forceinline__ bool step_any(const Bound<R>& b, const float (&cur)[R
 template <int R, bool MASK, bool PS, bool FIRST>
 __device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1], const float (&nxt)[R + 1],
                                            float scol, int row0, int j, float4 c0, float4 c1, float ej,
-                                           const float* my_rowe, const float2* P, unsigned long long& mykey)
+                                           const float* my_rowe, const float2* my_rowp, unsigned long long& mykey)
 {
     const float lim = ej + b.Bf + 0.5f;
     unsigned mask = 0;
@@ -198,7 +202,7 @@ __device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1
     while (mask) {  // ascending r == ascending cell number
         const int r = __ffs(mask) - 1;
         mask &= mask - 1;
-        const float2 pi = gld<PS>(P + row0 + r), pi1 = gld<PS>(P + row0 + r + 1);
+        const float2 pi = my_rowp[r], pi1 = my_rowp[r + 1];
         // nint from the float path when it is unambiguous: |sqrt_approx(s_f) - sqrt(s)|
         // < 0.03, so |r - m| < 0.45 for the nearest integer m
         // proves nint(sqrt(s)) == m.  Otherwise the integer nint (rare).
@@ -252,7 +256,7 @@ __device__ __forceinline__ int fill_colthr(int a2, float4* rec, int w, int count
 template <int R, bool MASK, bool PS, bool FIRST>
 __device__ __forceinline__ bool column_step(const Rows<R>& rows, Bound<R>& b, const float (&cur)[R + 1],
                                             float (&nxt)[R + 1], int row0, int j, float4* rec, int w, int left,
-                                            int& a2w, const float* my_rowe, const float2* P,
+                                            int& a2w, const float* my_rowe, const float2* my_rowp,
                                             unsigned long long& mykey)
 {
     const float4 c1 = rec[kColRec];
@@ -267,7 +271,8 @@ __device__ __forceinline__ bool column_step(const Rows<R>& rows, Bound<R>& b, co
         if ((threadIdx.x & 31) == 0) atomicAdd(&g_stats[1], 1ULL);
 #endif
         const int B0 = b.B;
-        if (any) exact_step<R, MASK, PS, FIRST>(b, cur, nxt, scol, row0, j, rec[0], c1, rec_e(rec), my_rowe, P, mykey);
+        if (any) exact_step<R, MASK, PS, FIRST>(b, cur, nxt, scol, row0, j, rec[0], c1, rec_e(rec), my_rowe, my_rowp,
+                                                mykey);
         if (FIRST) return __any_sync(0xffffffffu, mykey != kKeyNone);
         // share the warp's best: a lane may accept delta <= (best of another lane)
         const int wb = __reduce_min_sync(0xffffffffu, b.B);
@@ -283,7 +288,7 @@ __device__ __forceinline__ bool column_step(const Rows<R>& rows, Bound<R>& b, co
 // (the walk's arrays have moved on), then exactly as column_step's rare branch.
 template <int R, bool MASK, bool PS, bool FIRST>
 __device__ __forceinline__ bool rare_step(const Rows<R>& rows, Bound<R>& b, int row0, int j, float4* rec, int w,
-                                          int left, int& a2w, const float* my_rowe, const float2* P,
+                                          int left, int& a2w, const float* my_rowe, const float2* my_rowp,
                                           unsigned long long& mykey)
 {
     float cur[R + 1], nxt[R + 1];
@@ -297,7 +302,7 @@ __device__ __forceinline__ bool rare_step(const Rows<R>& rows, Bound<R>& b, int 
     if ((threadIdx.x & 31) == 0) atomicAdd(&g_stats[1], 1ULL);
 #endif
     const int B0 = b.B;
-    if (any) exact_step<R, MASK, PS, FIRST>(b, cur, nxt, scol, row0, j, rec[0], c1, rec_e(rec), my_rowe, P, mykey);
+    if (any) exact_step<R, MASK, PS, FIRST>(b, cur, nxt, scol, row0, j, rec[0], c1, rec_e(rec), my_rowe, my_rowp, mykey);
     if (FIRST) return __any_sync(0xffffffffu, mykey != kKeyNone);
     const int wb = __reduce_min_sync(0xffffffffu, b.B);
     const int nb = min(b.B, wb + 1);
@@ -313,7 +318,7 @@ __device__ __forceinline__ bool rare_step(const Rows<R>& rows, Bound<R>& b, int 
 
 template <int R, bool MASK, bool PS, bool FIRST>
 __device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0, int jstart, int J0, int J1,
-                                     const TileSmem& sm, const float* my_rowe, const float2* P,
+                                     const TileSmem& sm, const float* my_rowe, const float2* my_rowp,
                                      unsigned long long& mykey, int w)
 {
     float4* rec = sm.col + kColRec * (jstart - J0);
@@ -343,19 +348,21 @@ __device__ __forceinline__ void walk(const Rows<R>& rows, Bound<R>& b, int row0,
 #pragma unroll 1
                 for (int v = 0; v < V; v++)
                     if (rare_step<R, MASK, PS, FIRST>(rows, b, row0, j + v, rec + v * kColRec, w, J1 - j - v, a2w,
-                                                      my_rowe, P, mykey))
+                                                      my_rowe, my_rowp, mykey))
                         return;
                 column_sq<R>(sa, rows, rec[V * kColRec]);  // the next group's current column
             }
         }
     }
     for (; j + 1 < J1; j += 2, rec += 2 * kColRec) {
-        if (column_step<R, MASK, PS, FIRST>(rows, b, sa, sb, row0, j, rec, w, J1 - j, a2w, my_rowe, P, mykey)) return;
+        if (column_step<R, MASK, PS, FIRST>(rows, b, sa, sb, row0, j, rec, w, J1 - j, a2w, my_rowe, my_rowp, mykey))
+            return;
         if (column_step<R, MASK, PS, FIRST>(rows, b, sb, sa, row0, j + 1, rec + kColRec, w, J1 - j - 1, a2w, my_rowe,
-                                            P, mykey))
+                                            my_rowp, mykey))
             return;
     }
-    if (j < J1) column_step<R, MASK, PS, FIRST>(rows, b, sa, sb, row0, j, rec, w, J1 - j, a2w, my_rowe, P, mykey);
+    if (j < J1)
+        column_step<R, MASK, PS, FIRST>(rows, b, sa, sb, row0, j, rec, w, J1 - j, a2w, my_rowe, my_rowp, mykey);
 }
 
 // Tile-level form of the same exact necessary condition (a bound on all of the
@@ -417,7 +424,9 @@ __device__ __forceinline__ bool tile_may_pass(const Rows<R>& rows, const Bound<R
 // Shared memory bytes of a tile with TJ columns and TI rows.
 __host__ __device__ inline size_t tile_smem_bytes(int TJ, int TI)
 {
-    return (size_t)(TJ + 2) * kColRec * sizeof(float4) + (size_t)TI * sizeof(float);
+    // rowp: (TI / R) * (R + 1) <= TI + TI / 7 entries for R >= 7, plus slack
+    return (size_t)(TJ + 2) * kColRec * sizeof(float4) + (size_t)TI * sizeof(float) +
+           (size_t)(TI + TI / 7 + 32) * sizeof(float2);
 }
 
 // One tile.  All global loads of the tile (the lane's rows and row edges, the
@@ -446,6 +455,7 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     const int jstart = max(J0, wrow0 + 1);  // no pair of this warp has j <= wrow0
     const bool active = jstart < J1;        // warp-uniform
     float* my_rowe = sm.rowe + tid * R;  // stride R (odd): conflict-free
+    float2* my_rowp = sm.rowp + tid * (R + 1);
 
     Rows<R> rows;
     float erow[R];
@@ -455,6 +465,8 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
             const float2 p0 = gld<PS>(P + row0 + 2 * q), p1 = gld<PS>(P + row0 + 2 * q + 1);
             rows.xp[q] = make_float2(p0.x, p1.x);
             rows.yp[q] = make_float2(p0.y, p1.y);
+            my_rowp[2 * q] = p0;
+            my_rowp[2 * q + 1] = p1;
         }
 #pragma unroll
         for (int r = 0; r < R; r++) erow[r] = (float)gld<PS>(E + row0 + r);
@@ -500,8 +512,8 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
 #ifdef TSP2OPT_STATS
             if (lane == 0) atomicAdd(&g_stats[3], 1ULL);
 #endif
-            if (masked) walk<R, true, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey, warp);
-            else walk<R, false, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, P, mykey, warp);
+            if (masked) walk<R, true, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, my_rowp, mykey, warp);
+            else walk<R, false, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, my_rowp, mykey, warp);
         }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {

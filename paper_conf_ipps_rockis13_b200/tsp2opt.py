@@ -82,6 +82,7 @@ def _L():
             "tsp2opt_profile_read": ([P, ctypes.POINTER(ctypes.c_double), pI64], I32),
             "tsp2opt_launch_count": ([], I64),
             "tsp2opt_debug_stats": ([pI64, I32], I32),
+            "tsp2opt_debug_phases": ([P, I32], I32),
             "tsp2opt_selftest_sqrt": ([ctypes.POINTER(ctypes.c_double), pI32], I32),
             "tsp2opt_strerror": ([I32], ctypes.c_char_p),
             "tsp2opt_last_error": ([], ctypes.c_char_p),
@@ -527,6 +528,13 @@ class TSP2Opt:
 
     def profile_read(self):
         return profile_read(self.h)
+
+
+def debug_phases(reset: bool = True) -> list:
+    """Phase clocks of the persistent incremental search (instrumented builds; -1 otherwise)."""
+    out = np.zeros(8, dtype=np.int64)
+    _check(_L().tsp2opt_debug_phases(_ptr(out), 1 if reset else 0), "tsp2opt_debug_phases")
+    return out.tolist()
 
 
 def debug_stats(reset: bool = True) -> dict:
