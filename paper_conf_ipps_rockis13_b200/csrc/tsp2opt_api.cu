@@ -85,6 +85,8 @@ struct tsp2opt_ctx {
     int inc_grid = 0;           // one-warp CTAs of the fused incremental sweep (co-resident)
     bool inc_fused = true;      // TSP2OPT_INC_FUSED=0: the box + cull + list kernels on every iteration
     bool inc_persistent = true; // TSP2OPT_INC_PERSISTENT=0: per-iteration launches instead of one cooperative launch
+    int inc_parts = 1;          // TSP2OPT_INC_PARTS: column parts per kept tile in the persistent search (work queue)
+    int4* d_incq = nullptr;     // its queue: [0] = (count, next, culled warps), then nctiles * inc_parts items
     int nctiles = 0;
     int list_grid = 0;          // CTAs of the culled sweep (co-resident)
     int list25_grid = 0;        // CTAs of the 2.5-opt culled sweep
@@ -233,6 +235,7 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
         std::vector<Tile> mine = shard_tiles(h->all_ctiles, rank, world, &unused);
         for (size_t k = 0; k < mine.size(); k++) map[(size_t)(mine[k].i0 / TI) * ncc + mine[k].j0 / TJ] = (int)k;
         cudaFree(h->d_tmap);
+    cudaFree(h->d_incq);
     for (void* p : h->p2p_opened)
         if (p) cudaIpcCloseMemHandle(p);
     cudaFree(h->d_peers);
@@ -241,6 +244,13 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
         CUDA_TRY(cudaMalloc(&h->d_tmap, sizeof(int) * map.size()));
         CUDA_TRY(cudaMemcpy(h->d_tmap, map.data(), sizeof(int) * map.size(), cudaMemcpyHostToDevice));
         h->inc_grid = inc_sweep_grid(h->cgeo);
+        cudaFree(h->d_incq);
+        h->d_incq = nullptr;
+        if (h->inc_parts > 1) {
+            const size_t items = 1 + (size_t)h->inc_parts * std::max(1, h->nctiles) + 8192;  // + over-claims
+            CUDA_TRY(cudaMalloc(&h->d_incq, sizeof(int4) * items));
+            CUDA_TRY(cudaMemset(h->d_incq, 0, sizeof(int4) * items));
+        }
     }
     h->list_grid = sweep_list_grid(h->cgeo, h->nctiles);
     if (const char* el = getenv("TSP2OPT_LIST_GRID"))  // experiment: cap the list sweep's co-resident grid
@@ -274,6 +284,7 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_ctilebest);
     cudaFree(h->d_list);
     cudaFree(h->d_tmap);
+    cudaFree(h->d_incq);
     for (void* p : h->p2p_opened)
         if (p) cudaIpcCloseMemHandle(p);
     cudaFree(h->d_peers);
@@ -485,7 +496,8 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
             }
             CUDA_TRY(launch_inc_ls(h->cgeo, h->d_P, h->d_E, h->d_tour, h->n, h->d_ctiles, h->nctiles, h->d_tmap,
                                    h->d_rbox, h->d_cbox, h->d_slots, h->parity, max_iters, 1LL << 20, full, h->d_bar,
-                                   h->d_ctl, h->d_ctilebest, flags, h->d_trace, h->trace_cap, h->stream));
+                                   h->d_ctl, h->d_ctilebest, flags, h->d_trace, h->trace_cap, h->inc_parts,
+                                   h->d_incq, h->stream));
             full = 0;
             CUDA_TRY(cudaMemcpyAsync(h->h_ctl, h->d_ctl, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
             CUDA_TRY(cudaStreamSynchronize(h->stream));
@@ -626,6 +638,10 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     if (const char* eg = getenv("TSP2OPT_GLOBAL_SEED")) h->global_seed = atoi(eg) != 0;
     if (const char* ef = getenv("TSP2OPT_INC_FUSED")) h->inc_fused = atoi(ef) != 0;
     if (const char* ei = getenv("TSP2OPT_INC_PERSISTENT")) h->inc_persistent = atoi(ei) != 0;
+    if (const char* ep2 = getenv("TSP2OPT_INC_PARTS")) {
+        const int v = atoi(ep2);
+        if (v == 1 || v == 2 || v == 4 || v == 8) h->inc_parts = v;
+    }
 
     CTRY(cudaMemset(h->d_slots, 0, sizeof(Slot) * 2));
     {

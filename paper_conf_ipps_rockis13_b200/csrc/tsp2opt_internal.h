@@ -124,7 +124,7 @@ int inc_sweep_grid(const Geometry& g);
 cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
                           const int* tmap, Box* rbox, Box* cbox, Slot* slots, int parity, long long max_moves,
                           long long budget, int full, unsigned* bar, int* ctl, unsigned long long* tilebest, int flags,
-                          unsigned long long* trace, long long trace_cap, cudaStream_t st);
+                          unsigned long long* trace, long long trace_cap, int nparts, int4* queue, cudaStream_t st);
 cudaError_t launch_inc_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
                              const int* tmap, int grid, Box* rbox, Box* cbox, Slot* slot, int respect_done,
                              unsigned long long* tilebest, int flags, cudaStream_t st);

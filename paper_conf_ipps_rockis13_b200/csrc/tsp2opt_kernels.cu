@@ -697,7 +697,7 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
                                                         int* __restrict__ ctl,
                                                         unsigned long long* __restrict__ tilebest, int flags,
                                                         unsigned long long* __restrict__ trace, long long trace_cap,
-                                                        int tile_bytes)
+                                                        int tile_bytes, int nparts, int4* __restrict__ queue)
 {
     extern __shared__ float4 smem[];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -740,6 +740,7 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
         }
         const int rlo = dlo >= 1 ? (dlo - 1) / TI : 0, rhi = min(nrb - 1, dhi / TI);
         const int clo = dlo >= 1 ? (dlo - 1) / TJ : 0, chi = min(ncc - 1, dhi / TJ);
+        if (gtid == 0 && nparts > 1) queue[0] = make_int4(0, 0, 0, 0);  // count, next, culled warps (seen after the barrier)
         // (B) boxes of the dirty blocks
         {
             const int nR = rhi - rlo + 1, nC = chi - clo + 1;
@@ -785,13 +786,75 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
                 if (!keep) tilebest[t] = kKeyNone;
             }
             unsigned kept = __ballot_sync(0xffffffffu, keep);
-            while (kept) {
-                const int src = __ffs(kept) - 1;
-                kept &= kept - 1;
-                const int kt = __shfl_sync(0xffffffffu, t, src);
-                const int krb = __shfl_sync(0xffffffffu, rb, src), kcc = __shfl_sync(0xffffffffu, cc, src);
-                sweep_tile<R, true, FIRST, true>(P, E, n, make_int2(krb * TI, kcc * TJ), TJ, in, sm, tilebest + kt,
-                                                 tflags);
+            if (nparts <= 1) {
+                while (kept) {  // this warp sweeps the kept tiles its lanes found
+                    const int src = __ffs(kept) - 1;
+                    kept &= kept - 1;
+                    const int kt = __shfl_sync(0xffffffffu, t, src);
+                    const int krb = __shfl_sync(0xffffffffu, rb, src), kcc = __shfl_sync(0xffffffffu, cc, src);
+                    sweep_tile<R, true, FIRST, true>(P, E, n, make_int2(krb * TI, kcc * TJ), TJ, in, sm,
+                                                     tilebest + kt, tflags);
+                }
+            } else if (kept) {
+                // publish nparts column parts per kept tile to the work queue: the tile's
+                // minimum is reset here, before any part can atomicMin into it
+                if (keep) tilebest[t] = kKeyNone;
+                int qb = 0;
+                if (lane == 0) qb = atomicAdd(&queue[0].x, __popc(kept) * nparts);
+                qb = __shfl_sync(0xffffffffu, qb, 0) + __popc(kept & ((1u << lane) - 1u)) * nparts;
+                if (keep) {
+                    __threadfence();
+                    for (int k = 0; k < nparts; k++) {
+                        int4* it = queue + 1 + qb + k;
+                        it->x = rb;
+                        it->y = cc;
+                        it->z = t;
+                        __threadfence();
+                        *(volatile int*)&it->w = k + 1;  // ready flag, written last
+                    }
+                }
+            }
+        }
+        if (nparts > 1) {
+            // consume: parts claimed one at a time until every warp has culled and the
+            // queue is drained; a claimed slot is cleared (w = 0) for the next iteration
+            __syncwarp();
+            if (lane == 0) {
+                __threadfence();
+                atomicAdd(&queue[0].z, 1);
+            }
+            const int TJp = TJ / nparts;
+            for (;;) {
+                int idx = 0;
+                if (lane == 0) idx = atomicAdd(&queue[0].y, 1);
+                idx = __shfl_sync(0xffffffffu, idx, 0);
+                int4 it = make_int4(0, 0, 0, 0);
+                int state = 0;  // 1 item ready, 2 no more items
+                if (lane == 0) {
+                    volatile int* w = &queue[1 + idx].w;
+                    for (;;) {
+                        if (*w) {
+                            __threadfence();
+                            it = __ldcg(queue + 1 + idx);
+                            state = 1;
+                            break;
+                        }
+                        if (*(volatile int*)&queue[0].z == nw && idx >= *(volatile int*)&queue[0].x) {
+                            state = 2;
+                            break;
+                        }
+                        __nanosleep(32);
+                    }
+                }
+                state = __shfl_sync(0xffffffffu, state, 0);
+                if (state == 2) break;
+                it.x = __shfl_sync(0xffffffffu, it.x, 0);
+                it.y = __shfl_sync(0xffffffffu, it.y, 0);
+                it.z = __shfl_sync(0xffffffffu, it.z, 0);
+                it.w = __shfl_sync(0xffffffffu, it.w, 0);
+                sweep_tile<R, true, FIRST, true>(P, E, n, make_int2(it.x * TI, it.y * TJ + (it.w - 1) * TJp), TJp, in,
+                                                 sm, tilebest + it.z, tflags | kSweepAtomicBest);
+                if (lane == 0) queue[1 + idx].w = 0;
             }
         }
         PHASE_MARK(2);
@@ -1023,6 +1086,7 @@ cudaError_t launch_reset_key(Slot* slot, cudaStream_t st)
 }
 
 size_t sweep_smem_bytes(const Geometry& g) { return tile_smem_bytes(g.tj, g.ti()); }
+size_t sweep_smem_bytes_ps(const Geometry& g) { return tile_smem_bytes(g.tj, g.ti(), true); }
 
 // The sweep is instantiated for R = 15 (large n: longest column steps) and
 // R = 7 (small / medium n: twice the warps per row block, lower latency per
@@ -1071,7 +1135,7 @@ cudaError_t sweep_prepare()
         }
         e = by_rows(R, [&](auto r) {
             return cudaFuncSetAttribute(local_search_kernel<decltype(r)::value>,
-                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sweep_smem_bytes(gmax));
+                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sweep_smem_bytes_ps(gmax));
         });
         if (e != cudaSuccess) return e;
     }
@@ -1126,11 +1190,12 @@ constexpr int kIncLsThreads = 512;  // 16 warps, one CTA per SM
 cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
                           const int* tmap, Box* rbox, Box* cbox, Slot* slots, int parity, long long max_moves,
                           long long budget, int full, unsigned* bar, int* ctl, unsigned long long* tilebest, int flags,
-                          unsigned long long* trace, long long trace_cap, cudaStream_t st)
+                          unsigned long long* trace, long long trace_cap, int nparts, int4* queue, cudaStream_t st)
 {
     if (g.rows != kRowsSmall || g.warps != 1) return cudaErrorInvalidValue;
+    if (nparts > 1 && (g.tj % nparts != 0 || !queue)) return cudaErrorInvalidValue;
     int TI = g.ti(), TJ = g.tj, nrb = (n - 1 + TI - 1) / TI, ncc = (n + TJ - 1) / TJ;
-    int tile_bytes = (int)((sweep_smem_bytes(g) + 15) / 16 * 16);
+    int tile_bytes = (int)((sweep_smem_bytes_ps(g) + 15) / 16 * 16);
     const size_t smem = (size_t)tile_bytes * (kIncLsThreads / 32);
     auto kern = (flags & kSweepFirst) ? inc_ls_kernel<kRowsSmall, true> : inc_ls_kernel<kRowsSmall, false>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -1144,7 +1209,8 @@ cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int grid = sms;  // one CTA per SM (co-resident: cooperative launch)
     void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &tmap, &TI, &TJ, &nrb, &ncc, &rbox, &cbox, &slots, &parity,
-                    &max_moves, &budget, &full, &bar, &ctl, &tilebest, &flags, &trace, &trace_cap, &tile_bytes};
+                    &max_moves, &budget, &full, &bar, &ctl, &tilebest, &flags, &trace, &trace_cap, &tile_bytes,
+                    &nparts, &queue};
     g_launches += 1;
     return cudaLaunchCooperativeKernel((const void*)kern, dim3(grid), dim3(kIncLsThreads), args, smem, st);
 }
@@ -1219,7 +1285,7 @@ int local_search_grid(const Geometry& g, int ntiles)
     int per_sm = 0;
     cudaError_t e = by_rows(g.rows, [&](auto r) {
         return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, local_search_kernel<decltype(r)::value>,
-                                                             32 * g.warps, sweep_smem_bytes(g));
+                                                             32 * g.warps, sweep_smem_bytes_ps(g));
     });
     if (e != cudaSuccess) return 0;
     int dev = 0, sms = 0;
@@ -1242,7 +1308,7 @@ cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour,
     g_launches += 1;
     return by_rows(g.rows, [&](auto r) {
         return cudaLaunchCooperativeKernel((const void*)local_search_kernel<decltype(r)::value>, dim3(grid),
-                                           dim3(32 * g.warps), args, sweep_smem_bytes(g), st);
+                                           dim3(32 * g.warps), args, sweep_smem_bytes_ps(g), st);
     });
 }
 

@@ -202,7 +202,9 @@ __device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1
     while (mask) {  // ascending r == ascending cell number
         const int r = __ffs(mask) - 1;
         mask &= mask - 1;
-        const float2 pi = my_rowp[r], pi1 = my_rowp[r + 1];
+        // PS (persistent kernels): the row cities staged in shared memory (P's L1 lines are
+        // invalidated by every grid barrier); otherwise my_rowp = P + row0, read through L1
+        const float2 pi = PS ? my_rowp[r] : __ldg(my_rowp + r), pi1 = PS ? my_rowp[r + 1] : __ldg(my_rowp + r + 1);
         // nint from the float path when it is unambiguous: |sqrt_approx(s_f) - sqrt(s)|
         // < 0.03, so |r - m| < 0.45 for the nearest integer m
         // proves nint(sqrt(s)) == m.  Otherwise the integer nint (rare).
@@ -421,12 +423,13 @@ __device__ __forceinline__ bool tile_may_pass(const Rows<R>& rows, const Bound<R
     return d2 * 0.99999904632568359375f <= thr;  // (1 - 2^-20)
 }
 
-// Shared memory bytes of a tile with TJ columns and TI rows.
-__host__ __device__ inline size_t tile_smem_bytes(int TJ, int TI)
+// Shared memory bytes of a tile with TJ columns and TI rows; rowp: the
+// persistent kernels' staged row cities, (TI / R) * (R + 1) <= TI + TI / 7
+// entries for R >= 7, plus slack.
+__host__ __device__ inline size_t tile_smem_bytes(int TJ, int TI, bool rowp = false)
 {
-    // rowp: (TI / R) * (R + 1) <= TI + TI / 7 entries for R >= 7, plus slack
     return (size_t)(TJ + 2) * kColRec * sizeof(float4) + (size_t)TI * sizeof(float) +
-           (size_t)(TI + TI / 7 + 32) * sizeof(float2);
+           (rowp ? (size_t)(TI + TI / 7 + 32) * sizeof(float2) : 0);
 }
 
 // One tile.  All global loads of the tile (the lane's rows and row edges, the
@@ -455,7 +458,7 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     const int jstart = max(J0, wrow0 + 1);  // no pair of this warp has j <= wrow0
     const bool active = jstart < J1;        // warp-uniform
     float* my_rowe = sm.rowe + tid * R;  // stride R (odd): conflict-free
-    float2* my_rowp = sm.rowp + tid * (R + 1);
+    float2* my_rowp = PS ? sm.rowp + tid * (R + 1) : const_cast<float2*>(P) + row0;
 
     Rows<R> rows;
     float erow[R];
@@ -465,8 +468,10 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
             const float2 p0 = gld<PS>(P + row0 + 2 * q), p1 = gld<PS>(P + row0 + 2 * q + 1);
             rows.xp[q] = make_float2(p0.x, p1.x);
             rows.yp[q] = make_float2(p0.y, p1.y);
-            my_rowp[2 * q] = p0;
-            my_rowp[2 * q + 1] = p1;
+            if (PS) {
+                my_rowp[2 * q] = p0;
+                my_rowp[2 * q + 1] = p1;
+            }
         }
 #pragma unroll
         for (int r = 0; r < R; r++) erow[r] = (float)gld<PS>(E + row0 + r);
@@ -525,7 +530,11 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     // The tile's best (a real pair of this sweep, or none) is kept for the next
     // iteration's seed (apply_phase: moves the applied reversal leaves intact).
     if (WT) {
-        if (lane == 0) *tilebest = active ? mykey : kKeyNone;  // mykey is the warp minimum here
+        if (flags & kSweepAtomicBest) {  // one of several parts of the tile: min into the tile's entry
+            if (lane == 0 && active && mykey != kKeyNone) atomicMin(tilebest, mykey);
+        } else if (lane == 0) {
+            *tilebest = active ? mykey : kKeyNone;  // mykey is the warp minimum here
+        }
         __syncwarp();
         return;
     }
