@@ -393,11 +393,13 @@ int tsp2opt_selftest_sqrt(double *max_rel_err, int32_t *zero_ok);
 int tsp2opt_debug_stats(int64_t *out4, int32_t reset);
 
 /* Phase clocks of the persistent incremental local search in an instrumented
- * build (-DTSP2OPT_PHASE_TIMING): out8[k] = SM clock cycles CTA 0 spent in
- * [0] dirty boxes, [1] barrier, [6] clean-minimum scan, [2] cull + kept-tile
- * sweeps, [3] barrier, [4] apply, [5] barrier, summed over iterations; -1 in
+ * build (-DTSP2OPT_PHASE_TIMING), summed over iterations: out16[k] = SM clock
+ * cycles CTA 0 spent in [0] dirty boxes, [1] barrier, [2] cull + kept-tile
+ * sweeps, [6] clean-minimum scan, [3] barrier, [4] apply, [5] barrier; over
+ * all warps, per iteration: [8] the longest cull + sweep, [9] the most kept
+ * tiles of one warp, [10] the longest cull alone, [11] the kept tiles; -1 in
  * product builds.  reset != 0 zeroes them afterwards. */
-int tsp2opt_debug_phases(int64_t *out8, int32_t reset);
+int tsp2opt_debug_phases(int64_t *out16, int32_t reset);
 
 /* Number of this library's kernel launches since load (for gpu_launches). */
 int64_t tsp2opt_launch_count(void);

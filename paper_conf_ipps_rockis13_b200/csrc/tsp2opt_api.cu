@@ -85,8 +85,7 @@ struct tsp2opt_ctx {
     int inc_grid = 0;           // one-warp CTAs of the fused incremental sweep (co-resident)
     bool inc_fused = true;      // TSP2OPT_INC_FUSED=0: the box + cull + list kernels on every iteration
     bool inc_persistent = true; // TSP2OPT_INC_PERSISTENT=0: per-iteration launches instead of one cooperative launch
-    int inc_parts = 1;          // TSP2OPT_INC_PARTS: column parts per kept tile in the persistent search (work queue)
-    int4* d_incq = nullptr;     // its queue: [0] = (count, next, culled warps), then nctiles * inc_parts items
+    bool dense_ls = true;       // TSP2OPT_DENSE_LS=0: per-iteration kernels for the dense loop above the persistent size
     int nctiles = 0;
     int list_grid = 0;          // CTAs of the culled sweep (co-resident)
     int list25_grid = 0;        // CTAs of the 2.5-opt culled sweep
@@ -235,7 +234,6 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
         std::vector<Tile> mine = shard_tiles(h->all_ctiles, rank, world, &unused);
         for (size_t k = 0; k < mine.size(); k++) map[(size_t)(mine[k].i0 / TI) * ncc + mine[k].j0 / TJ] = (int)k;
         cudaFree(h->d_tmap);
-    cudaFree(h->d_incq);
     for (void* p : h->p2p_opened)
         if (p) cudaIpcCloseMemHandle(p);
     cudaFree(h->d_peers);
@@ -244,13 +242,6 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
         CUDA_TRY(cudaMalloc(&h->d_tmap, sizeof(int) * map.size()));
         CUDA_TRY(cudaMemcpy(h->d_tmap, map.data(), sizeof(int) * map.size(), cudaMemcpyHostToDevice));
         h->inc_grid = inc_sweep_grid(h->cgeo);
-        cudaFree(h->d_incq);
-        h->d_incq = nullptr;
-        if (h->inc_parts > 1) {
-            const size_t items = 1 + (size_t)h->inc_parts * std::max(1, h->nctiles) + 8192;  // + over-claims
-            CUDA_TRY(cudaMalloc(&h->d_incq, sizeof(int4) * items));
-            CUDA_TRY(cudaMemset(h->d_incq, 0, sizeof(int4) * items));
-        }
     }
     h->list_grid = sweep_list_grid(h->cgeo, h->nctiles);
     if (const char* el = getenv("TSP2OPT_LIST_GRID"))  // experiment: cap the list sweep's co-resident grid
@@ -284,7 +275,6 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_ctilebest);
     cudaFree(h->d_list);
     cudaFree(h->d_tmap);
-    cudaFree(h->d_incq);
     for (void* p : h->p2p_opened)
         if (p) cudaIpcCloseMemHandle(p);
     cudaFree(h->d_peers);
@@ -479,6 +469,11 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
     // = 0 / 1 forces either loop, 2 (default) chooses by pair count.
     const bool use_persistent =
         !h->comm && !h->p2p && h->nbr_k == 0 && !h->or25 && !h->first && (h->persistent == 1 || (h->persistent == 2 && h->shard_pairs <= 4000000LL));
+    // dense best-improvement sweeps above that (n ~ 7e3, in-sweep tile bound): the
+    // persistent loop with dynamic warp-level claims (TSP2OPT_PERSISTENT = 3 forces it)
+    const bool use_dense_ls = !use_persistent && !h->comm && !h->p2p && h->nbr_k == 0 && !h->or25 && !h->first &&
+                              h->tile_bounds <= 1 && h->geo.warps == 1 && !h->profiling && h->shard_world == 1 &&
+                              (h->persistent == 3 || (h->persistent == 2 && h->dense_ls));
     // The incremental culled search of a single GPU in one cooperative launch per
     // ~1M iterations (launch_inc_ls): no per-iteration launches, three grid barriers
     // per move.  Sharded handles keep the per-iteration kernels (the exchange sits
@@ -496,14 +491,30 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
             }
             CUDA_TRY(launch_inc_ls(h->cgeo, h->d_P, h->d_E, h->d_tour, h->n, h->d_ctiles, h->nctiles, h->d_tmap,
                                    h->d_rbox, h->d_cbox, h->d_slots, h->parity, max_iters, 1LL << 20, full, h->d_bar,
-                                   h->d_ctl, h->d_ctilebest, flags, h->d_trace, h->trace_cap, h->inc_parts,
-                                   h->d_incq, h->stream));
+                                   h->d_ctl, h->d_ctilebest, flags, h->d_trace, h->trace_cap, h->stream));
             full = 0;
             CUDA_TRY(cudaMemcpyAsync(h->h_ctl, h->d_ctl, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
             CUDA_TRY(cudaStreamSynchronize(h->stream));
             h->parity = *h->h_ctl;
             h->inc_valid = true;  // the stored tile minima are tile-local and exact for the current tour
             h->last_tiling = 1;
+            rc = read_slot(h);
+            if (rc) return rc;
+            if (h->h_slot->done & 3) break;
+        }
+    } else if (use_dense_ls) {
+        h->inc_valid = false;
+        for (long long launches = 0;; launches++) {
+            if (launches > 1000000) {
+                g_last_error = "local search did not converge";
+                return TSP2OPT_ECUDA;
+            }
+            CUDA_TRY(launch_dense_ls(h->geo, h->d_P, h->d_E, h->d_tour, h->n, h->d_tiles, h->ntiles, h->d_slots,
+                                     h->parity, max_iters, 1LL << 20, h->d_bar, h->d_ctl, sweep_flags(h),
+                                     h->d_tilebest, h->d_trace, h->trace_cap, h->stream));
+            CUDA_TRY(cudaMemcpyAsync(h->h_ctl, h->d_ctl, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+            CUDA_TRY(cudaStreamSynchronize(h->stream));
+            h->parity = *h->h_ctl;
             rc = read_slot(h);
             if (rc) return rc;
             if (h->h_slot->done & 3) break;
@@ -638,10 +649,7 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     if (const char* eg = getenv("TSP2OPT_GLOBAL_SEED")) h->global_seed = atoi(eg) != 0;
     if (const char* ef = getenv("TSP2OPT_INC_FUSED")) h->inc_fused = atoi(ef) != 0;
     if (const char* ei = getenv("TSP2OPT_INC_PERSISTENT")) h->inc_persistent = atoi(ei) != 0;
-    if (const char* ep2 = getenv("TSP2OPT_INC_PARTS")) {
-        const int v = atoi(ep2);
-        if (v == 1 || v == 2 || v == 4 || v == 8) h->inc_parts = v;
-    }
+    if (const char* ed = getenv("TSP2OPT_DENSE_LS")) h->dense_ls = atoi(ed) != 0;
 
     CTRY(cudaMemset(h->d_slots, 0, sizeof(Slot) * 2));
     {
@@ -1334,12 +1342,12 @@ int tsp2opt_selftest_sqrt(double* max_rel_err, int32_t* zero_ok)
     return TSP2OPT_OK;
 }
 
-int tsp2opt_debug_phases(int64_t* out8, int32_t reset)
+int tsp2opt_debug_phases(int64_t* out16, int32_t reset)
 {
-    if (!out8) return TSP2OPT_EINVAL;
-    long long v[8];
+    if (!out16) return TSP2OPT_EINVAL;
+    long long v[16];
     CUDA_TRY(read_phases(v, reset));
-    for (int k = 0; k < 8; k++) out8[k] = v[k];
+    for (int k = 0; k < 16; k++) out16[k] = v[k];
     return TSP2OPT_OK;
 }
 

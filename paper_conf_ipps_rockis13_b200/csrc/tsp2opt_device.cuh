@@ -33,7 +33,6 @@ constexpr int kSweepFull = 16;       // incremental sweep whose stored minima ar
 // delta, so the min is the lowest cell; first_fix_kernel writes the real delta.
 constexpr int kFirstDelta = -1;
 constexpr int kSweepFirst = 32;      // first improvement: the lowest improving cell instead of the lowest delta
-constexpr int kSweepAtomicBest = 64; // the tile is swept in parts: each part atomicMins its minimum into the entry
 
 // Bounding box of a run of route positions (unbiased integer coordinates) and
 // the largest tour edge leaving it: the summaries the tile cull compares.
@@ -310,7 +309,7 @@ __device__ __forceinline__ void grid_sync(unsigned* bar, unsigned nblocks)
             __threadfence();
             atomicAdd(bar + 1, 1u);
         } else {
-            while (*vgen == gen) __nanosleep(32);
+            while (*vgen == gen) __nanosleep(32);  // (a busy spin measured the same, r02)
         }
         __threadfence();
     }

@@ -118,13 +118,18 @@ cudaError_t launch_cull_sweep(const Geometry& g, const float2* P, const int* E, 
 // dirty tiles enumerated from the last move via tmap, boxes recomputed in place, cull and sweep
 // in one launch of `grid` one-warp CTAs (inc_sweep_grid), clean minima folded into the key.
 int inc_sweep_grid(const Geometry& g);
+// Persistent dense local search with dynamic warp-level tile claims (one cooperative launch).
+cudaError_t launch_dense_ls(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
+                            Slot* slots, int parity, long long max_moves, long long budget, unsigned* bar, int* ctl,
+                            int flags, unsigned long long* tilebest, unsigned long long* trace, long long trace_cap,
+                            cudaStream_t st);
 // Persistent incremental local search (one cooperative launch, one CTA of 16 warps per SM):
 // up to `budget` iterations of {dirty boxes; clean minima + cull + kept-tile sweeps; apply};
 // full = 1 makes the first iteration the full culled sweep.  ctl[0] = the final slot parity.
 cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
                           const int* tmap, Box* rbox, Box* cbox, Slot* slots, int parity, long long max_moves,
                           long long budget, int full, unsigned* bar, int* ctl, unsigned long long* tilebest, int flags,
-                          unsigned long long* trace, long long trace_cap, int nparts, int4* queue, cudaStream_t st);
+                          unsigned long long* trace, long long trace_cap, cudaStream_t st);
 cudaError_t launch_inc_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
                              const int* tmap, int grid, Box* rbox, Box* cbox, Slot* slot, int respect_done,
                              unsigned long long* tilebest, int flags, cudaStream_t st);
@@ -140,7 +145,7 @@ cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour,
 cudaError_t launch_p2p_min(Slot* slot, Mailbox* const* peers, int rank, int world, int respect_done,
                            cudaStream_t st);
 cudaError_t read_stats(long long* out4, int reset);
-cudaError_t read_phases(long long* out8, int reset);
+cudaError_t read_phases(long long* out16, int reset);
 cudaError_t run_selftest_sqrt(double* max_rel, int* zero_ok);
 cudaError_t run_selftest(long long* out4);  // dist_bad, filter_bad, first bad s, first bad dx<<15|dy
 

@@ -19,7 +19,8 @@ namespace tsp2opt {
 // Instrumented builds only: clock cycles CTA 0 spends in each phase of the
 // persistent incremental local search (boxes, barrier, sweep, barrier, apply,
 // barrier), summed over the iterations; read by tsp2opt_debug_stats.
-__device__ unsigned long long g_phase[8];
+__device__ unsigned long long g_phase[16];
+__device__ unsigned long long g_phase_it[4];  // per-iteration maxima, folded into g_phase[8..11] by CTA 0
 #endif
 
 // ===========================================================================
@@ -697,7 +698,7 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
                                                         int* __restrict__ ctl,
                                                         unsigned long long* __restrict__ tilebest, int flags,
                                                         unsigned long long* __restrict__ trace, long long trace_cap,
-                                                        int tile_bytes, int nparts, int4* __restrict__ queue)
+                                                        int tile_bytes)
 {
     extern __shared__ float4 smem[];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -740,7 +741,6 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
         }
         const int rlo = dlo >= 1 ? (dlo - 1) / TI : 0, rhi = min(nrb - 1, dhi / TI);
         const int clo = dlo >= 1 ? (dlo - 1) / TJ : 0, chi = min(ncc - 1, dhi / TJ);
-        if (gtid == 0 && nparts > 1) queue[0] = make_int4(0, 0, 0, 0);  // count, next, culled warps (seen after the barrier)
         // (B) boxes of the dirty blocks
         {
             const int nR = rhi - rlo + 1, nC = chi - clo + 1;
@@ -760,6 +760,11 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
         grid_sync(bar, gridDim.x);
         PHASE_MARK(1);
         // (C2) the dirty tiles: cull per thread, sweep the kept ones per warp
+#ifdef TSP2OPT_PHASE_TIMING
+        const long long tw0 = clock64();
+        long long tcull = 0, tsweep = 0;
+        int nkept = 0;
+#endif
         const long long nA = (long long)(rhi - rlo + 1) * ncc;
         const long long nB = (long long)nrb * (chi - clo + 1);
         for (long long base = 0; base < nA + nB; base += (long long)nw * 32) {
@@ -786,77 +791,31 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
                 if (!keep) tilebest[t] = kKeyNone;
             }
             unsigned kept = __ballot_sync(0xffffffffu, keep);
-            if (nparts <= 1) {
-                while (kept) {  // this warp sweeps the kept tiles its lanes found
-                    const int src = __ffs(kept) - 1;
-                    kept &= kept - 1;
-                    const int kt = __shfl_sync(0xffffffffu, t, src);
-                    const int krb = __shfl_sync(0xffffffffu, rb, src), kcc = __shfl_sync(0xffffffffu, cc, src);
-                    sweep_tile<R, true, FIRST, true>(P, E, n, make_int2(krb * TI, kcc * TJ), TJ, in, sm,
-                                                     tilebest + kt, tflags);
-                }
-            } else if (kept) {
-                // publish nparts column parts per kept tile to the work queue: the tile's
-                // minimum is reset here, before any part can atomicMin into it
-                if (keep) tilebest[t] = kKeyNone;
-                int qb = 0;
-                if (lane == 0) qb = atomicAdd(&queue[0].x, __popc(kept) * nparts);
-                qb = __shfl_sync(0xffffffffu, qb, 0) + __popc(kept & ((1u << lane) - 1u)) * nparts;
-                if (keep) {
-                    __threadfence();
-                    for (int k = 0; k < nparts; k++) {
-                        int4* it = queue + 1 + qb + k;
-                        it->x = rb;
-                        it->y = cc;
-                        it->z = t;
-                        __threadfence();
-                        *(volatile int*)&it->w = k + 1;  // ready flag, written last
-                    }
-                }
+#ifdef TSP2OPT_PHASE_TIMING
+            if (base == 0) tcull = clock64() - tw0;  // the first round's cull
+            nkept += __popc(kept);
+            const long long ts0 = clock64();
+#endif
+            while (kept) {  // this warp sweeps the kept tiles its lanes found
+                const int src = __ffs(kept) - 1;
+                kept &= kept - 1;
+                const int kt = __shfl_sync(0xffffffffu, t, src);
+                const int krb = __shfl_sync(0xffffffffu, rb, src), kcc = __shfl_sync(0xffffffffu, cc, src);
+                sweep_tile<R, true, FIRST, true>(P, E, n, make_int2(krb * TI, kcc * TJ), TJ, in, sm, tilebest + kt,
+                                                 tflags);
             }
+#ifdef TSP2OPT_PHASE_TIMING
+            tsweep += clock64() - ts0;
+#endif
         }
-        if (nparts > 1) {
-            // consume: parts claimed one at a time until every warp has culled and the
-            // queue is drained; a claimed slot is cleared (w = 0) for the next iteration
-            __syncwarp();
-            if (lane == 0) {
-                __threadfence();
-                atomicAdd(&queue[0].z, 1);
-            }
-            const int TJp = TJ / nparts;
-            for (;;) {
-                int idx = 0;
-                if (lane == 0) idx = atomicAdd(&queue[0].y, 1);
-                idx = __shfl_sync(0xffffffffu, idx, 0);
-                int4 it = make_int4(0, 0, 0, 0);
-                int state = 0;  // 1 item ready, 2 no more items
-                if (lane == 0) {
-                    volatile int* w = &queue[1 + idx].w;
-                    for (;;) {
-                        if (*w) {
-                            __threadfence();
-                            it = __ldcg(queue + 1 + idx);
-                            state = 1;
-                            break;
-                        }
-                        if (*(volatile int*)&queue[0].z == nw && idx >= *(volatile int*)&queue[0].x) {
-                            state = 2;
-                            break;
-                        }
-                        __nanosleep(32);
-                    }
-                }
-                state = __shfl_sync(0xffffffffu, state, 0);
-                if (state == 2) break;
-                it.x = __shfl_sync(0xffffffffu, it.x, 0);
-                it.y = __shfl_sync(0xffffffffu, it.y, 0);
-                it.z = __shfl_sync(0xffffffffu, it.z, 0);
-                it.w = __shfl_sync(0xffffffffu, it.w, 0);
-                sweep_tile<R, true, FIRST, true>(P, E, n, make_int2(it.x * TI, it.y * TJ + (it.w - 1) * TJp), TJp, in,
-                                                 sm, tilebest + it.z, tflags | kSweepAtomicBest);
-                if (lane == 0) queue[1 + idx].w = 0;
-            }
+#ifdef TSP2OPT_PHASE_TIMING
+        if (lane == 0) {
+            atomicMax(&g_phase_it[0], (unsigned long long)(clock64() - tw0));
+            atomicMax(&g_phase_it[1], (unsigned long long)tsweep);
+            atomicMax(&g_phase_it[2], (unsigned long long)tcull);
+            atomicAdd(&g_phase_it[3], (unsigned long long)nkept);
         }
+#endif
         PHASE_MARK(2);
         // (C1) the clean tiles' stored minima -- after the sweeps, so that warps
         // without kept tiles do it while the others still sweep; loads batched
@@ -891,6 +850,13 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
         }
         grid_sync(bar, gridDim.x);
         PHASE_MARK(3);
+#ifdef TSP2OPT_PHASE_TIMING
+        if (blockIdx.x == 0 && threadIdx.x == 0)
+            for (int q = 0; q < 4; q++) {
+                g_phase[8 + q] += g_phase_it[q];
+                g_phase_it[q] = 0;
+            }
+#endif
         // (A) apply the winning move
         if (threadIdx.x == 0) {
             unsigned long long key = *(volatile unsigned long long*)&in->key;
@@ -913,6 +879,63 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
     }
     if (gtid == 0) ctl[0] = p;
 #undef PHASE_MARK
+}
+
+// ===========================================================================
+// Persistent dense local search with dynamic tile claims (medium n, one GPU):
+// one cooperative launch of one 16-warp CTA per SM; per iteration every WARP
+// claims tiles of the dense tiling from the slot's counter (largest first) and
+// sweeps each with its private shared memory and the in-sweep bound (the slot's
+// running key), then one grid barrier, the apply, another barrier.  The round-
+// robin tile assignment of local_search_kernel lost to the per-iteration
+// kernels from n ~ 7e3 because static shares of unequal tiles imbalance; the
+// claims balance them, and two barriers replace two launches per move.
+// ===========================================================================
+template <int R>
+__global__ void __launch_bounds__(512, 1) dense_ls_kernel(float2* __restrict__ P, int* __restrict__ E,
+                                                          int* __restrict__ tour, int n,
+                                                          const int2* __restrict__ tiles, int ntiles, int TJ,
+                                                          Slot* __restrict__ slots, int parity, long long max_moves,
+                                                          long long budget, unsigned* __restrict__ bar,
+                                                          int* __restrict__ ctl, int flags,
+                                                          unsigned long long* __restrict__ tilebest,
+                                                          unsigned long long* __restrict__ trace, long long trace_cap,
+                                                          int tile_bytes)
+{
+    extern __shared__ float4 smem[];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const TileSmem sm(reinterpret_cast<char*>(smem) + (size_t)wib * tile_bytes, TJ, 32 * R);
+    const int gtid = blockIdx.x * blockDim.x + threadIdx.x, stride = gridDim.x * blockDim.x;
+    const int tflags = flags & ~(kSweepSeed | kSweepLocal | kSweepIncremental);
+    __shared__ Slot s_in;
+    int p = parity;
+    for (long long it = 0; it < budget; it++) {
+        Slot* in = slots + p;
+        if (threadIdx.x == 0) s_in.done = *(volatile int*)&in->done;
+        __syncthreads();
+        if (s_in.done) break;  // uniform across the grid
+        for (;;) {
+            int t = 0;
+            if (lane == 0) t = (int)atomicAdd(&in->next_tile, 1u);
+            t = __shfl_sync(0xffffffffu, t, 0);
+            if (t >= ntiles) break;
+            sweep_tile<R, true, false, true>(P, E, n, tiles[t], TJ, in, sm, tilebest + t, tflags);
+        }
+        grid_sync(bar, gridDim.x);
+        if (threadIdx.x == 0) {
+            s_in.key = *(volatile unsigned long long*)&in->key;
+            s_in.last_key = in->last_key;
+            s_in.moves = *(volatile long long*)&in->moves;
+            s_in.length = *(volatile long long*)&in->length;
+            s_in.done = *(volatile int*)&in->done;
+            s_in.seed_ok = *(volatile int*)&in->seed_ok;
+        }
+        __syncthreads();
+        apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride, trace, trace_cap, nullptr);
+        p ^= 1;
+        grid_sync(bar, gridDim.x);
+    }
+    if (gtid == 0) ctl[0] = p;
 }
 
 // ===========================================================================
@@ -1190,10 +1213,9 @@ constexpr int kIncLsThreads = 512;  // 16 warps, one CTA per SM
 cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
                           const int* tmap, Box* rbox, Box* cbox, Slot* slots, int parity, long long max_moves,
                           long long budget, int full, unsigned* bar, int* ctl, unsigned long long* tilebest, int flags,
-                          unsigned long long* trace, long long trace_cap, int nparts, int4* queue, cudaStream_t st)
+                          unsigned long long* trace, long long trace_cap, cudaStream_t st)
 {
     if (g.rows != kRowsSmall || g.warps != 1) return cudaErrorInvalidValue;
-    if (nparts > 1 && (g.tj % nparts != 0 || !queue)) return cudaErrorInvalidValue;
     int TI = g.ti(), TJ = g.tj, nrb = (n - 1 + TI - 1) / TI, ncc = (n + TJ - 1) / TJ;
     int tile_bytes = (int)((sweep_smem_bytes_ps(g) + 15) / 16 * 16);
     const size_t smem = (size_t)tile_bytes * (kIncLsThreads / 32);
@@ -1209,10 +1231,34 @@ cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int grid = sms;  // one CTA per SM (co-resident: cooperative launch)
     void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &tmap, &TI, &TJ, &nrb, &ncc, &rbox, &cbox, &slots, &parity,
-                    &max_moves, &budget, &full, &bar, &ctl, &tilebest, &flags, &trace, &trace_cap, &tile_bytes,
-                    &nparts, &queue};
+                    &max_moves, &budget, &full, &bar, &ctl, &tilebest, &flags, &trace, &trace_cap, &tile_bytes};
     g_launches += 1;
     return cudaLaunchCooperativeKernel((const void*)kern, dim3(grid), dim3(kIncLsThreads), args, smem, st);
+}
+
+cudaError_t launch_dense_ls(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
+                            Slot* slots, int parity, long long max_moves, long long budget, unsigned* bar, int* ctl,
+                            int flags, unsigned long long* tilebest, unsigned long long* trace, long long trace_cap,
+                            cudaStream_t st)
+{
+    if (g.warps != 1) return cudaErrorInvalidValue;
+    int TJ = g.tj;
+    int tile_bytes = (int)((sweep_smem_bytes_ps(g) + 15) / 16 * 16);
+    const size_t smem = (size_t)tile_bytes * (kIncLsThreads / 32);
+    auto kern = g.rows == kRowsSmall ? dense_ls_kernel<kRowsSmall> : dense_ls_kernel<kRowsLarge>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kIncLsThreads, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) return cudaErrorInvalidConfiguration;
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &TJ, &slots, &parity, &max_moves, &budget, &bar, &ctl,
+                    &flags, &tilebest, &trace, &trace_cap, &tile_bytes};
+    g_launches += 1;
+    return cudaLaunchCooperativeKernel((const void*)kern, dim3(sms), dim3(kIncLsThreads), args, smem, st);
 }
 
 int inc_sweep_grid(const Geometry& g)
@@ -1330,21 +1376,21 @@ cudaError_t run_selftest_sqrt(double* max_rel, int* zero_ok)
     return err;
 }
 
-cudaError_t read_phases(long long* out8, int reset)
+cudaError_t read_phases(long long* out16, int reset)
 {
 #ifdef TSP2OPT_PHASE_TIMING
-    unsigned long long ph[8];
+    unsigned long long ph[16];
     cudaError_t ep = cudaMemcpyFromSymbol(ph, g_phase, sizeof(ph));
     if (ep != cudaSuccess) return ep;
-    for (int k = 0; k < 8; k++) out8[k] = (long long)ph[k];
+    for (int k = 0; k < 16; k++) out16[k] = (long long)ph[k];
     if (reset) {
-        const unsigned long long z[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        const unsigned long long z[16] = {};
         ep = cudaMemcpyToSymbol(g_phase, z, sizeof(z));
     }
     return ep;
 #else
     (void)reset;
-    for (int k = 0; k < 8; k++) out8[k] = -1;
+    for (int k = 0; k < 16; k++) out16[k] = -1;
     return cudaSuccess;
 #endif
 }

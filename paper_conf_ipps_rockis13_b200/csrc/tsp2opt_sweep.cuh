@@ -530,11 +530,7 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
     // The tile's best (a real pair of this sweep, or none) is kept for the next
     // iteration's seed (apply_phase: moves the applied reversal leaves intact).
     if (WT) {
-        if (flags & kSweepAtomicBest) {  // one of several parts of the tile: min into the tile's entry
-            if (lane == 0 && active && mykey != kKeyNone) atomicMin(tilebest, mykey);
-        } else if (lane == 0) {
-            *tilebest = active ? mykey : kKeyNone;  // mykey is the warp minimum here
-        }
+        if (lane == 0) *tilebest = active ? mykey : kKeyNone;  // mykey is the warp minimum here
         __syncwarp();
         return;
     }

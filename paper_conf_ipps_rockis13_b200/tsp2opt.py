@@ -532,7 +532,7 @@ class TSP2Opt:
 
 def debug_phases(reset: bool = True) -> list:
     """Phase clocks of the persistent incremental search (instrumented builds; -1 otherwise)."""
-    out = np.zeros(8, dtype=np.int64)
+    out = np.zeros(16, dtype=np.int64)
     _check(_L().tsp2opt_debug_phases(_ptr(out), 1 if reset else 0), "tsp2opt_debug_phases")
     return out.tolist()
 

@@ -8,7 +8,8 @@ import sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ipps_rockis13_b200 import inputs, tsp2opt  # noqa: E402
 
-names = ["boxes", "barrier1", "cull+sweep", "barrier2", "apply", "barrier3", "clean_scan", "-"]
+names = ["boxes", "barrier1", "cull+sweep", "barrier2", "apply", "barrier3", "clean_scan", "-",
+         "max_warp_cull+sweep", "max_warp_sweeps", "max_warp_first_cull", "kept_tiles(count)"]
 for cfg, tk in (("C4", "hilbert"), ("C5", "hilbert"), ("C5", "mf")):
     c, t = inputs.config_instance(cfg, "random" if tk == "mf" else tk)
     with tsp2opt.TSP2Opt(c) as g:
@@ -19,5 +20,6 @@ for cfg, tk in (("C4", "hilbert"), ("C5", "hilbert"), ("C5", "mf")):
         ph = tsp2opt.debug_phases(True)
     k = max(1, r["iterations"])
     print(json.dumps({"config": cfg, "start": tk, "moves": r["iterations"],
-                      "us_per_move_at_1.9GHz": {nm: round(v / k / 1900.0, 3) for nm, v in zip(names, ph) if nm != "-"}}),
+                      "us_per_move_at_1.9GHz": {nm: round(v / k / (1.0 if "count" in nm else 1900.0), 3)
+                                                for nm, v in zip(names, ph) if nm != "-"}}),
           flush=True)
