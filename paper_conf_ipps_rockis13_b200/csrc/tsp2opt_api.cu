@@ -85,7 +85,8 @@ struct tsp2opt_ctx {
     int inc_grid = 0;           // one-warp CTAs of the fused incremental sweep (co-resident)
     bool inc_fused = true;      // TSP2OPT_INC_FUSED=0: the box + cull + list kernels on every iteration
     bool inc_persistent = true; // TSP2OPT_INC_PERSISTENT=0: per-iteration launches instead of one cooperative launch
-    bool dense_ls = true;       // TSP2OPT_DENSE_LS=0: per-iteration kernels for the dense loop above the persistent size
+    bool dense_ls = false;      // TSP2OPT_DENSE_LS=1: the persistent dense loop with dynamic claims above the round-robin
+                                // persistent size (measured slower at C3: 30-38 vs 22 us per move, r02_exp_dense_ls.jsonl)
     int nctiles = 0;
     int list_grid = 0;          // CTAs of the culled sweep (co-resident)
     int list25_grid = 0;        // CTAs of the 2.5-opt culled sweep

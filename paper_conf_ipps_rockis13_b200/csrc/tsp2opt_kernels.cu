@@ -565,13 +565,21 @@ __device__ __forceinline__ bool apply_phase(float2* __restrict__ P, int* __restr
             else if (moves >= max_moves) o.done = 2;    // capped with an improving move left (R8)
         }
         if (apply) {
+            // thread 0 alone swaps positions i+1 <-> j and writes E[i], E[j], so these reads
+            // see the pre-move state even while other threads (and CTAs) reverse the rest
             const float2 pi = __ldcg(P + i), pj = __ldcg(P + j), pi1 = __ldcg(P + i + 1), pj1 = __ldcg(P + j + 1);
             const int ni = exact_dist_biased(pi, pj), nj = exact_dist_biased(pi1, pj1);
-            o.length += (long long)ni + nj - __ldcg(E + i) - __ldcg(E + j);
+            const int d = ni + nj - __ldcg(E + i) - __ldcg(E + j);
+            o.length += d;
             o.moves = moves + 1;
             E[i] = ni;
             E[j] = nj;
-            if (trace && !explicit_move && moves < trace_cap) trace[moves] = key;  // move trace (tests)
+            if (!explicit_move) {
+                // the applied move with its exact delta: a first-improvement key carries the
+                // marker delta (reading R20) until here; a best-improvement key already has d
+                o.last_key = pack_key(d, i, j);
+                if (trace && moves < trace_cap) trace[moves] = o.last_key;  // move trace (tests)
+            }
         }
         *out = o;
     }
@@ -859,14 +867,9 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
 #endif
         // (A) apply the winning move
         if (threadIdx.x == 0) {
-            unsigned long long key = *(volatile unsigned long long*)&in->key;
-            if (FIRST && key_delta(key) == kFirstDelta) {  // the marker delta: the winner's exact delta (R20)
-                const int i = key_i(key), j = key_j(key);
-                const int d = exact_dist_biased(__ldcg(P + i), __ldcg(P + j)) +
-                              exact_dist_biased(__ldcg(P + i + 1), __ldcg(P + j + 1)) - __ldcg(E + i) - __ldcg(E + j);
-                key = pack_key(d, i, j);
-            }
-            s_in.key = key;
+            // first improvement: the key keeps its marker delta (< 0, so every CTA applies);
+            // apply_phase's thread 0 derives the exact delta before its own swap (reading R20)
+            s_in.key = *(volatile unsigned long long*)&in->key;
             s_in.moves = *(volatile long long*)&in->moves;
             s_in.length = *(volatile long long*)&in->length;
         }
@@ -914,12 +917,27 @@ __global__ void __launch_bounds__(512, 1) dense_ls_kernel(float2* __restrict__ P
         if (threadIdx.x == 0) s_in.done = *(volatile int*)&in->done;
         __syncthreads();
         if (s_in.done) break;  // uniform across the grid
-        for (;;) {
-            int t = 0;
-            if (lane == 0) t = (int)atomicAdd(&in->next_tile, 1u);
-            t = __shfl_sync(0xffffffffu, t, 0);
-            if (t >= ntiles) break;
-            sweep_tile<R, true, false, true>(P, E, n, tiles[t], TJ, in, sm, tilebest + t, tflags);
+#ifndef TSP2OPT_DENSE_CLAIM
+#define TSP2OPT_DENSE_CLAIM 0  // tiles per claim (0: static round-robin by warp; measured best of 0 / 1 / 4 / 16)
+#endif
+        if (TSP2OPT_DENSE_CLAIM == 0) {
+            const int gw = blockIdx.x * (blockDim.x >> 5) + wib, nw = gridDim.x * (blockDim.x >> 5);
+            for (int t = gw; t < ntiles; t += nw)
+                sweep_tile<R, true, false, true>(P, E, n, tiles[t], TJ, in, sm, tilebest + t, tflags);
+        } else {
+            // the first chunk by warp index, then claims of TSP2OPT_DENSE_CLAIM consecutive
+            // (similar-sized) tiles: few atomics on the slot's counter per sweep
+            const int gw = blockIdx.x * (blockDim.x >> 5) + wib, nw = gridDim.x * (blockDim.x >> 5);
+            constexpr int C = TSP2OPT_DENSE_CLAIM > 0 ? TSP2OPT_DENSE_CLAIM : 1;
+            int t0 = gw * C;
+            for (;;) {
+                if (t0 >= ntiles) break;
+                for (int t = t0; t < min(t0 + C, ntiles); t++)
+                    sweep_tile<R, true, false, true>(P, E, n, tiles[t], TJ, in, sm, tilebest + t, tflags);
+                int c = 0;
+                if (lane == 0) c = (int)atomicAdd(&in->next_tile, 1u);
+                t0 = (nw + __shfl_sync(0xffffffffu, c, 0)) * C;
+            }
         }
         grid_sync(bar, gridDim.x);
         if (threadIdx.x == 0) {

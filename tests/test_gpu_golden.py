@@ -34,6 +34,8 @@ def _goldens():
         if len(parts) != 5:  # ls_C3_lattice_random_s1.npz (round 1, plain oracle): test_gpu_parity.py
             continue
         variant, cfg, _, tk, _ = parts
+        if variant == "oropt":  # the stateless Or-opt path: tests/test_gpu_oropt.py
+            continue
         out.append(pytest.param(variant, cfg, tk, p, id=f"{variant}-{cfg}-{tk}"))
     return out
 

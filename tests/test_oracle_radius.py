@@ -69,7 +69,7 @@ def test_radius_local_search_equals_plain_move_by_move(kind, n, seed):
     assert np.array_equal(a["tour"], b["tour"])
 
 
-@pytest.mark.parametrize("kind,n,seed", [("uniform", 100, 1), ("lattice", 150, 2), ("uniform", 300, 3)])
+@pytest.mark.parametrize("kind,n,seed", [("uniform", 100, 1), ("lattice", 150, 2), ("uniform", 240, 3)])
 def test_radius_first_and_25opt_equal_plain_move_by_move(kind, n, seed):
     """First improvement (R20) and 2.5-opt (R19): every move equals the plain oracle's."""
     coords = inputs.make_coords(kind, n, seed)
@@ -86,13 +86,13 @@ def test_radius_first_and_25opt_equal_plain_move_by_move(kind, n, seed):
 
 
 def test_radius_constructive_starts_equal_plain():
-    """From Hilbert and Multiple Fragment starts (the C4/C5 golden starts) at n = 2000:
+    """From Hilbert and Multiple Fragment starts (the C4/C5 golden starts) at n = 1200:
     every move equals the plain oracle's, for all three sweeps."""
-    coords = inputs.lattice_coords(2000, 7)
+    coords = inputs.lattice_coords(1200, 7)
     for tour in (inputs.hilbert_tour(coords), oracle.mf_tour(coords)):
         a = oracle.local_search(coords, tour, trace_cap=5000)
         b = oracle.radius_local_search(coords, tour, trace_cap=5000)
-        assert a["iterations"] > 50 and np.array_equal(a["trace"], b["trace"]) and np.array_equal(a["tour"], b["tour"])
+        assert a["iterations"] > 30 and np.array_equal(a["trace"], b["trace"]) and np.array_equal(a["tour"], b["tour"])
         a = oracle.local_search25(coords, tour, trace_cap=5000)
         b = oracle.radius_local_search(coords, tour, trace_cap=5000, node_insertion=True)
         assert np.array_equal(a["trace"], b["trace"]) and np.array_equal(a["tour"], b["tour"])

@@ -21,8 +21,9 @@ import numpy as np  # noqa: E402
 import oracle  # noqa: E402
 from paper_conf_ipps_rockis13_b200 import inputs, tsp2opt  # noqa: E402
 
-MODES = ["persistent", "kernels", "culled", "incremental", "graph_off", "25opt", "25opt_culled", "first",
-         "pruned", "mf", "ils", "batch", "batch_ils", "oropt", "oropt_filter", "shards"]
+MODES = ["persistent", "kernels", "culled", "incremental", "inc_fused", "dense_ls", "graph_off", "25opt",
+         "25opt_culled", "first", "first_inc", "pruned", "mf", "ils", "batch", "batch_ils", "oropt", "oropt_filter",
+         "shards", "p2p1"]
 
 # environment each mode needs (read by the library at handle creation)
 ENV = {
@@ -30,7 +31,12 @@ ENV = {
     "kernels": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "1"},
     "culled": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "2", "TSP2OPT_CULL_TJ": "16"},
     "incremental": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "3", "TSP2OPT_CULL_TJ": "16"},
-    "graph_off": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "3", "TSP2OPT_GRAPH": "0"},
+    "inc_fused": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "3", "TSP2OPT_CULL_TJ": "16",
+                  "TSP2OPT_INC_PERSISTENT": "0"},
+    "dense_ls": {"TSP2OPT_PERSISTENT": "3", "TSP2OPT_TILE_BOUNDS": "1"},
+    "first_inc": {"TSP2OPT_TILE_BOUNDS": "3", "TSP2OPT_CULL_TJ": "16"},
+    "graph_off": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "3", "TSP2OPT_GRAPH": "0",
+                  "TSP2OPT_INC_PERSISTENT": "0"},
     "25opt_culled": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "3", "TSP2OPT_CULL_TJ": "16"},
     "oropt_filter": {"TSP2OPT_OROPT_FILTER": "1"},
 }
@@ -46,7 +52,7 @@ def main(mode):
     n = 300
     c = inputs.lattice_coords(n, 3)
     t = inputs.random_tour(n, 3)
-    if mode in ("persistent", "kernels", "culled", "incremental", "graph_off"):
+    if mode in ("persistent", "kernels", "culled", "incremental", "inc_fused", "dense_ls", "graph_off"):
         with tsp2opt.TSP2Opt(c) as g:
             r = g.local_search(t)
         o = oracle.local_search(c, t)
@@ -58,7 +64,7 @@ def main(mode):
             r = g.local_search(t)
         o = oracle.local_search25(c, t)
         check(r["length"] == o["length"] and np.array_equal(r["tour"], o["tour"]), mode)
-    elif mode == "first":
+    elif mode in ("first", "first_inc"):
         with tsp2opt.TSP2Opt(c) as g:
             g.set_option(tsp2opt.OPT_FIRST_IMPROVEMENT, 1)
             r = g.local_search(t)
@@ -95,6 +101,11 @@ def main(mode):
     elif mode in ("oropt", "oropt_filter"):
         r = tsp2opt.oropt_local_search(c, t)
         o = oracle.local_search_or(c, t)
+        check(r["length"] == o["length"] and np.array_equal(r["tour"], o["tour"]), mode)
+    elif mode == "p2p1":  # the peer-memory exchange kernel, one rank
+        with tsp2opt.TSP2Opt(c, 0, 1, p2p_allgather=lambda b: [b]) as g:
+            r = g.local_search(t)
+        o = oracle.local_search(c, t)
         check(r["length"] == o["length"] and np.array_equal(r["tour"], o["tour"]), mode)
     elif mode == "shards":
         with tsp2opt.TSP2Opt(c) as g:
