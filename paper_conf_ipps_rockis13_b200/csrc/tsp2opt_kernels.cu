@@ -105,7 +105,11 @@ __global__ void reset_key_kernel(Slot* slot)
 #define TSP2OPT_MINB 4  // CTAs of 128 threads per SM the register allocation must allow
 #endif
 template <int R, bool FIRST>
-__global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_kernel(const float2* __restrict__ P, const int* __restrict__ E, int n,
+#ifndef TSP2OPT_SWEEP_LB_T
+#define TSP2OPT_SWEEP_LB_T 128  // experiment: (32, 20) forces 102 registers for 20 one-warp CTAs per SM
+#define TSP2OPT_SWEEP_LB_B TSP2OPT_MINB
+#endif
+__global__ void __launch_bounds__(TSP2OPT_SWEEP_LB_T, TSP2OPT_SWEEP_LB_B) sweep_kernel(const float2* __restrict__ P, const int* __restrict__ E, int n,
                                                      const int2* __restrict__ tiles, int TJ, Slot* __restrict__ slot,
                                                      int respect_done, unsigned long long* __restrict__ tilebest,
                                                      int flags)

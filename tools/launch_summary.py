@@ -14,7 +14,9 @@ def main(path):
             k = d["Kernel Name"].split("(")[0]
             agg[k][0] += 1
             agg[k][1] += float(d["Metric Value"]) * (1e-3 if d["Metric Unit"] == "ns" else 1.0)
-    ours = {k: v for k, v in agg.items() if "tsp2opt" in k or k.split("<")[0].split()[-1].startswith("or_")}
+    # every kernel of libtsp2opt.so; the rest (PyTorch / NCCL / CUB helpers) is reported as not ours
+    foreign = ("at::", "nccl", "cub::", "cutlass", "triton", "elementwise", "vectorized", "reduce_kernel", "CatArray")
+    ours = {k: v for k, v in agg.items() if not any(f in k for f in foreign)}
     tot_ours = sum(v[1] for v in ours.values())
     print(f"# {path}: per-kernel device time (cold-cache, serialised; compare shares)")
     print(f"{'launches':>8} {'total_us':>12} {'avg_us':>10} {'share_of_ours':>13}  kernel")
