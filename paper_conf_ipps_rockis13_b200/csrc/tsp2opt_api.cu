@@ -1397,16 +1397,24 @@ int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters
     int* d_xy = nullptr;
     int* d_t = nullptr;
     int* d_span = nullptr;
+    int* d_trace = nullptr;
     int2* d_q = nullptr;
     int4* d_c = nullptr;  // per-position sweep constants CR | CC
-    unsigned long long* d_slot = nullptr;  // [0] key, [1] length
+    unsigned long long* d_slot = nullptr;  // kOrSlotWords: key, length, moves, done, cap, move
+    unsigned long long* h_slot = nullptr;  // pinned readback
+    cudaStream_t st = nullptr;
+    cudaGraphExec_t gexec = nullptr;
     auto cleanup = [&]() {
+        if (gexec) cudaGraphExecDestroy(gexec);
+        if (st) cudaStreamDestroy(st);
         cudaFree(d_c);
         cudaFree(d_xy);
         cudaFree(d_t);
         cudaFree(d_span);
+        cudaFree(d_trace);
         cudaFree(d_q);
         cudaFree(d_slot);
+        cudaFreeHost(h_slot);
     };
     auto fail = [&](cudaError_t e, const char* what) {
         cleanup();
@@ -1414,41 +1422,84 @@ int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters
     };
     cudaError_t e;
     const size_t nb = sizeof(int) * (size_t)n;
+    const long long tcap = trace ? std::min<long long>(trace_cap, max_iters) : 0;
+    if ((e = cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking)) != cudaSuccess) return fail(e, "stream");
     if ((e = cudaMalloc(&d_xy, 2 * nb)) != cudaSuccess) return fail(e, "cudaMalloc");
     if ((e = cudaMalloc(&d_t, nb)) != cudaSuccess) return fail(e, "cudaMalloc");
     if ((e = cudaMalloc(&d_span, nb)) != cudaSuccess) return fail(e, "cudaMalloc");
+    if (tcap > 0 && (e = cudaMalloc(&d_trace, sizeof(int) * 4 * (size_t)tcap)) != cudaSuccess)
+        return fail(e, "cudaMalloc");
     if ((e = cudaMalloc(&d_q, sizeof(int2) * oropt_q_entries(n))) != cudaSuccess) return fail(e, "cudaMalloc");
-    if ((e = cudaMalloc(&d_slot, 2 * sizeof(unsigned long long))) != cudaSuccess) return fail(e, "cudaMalloc");
+    if ((e = cudaMalloc(&d_slot, kOrSlotWords * sizeof(unsigned long long))) != cudaSuccess) return fail(e, "cudaMalloc");
     if ((e = cudaMalloc(&d_c, 2 * sizeof(int4) * oropt_const_entries(n))) != cudaSuccess) return fail(e, "cudaMalloc");
-    if ((e = cudaMemcpy(d_xy, coords_xy, 2 * nb, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "H2D");
-    if ((e = cudaMemcpy(d_t, tour, nb, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "H2D");
-    if ((e = launch_or_load(d_xy, d_t, d_q, n, d_slot + 1, nullptr)) != cudaSuccess) return fail(e, "or_load");
-    unsigned long long len = 0;
-    if ((e = cudaMemcpy(&len, d_slot + 1, sizeof(len), cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
-    long long L = (long long)len, it = 0;
-    int status = TSP2OPT_OK;
-    std::vector<int32_t> tr;  // copied to the caller only on success (nothing is written on error)
-    for (;;) {
-        if ((e = launch_or_sweep(d_q, d_c, d_c + oropt_const_entries(n), n, d_slot, nullptr)) != cudaSuccess) return fail(e, "or_sweep_kernel");
-        unsigned long long key = 0;
-        if ((e = cudaMemcpy(&key, d_slot, sizeof(key), cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
-        if (first_key && it == 0) *first_key = key;
-        int i, j, type, d;
-        or_unpack(key, &i, &j, &type, &d);
-        if (d >= 0) break;
-        if (it >= max_iters) {  // reading R8
-            status = TSP2OPT_MAXITER;
-            break;
-        }
-        if ((e = launch_or_apply(d_xy, d_t, d_q, d_span, n, i, j, type, nullptr)) != cudaSuccess)
-            return fail(e, "or_apply");
-        if (trace && it < trace_cap) tr.insert(tr.end(), {i, j, d, type});
-        L += d;
-        it++;
+    if ((e = cudaHostAlloc(&h_slot, kOrSlotWords * sizeof(unsigned long long), cudaHostAllocDefault)) != cudaSuccess)
+        return fail(e, "cudaHostAlloc");
+    {
+        unsigned long long init[kOrSlotWords] = {};
+        init[kOrCap] = (unsigned long long)max_iters;
+        if ((e = cudaMemcpyAsync(d_slot, init, sizeof(init), cudaMemcpyHostToDevice, st)) != cudaSuccess)
+            return fail(e, "H2D");
+        if ((e = cudaMemcpyAsync(d_xy, coords_xy, 2 * nb, cudaMemcpyHostToDevice, st)) != cudaSuccess)
+            return fail(e, "H2D");
+        if ((e = cudaMemcpyAsync(d_t, tour, nb, cudaMemcpyHostToDevice, st)) != cudaSuccess) return fail(e, "H2D");
+        if ((e = launch_or_load(d_xy, d_t, d_q, n, d_slot + kOrLength, st)) != cudaSuccess) return fail(e, "or_load");
+        if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return fail(e, "sync");
     }
-    if ((e = cudaMemcpy(tour, d_t, nb, cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
+    // Device-resident loop (no host decision per move): each iteration is the sweep
+    // (constants + tile kernel), the decide kernel and the apply; batches of k
+    // iterations between host reads of the state, k doubling to 64, full batches
+    // replayed from one captured CUDA graph.  An iteration after convergence is a no-op.
+    auto enqueue = [&](long long k) -> cudaError_t {
+        for (long long c = 0; c < k; c++) {
+            cudaError_t x = launch_or_sweep(d_q, d_c, d_c + oropt_const_entries(n), n, d_slot, st);
+            if (x == cudaSuccess) x = launch_or_apply(d_xy, d_t, d_q, d_span, n, d_slot, d_trace, tcap, st);
+            if (x != cudaSuccess) return x;
+        }
+        return cudaSuccess;
+    };
+    long long k = 1;
+    for (long long batches = 0;; batches++) {
+        if (batches > (1LL << 26)) return fail(cudaErrorUnknown, "Or-opt local search did not converge");
+        if (k == 64 && graphs_enabled()) {
+            if (!gexec) {
+                cudaGraph_t graph = nullptr;
+                if ((e = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal)) != cudaSuccess)
+                    return fail(e, "capture");
+                const cudaError_t eq = enqueue(k);
+                e = cudaStreamEndCapture(st, &graph);
+                if (eq != cudaSuccess) {
+                    if (graph) cudaGraphDestroy(graph);
+                    return fail(eq, "Or-opt iteration");
+                }
+                if (e != cudaSuccess) return fail(e, "capture");
+                e = cudaGraphInstantiate(&gexec, graph, 0);
+                cudaGraphDestroy(graph);
+                if (e != cudaSuccess) return fail(e, "cudaGraphInstantiate");
+            }
+            if ((e = cudaGraphLaunch(gexec, st)) != cudaSuccess) return fail(e, "cudaGraphLaunch");
+        } else if ((e = enqueue(k)) != cudaSuccess) {
+            return fail(e, "Or-opt iteration");
+        }
+        if ((e = cudaMemcpyAsync(h_slot, d_slot, kOrSlotWords * sizeof(unsigned long long), cudaMemcpyDeviceToHost,
+                                 st)) != cudaSuccess)
+            return fail(e, "D2H");
+        if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return fail(e, "sync");
+        if (first_key && batches == 0) *first_key = h_slot[0];  // the first sweep's key (best_move: max_iters 0)
+        if (h_slot[kOrDone]) break;
+        if (k < 64) k *= 2;
+    }
+    const int status = h_slot[kOrDone] == 2 ? TSP2OPT_MAXITER : TSP2OPT_OK;
+    const long long it = (long long)h_slot[kOrMoves], L = (long long)h_slot[kOrLength];
+    std::vector<int32_t> tr(4 * (size_t)std::min<long long>(it, tcap));
+    if (!tr.empty() && (e = cudaMemcpy(tr.data(), d_trace, sizeof(int32_t) * tr.size(), cudaMemcpyDeviceToHost)) !=
+                           cudaSuccess)
+        return fail(e, "D2H");
+    std::vector<int32_t> out(n);
+    if ((e = cudaMemcpy(out.data(), d_t, nb, cudaMemcpyDeviceToHost)) != cudaSuccess) return fail(e, "D2H");
     cleanup();
-    if (trace && !tr.empty()) memcpy(trace, tr.data(), sizeof(int32_t) * tr.size());
+    // nothing is written to the caller before this point (errors leave tour / trace untouched)
+    memcpy(tour, out.data(), nb);
+    if (!tr.empty()) memcpy(trace, tr.data(), sizeof(int32_t) * tr.size());
     if (length) *length = L;
     if (iterations) *iterations = it;
     return status;

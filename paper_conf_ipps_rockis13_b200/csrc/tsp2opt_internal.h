@@ -86,13 +86,21 @@ cudaError_t launch_apply25(float2* P, int* E, int* G, int* tour, int n, const Sl
                            long long max_moves, int explicit_move, int ei, int ej, int etype,
                            unsigned long long* trace, int* ttype, long long trace_cap, unsigned* bar, cudaStream_t st);
 // Or-opt (tsp2opt_oropt.cu; reading R21): route-ordered int2 Q[n + 5], dense sweep, span apply.
+// Device state of the Or-opt loop, u64 words: [0] the sweep's key, then these.
+constexpr int kOrLength = 1;  // tour length (int64)
+constexpr int kOrMoves = 2;   // moves applied
+constexpr int kOrDone = 3;    // 0 running, 1 local minimum, 2 capped with an improving move left
+constexpr int kOrCap = 4;     // max_iters
+constexpr int kOrMove = 5;    // the key of the move the current iteration applies, 0 if none
+constexpr int kOrSlotWords = 8;
 size_t oropt_q_entries(int n);
 cudaError_t launch_or_load(const int* coords, const int* tour, int2* Q, int n, unsigned long long* len, cudaStream_t st);
 size_t oropt_const_entries(int n);
 void or_config(int filter, int naive);
 cudaError_t launch_or_sweep(const int2* Q, int4* CR, int4* CC, int n, unsigned long long* slot, cudaStream_t st);
-cudaError_t launch_or_apply(const int* coords, int* tour, int2* Q, int* span, int n, int i, int j, int type,
-                            cudaStream_t st);
+// decide (device: done / capped / record the move) + span + commit, all reading the slot
+cudaError_t launch_or_apply(const int* coords, int* tour, int2* Q, int* span, int n, unsigned long long* slot,
+                            int* trace, long long trace_cap, cudaStream_t st);
 void or_unpack(unsigned long long key, int* i, int* j, int* type, int* delta);
 size_t sweep_smem_bytes(const Geometry& g);
 cudaError_t sweep_prepare();

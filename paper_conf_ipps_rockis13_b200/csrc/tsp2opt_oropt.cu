@@ -62,6 +62,7 @@ __global__ void or_length_kernel(const int2* __restrict__ Q, int n, unsigned lon
 __global__ void __launch_bounds__(kOrThreads) or_sweep_kernel(const int2* __restrict__ Q, int n, long long cells,
                                                               unsigned long long* slot)
 {
+    if (*(volatile const unsigned long long*)(slot + kOrDone)) return;
     unsigned long long best = or_pack(0, 0, 1, 0);
     for (long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x; k < cells;
          k += (long long)gridDim.x * blockDim.x) {
@@ -120,6 +121,7 @@ __global__ void __launch_bounds__(kOrThreads) or_sweep_kernel(const int2* __rest
 __global__ void or_consts_kernel(const int2* __restrict__ Q, int n, int4* __restrict__ CR, int4* __restrict__ CC,
                                  unsigned long long* slot)
 {
+    if (*(volatile const unsigned long long*)(slot + kOrDone)) return;  // converged / capped: a no-op iteration
     if (blockIdx.x == 0 && threadIdx.x == 0) *slot = or_pack(0, 0, 1, 0);  // the sweep's seed key (reading R7)
     for (int p = blockIdx.x * blockDim.x + threadIdx.x; p < n; p += gridDim.x * blockDim.x) {
         const int e = or_d(Q[p], Q[p + 1]);
@@ -229,6 +231,7 @@ __global__ void __launch_bounds__(kOrMaxTI) or_tile_kernel(const int2* __restric
     const int ti = blockDim.x;
     const int row0 = blockIdx.y * ti, col1 = (blockIdx.x + 1) * tj;
     if (col1 - 1 <= row0) return;  // below the diagonal: no pair i < j (uniform over the CTA)
+    if (*(volatile const unsigned long long*)(slot + kOrDone)) return;  // converged / capped
     const int i = row0 + threadIdx.x;
     const int j0 = max(blockIdx.x * tj, i + 1), j1 = min(n, col1);
     // Seed the thread's bound with the sweep's best so far (other CTAs'
@@ -335,8 +338,47 @@ __global__ void __launch_bounds__(kOrMaxTI) or_tile_kernel(const int2* __restric
 }
 
 // span[p - i - 1] = the tour city that lands on position p in [i+1, j] (oracleor_apply's order)
-__global__ void or_span_kernel(const int* __restrict__ tour, int* __restrict__ span, int i, int j, int type)
+// The move decision of one iteration, on the device (one thread): the sweep's
+// key in slot[0]; slot[kOrDone] = 1 at a local minimum (delta >= 0, reading
+// R7), 2 when capped with an improving move left (R8); otherwise the move is
+// recorded (length, moves, trace row (i, j, delta, type)) and published in
+// slot[kOrMove] for the apply kernels (0: no move this iteration).
+__global__ void or_decide_kernel(unsigned long long* slot, int* __restrict__ trace, long long trace_cap)
 {
+    if (slot[kOrDone]) return;
+    const unsigned long long key = slot[0];
+    const int d = (int)(key >> 44) - kDeltaBias;
+    const long long moves = (long long)slot[kOrMoves];
+    if (d >= 0) {
+        slot[kOrDone] = 1;
+        slot[kOrMove] = 0;
+        return;
+    }
+    if (moves >= (long long)slot[kOrCap]) {
+        slot[kOrDone] = 2;
+        slot[kOrMove] = 0;
+        return;
+    }
+    const int j = (int)((key >> 24) & 0xFFFFF), i = (int)((key >> 4) & 0xFFFFF), type = (int)(key & 0xF);
+    if (trace && moves < trace_cap) {
+        trace[4 * moves] = i;
+        trace[4 * moves + 1] = j;
+        trace[4 * moves + 2] = d;
+        trace[4 * moves + 3] = type;
+    }
+    slot[kOrLength] = (unsigned long long)((long long)slot[kOrLength] + d);
+    slot[kOrMoves] = (unsigned long long)(moves + 1);
+    slot[kOrMove] = key;
+}
+
+// span[p - i - 1] = the tour city that lands on position p in [i+1, j] (oracleor_apply's order),
+// for the move the decide kernel published (none: a no-op)
+__global__ void or_span_kernel(const int* __restrict__ tour, int* __restrict__ span,
+                               const unsigned long long* __restrict__ slot)
+{
+    const unsigned long long key = slot[kOrMove];
+    if (!key) return;
+    const int j = (int)((key >> 24) & 0xFFFFF), i = (int)((key >> 4) & 0xFFFFF), type = (int)(key & 0xF);
     const int m = j - i;
     const int L = 1 + (type - 1) / 4, dir = ((type - 1) / 2) & 1, rev = (type - 1) & 1;
     for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < m; q += gridDim.x * blockDim.x) {
@@ -350,8 +392,11 @@ __global__ void or_span_kernel(const int* __restrict__ tour, int* __restrict__ s
 }
 
 __global__ void or_commit_kernel(const int* __restrict__ coords, const int* __restrict__ span, int* __restrict__ tour,
-                                 int2* __restrict__ Q, int n, int i, int j)
+                                 int2* __restrict__ Q, int n, const unsigned long long* __restrict__ slot)
 {
+    const unsigned long long key = slot[kOrMove];
+    if (!key) return;
+    const int j = (int)((key >> 24) & 0xFFFFF), i = (int)((key >> 4) & 0xFFFFF);
     for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < j - i; q += gridDim.x * blockDim.x) {
         const int p = i + 1 + q, c = span[q];
         tour[p] = c;
@@ -359,6 +404,11 @@ __global__ void or_commit_kernel(const int* __restrict__ coords, const int* __re
         Q[p] = v;
         if (p < kOrHalo) Q[n + p] = v;  // the halo copies of positions 1..4
     }
+}
+
+__global__ void or_seed_kernel(unsigned long long* slot)
+{
+    if (!slot[kOrDone]) slot[0] = or_pack(0, 0, 1, 0);
 }
 
 static int or_grid(long long work, int per_cta, int cap)
@@ -424,9 +474,7 @@ size_t oropt_const_entries(int n) { return (size_t)n; }
 cudaError_t launch_or_sweep(const int2* Q, int4* CR, int4* CC, int n, unsigned long long* slot, cudaStream_t st)
 {
     if (or_naive()) {  // TSP2OPT_OROPT_NAIVE=1: the one-thread-per-cell kernel (experiment switch, same result)
-        const unsigned long long seed = or_pack(0, 0, 1, 0);
-        cudaError_t e = cudaMemcpyAsync(slot, &seed, sizeof(seed), cudaMemcpyHostToDevice, st);
-        if (e != cudaSuccess) return e;
+        or_seed_kernel<<<1, 1, 0, st>>>(slot);
         const long long cells = (long long)n * (n - 1) / 2;
         or_sweep_kernel<<<or_grid(cells, kOrThreads, 8), kOrThreads, 0, st>>>(Q, n, cells, slot);
         count_launch();
@@ -444,13 +492,14 @@ cudaError_t launch_or_sweep(const int2* Q, int4* CR, int4* CC, int n, unsigned l
     return cudaGetLastError();
 }
 
-cudaError_t launch_or_apply(const int* coords, int* tour, int2* Q, int* span, int n, int i, int j, int type,
-                            cudaStream_t st)
+cudaError_t launch_or_apply(const int* coords, int* tour, int2* Q, int* span, int n, unsigned long long* slot,
+                            int* trace, long long trace_cap, cudaStream_t st)
 {
-    const int g = or_grid(j - i, 256, 4);
-    or_span_kernel<<<g, 256, 0, st>>>(tour, span, i, j, type);
-    or_commit_kernel<<<g, 256, 0, st>>>(coords, span, tour, Q, n, i, j);
-    count_launch(2);
+    const int g = or_grid(n, 256, 4);
+    or_decide_kernel<<<1, 1, 0, st>>>(slot, trace, trace_cap);
+    or_span_kernel<<<g, 256, 0, st>>>(tour, span, slot);
+    or_commit_kernel<<<g, 256, 0, st>>>(coords, span, tour, Q, n, slot);
+    count_launch(3);
     return cudaGetLastError();
 }
 
