@@ -1401,7 +1401,7 @@ int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters
     int2* d_q = nullptr;
     int4* d_c = nullptr;  // per-position sweep constants CR | CC
     unsigned long long* d_slot = nullptr;  // kOrSlotWords: key, length, moves, done, cap, move
-    unsigned long long* h_slot = nullptr;  // pinned readback
+    unsigned long long h_slot[kOrSlotWords] = {};  // readback (pageable: a pinned buffer costs ~1 ms per call)
     cudaStream_t st = nullptr;
     cudaGraphExec_t gexec = nullptr;
     auto cleanup = [&]() {
@@ -1414,7 +1414,6 @@ int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters
         cudaFree(d_trace);
         cudaFree(d_q);
         cudaFree(d_slot);
-        cudaFreeHost(h_slot);
     };
     auto fail = [&](cudaError_t e, const char* what) {
         cleanup();
@@ -1432,8 +1431,6 @@ int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters
     if ((e = cudaMalloc(&d_q, sizeof(int2) * oropt_q_entries(n))) != cudaSuccess) return fail(e, "cudaMalloc");
     if ((e = cudaMalloc(&d_slot, kOrSlotWords * sizeof(unsigned long long))) != cudaSuccess) return fail(e, "cudaMalloc");
     if ((e = cudaMalloc(&d_c, 2 * sizeof(int4) * oropt_const_entries(n))) != cudaSuccess) return fail(e, "cudaMalloc");
-    if ((e = cudaHostAlloc(&h_slot, kOrSlotWords * sizeof(unsigned long long), cudaHostAllocDefault)) != cudaSuccess)
-        return fail(e, "cudaHostAlloc");
     {
         unsigned long long init[kOrSlotWords] = {};
         init[kOrCap] = (unsigned long long)max_iters;
@@ -1457,10 +1454,11 @@ int or_run(const int32_t* coords_xy, int32_t n, int32_t* tour, int64_t max_iters
         }
         return cudaSuccess;
     };
-    long long k = 1;
+    long long k = 1, full_batches = 0;
     for (long long batches = 0;; batches++) {
         if (batches > (1LL << 26)) return fail(cudaErrorUnknown, "Or-opt local search did not converge");
-        if (k == 64 && graphs_enabled()) {
+        // (below n = 512 an iteration is a few microseconds: capturing costs more than it saves)
+        if (k == 64 && n >= 512 && graphs_enabled() && ++full_batches >= 1) {
             if (!gexec) {
                 cudaGraph_t graph = nullptr;
                 if ((e = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal)) != cudaSuccess)

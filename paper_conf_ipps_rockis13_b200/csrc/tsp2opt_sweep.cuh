@@ -178,6 +178,7 @@ __device__ __forceinline__ bool step_any(const Bound<R>& b, const float (&cur)[R
 // exhaustively by tsp2opt_selftest) is covered by a 0.5 slack.  Survivors are
 // evaluated with integer nint distances -- the oracle's arithmetic -- and
 // accepted iff delta < B, in increasing cell order.
+
 template <int R, bool MASK, bool PS, bool FIRST>
 __device__ __forceinline__ void exact_step(Bound<R>& b, const float (&cur)[R + 1], const float (&nxt)[R + 1],
                                            float scol, int row0, int j, float4 c0, float4 c1, float ej,
