@@ -119,6 +119,8 @@ __global__ void __launch_bounds__(TSP2OPT_SWEEP_LB_T, TSP2OPT_SWEEP_LB_B) sweep_
     pdl_trigger();
     pdl_wait();
     if (respect_done && *(volatile int*)&slot->done) return;  // converged: iteration is a no-op
+    // (the warp-tile form for one-warp CTAs -- compile-time warp index, 63-70 instead of
+    // about 71 instructions per step -- measured 1 % slower here, r02_exp_sweep.jsonl)
     sweep_tile<R, false, FIRST>(P, E, n, tiles[blockIdx.x], TJ, slot, sm, tilebest + blockIdx.x, flags);
 }
 
@@ -359,7 +361,10 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) sweep_list_kernel(const flo
         __syncthreads();
         const int4 e = s_t;
         if (e.z < 0) break;
-        sweep_tile<R, false, FIRST>(P, E, n, make_int2(e.x, e.y), TJ, slot, sm, tilebest + e.z, flags);
+        if (blockDim.x == 32)
+            sweep_tile<R, false, FIRST, true>(P, E, n, make_int2(e.x, e.y), TJ, slot, sm, tilebest + e.z, flags);
+        else
+            sweep_tile<R, false, FIRST>(P, E, n, make_int2(e.x, e.y), TJ, slot, sm, tilebest + e.z, flags);
         if (threadIdx.x == 0) k = gridDim.x + atomicAdd(&slot->next_tile, 1u);
         __syncthreads();  // before the next tile overwrites the shared chunk (and s_t)
     }
@@ -505,7 +510,7 @@ __global__ void __launch_bounds__(32, 16) inc_sweep_kernel(const float2* __restr
         const long long T = (long long)max(r.emax, c.emax) - 1;
         const bool keep = T >= 0 && gx * gx + gy * gy <= T * T + T;
         if (keep) {
-            sweep_tile<R, false, FIRST>(P, E, n, make_int2(rb * TI, cc * TJ), TJ, slot, sm, tilebest + t,
+            sweep_tile<R, false, FIRST, true>(P, E, n, make_int2(rb * TI, cc * TJ), TJ, slot, sm, tilebest + t,
                                         flags | kSweepLocal);
             __syncthreads();  // before the next tile overwrites the shared chunk
         } else if (lane == 0) {
