@@ -126,20 +126,23 @@ def run_ours(args):
     rank, world, local = dist_env()
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
-    torch.cuda.set_device(local)
+    p2p = args.exchange == "p2p"
+    # --exchange p2p: the per-sweep MIN over peer-memory mailboxes; ranks may then share a
+    # GPU (rank r on device r mod the visible count: a code-path check on a one-GPU box,
+    # the ranks time-slice), and gloo carries only the host-side collectives
+    torch.cuda.set_device(local % torch.cuda.device_count() if p2p else local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if p2p:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    hdev = "cpu" if p2p else "cuda"  # device of the tensors the host-side collectives reduce
     cfg = inputs.CONFIGS[args.config]
     n = cfg["n"]
     coords, tour = inputs.config_instance(args.config, args.tour)
     total_pairs = n * (n - 1) // 2
 
-    if world > 1:
-        obj = [tsp2opt.nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        g = tsp2opt.TSP2Opt(coords, rank, world, obj[0])
-    else:
-        g = tsp2opt.TSP2Opt(coords)
+    g = sharded_handle(tsp2opt, coords, rank, world, p2p) if world > 1 else tsp2opt.TSP2Opt(coords)
     stream = torch.cuda.Stream()  # a real stream: events and the library's launches share it
     torch.cuda.set_stream(stream)
     g.set_stream(stream.cuda_stream)
@@ -158,7 +161,7 @@ def run_ours(args):
             step()
         s = g.sync()
         first = s["last_move"]
-        sampler = ClockSampler(local) if sample_clocks else None
+        sampler = ClockSampler(torch.cuda.current_device()) if sample_clocks else None
         if sampler:
             sampler.start()
         starts = [torch.cuda.Event(enable_timing=True) for _ in range(nsteps)]
@@ -212,14 +215,14 @@ def run_ours(args):
     tb_steps = max(3, args.steps // 2)
 
     t = torch.tensor([total_ms, sweep_avg_ms, sum(e2e_ms), tb_total_ms, tb_sweep_ms], dtype=torch.float64,
-                     device="cuda")
+                     device=hdev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms, sweep_avg_ms, e2e_total, tb_total_ms, tb_sweep_ms = t.tolist()
 
     ls = ils = batch = batch_ils = pruned = or25 = first = oropt = sharded = balance = None
     if world > 1 and not args.no_ls:  # collective: every rank runs it
-        sharded = time_sharded_ls(tsp2opt, rank, world, args.sharded_config)
+        sharded = time_sharded_ls(tsp2opt, rank, world, args.sharded_config, p2p)
     if rank == 0 and world == 1 and not args.no_ls and args.balance_config:
         balance = shard_balance(tsp2opt, args.balance_config)
     if rank == 0 and world == 1 and not args.no_ls:
@@ -255,6 +258,7 @@ def run_ours(args):
             "ms_per_step": total_ms / args.steps,
             "higher_is_better": True,
             "scaling": "strong" if world > 1 else "weak",
+            "exchange": ("peer memory" if p2p else "NCCL") if world > 1 else None,
             "vs_baseline": None,
             "dtype": "int32+f32",
             "data": "synthetic",
@@ -427,7 +431,23 @@ def time_to_local_min(tsp2opt, cfg_name, with_oracle=True):
     return out
 
 
-def time_sharded_ls(tsp2opt, rank, world, spec):
+def sharded_handle(tsp2opt, coords, rank, world, p2p):
+    """A sharded handle on every rank: NCCL (unique id broadcast by torch.distributed) or
+    the peer-memory exchange (mailbox handles all-gathered)."""
+    import torch.distributed as dist
+
+    if p2p:
+        def allgather(b):
+            out = [None] * world
+            dist.all_gather_object(out, b)
+            return out
+        return tsp2opt.TSP2Opt(coords, rank, world, p2p_allgather=allgather)
+    obj = [tsp2opt.nccl_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0)
+    return tsp2opt.TSP2Opt(coords, rank, world, obj[0])
+
+
+def time_sharded_ls(tsp2opt, rank, world, spec, p2p=False):
     """Time to local minimum on sharded handles (§VI "dividing the 2-opt task
     between multiple devices"): every rank runs tsp2opt_local_search on its
     tile shard with one allreduce-min per sweep.  seconds = max over ranks of each rank's
@@ -445,9 +465,7 @@ def time_sharded_ls(tsp2opt, rank, world, spec):
             continue
         name, _, tk = item.partition(":")
         coords, tour = inputs.config_instance(name, "random" if tk == "mf" else (tk or None))
-        obj = [tsp2opt.nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        with tsp2opt.TSP2Opt(coords, rank, world, obj[0]) as g:
+        with sharded_handle(tsp2opt, coords, rank, world, p2p) as g:
             if tk == "mf":
                 tour = g.mf_tour()["tour"]
             g.local_search(tour, max_iters=2)  # warm-up (graphs, NCCL channels)
@@ -455,7 +473,7 @@ def time_sharded_ls(tsp2opt, rank, world, spec):
             t0 = time.perf_counter()
             r = g.local_search(tour)
             dt = time.perf_counter() - t0
-        t = torch.tensor([dt], dtype=torch.float64, device="cuda")
+        t = torch.tensor([dt], dtype=torch.float64, device="cpu" if p2p else "cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         h = hashlib.sha1(r["tour"].tobytes()).hexdigest()[:16]
         hs = [None] * world
@@ -465,6 +483,7 @@ def time_sharded_ls(tsp2opt, rank, world, spec):
                     "iterations": r["iterations"], "length": r["length"],
                     "us_per_move": 1e6 * t.item() / max(1, r["iterations"]),
                     "tours_agree": all(x == hs[0] for x in hs), "tour_sha1_16": h,
+                    "exchange": "peer memory" if p2p else "NCCL",
                     "timing": "max over ranks of the per-rank wall time of tsp2opt_local_search"})
     return out
 
@@ -869,7 +888,7 @@ def launch_ranks(n: int) -> int:
         have = torch.cuda.device_count()
     except Exception:  # pragma: no cover
         have = 0
-    if have < n:
+    if have < n and "--exchange=p2p" not in sys.argv and "p2p" not in sys.argv:
         print(json.dumps({"metric": METRIC, "error": f"--gpus {n} but {have} CUDA device(s) visible"}), flush=True)
         return 2
     with socket.socket() as so:
@@ -891,6 +910,8 @@ def main():
     ap.add_argument("--ls-config", default="C1,C2,C3,C4:hilbert,C5:hilbert,C2:mf,C3:mf,C4:mf,C5:mf", help="configs timed to a local minimum (rank 0, N=1)")
     ap.add_argument("--sharded-config", default="C4:hilbert,C5:hilbert,C4:mf,C5:mf",
                     help="time to local minimum on the sharded handle, N > 1 (every rank)")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p"],
+                    help="sharded exchange for N > 1; p2p also lets ranks share a GPU (a code-path check)")
     ap.add_argument("--balance-config", default="C4,C5", help="per-shard sweep times of the LPT split, N = 1")
     ap.add_argument("--ils-config", default="C1:200,C2:50", help="Iterated Local Search runs cfg:iterations")
     ap.add_argument("--pruned-config", default="C3:8,C4:8,C5:8,C5:16", help="pruned 2-opt from MF, cfg:K")

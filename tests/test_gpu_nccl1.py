@@ -52,11 +52,16 @@ def test_nccl_one_rank_modes(gpu):
 
 
 def test_nccl_one_rank_full_size_C4(gpu):
+    """C4 from the Hilbert start through the NCCL path (incremental culled sweep, the
+    allreduce captured in the graph batches): every move equals the oracle's golden."""
+    import os
+    gold = np.load(os.path.join(os.path.dirname(__file__), "golden", "ls_radius_C4_lattice_hilbert_s1.npz"))
+    k = int(gold["iterations"])
     c, t = inputs.config_instance("C4", "hilbert")
     with _handle(c) as g:
+        g.set_option(tsp2opt.OPT_TRACE, k + 8)
         res = g.local_search(t)
-    with tsp2opt.TSP2Opt(c) as g:
-        ref = g.local_search(t)  # the unsharded path (itself checked against the oracle in test_gpu_fullsize)
-    assert (res["iterations"], res["length"]) == (ref["iterations"], ref["length"])
-    assert np.array_equal(res["tour"], ref["tour"])
-    assert oracle.best_move(c, res["tour"]) == (0, 1, 0)
+        trace = g.get_trace(k + 8)
+    assert (res["iterations"], res["length"]) == (k, int(gold["length"]))
+    assert np.array_equal(np.asarray(trace, np.int64), gold["trace"][:k])
+    assert np.array_equal(res["tour"], gold["tour"])

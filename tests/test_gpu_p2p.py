@@ -93,3 +93,11 @@ def test_p2p_errors(gpu):
             tsp2opt.p2p_export(g)
     finally:
         tsp2opt.destroy(g)
+
+
+def test_p2p_c4_sharded_incremental(gpu):
+    """C4 (571 M pairs) on two ranks: the incremental culled sweep of each rank's half of
+    the tile list (the per-shard (row block, column chunk) map, the fused dirty-tile
+    kernel, the mailbox exchange between sweep and apply inside the captured graph
+    batches) -- every move equals the golden."""
+    _check_golden(_run(2, "C4:hilbert"))
