@@ -246,7 +246,9 @@ def run_ours(args):
         # fraction -- the warp instructions ONE sweep launch executes (ncu, committed
         # profile of this workload) over the live launch time, against 4 warp-inst/clk/SM.
         issue_peak = ISSUE_PER_CLK_SM * N_SM * sm_max * 1e6  # warp-instructions/s per GPU
-        winst = prof.get("warp_inst")
+        winst = prof.get("warp_inst")  # one full single-GPU sweep; a rank's shard does its share of it
+        if winst:
+            winst *= geo["pairs"] / total_pairs
         issue_rate = winst / (sweep_avg_ms * 1e-3) if winst else None
         line = {
             "metric": METRIC,
