@@ -676,7 +676,10 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     // local search from MF).
     // (incremental culled sweep, measured without per-sweep events: n = 85900 TJ 32 28.6 vs 64 30.6 us
     // per iteration, n = 33810 TJ 16 20.6 vs 32 22.7 us; profiles/r01_inc_tiling.jsonl)
-    h->cgeo = Geometry{kRowsSmall, 1, total_pairs >= 1000000000LL ? 32 : 16};
+    // Round 2, with the persistent incremental search (one warp per kept tile, the move's cost
+    // set by the slowest tile's walk): narrower chunks again -- C5 16 columns 21.9 vs 32 23.8 us
+    // per move, C4 8 columns 17.7 vs 16 18.9 (profiles/r02_exp_cull_tj.jsonl).
+    h->cgeo = Geometry{kRowsSmall, 1, total_pairs >= 1000000000LL ? 16 : 8};
     if (const char* er = getenv("TSP2OPT_CULL_ROWS")) h->cgeo.rows = atoi(er) == kRowsSmall ? kRowsSmall : kRowsLarge;
     if (const char* ec = getenv("TSP2OPT_CULL_TJ"))
         if (atoi(ec) >= 2 && atoi(ec) <= kMaxTJ) h->cgeo.tj = atoi(ec);
