@@ -60,6 +60,14 @@ struct tsp2opt_ctx {
     int* d_tour_in = nullptr;   // int32[n] staging for host tours
     float2* d_P = nullptr;      // [n + 1 + pad] biased route-ordered coordinates
     int* d_E = nullptr;         // [n + pad] edges
+    float2* d_P_alt = nullptr;  // alternate P / E / tour of the two-barrier persistent search (allocated on first use)
+    int* d_E_alt = nullptr;
+    int* d_tour_alt = nullptr;
+    void* d_inc2_ws = nullptr; // its barrier counter, dense tile minima and group minima (inc_ls2_ws_bytes)
+    int inc_barriers = 2;       // TSP2OPT_INC_BARRIERS=3: the three-barrier persistent kernel (in-place apply)
+    int inc_part = -1;          // TSP2OPT_INC_PART: columns per part of a kept tile (-1: the default; 0 with the
+                                // three-barrier kernel: one warp per whole tile)
+    int inc_part_bound = 0;     // TSP2OPT_INC_PART_BOUND=1: the tile bound on every part (measured 4 % slower)
     Slot* d_slots = nullptr;    // [2]
     unsigned* d_stamp = nullptr;  // [n] permutation check
     unsigned* d_bar = nullptr;    // [2] grid barrier of the persistent local search (count, generation)
@@ -265,6 +273,10 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_tour_in);
     cudaFree(h->d_P);
     cudaFree(h->d_E);
+    cudaFree(h->d_P_alt);
+    cudaFree(h->d_E_alt);
+    cudaFree(h->d_tour_alt);
+    cudaFree(h->d_inc2_ws);
     cudaFree(h->d_slots);
     cudaFree(h->d_stamp);
     cudaFree(h->d_bar);
@@ -484,21 +496,40 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
                             h->shard_world == 1;
     if (use_inc_ls) {
         const int flags = sweep_flags(h);
-        int full = (h->inc_valid && h->last_tiling == 1) ? 0 : 1;
+        // the two-barrier kernel keeps its minima in its own dense layout: tiling id 4
+        const int inc_tiling = h->inc_barriers == 2 ? 4 : 1;
+        int full = (h->inc_valid && h->last_tiling == inc_tiling) ? 0 : 1;
         for (long long launches = 0;; launches++) {
             if (launches > 1000000) {
                 g_last_error = "local search did not converge";
                 return TSP2OPT_ECUDA;
             }
-            CUDA_TRY(launch_inc_ls(h->cgeo, h->d_P, h->d_E, h->d_tour, h->n, h->d_ctiles, h->nctiles, h->d_tmap,
-                                   h->d_rbox, h->d_cbox, h->d_slots, h->parity, max_iters, 1LL << 20, full, h->d_bar,
-                                   h->d_ctl, h->d_ctilebest, flags, h->d_trace, h->trace_cap, h->stream));
+            if (h->inc_barriers == 2) {
+                const size_t np = (size_t)h->n + 1 + kPad;
+                if (!h->d_P_alt) {
+                    const size_t wsb = inc_ls2_ws_bytes(h->cgeo, h->n);
+                    CUDA_TRY(cudaMalloc(&h->d_P_alt, sizeof(float2) * np));
+                    CUDA_TRY(cudaMalloc(&h->d_E_alt, sizeof(int) * np));
+                    CUDA_TRY(cudaMalloc(&h->d_tour_alt, sizeof(int) * np));
+                    CUDA_TRY(cudaMalloc(&h->d_inc2_ws, wsb));
+                    CUDA_TRY(cudaMemsetAsync(h->d_inc2_ws, 0xFF, wsb, h->stream));  // minima: none
+                }
+                CUDA_TRY(launch_inc_ls2(h->cgeo, h->d_P, h->d_E, h->d_tour, h->d_P_alt, h->d_E_alt, h->d_tour_alt,
+                                        h->n, (int)np, h->d_tmap, h->d_rbox, h->d_cbox, h->d_inc2_ws, h->d_slots,
+                                        h->parity, max_iters, 1LL << 20, full, h->d_ctl, flags, h->d_trace,
+                                        h->trace_cap, h->inc_part, h->inc_part_bound, h->stream));
+            } else {
+                CUDA_TRY(launch_inc_ls(h->cgeo, h->d_P, h->d_E, h->d_tour, h->n, h->d_ctiles, h->nctiles, h->d_tmap,
+                                       h->d_rbox, h->d_cbox, h->d_slots, h->parity, max_iters, 1LL << 20, full,
+                                       h->d_bar, h->d_ctl, h->d_ctilebest, flags, h->d_trace, h->trace_cap,
+                                       h->inc_part < 0 ? 4 : h->inc_part, h->stream));
+            }
             full = 0;
             CUDA_TRY(cudaMemcpyAsync(h->h_ctl, h->d_ctl, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
             CUDA_TRY(cudaStreamSynchronize(h->stream));
             h->parity = *h->h_ctl;
             h->inc_valid = true;  // the stored tile minima are tile-local and exact for the current tour
-            h->last_tiling = 1;
+            h->last_tiling = inc_tiling;
             rc = read_slot(h);
             if (rc) return rc;
             if (h->h_slot->done & 3) break;
@@ -650,6 +681,9 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     if (const char* eg = getenv("TSP2OPT_GLOBAL_SEED")) h->global_seed = atoi(eg) != 0;
     if (const char* ef = getenv("TSP2OPT_INC_FUSED")) h->inc_fused = atoi(ef) != 0;
     if (const char* ei = getenv("TSP2OPT_INC_PERSISTENT")) h->inc_persistent = atoi(ei) != 0;
+    if (const char* eb = getenv("TSP2OPT_INC_BARRIERS")) h->inc_barriers = atoi(eb) == 3 ? 3 : 2;
+    if (const char* ep2 = getenv("TSP2OPT_INC_PART")) h->inc_part = atoi(ep2);
+    if (const char* eq = getenv("TSP2OPT_INC_PART_BOUND")) h->inc_part_bound = atoi(eq) != 0;
     if (const char* ed = getenv("TSP2OPT_DENSE_LS")) h->dense_ls = atoi(ed) != 0;
 
     CTRY(cudaMemset(h->d_slots, 0, sizeof(Slot) * 2));

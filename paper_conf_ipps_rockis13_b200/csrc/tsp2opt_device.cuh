@@ -33,6 +33,7 @@ constexpr int kSweepFull = 16;       // incremental sweep whose stored minima ar
 // delta, so the min is the lowest cell; first_fix_kernel writes the real delta.
 constexpr int kFirstDelta = -1;
 constexpr int kSweepFirst = 32;      // first improvement: the lowest improving cell instead of the lowest delta
+constexpr int kSweepPartBounds = 64; // inc_ls2: the bounding-box test of tile_may_pass on each column part
 
 // Bounding box of a run of route positions (unbiased integer coordinates) and
 // the largest tour edge leaving it: the summaries the tile cull compares.

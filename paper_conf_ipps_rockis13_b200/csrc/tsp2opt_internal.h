@@ -137,7 +137,19 @@ cudaError_t launch_dense_ls(const Geometry& g, float2* P, int* E, int* tour, int
 cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
                           const int* tmap, Box* rbox, Box* cbox, Slot* slots, int parity, long long max_moves,
                           long long budget, int full, unsigned* bar, int* ctl, unsigned long long* tilebest, int flags,
-                          unsigned long long* trace, long long trace_cap, cudaStream_t st);
+                          unsigned long long* trace, long long trace_cap, int part_cols, cudaStream_t st);
+// Same search with two grid barriers per move (inc_ls2_kernel): the move is applied out of place into
+// P1 / E1 / T1 (np entries each, alternating with P / E / tour), and the next sweep's boxes and clean
+// minima are computed in the same phase.  ws: inc_ls2_ws_bytes (the barrier counter, the dense tile
+// minima and their group minima; the minima initialised to all-ones once).  part_cols: columns per
+// part of a kept tile (0: the default); part_bound: the tile bound on every part.  P / E / tour hold the
+// current state when it returns.
+size_t inc_ls2_ws_bytes(const Geometry& g, int n);
+cudaError_t launch_inc_ls2(const Geometry& g, float2* P, int* E, int* tour, float2* P1, int* E1, int* T1, int n,
+                           int np, const int* tmap, Box* rbox, Box* cbox, void* ws, Slot* slots, int parity,
+                           long long max_moves, long long budget, int full, int* ctl, int flags,
+                           unsigned long long* trace, long long trace_cap, int part_cols, int part_bound,
+                           cudaStream_t st);
 cudaError_t launch_inc_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
                              const int* tmap, int grid, Box* rbox, Box* cbox, Slot* slot, int respect_done,
                              unsigned long long* tilebest, int flags, cudaStream_t st);

@@ -20,7 +20,7 @@ namespace tsp2opt {
 // persistent incremental local search (boxes, barrier, sweep, barrier, apply,
 // barrier), summed over the iterations; read by tsp2opt_debug_stats.
 __device__ unsigned long long g_phase[16];
-__device__ unsigned long long g_phase_it[4];  // per-iteration maxima, folded into g_phase[8..11] by CTA 0
+__device__ unsigned long long g_phase_it[8];  // per-iteration maxima, folded into g_phase[8..11] by CTA 0
 #endif
 
 // ===========================================================================
@@ -100,6 +100,9 @@ __global__ void reset_key_kernel(Slot* slot)
 }
 
 // a4 + a5: the sweep of one tile lives in tsp2opt_sweep.cuh.
+constexpr int kIncLsThreads = 512;     // persistent searches: 16 warps, one CTA per SM
+constexpr int kIncLsMaxThreads = 512;
+constexpr int kIncPartCols = 4;        // columns per part of a kept tile (inc_kept_parts)
 
 #ifndef TSP2OPT_MINB
 #define TSP2OPT_MINB 4  // CTAs of 128 threads per SM the register allocation must allow
@@ -685,6 +688,173 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
     if (gtid == 0) ctl[0] = p;
 }
 
+// Phase (C2) of the persistent incremental search with kept tiles split into
+// column parts: the CTA's threads cull the dirty tiles enumerated CTA-major
+// (u = thread * grid + CTA, so the clustered kept tiles of one move spread over
+// the CTAs; the tile index, both boxes loaded in one round trip), collect the
+// kept ones in a shared list, stage up to kStageTiles of them at once (every
+// thread loads; one L2 round trip) and the CTA's warps sweep (tile, part)
+// items with sweep_part; the tile minimum is the shared atomicMin over its
+// parts.  Same cull test, tile-local bound and stored minima as the per-warp
+// tile sweep, so the same moves.  Minima go to tilebest[t] (tb2 == nullptr) or,
+// for inc_ls2_kernel, to the dense per-(row block, column chunk) array tb2
+// plus an atomicMin into the tile's group minimum sm2 (64 chunks per group).
+constexpr int kStageTiles = 16;
+constexpr int kGroupChunks = 64;  // column chunks per group minimum (inc_ls2_kernel)
+template <int R, bool FIRST>
+__device__ __forceinline__ void inc_kept_parts(const float2* P, const int* E, int n,
+                                               const int* __restrict__ tmap, int TI, int TJ, int nrb, int ncc,
+                                               int rlo, int rhi, int clo, int chi, long long nA, long long nB,
+                                               const Box* rbox, const Box* cbox,
+                                               Slot* in, unsigned long long* tilebest,
+                                               int tflags, int part_cols, float4* smem, int tile_bytes,
+                                               unsigned long long* tb2 = nullptr, unsigned long long* sm2 = nullptr,
+                                               int nsc = 0)
+{
+    __shared__ int s_nk;
+    __shared__ int4 s_kt[kIncLsMaxThreads];  // kept tiles of this round: (t, rb, cc)
+    __shared__ unsigned long long s_tmin[kStageTiles];
+    const int tid = threadIdx.x, nthr = blockDim.x, wib = tid >> 5, nwb = nthr >> 5;
+    const int nparts = (TJ + part_cols - 1) / part_cols;
+    const long long step = (long long)nthr * gridDim.x;
+#ifdef TSP2OPT_PHASE_TIMING
+    // per CTA: [2] cull cycles, [3] staging, [4] part sweeps, [5] kept tiles -- maxima over CTAs per move
+    long long pt0 = clock64(), pcull = 0, pstage = 0, pitems = 0;
+    int pkept = 0;
+#endif
+    for (long long base = 0; base < nA + nB; base += step) {
+        if (tid == 0) s_nk = 0;
+        __syncthreads();
+        const long long u = base + (long long)tid * gridDim.x + blockIdx.x;
+        if (u < nA + nB) {
+            int rb, cc;
+            bool cand = true;
+            if (u < nA) {
+                rb = rlo + (int)(u / ncc);
+                cc = (int)(u % ncc);
+            } else {
+                const long long v = u - nA;
+                rb = (int)(v / (chi - clo + 1));
+                cc = clo + (int)(v % (chi - clo + 1));
+                cand = rb < rlo || rb > rhi;  // else already in part A
+            }
+            if (cand) {
+                const int t = tmap[(long long)rb * ncc + cc];  // issued together with the two boxes
+                const Box r = rbox[rb], c = cbox[cc];
+                if (t >= 0) {
+                    const long long gx = max(0, max(c.xlo - r.xhi, r.xlo - c.xhi));
+                    const long long gy = max(0, max(c.ylo - r.yhi, r.ylo - c.yhi));
+                    const long long T = (long long)max(r.emax, c.emax) - 1;
+                    if (T >= 0 && gx * gx + gy * gy <= T * T + T) s_kt[atomicAdd(&s_nk, 1)] = make_int4(t, rb, cc, 0);
+                    else if (tb2) tb2[(long long)rb * ncc + cc] = kKeyNone;
+                    else tilebest[t] = kKeyNone;
+                }
+            }
+        }
+        __syncthreads();
+        const int nk = s_nk;
+#ifdef TSP2OPT_PHASE_TIMING
+        {
+            const long long t1 = clock64();
+            pcull += t1 - pt0;
+            pt0 = t1;
+            pkept += nk;
+        }
+#endif
+        for (int b0 = 0; b0 < nk; b0 += kStageTiles) {
+            const int nb = min(kStageTiles, nk - b0);
+            // stage: per tile the column positions J0 .. J1 + 1 and the row positions I0 .. I0 + 32R
+            // (P and E of each), loads batched ahead of the shared stores
+            const int ncolp = TJ + 2, nrowp = 32 * R + 1, per = ncolp + nrowp;
+            constexpr int U = 8;
+            for (int x0 = 0; x0 < nb * per; x0 += U * nthr) {
+                float2 pv[U];
+                int ev[U];
+#pragma unroll
+                for (int v = 0; v < U; v++) {
+                    const int x = x0 + v * nthr + tid;
+                    pv[v] = make_float2(0.f, 0.f);
+                    ev[v] = 0;
+                    if (x < nb * per) {
+                        const int k = x / per, q = x - k * per;
+                        const int4 kt = s_kt[b0 + k];
+                        const int pos = q < ncolp ? kt.z * TJ + q : kt.y * TI + (q - ncolp);
+                        pv[v] = P[pos];
+                        ev[v] = E[pos];
+                    }
+                }
+#pragma unroll
+                for (int v = 0; v < U; v++) {
+                    const int x = x0 + v * nthr + tid;
+                    if (x < nb * per) {
+                        const int k = x / per, q = x - k * per;
+                        const TileSmem tsm(reinterpret_cast<char*>(smem) + (size_t)k * tile_bytes, TJ, 32 * R);
+                        if (q < ncolp) {
+                            tsm.put(q, pv[v], (float)ev[v]);
+                        } else {
+                            const int rq = q - ncolp;  // row position I0 + rq: lane rq / R, slot rq % R
+                            const int ln = rq / R, sl = rq - ln * R;
+                            if (ln < 32) {
+                                tsm.rowp[ln * (R + 1) + sl] = pv[v];
+                                tsm.rowe[rq] = (float)ev[v];
+                            }
+                            if (sl == 0 && ln > 0) tsm.rowp[(ln - 1) * (R + 1) + R] = pv[v];  // previous lane's row R
+                        }
+                    }
+                }
+            }
+            if (tid < nb) s_tmin[tid] = kKeyNone;
+            __syncthreads();
+#ifdef TSP2OPT_PHASE_TIMING
+            {
+                const long long t1 = clock64();
+                pstage += t1 - pt0;
+                pt0 = t1;
+            }
+#endif
+            for (int it = wib; it < nb * nparts; it += nwb) {
+                const int k = it / nparts, part = it - k * nparts;
+                const int4 kt = s_kt[b0 + k];
+                const TileSmem tsm(reinterpret_cast<char*>(smem) + (size_t)k * tile_bytes, TJ, 32 * R);
+                const int I0 = kt.y * TI, J0 = kt.z * TJ, J1 = min(J0 + TJ, n);
+                const int jb = J0 + part * part_cols, je = min(jb + part_cols, J1);
+                if (jb < je) {
+                    const unsigned long long mk = sweep_part<R, FIRST>(I0, J0, jb, je, tsm, tflags);
+                    if (mk != kKeyNone) atomicMin(&s_tmin[k], mk);
+                }
+            }
+            __syncthreads();
+#ifdef TSP2OPT_PHASE_TIMING
+            {
+                const long long t1 = clock64();
+                pitems += t1 - pt0;
+                pt0 = t1;
+            }
+#endif
+            if (tid < nb) {
+                const unsigned long long m = s_tmin[tid];
+                const int4 kt = s_kt[b0 + tid];
+                if (tb2) {
+                    tb2[(long long)kt.y * ncc + kt.z] = m;
+                    if (m != kKeyNone) atomicMin(&sm2[(long long)kt.y * nsc + kt.z / kGroupChunks], m);
+                } else {
+                    tilebest[kt.x] = m;
+                }
+                if (m != kKeyNone && m < *(volatile unsigned long long*)&in->key) atomicMin(&in->key, m);
+            }
+            __syncthreads();  // before the next batch restages the shared tiles
+        }
+    }
+#ifdef TSP2OPT_PHASE_TIMING
+    if (tid == 0) {
+        atomicMax(&g_phase_it[2], (unsigned long long)pcull);
+        atomicMax(&g_phase_it[3], (unsigned long long)pstage);
+        atomicMax(&g_phase_it[4], (unsigned long long)pitems);
+        atomicMax(&g_phase_it[5], (unsigned long long)pkept);
+    }
+#endif
+}
+
 // ===========================================================================
 // Persistent incremental local search (TSP2OPT_OPT_TILE_BOUNDS = 3, one GPU):
 // ONE cooperative launch runs the whole culled, incremental search of §5.6 --
@@ -715,7 +885,7 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
                                                         int* __restrict__ ctl,
                                                         unsigned long long* __restrict__ tilebest, int flags,
                                                         unsigned long long* __restrict__ trace, long long trace_cap,
-                                                        int tile_bytes)
+                                                        int tile_bytes, int part_cols)
 {
     extern __shared__ float4 smem[];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -784,6 +954,10 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
 #endif
         const long long nA = (long long)(rhi - rlo + 1) * ncc;
         const long long nB = (long long)nrb * (chi - clo + 1);
+        if (part_cols > 0) {
+            inc_kept_parts<R, FIRST>(P, E, n, tmap, TI, TJ, nrb, ncc, rlo, rhi, clo, chi, nA, nB, rbox, cbox, in,
+                                     tilebest, tflags, part_cols, smem, tile_bytes);
+        } else
         for (long long base = 0; base < nA + nB; base += (long long)nw * 32) {
             const long long u = base + (long long)lane * nw + gw;
             int t = -1, rb = 0, cc = 0;
@@ -891,6 +1065,388 @@ __global__ void __launch_bounds__(512, 1) inc_ls_kernel(float2* __restrict__ P, 
     }
     if (gtid == 0) ctl[0] = p;
 #undef PHASE_MARK
+}
+
+// ===========================================================================
+// Persistent incremental local search, two grid barriers per move
+// (inc_ls2_kernel; the default for TSP2OPT_OPT_TILE_BOUNDS = 3 on one GPU).
+// Per move:
+//   (C) the dirty tiles culled and the kept ones swept in column parts
+//       (inc_kept_parts)                                          grid barrier,
+//   (X) the move applied OUT OF PLACE -- the next state is written into the
+//       other of two P / E / tour buffers, read only from the current one --
+//       so that, in the same phase, the boxes of the blocks the move dirties
+//       are computed from the current buffer through the reversal's mirror map
+//       (new P[k] = P[i+j+1-k] on [i+1, j], new e[k] = e[i+j-k] on (i, j),
+//       the two new edges), and the clean tiles' stored minima are folded into
+//       the next sweep's key;                                      grid barrier.
+// The buffer written by a move holds the state two moves back, so it is
+// brought up to date on the previous move's positions and written on this
+// move's (a few hundred entries for a typical move).  The launch starts with
+// a full copy current -> alternate and ends by copying the last move's
+// positions back if the current state is in the alternate buffer, so the
+// handle's P / E / tour are current between launches.
+// Clean minima: tile minima live in a dense (row block, column chunk) array
+// tb2 and, per group of kGroupChunks chunks of one row block, in sm2 = the
+// min over the group's tiles.  (X) resets sm2 of the groups the move dirties
+// to the min over their clean tiles (none for a dirty row block) and (C)
+// atomicMins every re-swept tile into its group, so sm2 is exact after every
+// sweep; the clean scan reads one sm2 entry per clean group and the clean
+// tiles of the (at most two) partly dirty groups of each row block, instead of
+// every tile.  Same boxes, cull test, tile sweep, clean / dirty rule and
+// decisions as the three-barrier kernel (inc_ls_kernel): the same moves.
+// ===========================================================================
+// Box of positions k0..ke (cities) and edges k0..ke-1 of the state AFTER move
+// (i, j) (i < 0: no move), read from the state before it: city at k is
+// P[i+j+1-k] on [i+1, j]; edge k is di / dj at i / j, e[i+j-k] on (i, j).
+// di / dj are computed here from loads issued with the box's own.
+__device__ __forceinline__ Box warp_box_mirror(const float2* P, const int* E, int k0, int ke, int i, int j)
+{
+    constexpr int kWarpBoxBatch = 8;
+    const int lane = threadIdx.x & 31;
+    float2 pi = make_float2(0.f, 0.f), pj = pi, pi1 = pi, pj1 = pi;
+    const bool has_i = i >= k0 && i < ke, has_j = j >= k0 && j < ke;  // the new edges fall in this range
+    if (has_i || has_j) {
+        pi = P[i];
+        pj = P[j];
+        pi1 = P[i + 1];
+        pj1 = P[j + 1];
+    }
+    int xlo = 1 << 30, xhi = -1, ylo = 1 << 30, yhi = -1, emax = 0;
+    for (int k1 = k0; k1 <= ke; k1 += 32 * kWarpBoxBatch) {
+        float2 p[kWarpBoxBatch];
+        int e[kWarpBoxBatch];
+#pragma unroll
+        for (int b = 0; b < kWarpBoxBatch; b++) {
+            const int k = k1 + lane + 32 * b;
+            const int mk = (k > i && k <= j) ? i + j + 1 - k : k;
+            const int me = (k > i && k < j) ? i + j - k : k;
+            p[b] = k <= ke ? P[mk] : make_float2(0.f, 0.f);
+            e[b] = (k < ke && k != i && k != j) ? E[me] : 0;
+        }
+#pragma unroll
+        for (int b = 0; b < kWarpBoxBatch; b++) {
+            const int k = k1 + lane + 32 * b;
+            if (k <= ke) {
+                const int x = unbias(p[b].x), y = unbias(p[b].y);
+                xlo = min(xlo, x);
+                xhi = max(xhi, x);
+                ylo = min(ylo, y);
+                yhi = max(yhi, y);
+                emax = max(emax, e[b]);
+            }
+        }
+    }
+    if (has_i) emax = max(emax, exact_dist_biased(pi, pj));
+    if (has_j) emax = max(emax, exact_dist_biased(pi1, pj1));
+    const unsigned full = 0xffffffffu;
+    Box b;
+    b.xlo = __reduce_min_sync(full, xlo);
+    b.xhi = __reduce_max_sync(full, xhi);
+    b.ylo = __reduce_min_sync(full, ylo);
+    b.yhi = __reduce_max_sync(full, yhi);
+    b.emax = __reduce_max_sync(full, emax);
+    b.pad[0] = b.pad[1] = b.pad[2] = 0;
+    return b;
+}
+
+// Boxes of the blocks dirtied by move (i, j) over positions [dlo, dhi] (i < 0:
+// no mirror, plain reads), one warp per block, warps gw of nw.
+__device__ __forceinline__ void dirty_boxes(const float2* P, const int* E, int n, int TI, int TJ, int nrb, int ncc,
+                                            int dlo, int dhi, int i, int j, Box* rbox, Box* cbox, int gw, int nw)
+{
+    const int lane = threadIdx.x & 31;
+    const int rlo = dlo >= 1 ? (dlo - 1) / TI : 0, rhi = min(nrb - 1, dhi / TI);
+    const int clo = dlo >= 1 ? (dlo - 1) / TJ : 0, chi = min(ncc - 1, dhi / TJ);
+    const int nR = rhi - rlo + 1, nC = chi - clo + 1;
+    for (int task = gw; task < nR + nC; task += nw) {
+        if (task < nR) {
+            const int rb = rlo + task;
+            const Box b = warp_box_mirror(P, E, rb * TI, min(rb * TI + TI, n - 1), i, j);
+            if (lane == 0) rbox[rb] = b;
+        } else {
+            const int cc = clo + task - nR;
+            const Box b = warp_box_mirror(P, E, cc * TJ, min(cc * TJ + TJ, n), i, j);
+            if (lane == 0) cbox[cc] = b;
+        }
+    }
+}
+
+// Group minima for the sweep whose dirty positions are [dlo, dhi] (dirty row
+// blocks [rlo, rhi], chunks [clo, chi]), one warp per row block (warps gw of
+// nw): a dirty row block's groups are reset to none; in a clean row block a
+// group inside [clo, chi] is reset to none, a group partly inside is set to
+// the min over its clean tiles (read from tb2), and both those and the
+// untouched groups' sm2 enter the returned warp minimum (every lane).
+__device__ __forceinline__ unsigned long long group_minima(const unsigned long long* tb2, unsigned long long* sm2,
+                                                           int nrb, int ncc, int nsc, int rlo, int rhi, int clo,
+                                                           int chi, int gw, int nw)
+{
+    const int lane = threadIdx.x & 31;
+    unsigned long long m = kKeyNone;
+    const int sclo = clo / kGroupChunks, schi = chi / kGroupChunks;
+    for (int rb = gw; rb < nrb; rb += nw) {
+        unsigned long long* srow = sm2 + (long long)rb * nsc;
+        if (rb >= rlo && rb <= rhi) {
+            for (int sc = lane; sc < nsc; sc += 32) srow[sc] = kKeyNone;
+            continue;
+        }
+        // the partly dirty groups (sclo, schi): their clean tiles, two loads per lane each
+        unsigned long long ga = kKeyNone, gb = kKeyNone;
+        const unsigned long long* trow = tb2 + (long long)rb * ncc;
+#pragma unroll
+        for (int h = 0; h < kGroupChunks / 32; h++) {
+            const int ca = sclo * kGroupChunks + h * 32 + lane, cb = schi * kGroupChunks + h * 32 + lane;
+            const unsigned long long va = (ca < ncc && (ca < clo || ca > chi)) ? trow[ca] : kKeyNone;
+            const unsigned long long vb = (cb < ncc && (cb < clo || cb > chi)) ? trow[cb] : kKeyNone;
+            ga = min(ga, va);
+            gb = min(gb, vb);
+        }
+        for (int sc = lane; sc < nsc; sc += 32) {
+            if (sc == sclo || sc == schi) continue;
+            if (sc > sclo && sc < schi) srow[sc] = kKeyNone;  // every tile of the group is dirty
+            else m = min(m, srow[sc]);
+        }
+        for (int o = 16; o > 0; o >>= 1) {
+            ga = min(ga, __shfl_xor_sync(0xffffffffu, ga, o));
+            gb = min(gb, __shfl_xor_sync(0xffffffffu, gb, o));
+        }
+        if (lane == 0) {
+            srow[sclo] = ga;
+            if (schi != sclo) srow[schi] = gb;
+        }
+        m = min(m, min(ga, gb));
+    }
+    for (int o = 16; o > 0; o >>= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
+    return m;
+}
+
+// Grid barrier on a monotonic 64-bit arrival counter (reset to 0 before the
+// launch; every barrier of the launch adds gridDim.x): one atomic per CTA and
+// polling, no reset round trips.  `target` is the CTA's running count.
+__device__ __forceinline__ void grid_sync_mono(unsigned long long* ctr, unsigned long long& target)
+{
+    __syncthreads();
+    target += gridDim.x;
+    if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(ctr, 1ULL);
+        while (*(volatile unsigned long long*)ctr < target) {
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+constexpr int kBoxWarps = 4;  // (X): warps per CTA computing boxes; the others scan the group minima
+
+template <int R, bool FIRST>
+__global__ void __launch_bounds__(512, 1) inc_ls2_kernel(float2* P0, int* E0, int* T0, float2* P1, int* E1, int* T1,
+                                                         int n, int np, const int* __restrict__ tmap, int TI, int TJ,
+                                                         int nrb, int ncc, int nsc, Box* rbox, Box* cbox,
+                                                         unsigned long long* tb2, unsigned long long* sm2,
+                                                         unsigned long long* ctr, Slot* slots, int parity,
+                                                         long long max_moves, long long budget, int full, int* ctl,
+                                                         int flags, unsigned long long* trace, long long trace_cap,
+                                                         int tile_bytes, int part_cols)
+{
+    extern __shared__ float4 smem[];
+    const int wib = threadIdx.x >> 5, nwb = blockDim.x >> 5, lane = threadIdx.x & 31;
+    const int gw = blockIdx.x * nwb + wib, nw = gridDim.x * nwb;
+    const int gtid = blockIdx.x * blockDim.x + threadIdx.x, stride = gridDim.x * blockDim.x;
+    const bool boxw = wib < kBoxWarps;  // (X) role
+    const int gwb = blockIdx.x * kBoxWarps + wib, nwbx = gridDim.x * kBoxWarps;
+    const int gwc = blockIdx.x * (nwb - kBoxWarps) + (wib - kBoxWarps), nwc = gridDim.x * (nwb - kBoxWarps);
+    const int tflags = (flags | kSweepLocal) & ~kSweepSeed;
+    __shared__ Slot s_in;
+    __shared__ unsigned long long s_min[32];
+    unsigned long long target = 0;
+    int p = parity;
+    float2 *Pc = P0, *Pa = P1;
+    int *Ec = E0, *Ea = E1, *Tc = T0, *Ta = T1;
+#ifdef TSP2OPT_PHASE_TIMING
+    // CTA 0's cycles per phase ([0] C, [1] barrier, [2] X, [3] barrier) and the per-move
+    // maxima over CTAs ([8] C, [9] X); [10] moves counted
+    const bool t_lead = threadIdx.x == 0, t_cta0 = blockIdx.x == 0 && threadIdx.x == 0;
+#endif
+    // prologue: the first sweep's dirty set, its boxes and group minima; alternate := current
+    if (threadIdx.x == 0) {
+        s_in.done = *(volatile int*)&slots[p].done;
+        s_in.seed_ok = full ? 0 : *(volatile int*)&slots[p].seed_ok;
+        s_in.last_key = *(volatile unsigned long long*)&slots[p].last_key;
+    }
+    __syncthreads();
+    if (s_in.done) {
+        if (gtid == 0) ctl[0] = p;
+        return;  // uniform
+    }
+    int dlo = 0, dhi = n;
+    if (s_in.seed_ok) {
+        dlo = key_i(s_in.last_key);
+        dhi = key_j(s_in.last_key);
+    }
+    int rlo = dlo >= 1 ? (dlo - 1) / TI : 0, rhi = min(nrb - 1, dhi / TI);
+    int clo = dlo >= 1 ? (dlo - 1) / TJ : 0, chi = min(ncc - 1, dhi / TJ);
+    dirty_boxes(Pc, Ec, n, TI, TJ, nrb, ncc, dlo, dhi, -1, -1, rbox, cbox, gw, nw);
+    {
+        unsigned long long m = group_minima(tb2, sm2, nrb, ncc, nsc, rlo, rhi, clo, chi, gw, nw);
+        if (lane == 0) s_min[wib] = s_in.seed_ok ? m : kKeyNone;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            unsigned long long bm = s_min[0];
+            for (int w = 1; w < nwb; w++) bm = min(bm, s_min[w]);
+            if (!s_in.seed_ok) {
+                if (blockIdx.x == 0) slots[p].key = seed_key();  // full sweep: nothing is clean
+            } else if (bm != kKeyNone) {
+                atomicMin(&slots[p].key, bm);
+            }
+        }
+    }
+    for (int k = gtid; k < np; k += stride) {
+        Pa[k] = Pc[k];
+        Ea[k] = Ec[k];
+        Ta[k] = Tc[k];
+    }
+    grid_sync_mono(ctr, target);
+    int ip = -1, jp = -1;  // the launch's previous move: where the two buffers differ
+    for (long long it = 0; it < budget; it++) {
+        Slot* in = slots + p;
+        Slot* out = slots + (p ^ 1);
+#ifdef TSP2OPT_PHASE_TIMING
+        const long long tc0 = clock64();
+#endif
+        // (C) cull + sweep the dirty tiles of the current state into in->key
+        if (gtid == 0) out->key = seed_key();  // read last by the previous (X), before the barrier
+        {
+            const long long nA = (long long)(rhi - rlo + 1) * ncc;
+            const long long nB = (long long)nrb * (chi - clo + 1);
+            inc_kept_parts<R, FIRST>(Pc, Ec, n, tmap, TI, TJ, nrb, ncc, rlo, rhi, clo, chi, nA, nB, rbox, cbox, in,
+                                     nullptr, tflags, part_cols, smem, tile_bytes, tb2, sm2, nsc);
+        }
+#ifdef TSP2OPT_PHASE_TIMING
+        const long long tc1 = clock64();
+        if (t_lead) atomicMax(&g_phase_it[0], (unsigned long long)(tc1 - tc0));
+        if (t_cta0) atomicAdd(&g_phase[0], (unsigned long long)(tc1 - tc0));
+#endif
+        grid_sync_mono(ctr, target);
+#ifdef TSP2OPT_PHASE_TIMING
+        const long long tx0 = clock64();
+        if (t_cta0) {
+            atomicAdd(&g_phase[1], (unsigned long long)(tx0 - tc1));
+            g_phase[8] += g_phase_it[0];
+            g_phase_it[0] = 0;
+            for (int q = 2; q < 6; q++) {
+                g_phase[10 + q] += g_phase_it[q];
+                g_phase_it[q] = 0;
+            }
+        }
+#endif
+        // (X) decide and apply the winning move out of place; prepare the next sweep
+        if (threadIdx.x == 0) {
+            s_in.key = *(volatile unsigned long long*)&in->key;
+            s_in.moves = *(volatile long long*)&in->moves;
+            s_in.length = *(volatile long long*)&in->length;
+            s_in.done = *(volatile int*)&in->done;
+        }
+        __syncthreads();
+        const unsigned long long key = s_in.key;
+        const int i = key_i(key), j = key_j(key);
+        const long long moves = s_in.moves;
+        const bool apply = !s_in.done && key_delta(key) < 0 && moves < max_moves;
+        // the slot, the trace and the apply's few writes go to the last CTA's last threads: warps
+        // without a box or group task (the others' critical path is the box / group round trips)
+        const int rtid = stride - 1 - gtid;
+        if (rtid == 0) {
+            out->last_key = key;
+            out->moves = moves;
+            out->length = s_in.length;
+            out->done = s_in.done;
+            out->next_tile = 0;
+            out->ncull = 0;
+            out->mtype = 0;
+            out->seed_ok = apply ? 1 : 0;
+            if (!s_in.done) {
+                if (key_delta(key) >= 0) out->done = 1;      // local minimum (reading R7)
+                else if (moves >= max_moves) out->done = 2;  // capped with an improving move left (R8)
+            }
+            if (apply) {  // exact delta from the current state (a first-improvement key carries a marker)
+                const int di = exact_dist_biased(Pc[i], Pc[j]), dj = exact_dist_biased(Pc[i + 1], Pc[j + 1]);
+                const int d = di + dj - Ec[i] - Ec[j];
+                out->length = s_in.length + d;
+                out->moves = moves + 1;
+                out->last_key = pack_key(d, i, j);
+                if (trace && moves < trace_cap) trace[moves] = out->last_key;
+            }
+        }
+        if (apply) {
+            // P / tour: positions [i+1, j] reversed, [ip+1, jp] brought up to date
+            const int n1 = j - i, n2 = ip >= 0 ? jp - ip : 0;
+            for (int t = rtid; t < n1 + n2; t += stride) {
+                const int k = t < n1 ? i + 1 + t : ip + 1 + (t - n1);
+                const int mk = (k > i && k <= j) ? i + j + 1 - k : k;
+                Pa[k] = Pc[mk];
+                Ta[k] = Tc[mk];
+            }
+            // e: [i, j] (the two new edges, the inside reversed), [ip, jp] brought up to date
+            const int m1 = j - i + 1, m2 = ip >= 0 ? jp - ip + 1 : 0;
+            for (int t = rtid; t < m1 + m2; t += stride) {
+                const int k = t < m1 ? i + t : ip + (t - m1);
+                if (k == i) Ea[k] = exact_dist_biased(Pc[i], Pc[j]);
+                else if (k == j) Ea[k] = exact_dist_biased(Pc[i + 1], Pc[j + 1]);
+                else Ea[k] = (k > i && k < j) ? Ec[i + j - k] : Ec[k];
+            }
+            rlo = i >= 1 ? (i - 1) / TI : 0;
+            rhi = min(nrb - 1, j / TI);
+            clo = i >= 1 ? (i - 1) / TJ : 0;
+            chi = min(ncc - 1, j / TJ);
+            unsigned long long m = kKeyNone;
+            if (boxw) dirty_boxes(Pc, Ec, n, TI, TJ, nrb, ncc, i, j, i, j, rbox, cbox, gwb, nwbx);
+            else m = group_minima(tb2, sm2, nrb, ncc, nsc, rlo, rhi, clo, chi, gwc, nwc);
+            if (lane == 0) s_min[wib] = m;
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                unsigned long long bm = s_min[0];
+                for (int w = 1; w < nwb; w++) bm = min(bm, s_min[w]);
+                if (bm != kKeyNone) atomicMin(&out->key, bm);
+            }
+        }
+#ifdef TSP2OPT_PHASE_TIMING
+        const long long tx1 = clock64();
+        if (t_lead) atomicMax(&g_phase_it[1], (unsigned long long)(tx1 - tx0));
+        if (t_cta0) atomicAdd(&g_phase[2], (unsigned long long)(tx1 - tx0));
+#endif
+        p ^= 1;
+        grid_sync_mono(ctr, target);
+#ifdef TSP2OPT_PHASE_TIMING
+        if (t_cta0) {
+            atomicAdd(&g_phase[3], (unsigned long long)(clock64() - tx1));
+            g_phase[9] += g_phase_it[1];
+            g_phase_it[1] = 0;
+            g_phase[10] += 1;
+        }
+#endif
+        if (!apply) break;  // uniform: every CTA read the same key
+        ip = i;
+        jp = j;
+        float2* tp = Pc;
+        Pc = Pa;
+        Pa = tp;
+        int* te = Ec;
+        Ec = Ea;
+        Ea = te;
+        int* tt = Tc;
+        Tc = Ta;
+        Ta = tt;
+    }
+    // the handle's buffers: copy the last move's positions back if the current state is the alternate
+    if (Pc != P0 && ip >= 0) {
+        for (int t = gtid; t < jp - ip; t += stride) {
+            P0[ip + 1 + t] = Pc[ip + 1 + t];
+            T0[ip + 1 + t] = Tc[ip + 1 + t];
+        }
+        for (int t = gtid; t <= jp - ip; t += stride) E0[ip + t] = Ec[ip + t];
+    }
+    if (gtid == 0) ctl[0] = p;
 }
 
 // ===========================================================================
@@ -1235,12 +1791,11 @@ cudaError_t launch_inc_sweep(const Geometry& g, const float2* P, const int* E, i
     return e != cudaSuccess ? e : cudaGetLastError();
 }
 
-constexpr int kIncLsThreads = 512;  // 16 warps, one CTA per SM
 
 cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
                           const int* tmap, Box* rbox, Box* cbox, Slot* slots, int parity, long long max_moves,
                           long long budget, int full, unsigned* bar, int* ctl, unsigned long long* tilebest, int flags,
-                          unsigned long long* trace, long long trace_cap, cudaStream_t st)
+                          unsigned long long* trace, long long trace_cap, int part_cols, cudaStream_t st)
 {
     if (g.rows != kRowsSmall || g.warps != 1) return cudaErrorInvalidValue;
     int TI = g.ti(), TJ = g.tj, nrb = (n - 1 + TI - 1) / TI, ncc = (n + TJ - 1) / TJ;
@@ -1257,10 +1812,59 @@ cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int grid = sms;  // one CTA per SM (co-resident: cooperative launch)
-    void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &tmap, &TI, &TJ, &nrb, &ncc, &rbox, &cbox, &slots, &parity,
-                    &max_moves, &budget, &full, &bar, &ctl, &tilebest, &flags, &trace, &trace_cap, &tile_bytes};
+    // kept tiles split into column parts over the CTA's warps (part_cols columns per part; 0: one warp
+    // sweeps each whole kept tile)
+    part_cols = std::min(std::max(part_cols, 0), TJ);
+    if (flags & kSweepTileBounds) flags |= kSweepPartBounds;
+    void* args[] = {&P,     &E,    &tour,   &n,        &tiles,    &ntiles,    &tmap,   &TI,
+                    &TJ,    &nrb,  &ncc,    &rbox,     &cbox,     &slots,     &parity, &max_moves,
+                    &budget, &full, &bar,   &ctl,      &tilebest, &flags,     &trace,  &trace_cap,
+                    &tile_bytes, &part_cols};
     g_launches += 1;
     return cudaLaunchCooperativeKernel((const void*)kern, dim3(grid), dim3(kIncLsThreads), args, smem, st);
+}
+
+size_t inc_ls2_ws_bytes(const Geometry& g, int n)
+{
+    const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
+    const int nsc = (ncc + kGroupChunks - 1) / kGroupChunks;
+    return sizeof(unsigned long long) * (2 + (size_t)nrb * ncc + (size_t)nrb * nsc);
+}
+
+cudaError_t launch_inc_ls2(const Geometry& g, float2* P, int* E, int* tour, float2* P1, int* E1, int* T1, int n,
+                           int np, const int* tmap, Box* rbox, Box* cbox, void* ws, Slot* slots, int parity,
+                           long long max_moves, long long budget, int full, int* ctl, int flags,
+                           unsigned long long* trace, long long trace_cap, int part_cols, int part_bound,
+                           cudaStream_t st)
+{
+    if (g.rows != kRowsSmall || g.warps != 1) return cudaErrorInvalidValue;
+    int TI = g.ti(), TJ = g.tj, nrb = (n - 1 + TI - 1) / TI, ncc = (n + TJ - 1) / TJ;
+    int nsc = (ncc + kGroupChunks - 1) / kGroupChunks;
+    unsigned long long* ctr = static_cast<unsigned long long*>(ws);
+    unsigned long long* tb2 = ctr + 2;
+    unsigned long long* sm2 = tb2 + (size_t)nrb * ncc;
+    int tile_bytes = (int)((sweep_smem_bytes_ps(g) + 15) / 16 * 16);
+    const size_t smem = (size_t)tile_bytes * kStageTiles;
+    auto kern = (flags & kSweepFirst) ? inc_ls2_kernel<kRowsSmall, true> : inc_ls2_kernel<kRowsSmall, false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kIncLsThreads, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) return cudaErrorInvalidConfiguration;
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    part_cols = part_cols > 0 ? std::min(part_cols, TJ) : kIncPartCols;
+    if (part_bound && (flags & kSweepTileBounds)) flags |= kSweepPartBounds;
+    e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long), st);  // the barrier's arrival counter
+    if (e != cudaSuccess) return e;
+    void* args[] = {&P,   &E,   &tour, &P1,    &E1,        &T1,    &n,       &np,        &tmap,
+                    &TI,  &TJ,  &nrb,  &ncc,   &nsc,       &rbox,  &cbox,    &tb2,       &sm2,
+                    &ctr, &slots, &parity, &max_moves, &budget, &full, &ctl, &flags, &trace,
+                    &trace_cap, &tile_bytes, &part_cols};
+    g_launches += 1;
+    return cudaLaunchCooperativeKernel((const void*)kern, dim3(sms), dim3(kIncLsThreads), args, smem, st);
 }
 
 cudaError_t launch_dense_ls(const Geometry& g, float2* P, int* E, int* tour, int n, const int2* tiles, int ntiles,
@@ -1424,7 +2028,7 @@ cudaError_t read_phases(long long* out16, int reset)
 
 cudaError_t read_stats(long long* out4, int reset)
 {
-#if defined(TSP2OPT_STATS)
+#if defined(TSP2OPT_STATS) || defined(TSP2OPT_TILE_TIMING)
     unsigned long long h[4];
     cudaError_t e = cudaMemcpyFromSymbol(h, g_stats, sizeof(h));
     if (e != cudaSuccess) return e;

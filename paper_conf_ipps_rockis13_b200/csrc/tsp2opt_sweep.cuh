@@ -28,8 +28,9 @@
 
 namespace tsp2opt {
 
-#ifdef TSP2OPT_STATS
-// Instrumented builds only: [0] warp column steps, [1] steps taking the exact
+#if defined(TSP2OPT_STATS) || defined(TSP2OPT_TILE_TIMING)
+// Instrumented builds only (TSP2OPT_TILE_TIMING: [0] prologue cycles -- loads, staging,
+// the seed key --, [1] walk cycles, [2] tiles walked, [3] the slowest tile's cycles): [0] warp column steps, [1] steps taking the exact
 // path, [2] candidate pairs evaluated exactly, [3] warp tiles walked (not
 // skipped by the tile bound).
 __device__ unsigned long long g_stats[4];
@@ -449,6 +450,9 @@ template <int R, bool PS, bool FIRST = false, bool WT = false>
 __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n, int2 tile, int TJ, Slot* slot,
                                            const TileSmem& sm, unsigned long long* tilebest, int flags)
 {
+#ifdef TSP2OPT_TILE_TIMING
+    const long long tt0 = clock64();
+#endif
     const int I0 = tile.x, J0 = tile.y;
     const int J1 = min(J0 + TJ, n);  // columns j in [J0, J1), j <= n-1
     const int ncol = J1 - J0;
@@ -514,12 +518,24 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
         Bound<R> b;
         set_bound<R>(b, erow, FIRST ? 0 : (dg == 0 ? 0 : dg + 1));
         const bool masked = (wrow0 + 32 * R - 1) >= jstart;  // warp-uniform: some row >= some j
+#ifdef TSP2OPT_TILE_TIMING
+        const long long tt1 = clock64();
+#endif
         if (!(flags & kSweepTileBounds) || tile_may_pass<R>(rows, b, sm, jstart - J0, J1 - J0)) {
 #ifdef TSP2OPT_STATS
             if (lane == 0) atomicAdd(&g_stats[3], 1ULL);
 #endif
             if (masked) walk<R, true, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, my_rowp, mykey, warp);
             else walk<R, false, PS, FIRST>(rows, b, row0, jstart, J0, J1, sm, my_rowe, my_rowp, mykey, warp);
+#ifdef TSP2OPT_TILE_TIMING
+            const long long tt2 = clock64();
+            if (lane == 0) {
+                atomicAdd(&g_stats[0], (unsigned long long)(tt1 - tt0));
+                atomicAdd(&g_stats[1], (unsigned long long)(tt2 - tt1));
+                atomicAdd(&g_stats[2], 1ULL);
+                atomicMax(&g_stats[3], (unsigned long long)(tt2 - tt0));
+            }
+#endif
         }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
@@ -543,6 +559,47 @@ __device__ __forceinline__ void sweep_tile(const float2* P, const int* E, int n,
         for (int w = 1; w < (int)(blockDim.x >> 5); w++) m = s_red[w] < m ? s_red[w] : m;
         *tilebest = m;
     }
+}
+
+// One column part [jb, je) of a tile whose column chunk (from J0), row edges
+// and row cities (rows [I0, I0 + 32 R]) a whole CTA has staged in `sm`, swept by
+// ONE warp with the tile-local bound (kSweepLocal: delta < 0, the global key
+// ignored), so the tile's minimum is the min over its parts and stays exact on
+// its own.  The persistent incremental search splits each kept tile into parts
+// over several warps (a warp alone on its SMSP walks a column step in about 500
+// cycles of latency; the slowest whole-tile walk bounded the move).  The walk,
+// the filters and the exact path are sweep_tile's; each part's column
+// thresholds (slot 0 of the column records) are written only by the warp
+// walking it.  Returns the lane's key (kKeyNone if none).
+template <int R, bool FIRST>
+__device__ __forceinline__ unsigned long long sweep_part(int I0, int J0, int jb, int je, const TileSmem& sm,
+                                                         int flags)
+{
+    const int lane = threadIdx.x & 31;
+    const int row0 = I0 + lane * R;
+    const int jstart = max(jb, I0 + 1);  // no pair of the tile has j <= I0
+    unsigned long long mykey = kKeyNone;
+    if (jstart >= je) return mykey;  // warp-uniform
+    const float* my_rowe = sm.rowe + lane * R;
+    const float2* my_rowp = sm.rowp + lane * (R + 1);
+    Rows<R> rows;
+    float erow[R];
+#pragma unroll
+    for (int q = 0; q < (R + 1) / 2; q++) {
+        const float2 p0 = my_rowp[2 * q], p1 = my_rowp[2 * q + 1];
+        rows.xp[q] = make_float2(p0.x, p1.x);
+        rows.yp[q] = make_float2(p0.y, p1.y);
+    }
+#pragma unroll
+    for (int r = 0; r < R; r++) erow[r] = my_rowe[r];
+    Bound<R> b;
+    set_bound<R>(b, erow, 0);
+    const bool masked = (I0 + 32 * R - 1) >= jstart;  // some row >= some column
+    if (!(flags & kSweepPartBounds) || tile_may_pass<R>(rows, b, sm, jstart - J0, je - J0)) {
+        if (masked) walk<R, true, true, FIRST>(rows, b, row0, jstart, J0, je, sm, my_rowe, my_rowp, mykey, 0);
+        else walk<R, false, true, FIRST>(rows, b, row0, jstart, J0, je, sm, my_rowe, my_rowp, mykey, 0);
+    }
+    return mykey;
 }
 
 }  // namespace tsp2opt

@@ -1,5 +1,7 @@
 """Execution switches that must not change any result: CUDA-graph batches on
 and off, and the pruned sweep's threads per position (read per launch)."""
+import functools
+
 import numpy as np
 import pytest
 
@@ -65,3 +67,43 @@ def test_global_seed_switch(gpu, monkeypatch, kind, n, seed):
         trace = g.get_trace(10 * n)
     assert (res["iterations"], res["length"]) == (want["iterations"], want["length"])
     assert np.array_equal(np.asarray(trace, dtype=np.int64), want["trace"])
+
+
+@functools.lru_cache(maxsize=None)
+def _inc_case(first, start, cap):
+    c = inputs.make_coords("lattice", 1500, 5)  # 7 row blocks x 94 chunks: two groups of minima
+    t = inputs.make_tour(start, c, 3)
+    ls = oracle.first_local_search if first else oracle.local_search
+    return c, t, ls(c, t, max_iters=cap, trace_cap=20000)
+
+
+@pytest.mark.parametrize("barriers,part", [("2", "1"), ("2", "2"), ("2", "4"), ("2", "16"), ("3", "0"), ("3", "4")])
+@pytest.mark.parametrize("first", [0, 1])
+@pytest.mark.parametrize("start,cap", [("hilbert", -1), ("random", 400)])
+def test_incremental_persistent_variants(gpu, monkeypatch, barriers, part, first, start, cap):
+    """The persistent incremental search (TSP2OPT_OPT_TILE_BOUNDS = 3): two barriers per move with the
+    out-of-place apply and group minima, or three with the in-place apply; kept tiles split into column
+    parts of 1 / 2 / 4 / 16 columns or swept whole -- every move equal to the oracle's, with a move cap
+    that ends a search mid-way (the alternate buffer copied back) and (best improvement) a resumed search
+    after it.  (The first-improvement oracle from a random tour to the minimum takes minutes: capped only.)"""
+    monkeypatch.setenv("TSP2OPT_TILE_BOUNDS", "3")
+    monkeypatch.setenv("TSP2OPT_CULL_TJ", "16")
+    monkeypatch.setenv("TSP2OPT_INC_BARRIERS", barriers)
+    monkeypatch.setenv("TSP2OPT_INC_PART", part)
+    c, t, want = _inc_case(first, start, cap)
+    with tsp2opt.TSP2Opt(c) as g:
+        if first:
+            g.set_option(tsp2opt.OPT_FIRST_IMPROVEMENT, 1)
+        g.set_option(tsp2opt.OPT_TRACE, 20000)
+        res = g.local_search(t, max_iters=None if cap < 0 else cap)
+        got = np.asarray(g.get_trace(20000), dtype=np.int64)
+        assert (res["iterations"], res["length"]) == (want["iterations"], want["length"])
+        assert np.array_equal(res["tour"], want["tour"])
+        assert np.array_equal(got, want["trace"][: len(got)]) and len(got) == want["iterations"]
+        assert np.array_equal(g.get_tour()[0], want["tour"])
+        if cap > 0 and not first:  # resume to the local minimum from the capped state
+            full = _inc_case(first, start, -1)[2]
+            r2 = g.local_search_current()
+            assert res["iterations"] + r2["iterations"] == full["iterations"]
+            assert r2["length"] == full["length"]
+            assert np.array_equal(g.get_tour()[0], full["tour"])

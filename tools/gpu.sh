@@ -20,7 +20,7 @@ for task in "$@"; do
     smoke) timeout 600 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1
            echo "smoke rc=$? $(tail -1 gpurun_out/smoke.log)";;
     tests) k=(); [ -n "$arg" ] && k=(-k "$arg")
-           timeout 2400 python -m pytest tests -m gpu -q -x --durations=15 "${k[@]}" > gpurun_out/pytest_gpu.log 2>&1
+           timeout 2400 python -m pytest tests -m gpu -q -x --timeout 900 --durations=15 "${k[@]}" > gpurun_out/pytest_gpu.log 2>&1
            echo "tests rc=$? $(tail -1 gpurun_out/pytest_gpu.log)";;
     exp) for lib in ${arg//,/ }; do
            so=paper_conf_ipps_rockis13_b200/libtsp2opt.so; [ "$lib" != default ] && so=paper_conf_ipps_rockis13_b200/libtsp2opt_$lib.so

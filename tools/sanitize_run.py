@@ -21,7 +21,7 @@ import numpy as np  # noqa: E402
 import oracle  # noqa: E402
 from paper_conf_ipps_rockis13_b200 import inputs, tsp2opt  # noqa: E402
 
-MODES = ["persistent", "kernels", "culled", "incremental", "inc_fused", "dense_ls", "graph_off", "25opt",
+MODES = ["persistent", "kernels", "culled", "incremental", "inc3", "inc_fused", "dense_ls", "graph_off", "25opt",
          "25opt_culled", "first", "first_inc", "pruned", "mf", "ils", "batch", "batch_ils", "oropt", "oropt_filter",
          "shards", "p2p1"]
 
@@ -31,6 +31,8 @@ ENV = {
     "kernels": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "1"},
     "culled": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "2", "TSP2OPT_CULL_TJ": "16"},
     "incremental": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "3", "TSP2OPT_CULL_TJ": "16"},
+    "inc3": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "3", "TSP2OPT_CULL_TJ": "16",
+             "TSP2OPT_INC_BARRIERS": "3"},
     "inc_fused": {"TSP2OPT_PERSISTENT": "0", "TSP2OPT_TILE_BOUNDS": "3", "TSP2OPT_CULL_TJ": "16",
                   "TSP2OPT_INC_PERSISTENT": "0"},
     "dense_ls": {"TSP2OPT_PERSISTENT": "3", "TSP2OPT_TILE_BOUNDS": "1"},
@@ -52,7 +54,7 @@ def main(mode):
     n = 300
     c = inputs.lattice_coords(n, 3)
     t = inputs.random_tour(n, 3)
-    if mode in ("persistent", "kernels", "culled", "incremental", "inc_fused", "dense_ls", "graph_off"):
+    if mode in ("persistent", "kernels", "culled", "incremental", "inc3", "inc_fused", "dense_ls", "graph_off"):
         with tsp2opt.TSP2Opt(c) as g:
             r = g.local_search(t)
         o = oracle.local_search(c, t)
