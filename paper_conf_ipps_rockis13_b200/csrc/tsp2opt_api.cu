@@ -6,6 +6,7 @@
 // for sharded handles owns an NCCL communicator and performs one 8-byte
 // ncclAllReduce(MIN) of the packed best-move key per sweep.
 #include <algorithm>
+#include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -68,6 +69,12 @@ struct tsp2opt_ctx {
     int inc_part = -1;          // TSP2OPT_INC_PART: columns per part of a kept tile (-1: the default; 0 with the
                                 // three-barrier kernel: one warp per whole tile)
     int inc_part_bound = 0;     // TSP2OPT_INC_PART_BOUND=1: the tile bound on every part (measured 4 % slower)
+    // Automatic switch of the dense best-improvement loop (TILE_BOUNDS 1, n ~ 7e3) to the persistent
+    // incremental search once the tour is spatially coherent: length < kAutoIncRho * sqrt(n * A),
+    // A = the coordinates' bounding-box area (a random tour is ~0.5 sqrt(n) times that, a good one
+    // ~0.75-1).  Off when TILE_BOUNDS is set by option or environment (TSP2OPT_AUTO_INC=0: off).
+    bool auto_inc = false;
+    double rho_unit = 0.0;      // sqrt(n * A)
     Slot* d_slots = nullptr;    // [2]
     unsigned* d_stamp = nullptr;  // [n] permutation check
     unsigned* d_bar = nullptr;    // [2] grid barrier of the persistent local search (count, generation)
@@ -464,6 +471,7 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
 
 // CUDA graphs for the multi-kernel loop (TSP2OPT_GRAPH=0 disables them).
 constexpr long long kGraphBatch = 64;
+constexpr double kAutoIncRho = 2.0;  // coherent tour: length < 2 sqrt(n * A) (r02_exp_c3_switch.jsonl)
 bool graphs_enabled()
 {
     const char* e = getenv("TSP2OPT_GRAPH");
@@ -473,6 +481,75 @@ bool graphs_enabled()
 // Device-resident best-improvement loop on the loaded tour (a4-a8) until the
 // local minimum or max_iters moves; leaves the final state in h->h_slot.
 // Returns TSP2OPT_OK / TSP2OPT_MAXITER or a negative error.
+// Multi-kernel loop (per-iteration kernels, and sharded handles) until the local
+// minimum, the move cap or, if `leave` is given, the first batch boundary where
+// it returns true.  Leaves the final state in h->h_slot.
+template <typename Leave>
+static int run_multi_kernel_loop(tsp2opt_ctx* h, long long max_iters, const Leave* leave)
+{
+    int rc = 0;
+    // Multi-kernel loop (and sharded handles): batches of K iterations
+    // between host checks; an iteration after convergence is a no-op
+    // (sweep CTAs exit on the done flag).
+    // Full batches of kGraphBatch iterations are replayed from a CUDA graph
+    // captured once per search (one host call instead of ~4 launches per
+    // iteration); the graph starts and ends on the same slot parity.
+    long long k = 4;
+    cudaGraphExec_t gexec = nullptr;
+    int gparity = -1;
+    // Measured (profiles/r01_graph.jsonl): 2-6 % faster for the culled, pruned,
+    // first-improvement and 2.5-opt loops; 20 % slower for the dense best-improvement
+    // sweep (C3 from random), which keeps plain stream launches.
+    const bool dense_best = !h->or25 && h->nbr_k == 0 && !h->first && h->tile_bounds < 2;
+    // Sharded handles capture the ncclAllReduce into the same graph (NCCL supports
+    // stream capture of collectives): one graph launch per 64 iterations on every rank.
+    const bool use_graph = graphs_enabled() && !h->profiling && !dense_best;
+    auto drop_graph = [&]() {
+        if (gexec) cudaGraphExecDestroy(gexec);
+        gexec = nullptr;
+    };
+    for (;;) {
+        if (use_graph && k == kGraphBatch) {
+            if (!gexec || gparity != h->parity) {
+                drop_graph();
+                gparity = h->parity;
+                cudaGraph_t graph = nullptr;
+                CUDA_TRY(cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal));
+                for (long long c = 0; c < k && rc == 0; c++) rc = enqueue_iteration(h, max_iters, true);
+                const cudaError_t ec = cudaStreamEndCapture(h->stream, &graph);
+                if (rc) {
+                    if (graph) cudaGraphDestroy(graph);
+                    return rc;
+                }
+                if (ec != cudaSuccess) return cuda_fail(ec, "cudaStreamEndCapture");
+                const cudaError_t ei = cudaGraphInstantiate(&gexec, graph, 0);
+                cudaGraphDestroy(graph);
+                if (ei != cudaSuccess) return cuda_fail(ei, "cudaGraphInstantiate");
+            }
+            const cudaError_t el = cudaGraphLaunch(gexec, h->stream);
+            if (el != cudaSuccess) {
+                drop_graph();
+                return cuda_fail(el, "cudaGraphLaunch");
+            }
+        } else {
+            for (long long c = 0; c < k; c++) {
+                rc = enqueue_iteration(h, max_iters, true);
+                if (rc) return rc;
+            }
+        }
+        rc = read_slot(h);
+        if (rc) {
+            drop_graph();
+            return rc;
+        }
+        if (h->h_slot->done & 3) break;
+        if (leave && (*leave)()) break;  // the caller continues with another loop
+        if (k < kGraphBatch) k *= 2;
+    }
+    drop_graph();
+    return 0;
+}
+
 int run_local_search(tsp2opt_ctx* h, long long max_iters)
 {
     int rc;
@@ -488,13 +565,27 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
                               h->tile_bounds <= 1 && h->geo.warps == 1 && !h->profiling && h->shard_world == 1 &&
                               (h->persistent == 3 || (h->persistent == 2 && h->dense_ls));
     // The incremental culled search of a single GPU in one cooperative launch per
-    // ~1M iterations (launch_inc_ls): no per-iteration launches, three grid barriers
+    // ~1M iterations (launch_inc_ls2): no per-iteration launches, two grid barriers
     // per move.  Sharded handles keep the per-iteration kernels (the exchange sits
     // between sweep and apply).
-    const bool use_inc_ls = h->inc_persistent && !h->comm && !h->p2p && h->nbr_k == 0 && !h->or25 &&
-                            h->tile_bounds == 3 && h->cgeo.rows == kRowsSmall && h->cgeo.warps == 1 && !h->profiling &&
-                            h->shard_world == 1;
-    if (use_inc_ls) {
+    const bool inc_ok = h->inc_persistent && !h->comm && !h->p2p && h->nbr_k == 0 && !h->or25 &&
+                        h->cgeo.rows == kRowsSmall && h->cgeo.warps == 1 && !h->profiling && h->shard_world == 1;
+    bool use_inc_ls = inc_ok && h->tile_bounds == 3;
+    // Dense loop (TILE_BOUNDS 1 by default, n ~ 7e3) until the tour is coherent, then the
+    // incremental search (measured, C3: profiles/r02_exp_c3_switch.jsonl).
+    const bool auto_inc = inc_ok && h->auto_inc && h->tile_bounds == 1 && !use_persistent && !use_dense_ls;
+    auto coherent = [&]() { return (double)h->h_slot->length < kAutoIncRho * h->rho_unit; };
+    if (auto_inc) {
+        rc = read_slot(h);
+        if (rc) return rc;
+        if (coherent()) use_inc_ls = true;
+    }
+    if (!use_inc_ls && !use_dense_ls && !use_persistent) {
+        rc = run_multi_kernel_loop(h, max_iters, auto_inc ? &coherent : nullptr);
+        if (rc) return rc;
+        if (auto_inc && !(h->h_slot->done & 3)) use_inc_ls = true;  // left the loop: the tour became coherent
+    }
+    if (use_inc_ls && !(auto_inc && (h->h_slot->done & 3))) {
         const int flags = sweep_flags(h);
         // the two-barrier kernel keeps its minima in its own dense layout: tiling id 4
         const int inc_tiling = h->inc_barriers == 2 ? 4 : 1;
@@ -573,65 +664,6 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
             if (rc) return rc;
             if (h->h_slot->done & 3) break;
         }
-    } else {
-        // Multi-kernel loop (and sharded handles): batches of K iterations
-        // between host checks; an iteration after convergence is a no-op
-        // (sweep CTAs exit on the done flag).
-        // Full batches of kGraphBatch iterations are replayed from a CUDA graph
-        // captured once per search (one host call instead of ~4 launches per
-        // iteration); the graph starts and ends on the same slot parity.
-        long long k = 4;
-        cudaGraphExec_t gexec = nullptr;
-        int gparity = -1;
-        // Measured (profiles/r01_graph.jsonl): 2-6 % faster for the culled, pruned,
-        // first-improvement and 2.5-opt loops; 20 % slower for the dense best-improvement
-        // sweep (C3 from random), which keeps plain stream launches.
-        const bool dense_best = !h->or25 && h->nbr_k == 0 && !h->first && h->tile_bounds < 2;
-        // Sharded handles capture the ncclAllReduce into the same graph (NCCL supports
-        // stream capture of collectives): one graph launch per 64 iterations on every rank.
-        const bool use_graph = graphs_enabled() && !h->profiling && !dense_best;
-        auto drop_graph = [&]() {
-            if (gexec) cudaGraphExecDestroy(gexec);
-            gexec = nullptr;
-        };
-        for (;;) {
-            if (use_graph && k == kGraphBatch) {
-                if (!gexec || gparity != h->parity) {
-                    drop_graph();
-                    gparity = h->parity;
-                    cudaGraph_t graph = nullptr;
-                    CUDA_TRY(cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal));
-                    for (long long c = 0; c < k && rc == 0; c++) rc = enqueue_iteration(h, max_iters, true);
-                    const cudaError_t ec = cudaStreamEndCapture(h->stream, &graph);
-                    if (rc) {
-                        if (graph) cudaGraphDestroy(graph);
-                        return rc;
-                    }
-                    if (ec != cudaSuccess) return cuda_fail(ec, "cudaStreamEndCapture");
-                    const cudaError_t ei = cudaGraphInstantiate(&gexec, graph, 0);
-                    cudaGraphDestroy(graph);
-                    if (ei != cudaSuccess) return cuda_fail(ei, "cudaGraphInstantiate");
-                }
-                const cudaError_t el = cudaGraphLaunch(gexec, h->stream);
-                if (el != cudaSuccess) {
-                    drop_graph();
-                    return cuda_fail(el, "cudaGraphLaunch");
-                }
-            } else {
-                for (long long c = 0; c < k; c++) {
-                    rc = enqueue_iteration(h, max_iters, true);
-                    if (rc) return rc;
-                }
-            }
-            rc = read_slot(h);
-            if (rc) {
-                drop_graph();
-                return rc;
-            }
-            if (h->h_slot->done & 3) break;
-            if (k < kGraphBatch) k *= 2;
-        }
-        drop_graph();
     }
     return (h->h_slot->done & 3) == 2 ? TSP2OPT_MAXITER : TSP2OPT_OK;
 }
@@ -704,7 +736,23 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     // the tiles on EVERY rank, and a rank's shard of a large instance is still a spread-out
     // subset of its tiles, so C4 at 8 ranks keeps the incremental culled sweep.
     h->tile_bounds = total_pairs >= 100000000LL ? 3 : 1;
-    if (const char* eb = getenv("TSP2OPT_TILE_BOUNDS")) h->tile_bounds = std::min(3, std::max(0, atoi(eb)));
+    // from ~4e6 pairs (where the per-iteration loop takes over from the persistent dense kernel)
+    h->auto_inc = h->tile_bounds == 1 && total_pairs > 4000000LL;
+    if (const char* eb = getenv("TSP2OPT_TILE_BOUNDS")) {
+        h->tile_bounds = std::min(3, std::max(0, atoi(eb)));
+        h->auto_inc = false;
+    }
+    if (const char* ea = getenv("TSP2OPT_AUTO_INC")) h->auto_inc = h->auto_inc && atoi(ea) != 0;
+    {
+        int xlo = xy[0], xhi = xy[0], ylo = xy[1], yhi = xy[1];
+        for (int k = 1; k < n; k++) {
+            xlo = std::min(xlo, xy[2 * k]);
+            xhi = std::max(xhi, xy[2 * k]);
+            ylo = std::min(ylo, xy[2 * k + 1]);
+            yhi = std::max(yhi, xy[2 * k + 1]);
+        }
+        h->rho_unit = std::sqrt((double)n * std::max(1.0, (double)(xhi - xlo) * (double)(yhi - ylo)));
+    }
     h->all_tiles = build_tiles(n, h->geo);
     // Culled-sweep tiling: R = 7 rows per lane and narrow column chunks (measured,
     // local search from MF).
@@ -1130,6 +1178,7 @@ int tsp2opt_set_option(tsp2opt_t h, int32_t option, int64_t value)
     case TSP2OPT_OPT_TILE_BOUNDS:
         if (value < 0 || value > 3) return TSP2OPT_EINVAL;
         h->tile_bounds = (int)value;
+        h->auto_inc = false;
         break;
     case TSP2OPT_OPT_SEED: h->seed_next = value != 0; break;
     case TSP2OPT_OPT_TRACE: {

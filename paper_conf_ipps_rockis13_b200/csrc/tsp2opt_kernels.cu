@@ -112,7 +112,12 @@ template <int R, bool FIRST>
 #define TSP2OPT_SWEEP_LB_T 128  // experiment: (32, 20) forces 102 registers for 20 one-warp CTAs per SM
 #define TSP2OPT_SWEEP_LB_B TSP2OPT_MINB
 #endif
-__global__ void __launch_bounds__(TSP2OPT_SWEEP_LB_T, TSP2OPT_SWEEP_LB_B) sweep_kernel(const float2* __restrict__ P, const int* __restrict__ E, int n,
+#ifdef TSP2OPT_SWEEP_MAXNREG  // experiment: a register cap between the launch-bounds steps
+#define TSP2OPT_SWEEP_ATTR __maxnreg__(TSP2OPT_SWEEP_MAXNREG)
+#else
+#define TSP2OPT_SWEEP_ATTR __launch_bounds__(TSP2OPT_SWEEP_LB_T, TSP2OPT_SWEEP_LB_B)
+#endif
+__global__ void TSP2OPT_SWEEP_ATTR sweep_kernel(const float2* __restrict__ P, const int* __restrict__ E, int n,
                                                      const int2* __restrict__ tiles, int TJ, Slot* __restrict__ slot,
                                                      int respect_done, unsigned long long* __restrict__ tilebest,
                                                      int flags)
