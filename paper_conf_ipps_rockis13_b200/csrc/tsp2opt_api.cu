@@ -107,7 +107,8 @@ struct tsp2opt_ctx {
     int list25_grid = 0;        // CTAs of the 2.5-opt culled sweep
     int last_tiling = -1;       // tiling of the previous sweep (0 dense, 1 cull): seeds are per tiling
     bool inc_valid = false;     // the stored per-tile minima are those of an incremental sweep of the current tiling
-    bool global_seed = false;   // TSP2OPT_GLOBAL_SEED=1: dense sweeps start from the best surviving tile minimum
+    int global_seed = 0;        // TSP2OPT_GLOBAL_SEED=1: dense sweeps start from the best surviving tile minimum
+                                // (2: from every tile minimum's positions re-evaluated on the new tour)
                                 // (measured: C4 random 8 % faster, C2 / C3 2-10 % slower; profiles/r01_global_seed.jsonl)
     unsigned long long* d_trace = nullptr;  // [trace_cap] keys of the applied moves (TSP2OPT_OPT_TRACE)
     int* d_best = nullptr;      // [n] best tour of an ILS run
@@ -463,7 +464,8 @@ int enqueue_iteration(tsp2opt_ctx* h, long long max_moves, bool apply)
                               h->trace_cap, h->nbr_k > 0 ? h->d_pos : nullptr, h->stream));
         // dense best-improvement sweep: start the next one from the best surviving tile minimum
         if (tiling == 0 && !h->first && h->global_seed)
-            CUDA_TRY(launch_global_seed(h->d_tilebest, h->ntiles, out, h->stream));
+            CUDA_TRY(launch_global_seed(h->d_tilebest, h->ntiles, out, h->global_seed == 2 ? h->d_P : nullptr,
+                                        h->global_seed == 2 ? h->d_E : nullptr, h->stream));
         h->parity ^= 1;
     }
     return TSP2OPT_OK;
@@ -710,7 +712,7 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     CTRY(cudaHostAlloc(&h->h_ctl, sizeof(int), cudaHostAllocDefault));
     if (const char* ep = getenv("TSP2OPT_PERSISTENT")) h->persistent = atoi(ep);
     if (const char* es = getenv("TSP2OPT_SEED")) h->seed_next = atoi(es) != 0;
-    if (const char* eg = getenv("TSP2OPT_GLOBAL_SEED")) h->global_seed = atoi(eg) != 0;
+    if (const char* eg = getenv("TSP2OPT_GLOBAL_SEED")) h->global_seed = std::min(2, std::max(0, atoi(eg)));
     if (const char* ef = getenv("TSP2OPT_INC_FUSED")) h->inc_fused = atoi(ef) != 0;
     if (const char* ei = getenv("TSP2OPT_INC_PERSISTENT")) h->inc_persistent = atoi(ei) != 0;
     if (const char* eb = getenv("TSP2OPT_INC_BARRIERS")) h->inc_barriers = atoi(eb) == 3 ? 3 : 2;

@@ -107,7 +107,9 @@ cudaError_t sweep_prepare();
 cudaError_t launch_load_tour(const int* coords, const int* tour_src, int* tour_dst, float2* P, int* E, int n,
                              Slot* slot, unsigned* stamp, unsigned epoch, cudaStream_t st);
 cudaError_t launch_reset_key(Slot* slot, cudaStream_t st);
-cudaError_t launch_global_seed(const unsigned long long* tilebest, int ntiles, Slot* slot, cudaStream_t st);
+// P / E non-null: re-evaluate every tile minimum's positions on the new tour (else: surviving pairs only)
+cudaError_t launch_global_seed(const unsigned long long* tilebest, int ntiles, Slot* slot, const float2* P,
+                               const int* E, cudaStream_t st);
 cudaError_t launch_first_fix(const float2* P, const int* E, Slot* slot, int respect_done, cudaStream_t st);
 cudaError_t launch_double_bridge(const int* in, int* out, int n, int a, int b, int c, cudaStream_t st);
 cudaError_t launch_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,

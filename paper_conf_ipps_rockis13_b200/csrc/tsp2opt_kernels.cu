@@ -1656,8 +1656,12 @@ cudaError_t launch_first_fix(const float2* P, const int* E, Slot* slot, int resp
 // Their min starts the next sweep's bound for every tile at once, instead of
 // the seed (0, 1, 0) that only tightens as tiles finish.  The sweep still
 // examines every pair: any pair with a lower (delta, cell) replaces it.
+// reeval (P, E given): every tile minimum's POSITIONS (a, b) are re-evaluated
+// on the new tour instead -- (a, b) is a pair of the new tour whatever the
+// move did to it, and its exact delta there (the oracle's nint arithmetic) is
+// as valid a bound, from every tile instead of the surviving ones.
 __global__ void __launch_bounds__(256) global_seed_kernel(const unsigned long long* __restrict__ tilebest, int ntiles,
-                                                          Slot* __restrict__ slot)
+                                                          Slot* __restrict__ slot, const float2* P, const int* E)
 {
     pdl_trigger();
     pdl_wait();
@@ -1667,8 +1671,16 @@ __global__ void __launch_bounds__(256) global_seed_kernel(const unsigned long lo
     if (!ok || done) return;
     const int i = key_i(mv), j = key_j(mv);
     unsigned long long m = kKeyNone;
-    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < ntiles; t += gridDim.x * blockDim.x)
-        m = min(m, surviving_key(tilebest[t], i, j));
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < ntiles; t += gridDim.x * blockDim.x) {
+        const unsigned long long k = tilebest[t];
+        if (!P) {
+            m = min(m, surviving_key(k, i, j));
+        } else if (k != kKeyNone) {
+            const int a = key_i(k), b = key_j(k);
+            const int d = exact_dist_biased(P[a], P[b]) + exact_dist_biased(P[a + 1], P[b + 1]) - E[a] - E[b];
+            if (d < 0) m = min(m, pack_key(d, a, b));
+        }
+    }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
     __shared__ unsigned long long s_m[8];
@@ -1680,11 +1692,12 @@ __global__ void __launch_bounds__(256) global_seed_kernel(const unsigned long lo
     }
 }
 
-cudaError_t launch_global_seed(const unsigned long long* tilebest, int ntiles, Slot* slot, cudaStream_t st)
+cudaError_t launch_global_seed(const unsigned long long* tilebest, int ntiles, Slot* slot, const float2* P,
+                               const int* E, cudaStream_t st)
 {
     if (ntiles <= 0) return cudaSuccess;
     const int grid = std::max(1, std::min(148, (ntiles + 255) / 256));
-    cudaError_t e = launch_pdl(global_seed_kernel, dim3(grid), dim3(256), 0, st, tilebest, ntiles, slot);
+    cudaError_t e = launch_pdl(global_seed_kernel, dim3(grid), dim3(256), 0, st, tilebest, ntiles, slot, P, E);
     g_launches += 1;
     return e != cudaSuccess ? e : cudaGetLastError();
 }
