@@ -65,6 +65,10 @@ struct tsp2opt_ctx {
     int* d_E_alt = nullptr;
     int* d_tour_alt = nullptr;
     void* d_inc2_ws = nullptr; // its barrier counter, dense tile minima and group minima (inc_ls2_ws_bytes)
+    Geometry igeo{};            // its culled tiling (own tile map and boxes)
+    int* d_itmap = nullptr;
+    Box* d_irbox = nullptr;
+    Box* d_icbox = nullptr;
     int inc_barriers = 2;       // TSP2OPT_INC_BARRIERS=3: the three-barrier persistent kernel (in-place apply)
     int inc_part = -1;          // TSP2OPT_INC_PART: columns per part of a kept tile (-1: the default; 0 with the
                                 // three-barrier kernel: one warp per whole tile)
@@ -251,10 +255,6 @@ int upload_shard(tsp2opt_ctx* h, int rank, int world)
         std::vector<Tile> mine = shard_tiles(h->all_ctiles, rank, world, &unused);
         for (size_t k = 0; k < mine.size(); k++) map[(size_t)(mine[k].i0 / TI) * ncc + mine[k].j0 / TJ] = (int)k;
         cudaFree(h->d_tmap);
-    for (void* p : h->p2p_opened)
-        if (p) cudaIpcCloseMemHandle(p);
-    cudaFree(h->d_peers);
-    cudaFree(h->d_mbox);
         h->d_tmap = nullptr;
         CUDA_TRY(cudaMalloc(&h->d_tmap, sizeof(int) * map.size()));
         CUDA_TRY(cudaMemcpy(h->d_tmap, map.data(), sizeof(int) * map.size(), cudaMemcpyHostToDevice));
@@ -285,6 +285,9 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_E_alt);
     cudaFree(h->d_tour_alt);
     cudaFree(h->d_inc2_ws);
+    cudaFree(h->d_itmap);
+    cudaFree(h->d_irbox);
+    cudaFree(h->d_icbox);
     cudaFree(h->d_slots);
     cudaFree(h->d_stamp);
     cudaFree(h->d_bar);
@@ -483,6 +486,39 @@ bool graphs_enabled()
 // Device-resident best-improvement loop on the loaded tour (a4-a8) until the
 // local minimum or max_iters moves; leaves the final state in h->h_slot.
 // Returns TSP2OPT_OK / TSP2OPT_MAXITER or a negative error.
+// Workspace of the two-barrier persistent search (inc_ls2_kernel): alternate P / E / tour, its
+// own tile map (which (row block, chunk) tiles of igeo exist; one GPU) and boxes, the barrier
+// counter and the dense / group minima.  Allocated at creation for sizes that use it, so that no
+// timed search pays for it.
+static int alloc_inc2(tsp2opt_ctx* h)
+{
+    const size_t np = (size_t)h->n + 1 + kPad;
+    const size_t wsb = inc_ls2_ws_bytes(h->igeo, h->n);
+    const int TI = h->igeo.ti(), TJ = h->igeo.tj;
+    const int nrb = (h->n - 1 + TI - 1) / TI, ncc = (h->n + TJ - 1) / TJ;
+    std::vector<int> map((size_t)nrb * ncc, -1);
+    {
+        const int n = h->n;
+        for (int I0 = 0, rb = 0; I0 <= n - 2; I0 += TI, rb++) {  // the tiles build_tiles keeps (pairs > 0)
+            const int rows = std::min(I0 + TI, n - 1) - I0;
+            for (int J0 = ((I0 + 1) / TJ) * TJ; J0 < n; J0 += TJ) {
+                const int J1 = std::min(J0 + TJ, n);
+                if (J1 - 1 > I0 && rows > 0) map[(size_t)rb * ncc + J0 / TJ] = 1;
+            }
+        }
+    }
+    CUDA_TRY(cudaMalloc(&h->d_P_alt, sizeof(float2) * np));
+    CUDA_TRY(cudaMalloc(&h->d_E_alt, sizeof(int) * np));
+    CUDA_TRY(cudaMalloc(&h->d_tour_alt, sizeof(int) * np));
+    CUDA_TRY(cudaMalloc(&h->d_inc2_ws, wsb));
+    CUDA_TRY(cudaMalloc(&h->d_itmap, sizeof(int) * map.size()));
+    CUDA_TRY(cudaMalloc(&h->d_irbox, sizeof(Box) * (size_t)nrb));
+    CUDA_TRY(cudaMalloc(&h->d_icbox, sizeof(Box) * (size_t)ncc));
+    CUDA_TRY(cudaMemcpy(h->d_itmap, map.data(), sizeof(int) * map.size(), cudaMemcpyHostToDevice));
+    CUDA_TRY(cudaMemset(h->d_inc2_ws, 0xFF, wsb));  // minima: none
+    return TSP2OPT_OK;
+}
+
 // Multi-kernel loop (per-iteration kernels, and sharded handles) until the local
 // minimum, the move cap or, if `leave` is given, the first batch boundary where
 // it returns true.  Leaves the final state in h->h_slot.
@@ -600,15 +636,11 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
             if (h->inc_barriers == 2) {
                 const size_t np = (size_t)h->n + 1 + kPad;
                 if (!h->d_P_alt) {
-                    const size_t wsb = inc_ls2_ws_bytes(h->cgeo, h->n);
-                    CUDA_TRY(cudaMalloc(&h->d_P_alt, sizeof(float2) * np));
-                    CUDA_TRY(cudaMalloc(&h->d_E_alt, sizeof(int) * np));
-                    CUDA_TRY(cudaMalloc(&h->d_tour_alt, sizeof(int) * np));
-                    CUDA_TRY(cudaMalloc(&h->d_inc2_ws, wsb));
-                    CUDA_TRY(cudaMemsetAsync(h->d_inc2_ws, 0xFF, wsb, h->stream));  // minima: none
+                    rc = alloc_inc2(h);
+                    if (rc) return rc;
                 }
-                CUDA_TRY(launch_inc_ls2(h->cgeo, h->d_P, h->d_E, h->d_tour, h->d_P_alt, h->d_E_alt, h->d_tour_alt,
-                                        h->n, (int)np, h->d_tmap, h->d_rbox, h->d_cbox, h->d_inc2_ws, h->d_slots,
+                CUDA_TRY(launch_inc_ls2(h->igeo, h->d_P, h->d_E, h->d_tour, h->d_P_alt, h->d_E_alt, h->d_tour_alt,
+                                        h->n, (int)np, h->d_itmap, h->d_irbox, h->d_icbox, h->d_inc2_ws, h->d_slots,
                                         h->parity, max_iters, 1LL << 20, full, h->d_ctl, flags, h->d_trace,
                                         h->trace_cap, h->inc_part, h->inc_part_bound, h->stream));
             } else {
@@ -764,9 +796,17 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     // set by the slowest tile's walk): narrower chunks again -- C5 16 columns 21.9 vs 32 23.8 us
     // per move, C4 8 columns 17.7 vs 16 18.9 (profiles/r02_exp_cull_tj.jsonl).
     h->cgeo = Geometry{kRowsSmall, 1, total_pairs >= 1000000000LL ? 16 : 8};
+    // The two-barrier persistent search has its own culled tiling: with kept tiles split into
+    // 4-column parts over a CTA's warps and group minima, wider chunks pay again -- 32 columns from
+    // 1e8 pairs: C5 Hilbert 14.6 vs 15.0 (16) / 15.5 (64) us per move, C5 MF 18.5 vs 19.8, C4 MF 15.2
+    // vs 16.9 (8); C3 keeps 8 (profiles/r02_exp_inc_parts.jsonl, r02_exp_c3_inc.jsonl).  The 2.5-opt
+    // and per-iteration culled sweeps keep cgeo (32 columns cost 2.5-opt at C4 35 %).
+    h->igeo = Geometry{kRowsSmall, 1, total_pairs >= 100000000LL ? 32 : 8};
     if (const char* er = getenv("TSP2OPT_CULL_ROWS")) h->cgeo.rows = atoi(er) == kRowsSmall ? kRowsSmall : kRowsLarge;
     if (const char* ec = getenv("TSP2OPT_CULL_TJ"))
-        if (atoi(ec) >= 2 && atoi(ec) <= kMaxTJ) h->cgeo.tj = atoi(ec);
+        if (atoi(ec) >= 2 && atoi(ec) <= kMaxTJ) h->cgeo.tj = h->igeo.tj = atoi(ec);
+    if (const char* ei2 = getenv("TSP2OPT_INC_TJ"))
+        if (atoi(ei2) >= 2 && atoi(ei2) <= kMaxTJ) h->igeo.tj = atoi(ei2);
     h->all_ctiles = build_tiles(n, h->cgeo);
     {
         const int nrb = (n - 1 + h->cgeo.ti() - 1) / h->cgeo.ti(), ncc = (n + h->cgeo.tj - 1) / h->cgeo.tj;
@@ -775,6 +815,10 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     }
     rc = upload_shard(h, rank, world);
     if (rc) return fail(rc);
+    if (world == 1 && !nccl_id && !p2p && total_pairs > 4000000LL) {  // sizes that run the persistent search
+        rc = alloc_inc2(h);
+        if (rc) return fail(rc);
+    }
     if (p2p) {  // peer-memory exchange: the mailbox now, the peers at tsp2opt_p2p_connect
         h->p2p = true;
         CTRY(cudaMalloc(&h->d_mbox, sizeof(Mailbox)));
