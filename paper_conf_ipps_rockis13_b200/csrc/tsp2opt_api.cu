@@ -69,7 +69,9 @@ struct tsp2opt_ctx {
     int* d_itmap = nullptr;
     Box* d_irbox = nullptr;
     Box* d_icbox = nullptr;
-    int inc_barriers = 2;       // TSP2OPT_INC_BARRIERS=3: the three-barrier persistent kernel (in-place apply)
+    int inc_barriers = 1;       // TSP2OPT_INC_BARRIERS=2: two grid barriers per move (inc_ls2_kernel); 3: the
+                                // three-barrier kernel (in-place apply)
+    void* d_inc1_ws = nullptr;  // inc_ls1_kernel workspace (inc_ls1_ws_bytes), allocated with the inc2 one
     int inc_part = -1;          // TSP2OPT_INC_PART: columns per part of a kept tile (-1: the default; 0 with the
                                 // three-barrier kernel: one warp per whole tile)
     int inc_part_bound = 0;     // TSP2OPT_INC_PART_BOUND=1: the tile bound on every part (measured 4 % slower)
@@ -285,6 +287,7 @@ void free_ctx(tsp2opt_ctx* h)
     cudaFree(h->d_E_alt);
     cudaFree(h->d_tour_alt);
     cudaFree(h->d_inc2_ws);
+    cudaFree(h->d_inc1_ws);
     cudaFree(h->d_itmap);
     cudaFree(h->d_irbox);
     cudaFree(h->d_icbox);
@@ -516,6 +519,9 @@ static int alloc_inc2(tsp2opt_ctx* h)
     CUDA_TRY(cudaMalloc(&h->d_icbox, sizeof(Box) * (size_t)ncc));
     CUDA_TRY(cudaMemcpy(h->d_itmap, map.data(), sizeof(int) * map.size(), cudaMemcpyHostToDevice));
     CUDA_TRY(cudaMemset(h->d_inc2_ws, 0xFF, wsb));  // minima: none
+    CUDA_TRY(cudaMalloc(&h->d_inc1_ws, inc_ls1_ws_bytes(h->igeo, h->n)));
+    CUDA_TRY(cudaMemset(h->d_inc1_ws, 0xFF, inc_ls1_ws_bytes(h->igeo, h->n)));  // tile minima of tiles that
+                                                                                    // do not exist: none
     return TSP2OPT_OK;
 }
 
@@ -626,14 +632,24 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
     if (use_inc_ls && !(auto_inc && (h->h_slot->done & 3))) {
         const int flags = sweep_flags(h);
         // the two-barrier kernel keeps its minima in its own dense layout: tiling id 4
-        const int inc_tiling = h->inc_barriers == 2 ? 4 : 1;
+        const int inc_tiling = h->inc_barriers == 1 ? 5 : h->inc_barriers == 2 ? 4 : 1;
         int full = (h->inc_valid && h->last_tiling == inc_tiling) ? 0 : 1;
         for (long long launches = 0;; launches++) {
             if (launches > 1000000) {
                 g_last_error = "local search did not converge";
                 return TSP2OPT_ECUDA;
             }
-            if (h->inc_barriers == 2) {
+            if (h->inc_barriers == 1) {
+                const size_t np = (size_t)h->n + 1 + kPad;
+                if (!h->d_P_alt) {
+                    rc = alloc_inc2(h);
+                    if (rc) return rc;
+                }
+                CUDA_TRY(launch_inc_ls1(h->igeo, h->d_P, h->d_E, h->d_tour, h->d_P_alt, h->d_E_alt, h->d_tour_alt,
+                                        h->n, (int)np, h->d_itmap, h->d_inc1_ws, h->d_slots, h->parity, max_iters,
+                                        1LL << 20, h->d_ctl, flags, h->d_trace, h->trace_cap, h->inc_part,
+                                        h->stream));
+            } else if (h->inc_barriers == 2) {
                 const size_t np = (size_t)h->n + 1 + kPad;
                 if (!h->d_P_alt) {
                     rc = alloc_inc2(h);
@@ -747,7 +763,7 @@ int create_common(const int32_t* xy, int32_t n, int rank, int world, const void*
     if (const char* eg = getenv("TSP2OPT_GLOBAL_SEED")) h->global_seed = std::min(2, std::max(0, atoi(eg)));
     if (const char* ef = getenv("TSP2OPT_INC_FUSED")) h->inc_fused = atoi(ef) != 0;
     if (const char* ei = getenv("TSP2OPT_INC_PERSISTENT")) h->inc_persistent = atoi(ei) != 0;
-    if (const char* eb = getenv("TSP2OPT_INC_BARRIERS")) h->inc_barriers = atoi(eb) == 3 ? 3 : 2;
+    if (const char* eb = getenv("TSP2OPT_INC_BARRIERS")) h->inc_barriers = std::min(3, std::max(1, atoi(eb)));
     if (const char* ep2 = getenv("TSP2OPT_INC_PART")) h->inc_part = atoi(ep2);
     if (const char* eq = getenv("TSP2OPT_INC_PART_BOUND")) h->inc_part_bound = atoi(eq) != 0;
     if (const char* ed = getenv("TSP2OPT_DENSE_LS")) h->dense_ls = atoi(ed) != 0;

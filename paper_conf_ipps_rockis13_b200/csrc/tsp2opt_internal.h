@@ -152,6 +152,16 @@ cudaError_t launch_inc_ls2(const Geometry& g, float2* P, int* E, int* tour, floa
                            long long max_moves, long long budget, int full, int* ctl, int flags,
                            unsigned long long* trace, long long trace_cap, int part_cols, int part_bound,
                            cudaStream_t st);
+// One grid barrier per move (inc_ls1_kernel): the dirty tiles of move m are swept in the same phase as
+// its out-of-place apply, reading the pre-move buffers through the mirror map, with conservative boxes
+// for the cull.  ws: inc_ls1_ws_bytes (barrier counter, keys, dense tile and group minima, two box
+// buffers; all-ones once, so that the minima of tiles that do not exist read as none).  Every launch starts with a full sweep; the slot comes back with
+// seed_ok = 0.
+size_t inc_ls1_ws_bytes(const Geometry& g, int n);
+cudaError_t launch_inc_ls1(const Geometry& g, float2* P, int* E, int* tour, float2* P1, int* E1, int* T1, int n,
+                           int np, const int* tmap, void* ws, Slot* slots, int parity, long long max_moves,
+                           long long budget, int* ctl, int flags, unsigned long long* trace, long long trace_cap,
+                           int part_cols, cudaStream_t st);
 cudaError_t launch_inc_sweep(const Geometry& g, const float2* P, const int* E, int n, const int2* tiles, int ntiles,
                              const int* tmap, int grid, Box* rbox, Box* cbox, Slot* slot, int respect_done,
                              unsigned long long* tilebest, int flags, cudaStream_t st);

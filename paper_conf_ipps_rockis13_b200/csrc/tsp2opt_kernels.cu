@@ -1455,6 +1455,440 @@ __global__ void __launch_bounds__(512, 1) inc_ls2_kernel(float2* P0, int* E0, in
 }
 
 // ===========================================================================
+// Persistent incremental local search, ONE grid barrier per move
+// (inc_ls1_kernel).  Phase m decides move m from the key the previous phase
+// completed, then, all reading only the pre-move state S_{m-1}:
+//   * item warps (12 per CTA) cull the tiles move m dirties, stage the kept
+//     ones through the reversal's mirror map (new P[k] = P[i+j+1-k] on
+//     [i+1, j], new e[k] = e[i+j-k] on (i, j), the two new edges) and sweep
+//     them in column parts: the minima of S_m, written to the dense tile
+//     minima and the next key.  The cull uses CONSERVATIVE boxes for the
+//     dirty blocks: the union of the stored boxes of the block and of the
+//     blocks its new cities and edges come from, and the largest of their
+//     edges and the two new ones -- a superset of what S_m's exact boxes keep,
+//     so every tile that can hold an improving pair is swept;
+//   * side warps (4 per CTA) write S_m into the other P / E / tour buffer (the
+//     positions of moves m-1 and m), compute S_m's exact boxes of the dirty
+//     blocks into the other box buffer (copying the blocks move m-1 dirtied),
+//     and fold the clean tiles' minima into the next key through the group
+//     minima (a group touched by move m is marked invalid; an invalid group
+//     that move m leaves clean is recomputed from its tiles first).
+// The key is triple-buffered (read, written, reset in the same phase), so one
+// barrier per move orders everything; the result is the same move sequence as
+// the two- and three-barrier kernels.  A launch starts with a full sweep of its
+// state and leaves seed_ok = 0 (the next launch starts full).
+// ===========================================================================
+constexpr int kSideWarps = 4;                 // inc_ls1: per CTA, the rest sweep
+constexpr unsigned long long kGroupInvalid = 0;  // not a key (delta + 2^18 > 0): "recompute this group"
+
+// Conservative box of block `b` (positions [b*B, min(b*B + B, last)], edges up
+// to the block end - 1) of the state after move (i, j), from the stored boxes
+// of the state before it: the union with the blocks whose positions the
+// reversal maps into this block, and the two new edges.
+__device__ __forceinline__ Box cons_box(const Box* boxes, int b, int B, int nb, int last, int i, int j, int di,
+                                        int dj)
+{
+    if (i < 0) return boxes[b];
+    const int a0 = b * B, a1 = min(a0 + B, last);
+    Box r;
+    if (a0 >= i + 1 && a1 <= j) {  // every city and edge of the block is replaced: the sources only
+        r.xlo = r.ylo = 1 << 30;
+        r.xhi = r.yhi = -1;
+        r.emax = 0;
+    } else {
+        r = boxes[b];
+    }
+    const int lo = max(a0, i + 1), hi = min(a1, j);
+    if (lo <= hi) {  // positions [lo, hi] receive cities from [i+j+1-hi, i+j+1-lo], edges from one lower
+        const int s0 = max(0, (i + j - hi) / B), s1 = min(nb - 1, (i + j + 1 - lo) / B);
+        for (int s = s0; s <= s1; s++) {
+            const Box q = boxes[s];
+            r.xlo = min(r.xlo, q.xlo);
+            r.xhi = max(r.xhi, q.xhi);
+            r.ylo = min(r.ylo, q.ylo);
+            r.yhi = max(r.yhi, q.yhi);
+            r.emax = max(r.emax, q.emax);
+        }
+    }
+    if (i >= a0 && i < a1) r.emax = max(r.emax, di);
+    if (j >= a0 && j < a1) r.emax = max(r.emax, dj);
+    return r;
+}
+
+template <int NT>
+__device__ __forceinline__ void bar_items()
+{
+    asm volatile("bar.sync 1, %0;" ::"n"(NT) : "memory");
+}
+
+// The item warps' share of phase m: cull / stage / sweep the tiles move (i, j)
+// dirties (i < 0: every tile, plain reads), into tb2 and *key.
+template <int R, bool FIRST, int NT>
+__device__ __forceinline__ void inc1_items(const float2* P, const int* E, int n, const int* __restrict__ tmap, int TI,
+                                           int TJ, int nrb, int ncc, int i, int j, int di, int dj, const Box* rbox,
+                                           const Box* cbox, unsigned long long* key, unsigned long long* tb2,
+                                           int tflags, int part_cols, float4* smem, int tile_bytes)
+{
+    __shared__ int s_nk;
+    __shared__ int4 s_kt[NT];
+    __shared__ unsigned long long s_tmin[kStageTiles];
+    const int tid = threadIdx.x, wib = tid >> 5, nwi = NT / 32;
+    const int dlo = i < 0 ? 0 : i, dhi = i < 0 ? n : j;
+    const int rlo = dlo >= 1 ? (dlo - 1) / TI : 0, rhi = min(nrb - 1, dhi / TI);
+    const int clo = dlo >= 1 ? (dlo - 1) / TJ : 0, chi = min(ncc - 1, dhi / TJ);
+    const long long nA = (long long)(rhi - rlo + 1) * ncc, nB = (long long)nrb * (chi - clo + 1);
+    const int nparts = (TJ + part_cols - 1) / part_cols;
+    const long long step = (long long)NT * gridDim.x;
+    for (long long base = 0; base < nA + nB; base += step) {
+        if (tid == 0) s_nk = 0;
+        bar_items<NT>();
+        const long long u = base + (long long)tid * gridDim.x + blockIdx.x;
+        if (u < nA + nB) {
+            int rb, cc;
+            bool cand = true;
+            if (u < nA) {
+                rb = rlo + (int)(u / ncc);
+                cc = (int)(u % ncc);
+            } else {
+                const long long v = u - nA;
+                rb = (int)(v / (chi - clo + 1));
+                cc = clo + (int)(v % (chi - clo + 1));
+                cand = rb < rlo || rb > rhi;
+            }
+            if (cand) {
+                const int t = tmap[(long long)rb * ncc + cc];
+                const Box r = (rb >= rlo && rb <= rhi) ? cons_box(rbox, rb, TI, nrb, n - 1, i, j, di, dj) : rbox[rb];
+                const Box c = (cc >= clo && cc <= chi) ? cons_box(cbox, cc, TJ, ncc, n, i, j, di, dj) : cbox[cc];
+                if (t >= 0) {
+                    const long long gx = max(0, max(c.xlo - r.xhi, r.xlo - c.xhi));
+                    const long long gy = max(0, max(c.ylo - r.yhi, r.ylo - c.yhi));
+                    const long long T = (long long)max(r.emax, c.emax) - 1;
+                    if (T >= 0 && gx * gx + gy * gy <= T * T + T) s_kt[atomicAdd(&s_nk, 1)] = make_int4(t, rb, cc, 0);
+                    else tb2[(long long)rb * ncc + cc] = kKeyNone;
+                }
+            }
+        }
+        bar_items<NT>();
+        const int nk = s_nk;
+        for (int b0 = 0; b0 < nk; b0 += kStageTiles) {
+            const int nb = min(kStageTiles, nk - b0);
+            const int ncolp = TJ + 2, nrowp = 32 * R + 1, per = ncolp + nrowp;
+            constexpr int U = 8;
+            for (int x0 = 0; x0 < nb * per; x0 += U * NT) {
+                float2 pv[U];
+                int ev[U];
+#pragma unroll
+                for (int v = 0; v < U; v++) {
+                    const int x = x0 + v * NT + tid;
+                    pv[v] = make_float2(0.f, 0.f);
+                    ev[v] = 0;
+                    if (x < nb * per) {
+                        const int k = x / per, q = x - k * per;
+                        const int4 kt = s_kt[b0 + k];
+                        const int pos = q < ncolp ? kt.z * TJ + q : kt.y * TI + (q - ncolp);
+                        // the state after the move, read through the mirror map
+                        const int mp = (pos > i && pos <= j) ? i + j + 1 - pos : pos;
+                        pv[v] = P[mp];
+                        ev[v] = (pos == i) ? di : (pos == j) ? dj : E[(pos > i && pos < j) ? i + j - pos : pos];
+                    }
+                }
+#pragma unroll
+                for (int v = 0; v < U; v++) {
+                    const int x = x0 + v * NT + tid;
+                    if (x < nb * per) {
+                        const int k = x / per, q = x - k * per;
+                        const TileSmem tsm(reinterpret_cast<char*>(smem) + (size_t)k * tile_bytes, TJ, 32 * R);
+                        if (q < ncolp) {
+                            tsm.put(q, pv[v], (float)ev[v]);
+                        } else {
+                            const int rq = q - ncolp;
+                            const int ln = rq / R, sl = rq - ln * R;
+                            if (ln < 32) {
+                                tsm.rowp[ln * (R + 1) + sl] = pv[v];
+                                tsm.rowe[rq] = (float)ev[v];
+                            }
+                            if (sl == 0 && ln > 0) tsm.rowp[(ln - 1) * (R + 1) + R] = pv[v];
+                        }
+                    }
+                }
+            }
+            if (tid < nb) s_tmin[tid] = kKeyNone;
+            bar_items<NT>();
+            for (int it = wib; it < nb * nparts; it += nwi) {
+                const int k = it / nparts, part = it - k * nparts;
+                const int4 kt = s_kt[b0 + k];
+                const TileSmem tsm(reinterpret_cast<char*>(smem) + (size_t)k * tile_bytes, TJ, 32 * R);
+                const int I0 = kt.y * TI, J0 = kt.z * TJ, J1 = min(J0 + TJ, n);
+                const int jb = J0 + part * part_cols, je = min(jb + part_cols, J1);
+                if (jb < je) {
+                    const unsigned long long mk = sweep_part<R, FIRST>(I0, J0, jb, je, tsm, tflags);
+                    if (mk != kKeyNone) atomicMin(&s_tmin[k], mk);
+                }
+            }
+            bar_items<NT>();
+            if (tid < nb) {
+                const unsigned long long m = s_tmin[tid];
+                const int4 kt = s_kt[b0 + tid];
+                tb2[(long long)kt.y * ncc + kt.z] = m;
+                if (m != kKeyNone) atomicMin(key, m);
+            }
+            bar_items<NT>();
+        }
+    }
+}
+
+// The side warps' group minima for the sweep after move (i, j) (i < 0: none --
+// everything is dirty and was invalidated): one lane per group, the groups
+// that need their tiles read (invalid ones move m leaves clean: recomputed and
+// stored; partly dirty ones: their clean tiles) collected per warp and read by
+// the whole warp.  Returns the warp's minimum over the clean tiles (all lanes).
+__device__ __forceinline__ unsigned long long inc1_groups(unsigned long long* tb2, unsigned long long* sm2, int nrb,
+                                                          int ncc, int nsc, int TI, int TJ, int n, int i, int j,
+                                                          int gw, int nw)
+{
+    const int lane = threadIdx.x & 31;
+    const int rlo = i >= 1 ? (i - 1) / TI : 0, rhi = min(nrb - 1, j / TI);
+    const int clo = i >= 1 ? (i - 1) / TJ : 0, chi = min(ncc - 1, j / TJ);
+    const long long G = (long long)nrb * nsc;
+    unsigned long long m = kKeyNone;
+    // group g = gw + nw * (k0 + lane): consecutive groups (a whole invalid row block) on different warps
+    for (long long k0 = 0; gw + (long long)nw * k0 < G; k0 += 32) {
+        const long long g = gw + (long long)nw * (k0 + lane);
+        bool heavy = false, store = false;
+        if (g < G) {
+            const int rb = (int)(g / nsc), sc = (int)(g % nsc);
+            const int c0 = sc * kGroupChunks, c1 = min(c0 + kGroupChunks, ncc) - 1;
+            if (rb >= rlo && rb <= rhi) {
+                sm2[g] = kGroupInvalid;
+            } else if (c0 <= chi && c1 >= clo) {
+                if (c0 >= clo && c1 <= chi) sm2[g] = kGroupInvalid;
+                else {
+                    heavy = true;  // partly dirty: its clean tiles; stays invalid
+                    sm2[g] = kGroupInvalid;
+                }
+            } else {
+                const unsigned long long v = sm2[g];
+                if (v == kGroupInvalid) heavy = store = true;
+                else m = min(m, v);
+            }
+        }
+        unsigned hv = __ballot_sync(0xffffffffu, heavy);
+        const unsigned sv = __ballot_sync(0xffffffffu, store);
+        while (hv) {
+            const int src = __ffs(hv) - 1;
+            hv &= hv - 1;
+            const long long gg = gw + (long long)nw * (k0 + src);
+            const int rb = (int)(gg / nsc), sc = (int)(gg % nsc);
+            const unsigned long long* trow = tb2 + (long long)rb * ncc;
+            unsigned long long gm = kKeyNone;
+#pragma unroll
+            for (int h = 0; h < kGroupChunks / 32; h++) {
+                const int cc = sc * kGroupChunks + h * 32 + lane;
+                if (cc < ncc && (cc < clo || cc > chi)) gm = min(gm, trow[cc]);
+            }
+            for (int o = 16; o > 0; o >>= 1) gm = min(gm, __shfl_xor_sync(0xffffffffu, gm, o));
+            if (lane == src && ((sv >> src) & 1u)) sm2[gg] = gm;  // recomputed (all its tiles are clean)
+            m = min(m, gm);
+        }
+    }
+    for (int o = 16; o > 0; o >>= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
+    return m;
+}
+
+template <int R, bool FIRST>
+__global__ void __launch_bounds__(512, 1) inc_ls1_kernel(float2* P0, int* E0, int* T0, float2* P1, int* E1, int* T1,
+                                                         int n, int np, const int* __restrict__ tmap, int TI, int TJ,
+                                                         int nrb, int ncc, int nsc, Box* rboxA, Box* cboxA,
+                                                         Box* rboxB, Box* cboxB, unsigned long long* tb2,
+                                                         unsigned long long* sm2, unsigned long long* ctr,
+                                                         unsigned long long* keys3, Slot* slots, int parity,
+                                                         long long max_moves, long long budget, int* ctl, int flags,
+                                                         unsigned long long* trace, long long trace_cap,
+                                                         int tile_bytes, int part_cols)
+{
+    extern __shared__ float4 smem[];
+    constexpr int NT = 32 * (16 - kSideWarps);  // item threads per CTA
+    const int wib = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int gtid = blockIdx.x * blockDim.x + threadIdx.x, stride = gridDim.x * blockDim.x;
+    const bool side = wib >= 16 - kSideWarps;
+    const int gws = blockIdx.x * kSideWarps + (wib - (16 - kSideWarps)), nws = gridDim.x * kSideWarps;
+    const int gw = blockIdx.x * 16 + wib, nw = gridDim.x * 16;
+    const int tflags = (flags | kSweepLocal) & ~kSweepSeed;
+    __shared__ Slot s_in;
+    __shared__ int s_d[2];
+    unsigned long long target = 0;
+    float2 *Pc = P0, *Pa = P1;
+    int *Ec = E0, *Ea = E1, *Tc = T0, *Ta = T1;
+    Box *rbc = rboxA, *cbc = cboxA, *rba = rboxB, *cba = cboxB;
+    if (threadIdx.x == 0) {
+        s_in.done = *(volatile int*)&slots[parity].done;
+        s_in.moves = *(volatile long long*)&slots[parity].moves;
+        s_in.length = *(volatile long long*)&slots[parity].length;
+    }
+    __syncthreads();
+    if (s_in.done) {
+        if (gtid == 0) ctl[0] = parity;
+        return;  // uniform
+    }
+    long long moves = s_in.moves, length = s_in.length;
+    int done = 0;
+    unsigned long long klast = seed_key();
+    // prologue: every block's box (both buffers), alternate := current, all groups invalid
+    {
+        for (int task = gw; task < nrb + ncc; task += nw) {
+            if (task < nrb) {
+                const Box b = warp_box_mirror(Pc, Ec, task * TI, min(task * TI + TI, n - 1), -1, -1);
+                if (lane == 0) rbc[task] = rba[task] = b;
+            } else {
+                const int cc = task - nrb;
+                const Box b = warp_box_mirror(Pc, Ec, cc * TJ, min(cc * TJ + TJ, n), -1, -1);
+                if (lane == 0) cbc[cc] = cba[cc] = b;
+            }
+        }
+        for (long long g = gtid; g < (long long)nrb * nsc; g += stride) sm2[g] = kGroupInvalid;
+        for (int k = gtid; k < np; k += stride) {
+            Pa[k] = Pc[k];
+            Ea[k] = Ec[k];
+            Ta[k] = Tc[k];
+        }
+        if (gtid == 0) keys3[1] = seed_key();
+    }
+    grid_sync_mono(ctr, target);
+    int ip = -1, jp = -1;  // the previous move: where the two P / E / tour buffers differ
+    int kr = 0, kw = 1, kz = 2;
+    for (long long it = 0; it <= budget; it++) {
+        int i = -1, j = -1, di = 0, dj = 0;
+        bool apply = false;
+        if (it > 0) {  // decide move m from the completed key
+            if (threadIdx.x == 0) {
+                s_in.key = *(volatile unsigned long long*)&keys3[kr];
+                const int ki = key_i(s_in.key), kj = key_j(s_in.key);
+                s_d[0] = exact_dist_biased(Pc[ki], Pc[kj]);
+                s_d[1] = exact_dist_biased(Pc[ki + 1], Pc[kj + 1]);
+            }
+            __syncthreads();
+            const unsigned long long key = s_in.key;
+            klast = key;
+            if (key_delta(key) >= 0) done = 1;         // local minimum (reading R7)
+            else if (moves >= max_moves) done = 2;     // capped with an improving move left (R8)
+            else if (it == budget) done = 0;           // launch budget: the next launch resumes (full)
+            else apply = true;
+            if (!apply) break;  // uniform
+            i = key_i(key);
+            j = key_j(key);
+            di = s_d[0];
+            dj = s_d[1];
+            if (gtid == 0) {  // the exact delta (a first-improvement key carries a marker): thread 0 only
+                const int d = di + dj - Ec[i] - Ec[j];
+                klast = pack_key(d, i, j);
+                if (trace && moves < trace_cap) trace[moves] = klast;
+                length += d;
+            }
+            moves += 1;
+        }
+        if (gtid == 0) keys3[kz] = seed_key();  // read in the previous phase, written in the next
+        if (!side) {
+            inc1_items<R, FIRST, NT>(Pc, Ec, n, tmap, TI, TJ, nrb, ncc, i, j, di, dj, rbc, cbc, &keys3[kw], tb2,
+                                     tflags, part_cols, smem, tile_bytes);
+        } else if (apply) {
+            // (1) S_m into the alternate buffers: positions of moves m-1 and m
+            const int sid = gws * 32 + lane, sn = nws * 32;
+            const int n1 = j - i, n2 = ip >= 0 ? jp - ip : 0;
+            for (int t = sid; t < n1 + n2; t += sn) {
+                const int k = t < n1 ? i + 1 + t : ip + 1 + (t - n1);
+                const int mk = (k > i && k <= j) ? i + j + 1 - k : k;
+                Pa[k] = Pc[mk];
+                Ta[k] = Tc[mk];
+            }
+            const int m1 = j - i + 1, m2 = ip >= 0 ? jp - ip + 1 : 0;
+            for (int t = sid; t < m1 + m2; t += sn) {
+                const int k = t < m1 ? i + t : ip + (t - m1);
+                Ea[k] = k == i ? di : k == j ? dj : (k > i && k < j) ? Ec[i + j - k] : Ec[k];
+            }
+            // (2) S_m's exact boxes of the blocks move m dirties; move m-1's blocks copied over
+            {
+                const int rlo = i >= 1 ? (i - 1) / TI : 0, rhi = min(nrb - 1, j / TI);
+                const int clo = i >= 1 ? (i - 1) / TJ : 0, chi = min(ncc - 1, j / TJ);
+                const int nR = rhi - rlo + 1, nC = chi - clo + 1;
+                for (int task = gws; task < nR + nC; task += nws) {
+                    if (task < nR) {
+                        const int rb = rlo + task;
+                        const Box b = warp_box_mirror(Pc, Ec, rb * TI, min(rb * TI + TI, n - 1), i, j);
+                        if (lane == 0) rba[rb] = b;
+                    } else {
+                        const int cc = clo + task - nR;
+                        const Box b = warp_box_mirror(Pc, Ec, cc * TJ, min(cc * TJ + TJ, n), i, j);
+                        if (lane == 0) cba[cc] = b;
+                    }
+                }
+                if (ip >= 0) {
+                    const int qlo = ip >= 1 ? (ip - 1) / TI : 0, qhi = min(nrb - 1, jp / TI);
+                    const int plo = ip >= 1 ? (ip - 1) / TJ : 0, phi = min(ncc - 1, jp / TJ);
+                    const int sid2 = gws * 32 + lane;
+                    for (int t = sid2; t < (qhi - qlo + 1) + (phi - plo + 1); t += sn) {
+                        if (t <= qhi - qlo) {
+                            const int rb = qlo + t;
+                            if (rb < rlo || rb > rhi) rba[rb] = rbc[rb];
+                        } else {
+                            const int cc = plo + t - (qhi - qlo + 1);
+                            if (cc < clo || cc > chi) cba[cc] = cbc[cc];
+                        }
+                    }
+                }
+            }
+            // (3) the clean tiles' minima of S_m
+            const unsigned long long m = inc1_groups(tb2, sm2, nrb, ncc, nsc, TI, TJ, n, i, j, gws, nws);
+            if (lane == 0 && m != kKeyNone) atomicMin(&keys3[kw], m);
+        }
+        grid_sync_mono(ctr, target);
+        kr = (kr + 1) % 3;
+        kw = (kw + 1) % 3;
+        kz = (kz + 1) % 3;
+        if (apply) {
+            ip = i;
+            jp = j;
+            float2* tp = Pc;
+            Pc = Pa;
+            Pa = tp;
+            int* te = Ec;
+            Ec = Ea;
+            Ea = te;
+            int* tt = Tc;
+            Tc = Ta;
+            Ta = tt;
+            Box* tb = rbc;
+            rbc = rba;
+            rba = tb;
+            tb = cbc;
+            cbc = cba;
+            cba = tb;
+        }
+    }
+    // the handle's buffers: copy the last move's positions back if the current state is the alternate
+    if (Pc != P0 && ip >= 0) {
+        for (int t = gtid; t < jp - ip; t += stride) {
+            P0[ip + 1 + t] = Pc[ip + 1 + t];
+            T0[ip + 1 + t] = Tc[ip + 1 + t];
+        }
+        for (int t = gtid; t <= jp - ip; t += stride) E0[ip + t] = Ec[ip + t];
+    }
+    if (gtid == 0) {
+        Slot o;
+        o.key = seed_key();
+        o.last_key = klast;
+        o.moves = moves;
+        o.length = length;
+        o.done = done;
+        o.next_tile = 0;
+        o.ncull = 0;
+        o.seed_ok = 0;  // the next launch starts with a full sweep
+        o.mtype = 0;
+        slots[parity] = o;
+        ctl[0] = parity;
+    }
+}
+
+// ===========================================================================
 // Persistent dense local search with dynamic tile claims (medium n, one GPU):
 // one cooperative launch of one 16-warp CTA per SM; per iteration every WARP
 // claims tiles of the dense tiling from the slot's counter (largest first) and
@@ -1881,6 +2315,54 @@ cudaError_t launch_inc_ls2(const Geometry& g, float2* P, int* E, int* tour, floa
                     &TI,  &TJ,  &nrb,  &ncc,   &nsc,       &rbox,  &cbox,    &tb2,       &sm2,
                     &ctr, &slots, &parity, &max_moves, &budget, &full, &ctl, &flags, &trace,
                     &trace_cap, &tile_bytes, &part_cols};
+    g_launches += 1;
+    return cudaLaunchCooperativeKernel((const void*)kern, dim3(sms), dim3(kIncLsThreads), args, smem, st);
+}
+
+size_t inc_ls1_ws_bytes(const Geometry& g, int n)
+{
+    const int TI = g.ti(), nrb = (n - 1 + TI - 1) / TI, ncc = (n + g.tj - 1) / g.tj;
+    const int nsc = (ncc + kGroupChunks - 1) / kGroupChunks;
+    const size_t words = (4 + 4 + (size_t)nrb * ncc + (size_t)nrb * nsc + 3) / 4 * 4;  // boxes 32-byte aligned
+    return sizeof(unsigned long long) * words + sizeof(Box) * 2 * ((size_t)nrb + ncc);
+}
+
+cudaError_t launch_inc_ls1(const Geometry& g, float2* P, int* E, int* tour, float2* P1, int* E1, int* T1, int n,
+                           int np, const int* tmap, void* ws, Slot* slots, int parity, long long max_moves,
+                           long long budget, int* ctl, int flags, unsigned long long* trace, long long trace_cap,
+                           int part_cols, cudaStream_t st)
+{
+    if (g.rows != kRowsSmall || g.warps != 1) return cudaErrorInvalidValue;
+    int TI = g.ti(), TJ = g.tj, nrb = (n - 1 + TI - 1) / TI, ncc = (n + TJ - 1) / TJ;
+    int nsc = (ncc + kGroupChunks - 1) / kGroupChunks;
+    unsigned long long* ctr = static_cast<unsigned long long*>(ws);
+    unsigned long long* keys3 = ctr + 4;
+    unsigned long long* tb2 = keys3 + 4;
+    unsigned long long* sm2 = tb2 + (size_t)nrb * ncc;
+    const size_t words = (4 + 4 + (size_t)nrb * ncc + (size_t)nrb * nsc + 3) / 4 * 4;  // Box is 32-byte aligned
+    Box* rboxA = reinterpret_cast<Box*>(ctr + words);
+    Box* cboxA = rboxA + nrb;
+    Box* rboxB = cboxA + ncc;
+    Box* cboxB = rboxB + nrb;
+    int tile_bytes = (int)((sweep_smem_bytes_ps(g) + 15) / 16 * 16);
+    const size_t smem = (size_t)tile_bytes * kStageTiles;
+    auto kern = (flags & kSweepFirst) ? inc_ls1_kernel<kRowsSmall, true> : inc_ls1_kernel<kRowsSmall, false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kIncLsThreads, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) return cudaErrorInvalidConfiguration;
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    part_cols = part_cols > 0 ? std::min(part_cols, TJ) : kIncPartCols;
+    e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long), st);
+    if (e != cudaSuccess) return e;
+    void* args[] = {&P,     &E,     &tour,  &P1,    &E1,       &T1,    &n,      &np,        &tmap,   &TI,
+                    &TJ,    &nrb,   &ncc,   &nsc,   &rboxA,    &cboxA, &rboxB,  &cboxB,     &tb2,    &sm2,
+                    &ctr,   &keys3, &slots, &parity, &max_moves, &budget, &ctl,  &flags,     &trace,  &trace_cap,
+                    &tile_bytes, &part_cols};
     g_launches += 1;
     return cudaLaunchCooperativeKernel((const void*)kern, dim3(sms), dim3(kIncLsThreads), args, smem, st);
 }

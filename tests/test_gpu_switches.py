@@ -77,11 +77,13 @@ def _inc_case(first, start, cap):
     return c, t, ls(c, t, max_iters=cap, trace_cap=20000)
 
 
-@pytest.mark.parametrize("barriers,part", [("2", "1"), ("2", "2"), ("2", "4"), ("2", "16"), ("3", "0"), ("3", "4")])
+@pytest.mark.parametrize("barriers,part", [("1", "1"), ("1", "4"), ("1", "16"), ("2", "1"), ("2", "2"), ("2", "4"),
+                                           ("2", "16"), ("3", "0"), ("3", "4")])
 @pytest.mark.parametrize("first", [0, 1])
 @pytest.mark.parametrize("start,cap", [("hilbert", -1), ("random", 400)])
 def test_incremental_persistent_variants(gpu, monkeypatch, barriers, part, first, start, cap):
-    """The persistent incremental search (TSP2OPT_OPT_TILE_BOUNDS = 3): two barriers per move with the
+    """The persistent incremental search (TSP2OPT_OPT_TILE_BOUNDS = 3): one barrier per move (the dirty
+    tiles swept from the pre-move state through the mirror map, conservative boxes), two with the
     out-of-place apply and group minima, or three with the in-place apply; kept tiles split into column
     parts of 1 / 2 / 4 / 16 columns or swept whole -- every move equal to the oracle's, with a move cap
     that ends a search mid-way (the alternate buffer copied back) and (best improvement) a resumed search
