@@ -618,7 +618,11 @@ int run_local_search(tsp2opt_ctx* h, long long max_iters)
     // Dense loop (TILE_BOUNDS 1 by default, n ~ 7e3) until the tour is coherent, then the
     // incremental search (measured, C3: profiles/r02_exp_c3_switch.jsonl).
     const bool auto_inc = inc_ok && h->auto_inc && h->tile_bounds == 1 && !use_persistent && !use_dense_ls;
-    auto coherent = [&]() { return (double)h->h_slot->length < kAutoIncRho * h->rho_unit; };
+    static const double auto_rho = [] {
+        const char* e = getenv("TSP2OPT_AUTO_INC_RHO");  // experiment: the hand-over threshold
+        return e ? atof(e) : kAutoIncRho;
+    }();
+    auto coherent = [&]() { return (double)h->h_slot->length < auto_rho * h->rho_unit; };
     if (auto_inc) {
         rc = read_slot(h);
         if (rc) return rc;
