@@ -1478,7 +1478,10 @@ __global__ void __launch_bounds__(512, 1) inc_ls2_kernel(float2* P0, int* E0, in
 // the two- and three-barrier kernels.  A launch starts with a full sweep of its
 // state and leaves seed_ok = 0 (the next launch starts full).
 // ===========================================================================
-constexpr int kSideWarps = 4;                 // inc_ls1: per CTA, the rest sweep
+#ifndef TSP2OPT_SIDE_WARPS
+#define TSP2OPT_SIDE_WARPS 4
+#endif
+constexpr int kSideWarps = TSP2OPT_SIDE_WARPS;  // inc_ls1: per CTA, the rest sweep
 constexpr unsigned long long kGroupInvalid = 0;  // not a key (delta + 2^18 > 0): "recompute this group"
 
 // Conservative box of block `b` (positions [b*B, min(b*B + B, last)], edges up
