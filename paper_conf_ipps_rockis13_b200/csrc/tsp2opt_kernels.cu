@@ -1479,7 +1479,7 @@ __global__ void __launch_bounds__(512, 1) inc_ls2_kernel(float2* P0, int* E0, in
 // state and leaves seed_ok = 0 (the next launch starts full).
 // ===========================================================================
 #ifndef TSP2OPT_SIDE_WARPS
-#define TSP2OPT_SIDE_WARPS 4
+#define TSP2OPT_SIDE_WARPS 2  // measured: 2 of 16 warps for the apply, boxes and group minima beat 4 and 1
 #endif
 constexpr int kSideWarps = TSP2OPT_SIDE_WARPS;  // inc_ls1: per CTA, the rest sweep
 constexpr unsigned long long kGroupInvalid = 0;  // not a key (delta + 2^18 > 0): "recompute this group"
@@ -2359,7 +2359,9 @@ cudaError_t launch_inc_ls1(const Geometry& g, float2* P, int* E, int* tour, floa
     int dev = 0, sms = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    part_cols = part_cols > 0 ? std::min(part_cols, TJ) : kIncPartCols;
+    // parts of a quarter tile, at least 4 columns (measured with one barrier: 8 of 32 columns, C5 MF 17.4
+    // vs 18.3 us per move with 4; profiles/r02_exp_inc_parts.jsonl)
+    part_cols = part_cols > 0 ? std::min(part_cols, TJ) : std::max(kIncPartCols, TJ / 4);
     e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long), st);
     if (e != cudaSuccess) return e;
     void* args[] = {&P,     &E,     &tour,  &P1,    &E1,       &T1,    &n,      &np,        &tmap,   &TI,
