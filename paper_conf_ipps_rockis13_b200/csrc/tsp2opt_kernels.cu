@@ -1458,7 +1458,7 @@ __global__ void __launch_bounds__(512, 1) inc_ls2_kernel(float2* P0, int* E0, in
 // Persistent incremental local search, ONE grid barrier per move
 // (inc_ls1_kernel).  Phase m decides move m from the key the previous phase
 // completed, then, all reading only the pre-move state S_{m-1}:
-//   * item warps (12 per CTA) cull the tiles move m dirties, stage the kept
+//   * item warps (14 per CTA) cull the tiles move m dirties, stage the kept
 //     ones through the reversal's mirror map (new P[k] = P[i+j+1-k] on
 //     [i+1, j], new e[k] = e[i+j-k] on (i, j), the two new edges) and sweep
 //     them in column parts: the minima of S_m, written to the dense tile
@@ -1467,7 +1467,7 @@ __global__ void __launch_bounds__(512, 1) inc_ls2_kernel(float2* P0, int* E0, in
 //     blocks its new cities and edges come from, and the largest of their
 //     edges and the two new ones -- a superset of what S_m's exact boxes keep,
 //     so every tile that can hold an improving pair is swept;
-//   * side warps (4 per CTA) write S_m into the other P / E / tour buffer (the
+//   * side warps (2 per CTA) write S_m into the other P / E / tour buffer (the
 //     positions of moves m-1 and m), compute S_m's exact boxes of the dirty
 //     blocks into the other box buffer (copying the blocks move m-1 dirtied),
 //     and fold the clean tiles' minima into the next key through the group
