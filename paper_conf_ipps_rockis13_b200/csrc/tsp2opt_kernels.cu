@@ -1463,10 +1463,11 @@ __global__ void __launch_bounds__(512, 1) inc_ls2_kernel(float2* P0, int* E0, in
 //     [i+1, j], new e[k] = e[i+j-k] on (i, j), the two new edges) and sweep
 //     them in column parts: the minima of S_m, written to the dense tile
 //     minima and the next key.  The cull uses CONSERVATIVE boxes for the
-//     dirty blocks: the union of the stored boxes of the block and of the
-//     blocks its new cities and edges come from, and the largest of their
-//     edges and the two new ones -- a superset of what S_m's exact boxes keep,
-//     so every tile that can hold an improving pair is swept;
+//     dirty blocks: the union of the stored boxes of the blocks its new
+//     cities and edges come from (and of the block itself unless the move
+//     replaces all of it), and the largest of their edges and the two new
+//     ones -- a superset of what S_m's exact boxes keep, so every tile that
+//     can hold an improving pair is swept;
 //   * side warps (2 per CTA) write S_m into the other P / E / tour buffer (the
 //     positions of moves m-1 and m), compute S_m's exact boxes of the dirty
 //     blocks into the other box buffer (copying the blocks move m-1 dirtied),
