@@ -317,4 +317,33 @@ __device__ __forceinline__ void grid_sync(unsigned* bar, unsigned nblocks)
     __syncthreads();
 }
 
+#ifndef TSP2OPT_BAR_ACQREL
+#define TSP2OPT_BAR_ACQREL 1  // measured 2 % faster per move than two __threadfence()s (MEMBAR.ALL vs .SC)
+#endif
+// Grid barrier on a monotonic 64-bit arrival counter (reset to 0 before the
+// launch; every barrier of the launch adds gridDim.x): one atomic per CTA and
+// polling, no reset round trips.  `target` is the CTA's running count.
+__device__ __forceinline__ void grid_sync_mono(unsigned long long* ctr, unsigned long long& target)
+{
+    __syncthreads();
+    target += gridDim.x;
+    if (threadIdx.x == 0) {
+#if TSP2OPT_BAR_ACQREL
+        // release-add / acquire-poll at gpu scope instead of two full fences
+        asm volatile("red.release.gpu.global.add.u64 [%0], 1;" ::"l"(ctr) : "memory");
+        unsigned long long v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(ctr) : "memory");
+        } while (v < target);
+#else
+        __threadfence();
+        atomicAdd(ctr, 1ULL);
+        while (*(volatile unsigned long long*)ctr < target) {
+        }
+        __threadfence();
+#endif
+    }
+    __syncthreads();
+}
+
 }  // namespace tsp2opt

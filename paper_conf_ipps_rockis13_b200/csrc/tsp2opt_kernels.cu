@@ -665,6 +665,8 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
     const int gtid = blockIdx.x * blockDim.x + threadIdx.x;
     const int stride = gridDim.x * blockDim.x;
     int p = parity;
+    unsigned long long target = 0;  // monotonic barrier on bar (reset to 0 before the launch)
+    unsigned long long* ctr = reinterpret_cast<unsigned long long*>(bar);
     for (long long it = 0; it < budget; it++) {
         Slot* in = slots + p;
         // one read of the settled state per block (not one per thread: a single hot address)
@@ -676,7 +678,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
             sweep_tile<R, true>(P, E, n, tiles[t], TJ, in, sm, tilebest + t, flags);
             __syncthreads();  // before the next tile overwrites the shared chunk
         }
-        grid_sync(bar, gridDim.x);
+        grid_sync_mono(ctr, target);
         if (threadIdx.x == 0) {
             s_in.key = *(volatile unsigned long long*)&in->key;
             s_in.last_key = in->last_key;
@@ -688,7 +690,7 @@ __global__ void __launch_bounds__(128, TSP2OPT_MINB) local_search_kernel(float2*
         __syncthreads();
         apply_phase(P, E, tour, &s_in, slots + (p ^ 1), max_moves, 0, 0, 0, gtid, stride, trace, trace_cap, nullptr);
         p ^= 1;
-        grid_sync(bar, gridDim.x);
+        grid_sync_mono(ctr, target);
     }
     if (gtid == 0) ctl[0] = p;
 }
@@ -1224,35 +1226,6 @@ __device__ __forceinline__ unsigned long long group_minima(const unsigned long l
     }
     for (int o = 16; o > 0; o >>= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
     return m;
-}
-
-#ifndef TSP2OPT_BAR_ACQREL
-#define TSP2OPT_BAR_ACQREL 1  // measured 2 % faster per move than two __threadfence()s (MEMBAR.ALL vs .SC)
-#endif
-// Grid barrier on a monotonic 64-bit arrival counter (reset to 0 before the
-// launch; every barrier of the launch adds gridDim.x): one atomic per CTA and
-// polling, no reset round trips.  `target` is the CTA's running count.
-__device__ __forceinline__ void grid_sync_mono(unsigned long long* ctr, unsigned long long& target)
-{
-    __syncthreads();
-    target += gridDim.x;
-    if (threadIdx.x == 0) {
-#if TSP2OPT_BAR_ACQREL
-        // release-add / acquire-poll at gpu scope instead of two full fences
-        asm volatile("red.release.gpu.global.add.u64 [%0], 1;" ::"l"(ctr) : "memory");
-        unsigned long long v;
-        do {
-            asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(ctr) : "memory");
-        } while (v < target);
-#else
-        __threadfence();
-        atomicAdd(ctr, 1ULL);
-        while (*(volatile unsigned long long*)ctr < target) {
-        }
-        __threadfence();
-#endif
-    }
-    __syncthreads();
 }
 
 constexpr int kBoxWarps = 4;  // (X): warps per CTA computing boxes; the others scan the group minima
@@ -2284,6 +2257,8 @@ cudaError_t launch_inc_ls(const Geometry& g, float2* P, int* E, int* tour, int n
     // sweeps each whole kept tile)
     part_cols = std::min(std::max(part_cols, 0), TJ);
     if (flags & kSweepTileBounds) flags |= kSweepPartBounds;
+    e = cudaMemsetAsync(bar, 0, 2 * sizeof(unsigned), st);  // count 0 (local_search_kernel leaves a counter)
+    if (e != cudaSuccess) return e;
     void* args[] = {&P,     &E,    &tour,   &n,        &tiles,    &ntiles,    &tmap,   &TI,
                     &TJ,    &nrb,  &ncc,    &rbox,     &cbox,     &slots,     &parity, &max_moves,
                     &budget, &full, &bar,   &ctl,      &tilebest, &flags,     &trace,  &trace_cap,
@@ -2404,6 +2379,8 @@ cudaError_t launch_dense_ls(const Geometry& g, float2* P, int* E, int* tour, int
     int dev = 0, sms = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    e = cudaMemsetAsync(bar, 0, 2 * sizeof(unsigned), st);  // count 0 (local_search_kernel leaves a counter)
+    if (e != cudaSuccess) return e;
     void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &TJ, &slots, &parity, &max_moves, &budget, &bar, &ctl,
                     &flags, &tilebest, &trace, &trace_cap, &tile_bytes};
     g_launches += 1;
@@ -2498,6 +2475,10 @@ cudaError_t launch_local_search(const Geometry& g, float2* P, int* E, int* tour,
     int grid = local_search_grid(g, ntiles);
     if (grid < 1) return cudaErrorInvalidConfiguration;
     int TJ = g.tj;
+    // the barrier's arrival counter (the other persistent kernels' (count, generation) pair reads as
+    // count 0 after this as well)
+    cudaError_t e = cudaMemsetAsync(bar, 0, 2 * sizeof(unsigned), st);
+    if (e != cudaSuccess) return e;
     void* args[] = {&P, &E, &tour, &n, &tiles, &ntiles, &TJ, &slots, &parity, &max_moves, &budget, &bar, &ctl,
                     &tilebest, &flags, &trace, &trace_cap};
     g_launches += 1;
