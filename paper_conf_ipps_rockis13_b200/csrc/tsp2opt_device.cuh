@@ -346,4 +346,23 @@ __device__ __forceinline__ void grid_sync_mono(unsigned long long* ctr, unsigned
     __syncthreads();
 }
 
+// Grid barrier on a monotonic 64-bit counter that is never reset: the arrival's
+// old value gives the generation (every launch on the counter uses the same grid
+// and passes every barrier, so the counter is a multiple of the grid between
+// launches).  Release-add / acquire-poll at gpu scope, as grid_sync_mono.
+__device__ __forceinline__ void grid_sync_gen(unsigned long long* ctr)
+{
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long old;
+        asm volatile("atom.release.gpu.global.add.u64 %0, [%1], 1;" : "=l"(old) : "l"(ctr) : "memory");
+        const unsigned long long target = (old / gridDim.x + 1) * gridDim.x;
+        unsigned long long v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(ctr) : "memory");
+        } while (v < target);
+    }
+    __syncthreads();
+}
+
 }  // namespace tsp2opt

@@ -484,12 +484,12 @@ __global__ void __launch_bounds__(256) apply25_kernel(float2* __restrict__ P, in
     const int i = s_i, j = s_j, t = s_t;
     if (!s_apply) return;  // grid-uniform: every block decided the same
     const int gtid = blockIdx.x * blockDim.x + threadIdx.x, stride = gridDim.x * blockDim.x;
-    grid_sync(bar, gridDim.x);  // all blocks have read the pre-move state
+    grid_sync_gen(reinterpret_cast<unsigned long long*>(bar));  // all blocks have read the pre-move state
     reverse_range(P, tour, i + 1, j, gtid, stride);
-    grid_sync(bar, gridDim.x);
+    grid_sync_gen(reinterpret_cast<unsigned long long*>(bar));
     if (t == 1) reverse_range(P, tour, i + 1, j - 1, gtid, stride);
     else if (t == 2) reverse_range(P, tour, i + 2, j, gtid, stride);
-    grid_sync(bar, gridDim.x);
+    grid_sync_gen(reinterpret_cast<unsigned long long*>(bar));
     for (int k = i + gtid; k <= j; k += stride) E[k] = exact_dist_biased(__ldcg(P + k), __ldcg(P + k + 1));
     for (int x = i + gtid; x <= j + 1; x += stride) {
         const int k = x == n ? 0 : x;
